@@ -1,0 +1,193 @@
+"""ORACLE — TEST INFRASTRUCTURE ONLY (see oracle/sq_oracle.c header).
+
+Thin numpy/ctypes wrapper over liboracle.so plus the sequential pipeline
+simulation O7.  Only tests/, __graft_entry__.smoke()
+and bench.py's cpu_baseline / --impl reference legs may import this module.
+It never imports the CUDA package, and the CUDA package never imports it.
+
+Functions whose pin is missing are marked "parity unpinned" (none at present;
+throughput has no paper number to pin).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "liboracle.so")
+_SRC = os.path.join(_HERE, "sq_oracle.c")
+CFLAGS = ["-O2", "-fopenmp", "-ffp-contract=off", "-fno-fast-math", "-fPIC", "-shared", "-std=gnu11"]
+
+
+def build(force: bool = False) -> str:
+    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
+        subprocess.check_call(["gcc", *CFLAGS, _SRC, "-o", _SO, "-lm"])
+    return _SO
+
+
+_L = None
+P = ctypes.c_void_p
+I64 = ctypes.c_int64
+
+
+def _lib() -> ctypes.CDLL:
+    global _L
+    if _L is None:
+        L = ctypes.CDLL(build())
+        L.oq_quantize_groups.argtypes = [P, I64, I64, ctypes.c_int, ctypes.c_int, P, P, P]
+        L.oq_pack.argtypes = [P, P, P, I64, I64, ctypes.c_int, ctypes.c_int, P, P]
+        L.oq_unpack.argtypes = [P, I64, I64, ctypes.c_int, P]
+        L.oq_dequant.argtypes = [P, P, I64, I64, ctypes.c_int, ctypes.c_int, P]
+        L.oq_linear.argtypes = [P, I64, I64, P, P, I64, ctypes.c_int, ctypes.c_int, P, P]
+        L.oq_layernorm.argtypes = [P, I64, I64, ctypes.c_double, P]
+        L.oq_layernorm.restype = None
+        L.oq_stage.argtypes = [P, ctypes.c_int, P, I64, I64, P]
+        L.oq_packed_bytes.argtypes = [I64, I64, ctypes.c_int]
+        L.oq_packed_bytes.restype = ctypes.c_size_t
+        _L = L
+    return _L
+
+
+def _p(a: np.ndarray | None):
+    return None if a is None else a.ctypes.data_as(ctypes.c_void_p)
+
+
+def _check(rc: int, what: str) -> None:
+    if rc != 0:
+        raise RuntimeError(f"oracle {what} failed rc={rc}")
+
+
+def quantize_groups(w: np.ndarray, bits: int, group: int = 128):
+    """O1.  w fp16 [n, k] -> (codes u8 [n,k], scales fp16 [n,k/g], zeros fp16 [n,k/g])."""
+    w = np.ascontiguousarray(w, dtype=np.float16)
+    n, k = w.shape
+    codes = np.empty((n, k), np.uint8)
+    s = np.empty((n, k // group), np.float16)
+    z = np.empty((n, k // group), np.float16)
+    _check(_lib().oq_quantize_groups(_p(w), n, k, bits, group, _p(codes), _p(s), _p(z)), "quantize")
+    return codes, s, z
+
+
+def pack(codes: np.ndarray, scales: np.ndarray, zeros: np.ndarray, bits: int, group: int = 128):
+    """O2 (DESIGN.md layouts).  -> (packed u8 [n, k*bits/8], meta u32 [k/g, n])."""
+    codes = np.ascontiguousarray(codes, np.uint8)
+    n, k = codes.shape
+    packed = np.empty((n, k * bits // 8), np.uint8)
+    meta = np.empty((k // group, n), np.uint32)
+    _check(_lib().oq_pack(_p(codes), _p(np.ascontiguousarray(scales, np.float16)),
+                          _p(np.ascontiguousarray(zeros, np.float16)), n, k, bits, group,
+                          _p(packed), _p(meta)), "pack")
+    return packed, meta
+
+
+def unpack(packed: np.ndarray, n: int, k: int, bits: int) -> np.ndarray:
+    """O3: inverse of the code packing."""
+    packed = np.ascontiguousarray(packed, np.uint8)
+    codes = np.empty((n, k), np.uint8)
+    _check(_lib().oq_unpack(_p(packed), n, k, bits, _p(codes)), "unpack")
+    return codes
+
+
+def packed_bytes(n: int, k: int, bits: int) -> int:
+    return int(_lib().oq_packed_bytes(n, k, bits))
+
+
+class QWeight:
+    """Oracle-side quantized linear: packed codes + meta (or fp16 W at bits 16)."""
+
+    def __init__(self, w16: np.ndarray, bits: int, group: int = 128, bias: np.ndarray | None = None):
+        self.n, self.k = w16.shape
+        self.bits, self.group = bits, group
+        self.bias = None if bias is None else np.ascontiguousarray(bias, np.float16)
+        if bits == 16:
+            self.packed = np.ascontiguousarray(w16, np.float16).view(np.uint8)
+            self.meta = None
+            self.codes = self.scales = self.zeros = None
+        else:
+            self.codes, self.scales, self.zeros = quantize_groups(w16, bits, group)
+            self.packed, self.meta = pack(self.codes, self.scales, self.zeros, bits, group)
+
+    def dequant(self) -> np.ndarray:
+        """O4: W~ in fp64 [n, k]."""
+        out = np.empty((self.n, self.k), np.float64)
+        _check(_lib().oq_dequant(_p(self.packed), _p(self.meta), self.n, self.k, self.bits,
+                                 self.group, _p(out)), "dequant")
+        return out
+
+    def c_struct(self):
+        return _OqWeight(self.bits, self.group, self.n, self.k, _p(self.packed), _p(self.meta), _p(self.bias))
+
+
+def linear(x: np.ndarray, qw: QWeight) -> np.ndarray:
+    """O5: y = x W~^T (+bias) in fp64.  x: [m, k] (any float dtype, taken exactly)."""
+    x = np.ascontiguousarray(x, np.float64)
+    m, k = x.shape
+    assert k == qw.k
+    y = np.empty((m, qw.n), np.float64)
+    _check(_lib().oq_linear(_p(x), m, k, _p(qw.packed), _p(qw.meta), qw.n, qw.bits, qw.group,
+                            _p(qw.bias), _p(y)), "linear")
+    return y
+
+
+def layernorm(x: np.ndarray, eps: float = 1e-5) -> np.ndarray:
+    x = np.ascontiguousarray(x, np.float64)
+    out = np.empty_like(x)
+    _lib().oq_layernorm(_p(x), x.shape[0], x.shape[1], eps, _p(out))
+    return out
+
+
+class _OqWeight(ctypes.Structure):
+    _fields_ = [("bits", ctypes.c_int32), ("group", ctypes.c_int32), ("n", ctypes.c_int64),
+                ("k", ctypes.c_int64), ("packed", ctypes.c_void_p), ("meta", ctypes.c_void_p),
+                ("bias", ctypes.c_void_p)]
+
+
+class _OqLayer(ctypes.Structure):
+    _fields_ = [("bits", ctypes.c_int32), ("act", ctypes.c_int32), ("qkv", _OqWeight),
+                ("o", _OqWeight), ("fc1", _OqWeight), ("fc2", _OqWeight)]
+
+
+class Layer:
+    """Oracle decoder layer (P:160 linear set; R11/R12)."""
+
+    def __init__(self, bits: int, act: int, qkv: QWeight, o: QWeight, fc1: QWeight, fc2: QWeight):
+        self.bits, self.act = bits, act
+        self.qkv, self.o, self.fc1, self.fc2 = qkv, o, fc1, fc2
+
+    def c_struct(self):
+        return _OqLayer(self.bits, self.act, self.qkv.c_struct(), self.o.c_struct(),
+                        self.fc1.c_struct(), self.fc2.c_struct())
+
+
+def stage(layers: list[Layer], x: np.ndarray, want_qkv: bool = False):
+    """O6: run consecutive layers on x fp64 [t, h1]; returns (x_out, qkv of last layer | None)."""
+    x = np.array(x, dtype=np.float64, order="C", copy=True)
+    t, h1 = x.shape
+    arr = (_OqLayer * len(layers))(*[L.c_struct() for L in layers])
+    qkv = np.empty((t, 3 * h1), np.float64) if want_qkv else None
+    _check(_lib().oq_stage(arr, len(layers), _p(x), t, h1, _p(qkv)), "stage")
+    return x, qkv
+
+
+def pipeline(layers: list[Layer], x0: np.ndarray, n_decode: int) -> np.ndarray:
+    """O7: sequential simulation of the pipelined generation (R13/R14).
+
+    x0: fp32/fp64 embeddings [B, s, h1].  Prefill runs every prompt row through all
+    layers (rows are independent under the attention stub, so micro-batching and the
+    stage partition cannot change the result).  out[b, 0] = hidden at the last prompt
+    position; decode input e_1 = LN(out[b, 0]); out[b, t] = F(e_t), e_{t+1} = LN(out[b, t]).
+    Returns out [B, 1 + n_decode, h1] in fp64."""
+    B, s, h1 = x0.shape
+    # prefill only needs the last prompt position of each sequence (rows independent)
+    last = np.ascontiguousarray(x0[:, s - 1, :], np.float64)
+    out = np.empty((B, 1 + n_decode, h1), np.float64)
+    h, _ = stage(layers, last)
+    out[:, 0] = h
+    for t in range(1, n_decode + 1):
+        e = layernorm(out[:, t - 1])
+        h, _ = stage(layers, e)
+        out[:, t] = h
+    return out

@@ -1,0 +1,303 @@
+/*
+ * ORACLE — TEST INFRASTRUCTURE ONLY.  Plain, slow, obviously-correct CPU
+ * reference for the SplitQuant hot path (DESIGN.md
+ * "Oracle").  Only tests/, __graft_entry__.smoke() and bench.py's
+ * cpu_baseline / --impl reference legs may load it.  It shares no code with
+ * the CUDA path (paper_conf_cluster_zhaowplw25_b200/csrc); neither side
+ * includes or calls the other.
+ *
+ * Build: gcc -O2 -fopenmp -ffp-contract=off -fno-fast-math -shared -fPIC
+ * (no FMA contraction: the quantizer is defined by single-rounded IEEE fp32
+ * operations, one rounding per operation).
+ *
+ * Citations are PAPER.md line numbers ("P:<line>") in /root/reference.
+ *
+ * Functions and what pins them (tests/test_oracle_pins.py):
+ *   oq_quantize_groups  P:91 (x^ = round((x - q_x)/s_x), s_x = (x_max - x_min)/(2^b - 1)),
+ *                       asymmetric S_W of P:184; readings R1-R6 of DESIGN.md.
+ *                       Pinned by brute-force argmin, |w - w~| <= s/2, grid-aligned
+ *                       recovery, constant groups, closed-form scale bound.
+ *   oq_pack/oq_unpack   Layout L3/L4/L8 of DESIGN.md (paper silent).  Pinned by
+ *                       hand-derived golden words (tests/golden/pack_words.txt),
+ *                       round trip, and the P:160 byte count.
+ *   oq_dequant_row      x~ = s_x x^ + q_x, exact in fp64.
+ *   oq_linear           y = x W~^T (+ bias) in fp64 (weight-only W.A16).  Pinned by
+ *                       numpy fp64 matmul at bits = 16 and on grid-aligned weights,
+ *                       Theorem 1 variance bound.
+ *   oq_layernorm        pre-LN block glue (R11), pinned by mean 0 / var 1.
+ *   oq_stage            one pipeline stage = layers of P:160's linear set with the
+ *                       attention stub (R12); pinned by composition checks.
+ */
+#include <math.h>
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+
+/* ---------------- fp16 <-> fp32 (IEEE binary16, round-to-nearest-even) ---------------- */
+static float h2f(uint16_t h) {
+  _Float16 v;
+  memcpy(&v, &h, 2);
+  return (float)v;
+}
+static uint16_t f2h(float f) {
+  _Float16 v = (_Float16)f; /* RNE */
+  uint16_t h;
+  memcpy(&h, &v, 2);
+  return h;
+}
+
+float oq_h2f(uint16_t h) { return h2f(h); }
+uint16_t oq_f2h(float f) { return f2h(f); }
+
+/* ---------------- O1: round-to-nearest per-group min/max quantization ----------------
+ * x^ = round((x - q_x) / s_x),  s_x = (x_max - x_min) / (2^b - 1),  x~ = s_x x^ + q_x.
+ * Group = `group` contiguous weights of one output row (reading R4).  All arithmetic is
+ * IEEE binary32 with one rounding per operation; the code is computed against the
+ * fp16-ROUNDED scale that is stored (R5); q_x = group minimum (R3, fp16 exact, -0 -> +0);
+ * ties round half to even (R1); s == 0 (constant group or underflow) gives code 0 (R6).
+ */
+int oq_quantize_groups(const uint16_t* w, int64_t n, int64_t k, int bits, int group,
+                       uint8_t* codes, uint16_t* scales, uint16_t* zeros) {
+  if (!(bits == 3 || bits == 4 || bits == 8) || group <= 0 || k % group) return 1;
+  const int64_t ng = k / group;
+  const int qmax_i = (1 << bits) - 1;
+  const float qmax = (float)qmax_i;
+  for (int64_t r = 0; r < n; ++r) {
+    for (int64_t g = 0; g < ng; ++g) {
+      const uint16_t* p = w + r * k + g * group;
+      float mn = h2f(p[0]), mx = mn;
+      for (int j = 1; j < group; ++j) {
+        float v = h2f(p[j]);
+        if (v < mn) mn = v;
+        if (v > mx) mx = v;
+      }
+      mn = mn + 0.0f;                       /* canonical zeros: -0 -> +0 */
+      mx = mx + 0.0f;
+      float sf = (mx - mn) / qmax;          /* two single-rounded fp32 ops */
+      uint16_t s16 = f2h(sf);
+      float s = h2f(s16);
+      scales[r * ng + g] = s16;
+      zeros[r * ng + g] = f2h(mn);          /* exact: mn is an fp16 value */
+      for (int j = 0; j < group; ++j) {
+        int c = 0;
+        if (s != 0.0f) {
+          float d = (h2f(p[j]) - mn) / s;   /* fp32 sub, fp32 div */
+          float q = rintf(d);               /* round half to even */
+          if (q < 0.0f) q = 0.0f;
+          if (q > qmax) q = qmax;
+          c = (int)q;
+        }
+        codes[r * k + g * group + j] = (uint8_t)c;
+      }
+    }
+  }
+  return 0;
+}
+
+/* ---------------- O2/O3: bit packing (DESIGN.md layouts L8, L4, L3) ----------------
+ * Rows are contiguous, row pitch = k*bits/8 bytes, codes in k order within a row.
+ * L8: byte k.
+ * L4: 32-bit little-endian word k/8, nibble (k%8)/2 + 4*(k%2)   (even k in the low
+ *     four nibbles, odd k in the high four).
+ * L3: blocks of 32 codes = 3 words [L0, L1, H]; for k' = k%32: a = k'/16,
+ *     i = (k'%16)/2, e = k'%2; low two bits at word La, bits 2i + 16e;
+ *     high bit at word H, bit i + 8a + 16e.
+ * meta: uint32 [k/group][n], low half = scale, high half = zero (group-major).
+ */
+size_t oq_packed_bytes(int64_t n, int64_t k, int bits) { return (size_t)(n * k * bits / 8); }
+
+int oq_pack(const uint8_t* codes, const uint16_t* scales, const uint16_t* zeros, int64_t n,
+            int64_t k, int bits, int group, uint8_t* packed, uint32_t* meta) {
+  if (!(bits == 3 || bits == 4 || bits == 8) || k % 32 || k % group) return 1;
+  const int64_t pitch = k * bits / 8;
+  memset(packed, 0, (size_t)(n * pitch));
+  for (int64_t r = 0; r < n; ++r) {
+    uint8_t* row = packed + r * pitch;
+    for (int64_t kk = 0; kk < k; ++kk) {
+      uint32_t c = codes[r * k + kk];
+      if (bits == 8) {
+        row[kk] = (uint8_t)c;
+      } else if (bits == 4) {
+        uint32_t word;
+        int64_t wi = kk / 8;
+        int nib = (int)((kk % 8) / 2 + 4 * (kk % 2));
+        memcpy(&word, row + 4 * wi, 4);
+        word |= (c & 0xF) << (4 * nib);
+        memcpy(row + 4 * wi, &word, 4);
+      } else {
+        int64_t blk = kk / 32;
+        int kp = (int)(kk % 32), a = kp / 16, i = (kp % 16) / 2, e = kp % 2;
+        uint32_t lw, hw;
+        memcpy(&lw, row + 4 * (3 * blk + a), 4);
+        memcpy(&hw, row + 4 * (3 * blk + 2), 4);
+        lw |= (c & 3u) << (2 * i + 16 * e);
+        hw |= ((c >> 2) & 1u) << (i + 8 * a + 16 * e);
+        memcpy(row + 4 * (3 * blk + a), &lw, 4);
+        memcpy(row + 4 * (3 * blk + 2), &hw, 4);
+      }
+    }
+  }
+  const int64_t ng = k / group;
+  for (int64_t g = 0; g < ng; ++g)
+    for (int64_t r = 0; r < n; ++r)
+      meta[g * n + r] = (uint32_t)scales[r * ng + g] | ((uint32_t)zeros[r * ng + g] << 16);
+  return 0;
+}
+
+int oq_unpack(const uint8_t* packed, int64_t n, int64_t k, int bits, uint8_t* codes) {
+  if (!(bits == 3 || bits == 4 || bits == 8) || k % 32) return 1;
+  const int64_t pitch = k * bits / 8;
+  for (int64_t r = 0; r < n; ++r) {
+    const uint8_t* row = packed + r * pitch;
+    for (int64_t kk = 0; kk < k; ++kk) {
+      uint32_t c;
+      if (bits == 8) {
+        c = row[kk];
+      } else if (bits == 4) {
+        uint32_t word;
+        memcpy(&word, row + 4 * (kk / 8), 4);
+        int nib = (int)((kk % 8) / 2 + 4 * (kk % 2));
+        c = (word >> (4 * nib)) & 0xF;
+      } else {
+        int64_t blk = kk / 32;
+        int kp = (int)(kk % 32), a = kp / 16, i = (kp % 16) / 2, e = kp % 2;
+        uint32_t lw, hw;
+        memcpy(&lw, row + 4 * (3 * blk + a), 4);
+        memcpy(&hw, row + 4 * (3 * blk + 2), 4);
+        c = ((lw >> (2 * i + 16 * e)) & 3u) | (((hw >> (i + 8 * a + 16 * e)) & 1u) << 2);
+      }
+      codes[r * k + kk] = (uint8_t)c;
+    }
+  }
+  return 0;
+}
+
+/* ---------------- O4: dequantize one row of a packed weight into fp64 ----------------
+ * x~ = s x^ + q, exact in fp64 (s, q fp16; x^ < 256).  bits == 16: the fp16
+ * weight itself (reading R7: FP16 layers are not quantized).
+ */
+static void dequant_row(const uint8_t* packed, const uint32_t* meta, int64_t n, int64_t k,
+                        int bits, int group, int64_t r, double* out, uint8_t* tmp_codes) {
+  if (bits == 16) {
+    const uint16_t* wrow = (const uint16_t*)packed + r * k;
+    for (int64_t kk = 0; kk < k; ++kk) out[kk] = (double)h2f(wrow[kk]);
+    return;
+  }
+  const int64_t pitch = k * bits / 8;
+  oq_unpack(packed + r * pitch, 1, k, bits, tmp_codes);
+  for (int64_t kk = 0; kk < k; ++kk) {
+    uint32_t m = meta[(kk / group) * n + r];
+    double s = (double)h2f((uint16_t)(m & 0xFFFF));
+    double z = (double)h2f((uint16_t)(m >> 16));
+    out[kk] = s * (double)tmp_codes[kk] + z;
+  }
+}
+
+int oq_dequant(const uint8_t* packed, const uint32_t* meta, int64_t n, int64_t k, int bits,
+               int group, double* w_out) {
+  uint8_t* tmp = (uint8_t*)malloc((size_t)k);
+  if (!tmp) return 2;
+  for (int64_t r = 0; r < n; ++r) dequant_row(packed, meta, n, k, bits, group, r, w_out + r * k, tmp);
+  free(tmp);
+  return 0;
+}
+
+/* ---------------- O5: weight-only linear, fp64 ----------------
+ * y[i][j] = sum_k x[i][k] * w~[j][k] (+ bias[j]);  x given in fp64 (fp16 values when the
+ * caller passes fp16 activations).  Plain loops, parallel over output rows only.
+ */
+int oq_linear(const double* x, int64_t m, int64_t k, const uint8_t* packed, const uint32_t* meta,
+              int64_t n, int bits, int group, const uint16_t* bias_f16, double* y) {
+  int err = 0;
+#pragma omp parallel
+  {
+    double* wrow = (double*)malloc((size_t)k * sizeof(double));
+    uint8_t* tmp = (uint8_t*)malloc((size_t)k);
+    if (!wrow || !tmp) err = 2;
+#pragma omp for schedule(static)
+    for (int64_t j = 0; j < n; ++j) {
+      if (!wrow || !tmp) continue;
+      dequant_row(packed, meta, n, k, bits, group, j, wrow, tmp);
+      double b = bias_f16 ? (double)h2f(bias_f16[j]) : 0.0;
+      for (int64_t i = 0; i < m; ++i) {
+        double acc = 0.0;
+        for (int64_t kk = 0; kk < k; ++kk) acc += x[i * k + kk] * wrow[kk];
+        y[i * n + j] = acc + b;
+      }
+    }
+    free(wrow);
+    free(tmp);
+  }
+  return err;
+}
+
+/* ---------------- glue (R11/R12) ---------------- */
+void oq_layernorm(const double* x, int64_t t, int64_t d, double eps, double* out) {
+  for (int64_t i = 0; i < t; ++i) {
+    const double* r = x + i * d;
+    double mean = 0.0, var = 0.0;
+    for (int64_t j = 0; j < d; ++j) mean += r[j];
+    mean /= (double)d;
+    for (int64_t j = 0; j < d; ++j) var += (r[j] - mean) * (r[j] - mean);
+    var /= (double)d;
+    double inv = 1.0 / sqrt(var + eps);
+    for (int64_t j = 0; j < d; ++j) out[i * d + j] = (r[j] - mean) * inv;
+  }
+}
+
+static double act_fn(double v, int act) {
+  if (act == 0) return v > 0.0 ? v : 0.0;                         /* ReLU (OPT) */
+  const double c = 0.7978845608028654;                             /* sqrt(2/pi) */
+  return 0.5 * v * (1.0 + tanh(c * (v + 0.044715 * v * v * v)));  /* tanh-GeLU (BLOOM) */
+}
+
+typedef struct {
+  int32_t bits, group;
+  int64_t n, k;
+  const uint8_t* packed; /* bits<16: packed codes; bits==16: fp16 W [n,k] */
+  const uint32_t* meta;  /* NULL iff bits == 16 */
+  const uint16_t* bias;  /* fp16 [n] or NULL */
+} oq_weight;
+
+typedef struct {
+  int32_t bits, act;
+  oq_weight qkv, o, fc1, fc2; /* qkv: [3*h1, h1]; o: [h1, h1]; fc1: [h2, h1]; fc2: [h1, h2] */
+} oq_layer;
+
+/* One stage = consecutive layers of a pre-LN decoder block with the attention stub
+ * (attention output = V, R12).  For each layer (bits b):
+ *   a = LN(x); [q k v] = a Wqkv^T (+b); h = x + v Wo^T (+b);
+ *   u = act(LN(h) W1^T + b1); x = h + u W2^T (+b2)
+ * x: fp64 [t, h1], updated in place.  qkv_dbg (optional): last layer's [t, 3*h1].
+ */
+int oq_stage(const oq_layer* layers, int n_layers, double* x, int64_t t, int64_t h1,
+             double* qkv_dbg) {
+  const int64_t h2 = layers[0].fc1.n;
+  double* a = (double*)malloc((size_t)(t * h1) * sizeof(double));
+  double* qkv = (double*)malloc((size_t)(t * 3 * h1) * sizeof(double));
+  double* v = (double*)malloc((size_t)(t * h1) * sizeof(double));
+  double* o = (double*)malloc((size_t)(t * h1) * sizeof(double));
+  double* u = (double*)malloc((size_t)(t * h2) * sizeof(double));
+  int err = (!a || !qkv || !v || !o || !u) ? 2 : 0;
+  for (int l = 0; l < n_layers && !err; ++l) {
+    const oq_layer* L = &layers[l];
+    oq_layernorm(x, t, h1, 1e-5, a);
+    err |= oq_linear(a, t, h1, L->qkv.packed, L->qkv.meta, 3 * h1, L->qkv.bits, L->qkv.group, L->qkv.bias, qkv);
+    for (int64_t i = 0; i < t; ++i)
+      for (int64_t j = 0; j < h1; ++j) v[i * h1 + j] = qkv[i * 3 * h1 + 2 * h1 + j];
+    err |= oq_linear(v, t, h1, L->o.packed, L->o.meta, h1, L->o.bits, L->o.group, L->o.bias, o);
+    for (int64_t i = 0; i < t * h1; ++i) x[i] += o[i];
+    oq_layernorm(x, t, h1, 1e-5, a);
+    err |= oq_linear(a, t, h1, L->fc1.packed, L->fc1.meta, h2, L->fc1.bits, L->fc1.group, L->fc1.bias, u);
+    for (int64_t i = 0; i < t * h2; ++i) u[i] = act_fn(u[i], L->act);
+    err |= oq_linear(u, t, h2, L->fc2.packed, L->fc2.meta, h1, L->fc2.bits, L->fc2.group, L->fc2.bias, o);
+    for (int64_t i = 0; i < t * h1; ++i) x[i] += o[i];
+    if (qkv_dbg && l == n_layers - 1) memcpy(qkv_dbg, qkv, (size_t)(t * 3 * h1) * sizeof(double));
+  }
+  free(a);
+  free(qkv);
+  free(v);
+  free(o);
+  free(u);
+  return err;
+}
