@@ -1,0 +1,423 @@
+#!/usr/bin/env python
+"""bench.py — SplitQuant hot path on B200 (BASELINE.json metric).
+
+Metric: "decode dequant-GEMV GB/s vs HBM peak; pipeline tokens/s at 1/2/4/8 B200".
+value = pipeline output tokens/s of the whole job on configs[3] (OPT-66B-shaped,
+64 layers, mixed bits 16 x {3,4,8,16}, prompt 512, 128 decode steps, prefill
+micro-batch eta = 8, decode micro-batch xi = 32), weak scaling B = 32 * N
+(SURVEY.md 8(d) D-4).  A step = one full generation run (prefill + decode) through
+sq_pipeline_run, inputs resident in HBM.  The decode dequant-GEMV GB/s (configs[1]
+OPT-13B shapes) is reported beside it in "decode_gemv" and as the roofline when it
+is the dominant kernel.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+  torchrun --nproc-per-node N bench.py --gpus N ...   (one rank per GPU)
+
+--impl reference times the CPU oracle (oracle/, the only other place this file
+executes it) on a bounded sample of the same workload on the host cores.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "decode dequant-GEMV GB/s vs HBM peak; pipeline tokens/s at 1/2/4/8 B200"
+
+WORKLOADS = {
+    # BASELINE.json configs[3]
+    "opt66b": dict(name="configs[3] OPT-66B-shaped 64 layers, uneven mixed-bit pipeline, prompt 512 + 128 decode tokens",
+                   h1=9216, h2=36864, L=64, act=0, eta=8, xi=32, s=512, n_dec=128, b_per_gpu=32, balanced=True),
+    # BASELINE.json configs[0] (small; for quick runs)
+    "opt125m": dict(name="configs[0] OPT-125m-shaped 12 layers, bits {3,4,8,16}, prefill 1x32 + 8 decode steps",
+                    h1=768, h2=3072, L=12, act=0, eta=1, xi=1, s=32, n_dec=8, b_per_gpu=1, balanced=False),
+}
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return {"hbm_gbs": float(d["hbm_gbs"]), "tflops": float(d["bf16_tflops"]),
+                "tflops_sustained": float(d.get("bf16_tflops_sustained", d["bf16_tflops"])), "src": "measured"}
+    except Exception:
+        return {"hbm_gbs": 6650.0, "tflops": 1590.0, "tflops_sustained": 1400.0, "src": "fallback"}
+
+
+def dist_env():
+    return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
+
+
+# ------------------------------------------------------------------ clocks sampler
+class ClockSampler:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu: int):
+        self.gpu, self.proc, self.lines = gpu, None, []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                                          "-lms", "200", "-i", str(self.gpu)], stdout=subprocess.PIPE,
+                                         stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sms, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            p = [x.strip() for x in ln.split(",")]
+            if len(p) < 9:
+                continue
+            try:
+                sms.append(float(p[1]))
+                mx = float(p[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, p[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sms) if sms else None, "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sms)}
+
+
+# ------------------------------------------------------------------ CPU oracle sample
+def oracle_sample(wl: dict, tokens: int = 16, row_frac: int = 8):
+    """Bounded oracle sample: oq_linear (fp64, plain loops) on the first n/row_frac rows of each
+    of the 4 linears of one 4-bit layer of the workload, `tokens` tokens.  Returns
+    (seconds, token-layer passes represented = tokens * row_frac... scaled by caller)."""
+    import numpy as np
+    import synth
+    from oracle import oracle as O
+    h1, h2 = wl["h1"], wl["h2"]
+    dims = {"qkv": (3 * h1, h1), "o": (h1, h1), "fc1": (h2, h1), "fc2": (h1, h2)}
+    qws = {}
+    for name, (n, k) in dims.items():
+        rows = np.arange(n // row_frac)
+        w = synth.weight_f16(synth.weight_seed(0, name), n, k, rows=rows)
+        qws[name] = O.QWeight(w, 4)
+    x1 = synth.act_f16(5, tokens, h1)
+    x2 = synth.act_f16(6, tokens, h2)
+    t0 = time.perf_counter()
+    for name, (n, k) in dims.items():
+        O.linear(x1 if k == h1 else x2, qws[name])
+    dt = time.perf_counter() - t0
+    return dt
+
+
+def cpu_tokens_per_s(wl: dict, dt: float, tokens: int, row_frac: int, B: int) -> float:
+    # one full layer for `tokens` tokens ~ dt * row_frac; the workload runs L layers over
+    # (B*s prefill + B*n_dec decode) token rows and yields B*(1+n_dec) output tokens
+    per_token_layer = dt * row_frac / tokens
+    total = per_token_layer * wl["L"] * (B * wl["s"] + B * wl["n_dec"])
+    return B * (1 + wl["n_dec"]) / total
+
+
+def run_reference(args, wl):
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return
+    ncores = len(os.sched_getaffinity(0))
+    os.environ.setdefault("OMP_NUM_THREADS", str(ncores))
+    B = wl["b_per_gpu"] * max(1, args.gpus)
+    tokens, frac = args.cpu_tokens, args.cpu_row_frac
+    for _ in range(args.warmup):
+        oracle_sample(wl, tokens, frac)
+    vals, ts = [], []
+    for _ in range(args.steps):
+        dt = oracle_sample(wl, tokens, frac)
+        ts.append(dt)
+        vals.append(cpu_tokens_per_s(wl, dt, tokens, frac, B))
+    v = statistics.median(vals)
+    sample = (f"oq_linear fp64 on the first 1/{frac} of the rows of the 4 linears of one 4-bit "
+              f"{wl['name'].split(' ')[1]} layer, {tokens} tokens, extrapolated to L={wl['L']} layers x "
+              f"(B*s + B*n_dec) token rows")
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "tokens/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * statistics.median(ts),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": wl["name"], "B": B},
+            "cpu_baseline": {"value": v, "unit": "tokens/s", "cores": int(os.environ["OMP_NUM_THREADS"]),
+                             "kind": "oracle", "sample": sample},
+            "e2e": {"value": v, "unit": "tokens/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------ decode GEMV sweep (configs[1])
+def gemv_sweep(reps=10):
+    import torch
+    import synth
+    import paper_conf_cluster_zhaowplw25_b200 as sq
+    pk = peaks()
+    dev = torch.device("cuda")
+    l2 = torch.cuda.get_device_properties(0).L2_cache_size
+    flush = torch.empty(2 * l2 // 4 + 1024, dtype=torch.float32, device=dev)
+    out = []
+    for (n, k) in ((5120, 5120), (20480, 5120), (5120, 20480)):
+        wd = torch.empty((n, k), dtype=torch.float16, device=dev)
+        synth.device_weight_f16(wd.data_ptr(), 4242, n, k)
+        for bits in (3, 4, 8):
+            q = sq.QLinear.from_fp16(wd, bits)
+            for m in (1, 8):
+                x = torch.randn(m, k, device=dev).half()
+                y = torch.empty(m, n, device=dev, dtype=torch.float16)
+                ws = torch.zeros(sq.sq_linear_workspace_bytes(q, m), dtype=torch.uint8, device=dev)
+                xs = sq.sq_xsum(x)
+                for _ in range(3):
+                    sq.sq_linear_decode(q, x, y, 0, xsum=xs, ws=ws)
+                ts = []
+                for _ in range(reps):
+                    flush.zero_()
+                    e0 = torch.cuda.Event(enable_timing=True)
+                    e1 = torch.cuda.Event(enable_timing=True)
+                    e0.record()
+                    sq.sq_linear_decode(q, x, y, 0, xsum=xs, ws=ws)
+                    e1.record()
+                    torch.cuda.synchronize()
+                    ts.append(e0.elapsed_time(e1))
+                med = statistics.median(ts)
+                gbs = q.nbytes() / med / 1e6
+                out.append({"n": n, "k": k, "bits": bits, "m": m, "us": round(med * 1e3, 2), "GBps": round(gbs, 1),
+                            "frac": round(gbs / pk["hbm_gbs"], 3)})
+            del q
+        del wd
+    return out
+
+
+# ------------------------------------------------------------------ our arm
+def run_ours(args, wl):
+    import torch
+    import synth
+    import paper_conf_cluster_zhaowplw25_b200 as sq
+    from paper_conf_cluster_zhaowplw25_b200 import runtime as R
+    from paper_conf_cluster_zhaowplw25_b200 import plan as PL
+
+    rank, world, local = dist_env()
+    assert world == args.gpus or world == 1, "launch N>1 with torchrun --nproc-per-node N"
+    P = world
+    torch.cuda.set_device(local)
+    dist = None
+    if P > 1:
+        import torch.distributed as dist
+        dist.init_process_group("gloo")
+    pk = peaks()
+
+    B = wl["b_per_gpu"] * P
+    L, h1, h2 = wl["L"], wl["h1"], wl["h2"]
+    bits = [int(b) for b in synth.bits_plan(2, L, balanced=wl["balanced"])]
+    costs = PL.phase_costs(bits, h1, h2, B, wl["eta"], wl["xi"], wl["s"], wl["n_dec"], pk["hbm_gbs"],
+                           pk["tflops_sustained"])
+    sol = PL.partition_layers(costs, P)
+    plan = R.Plan(bits, sol, h1, h2, B, wl["eta"], wl["xi"], wl["s"], wl["n_dec"])
+    R.sq_plan_check(plan)
+    mine = plan.layers_of(rank) if P > 1 else list(range(L))
+    layers = R.build_layers(len(mine), h1, h2, [bits[l] for l in mine], act=wl["act"], layer_offset=mine[0])
+    arr = R.layer_array(layers)
+    first, last = (rank == 0), (rank == P - 1)
+
+    comm = None
+    if P > 1:
+        uid = [sq.runtime.sq_comm_get_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        comm = R.Comm.nccl(uid[0], P, rank)
+    ws = R.PipelineWorkspace(plan, layers, rank if P > 1 else 0)
+    x0 = out = None
+    if first:
+        x0 = torch.empty((B, wl["s"], h1), dtype=torch.float32, device="cuda")
+        synth.device_fill_f32(x0.data_ptr(), 1, 0, x0.numel(), 1.0, False)
+    if last:
+        out = torch.zeros((B, 1 + wl["n_dec"], h1), dtype=torch.float32, device="cuda")
+    rk = rank if P > 1 else 0
+
+    def step():
+        return R.sq_pipeline_run(plan, rk, layers, comm, x0, out, ws, arr=arr)
+
+    def barrier():
+        torch.cuda.synchronize()
+        if dist:
+            dist.barrier()
+
+    def max_over_ranks(v: float) -> float:
+        if not dist:
+            return v
+        t = torch.tensor([v], dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def sum_over_ranks(v: float) -> float:
+        if not dist:
+            return v
+        t = torch.tensor([v], dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        return float(t.item())
+
+    for _ in range(args.warmup):
+        step()
+    # ---------------- timed region: device-resident inputs
+    barrier()
+    clocks = ClockSampler(local)
+    if rank == 0:
+        clocks.start()
+    sq.sq_profile_enable(True)
+    launches0 = sq.sq_launch_count()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    barrier()
+    e0.record()
+    stats = [step() for _ in range(args.steps)]
+    e1.record()
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1)
+    launches = sq.sq_launch_count() - launches0
+    sq.sq_profile_enable(False)
+    prof = sq.sq_profile_read()
+    clk = clocks.stop() if rank == 0 else None
+    ms = max_over_ranks(ms)
+    launches = int(sum_over_ranks(launches))
+    tokens = args.steps * B * (1 + wl["n_dec"])
+    value = tokens / (ms / 1e3)
+
+    # dominant kernel class on this rank (rank 0 reports)
+    kern = {}
+    for name, bound in (("gemv", "hbm"), ("gemm", "tensor")):
+        d = prof[name]
+        if d["launches"] and d["ms"] > 0:
+            if bound == "hbm":
+                ach = d["bytes"] / (d["ms"] / 1e3) / 1e9
+                kern[name] = {"bound": "hbm", "achieved": ach, "peak": pk["hbm_gbs"], "unit": "GB/s",
+                              "frac": ach / pk["hbm_gbs"], "launches": d["launches"], "ms": d["ms"],
+                              "bytes_per_launch": d["bytes"] / d["launches"]}
+            else:
+                ach = d["flops"] / (d["ms"] / 1e3) / 1e12
+                kern[name] = {"bound": "tensor", "achieved": ach, "peak": pk["tflops_sustained"], "unit": "TFLOP/s",
+                              "frac": ach / pk["tflops_sustained"], "launches": d["launches"], "ms": d["ms"],
+                              "flops_per_launch": d["flops"] / d["launches"]}
+    kern["glue_ms"] = prof["glue"]["ms"]
+    dom = max((k for k in ("gemv", "gemm") if k in kern), key=lambda k: kern[k]["ms"], default=None)
+    roof = None
+    if dom:
+        r = kern[dom]
+        roof = {"bound": r["bound"], "achieved": round(r["achieved"], 2), "peak": r["peak"], "unit": r["unit"],
+                "frac": round(r["frac"], 4), "traffic": traffic_for(dom), "kernel": dom,
+                "peak_src": pk["src"] + (" sustained" if r["bound"] == "tensor" else " copy")}
+
+    # ---------------- e2e: host buffers through the C-ABI, copies inside the timed region
+    e2e = None
+    if not args.no_e2e:
+        hx = torch.empty(x0.shape, dtype=torch.float32).pin_memory() if first else None
+        if first:
+            hx.copy_(x0.cpu())
+        hout = torch.empty(out.shape, dtype=torch.float32).pin_memory() if last else None
+        barrier()
+        f0 = torch.cuda.Event(enable_timing=True)
+        f1 = torch.cuda.Event(enable_timing=True)
+        f0.record()
+        for _ in range(args.steps):
+            if first:
+                x0.copy_(hx, non_blocking=True)
+            step()
+            if last:
+                hout.copy_(out, non_blocking=True)
+        f1.record()
+        torch.cuda.synchronize()
+        ems = max_over_ranks(f0.elapsed_time(f1))
+        e2e = {"value": tokens / (ems / 1e3), "unit": "tokens/s",
+               "h2d_bytes_per_step": int(sum_over_ranks(x0.numel() * 4 if first else 0)),
+               "d2h_bytes_per_step": int(sum_over_ranks(out.numel() * 4 if last else 0))}
+
+    # ---------------- side measurements on rank 0 at N = 1
+    extra = {}
+    cpu = None
+    if rank == 0 and P == 1:
+        if not args.no_gemv_sweep:
+            extra["decode_gemv"] = {"workload": "configs[1] OPT-13B linear shapes, L2 flushed, median of 10",
+                                    "results": gemv_sweep()}
+        if not args.no_cpu:
+            ncores = len(os.sched_getaffinity(0))
+            os.environ["OMP_NUM_THREADS"] = str(ncores)
+            dt = oracle_sample(wl, args.cpu_tokens, args.cpu_row_frac)
+            cpu = {"value": cpu_tokens_per_s(wl, dt, args.cpu_tokens, args.cpu_row_frac, B), "unit": "tokens/s",
+                   "cores": ncores, "kind": "oracle",
+                   "sample": (f"oq_linear fp64 on the first 1/{args.cpu_row_frac} of the rows of the 4 linears of "
+                              f"one 4-bit layer, {args.cpu_tokens} tokens, {dt:.2f} s, extrapolated to the workload")}
+    if rank == 0:
+        st = stats[-1]
+        line = {
+            "metric": METRIC, "value": value, "unit": "tokens/s", "n_gpus": P, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f16", "data": "synthetic",
+            "config": {"workload": wl["name"], "B": B, "eta": wl["eta"], "xi": wl["xi"], "prompt_len": wl["s"],
+                       "n_decode": wl["n_dec"], "layers": L, "hidden": h1, "ffn": h2,
+                       "bits_histogram": {str(b): bits.count(b) for b in (3, 4, 8, 16)},
+                       "stage_sizes": [sol.count(s) for s in range(P)],
+                       "weights_GB": round(sum(PL.layer_bytes(h1, h2, b) for b in bits) / 1e9, 2),
+                       "l2": "inputs larger than L2: every step streams all packed weights (tens of GB)",
+                       "parallelism": f"pp{P}"},
+            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk,
+            "kernels": kern,
+            "phase_ms_rank0": {"prefill": st["t_prefill_ms"], "decode": st["t_decode_ms"]},
+        }
+        line.update(extra)
+        print(json.dumps(line), flush=True)
+    if comm:
+        comm.destroy()
+    if dist:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def traffic_for(kernel: str):
+    """dram bytes per launch of the dominant kernel from the committed ncu capture (profiles/)."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            return json.load(f).get(kernel)
+    except Exception:
+        return None
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=3)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--workload", choices=sorted(WORKLOADS), default="opt66b")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-gemv-sweep", action="store_true")
+    ap.add_argument("--cpu-tokens", type=int, default=8)
+    ap.add_argument("--cpu-row-frac", type=int, default=8)
+    args = ap.parse_args()
+    wl = WORKLOADS[args.workload]
+    if args.impl == "reference":
+        run_reference(args, wl)
+    else:
+        run_ours(args, wl)
+
+
+if __name__ == "__main__":
+    main()

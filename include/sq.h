@@ -1,0 +1,237 @@
+/*
+ * sq.h — C-ABI of the SplitQuant hot path on B200 (libsq.so, sm_100a).
+ *
+ * Paper: Zhao et al., "SplitQuant" (PAPER.md in /root/reference; "P:<line>"
+ * below are its line numbers).  The library executes a plan (per-layer
+ * bit-widths, layer->stage partition, micro-batch sizes) produced host-side
+ * (P:133); it does not plan.
+ *
+ * Conventions for every entry point
+ *  - Pointers named *_dev are DEVICE pointers (any CUDA allocation on the
+ *    current device); *_host are host pointers.  The caller owns all memory;
+ *    the library never allocates in a hot call (only sq_comm_* and the first
+ *    TMA-descriptor cache fill allocate host memory).
+ *  - `stream` is a cudaStream_t (NULL = legacy default stream).  Kernels are
+ *    enqueued asynchronously; device faults surface at the next sync.
+ *  - Every call returns sq_status and never throws.  All validation happens
+ *    before any launch: SQ_EINVAL has no side effects.  The message of the last
+ *    non-OK status of the calling thread is in sq_last_error().
+ *  - Inputs must be finite (NaN/Inf behaviour of the quantizer is unspecified).
+ *  - Matrices are row-major.  A linear weight W is [n, k] (n = out_features,
+ *    k = in_features); y[m, n] = x[m, k] . W~^T.
+ */
+#ifndef SQ_H_
+#define SQ_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st* sq_stream_t; /* == cudaStream_t */
+
+typedef enum {
+  SQ_OK = 0,
+  SQ_EINVAL = 1,    /* bad argument (null, misaligned, unsupported bits/shape, bad plan) */
+  SQ_ENOTSUP = 2,   /* valid but not implemented (e.g. group != 128 in a linear) */
+  SQ_ENOMEM = 3,    /* workspace too small / host allocation failed */
+  SQ_ECUDA = 4,     /* CUDA runtime/driver error (message in sq_last_error) */
+  SQ_ENCCL = 5,     /* NCCL error */
+  SQ_EINTERNAL = 6
+} sq_status;
+
+const char* sq_last_error(void);
+const char* sq_version(void);
+int sq_abi_version(void); /* bumped on any incompatible change of this header */
+
+/* ------------------------------------------------------------------------
+ * Sizes.  P:160: a decoder layer with precision `bit` stores
+ * (4 h1^2 + 2 h1 h2) * bit/8 bytes of weights; sq_packed_bytes is that count
+ * for one [n,k] linear (codes only).  Group metadata is separate.
+ * Returns 0 on invalid input.
+ * ------------------------------------------------------------------------ */
+size_t sq_packed_bytes(int64_t n, int64_t k, int bits);        /* n*k*bits/8; bits in {3,4,8,16} */
+size_t sq_meta_bytes(int64_t n, int64_t k, int group);         /* n*(k/group)*4 */
+
+/* ------------------------------------------------------------------------
+ * a1 — per-group round-to-nearest min/max quantization (S_W of P:184).
+ *   For row r, group g (k in [g*group, (g+1)*group)), IEEE fp32, one rounding/op:
+ *     mn = min w, mx = max w (canonical +0);  s = fp16((mx - mn) / (2^bits - 1));
+ *     z = mn;  c = s == 0 ? 0 : clamp(rint_half_even((w - z) / s), 0, 2^bits - 1)
+ *   (readings R1-R6).
+ *   w_dev     fp16 [n, k], 16-B aligned.       codes_dev  u8 [n, k]
+ *   scales_dev, zeros_dev  fp16 [n, k/group]
+ *   bits in {3,4,8}; group in {32,64,128}; k % group == 0; n >= 1.
+ *   Result is bit-exact with the CPU oracle.
+ * ------------------------------------------------------------------------ */
+sq_status sq_quantize_groups(const void* w_dev, int64_t n, int64_t k, int bits, int group,
+                             uint8_t* codes_dev, void* scales_dev, void* zeros_dev,
+                             sq_stream_t stream);
+
+/* ------------------------------------------------------------------------
+ * a2 — bit packing (layouts L8/L4/L3 + tile placement T16 of DESIGN.md
+ *   section 4; the paper is silent on packing; P:160 fixes bits/8 bytes
+ *   per weight).  codes_dev u8 [n,k]; scales/zeros fp16 [n, k/128] ->
+ *   packed_dev n*k*bits/8 bytes (16-B aligned): unit (tile t = rows 16t..16t+15,
+ *   group g) is a contiguous chunk of 16 x (128*bits/8) bytes at unit index
+ *   t*(k/128) + g; meta_dev u32 [n/16][k/128][16] (low half = scale, high half =
+ *   zero).  bits in {3,4,8}; group == 128; n % 16 == 0; k % 128 == 0.
+ *   Bit-exact with the CPU oracle.
+ * ------------------------------------------------------------------------ */
+sq_status sq_pack(const uint8_t* codes_dev, const void* scales_dev, const void* zeros_dev,
+                  int64_t n, int64_t k, int bits, int group, void* packed_dev, void* meta_dev,
+                  sq_stream_t stream);
+
+/* One quantized linear: non-owning view of device memory. */
+typedef struct {
+  int32_t bits;          /* 3, 4, 8, or 16 (16 = fp16 weight, not quantized, R7) */
+  int32_t group;         /* 128 (only value the linear kernels implement) */
+  int64_t n, k;          /* n % 16 == 0, k % 128 == 0 */
+  const void* packed;    /* bits<16: packed codes (sq_pack, T16); bits==16: fp16 W [n,k] row-major */
+  const void* meta;      /* bits<16: u32 [n/16][k/128][16] (sq_pack); NULL when bits == 16 */
+  const void* bias;      /* fp16 [n] or NULL */
+} sq_qweight;
+
+/* Epilogue of a linear (fused into the kernel). */
+typedef enum {
+  SQ_EPI_F16 = 0,       /* y fp16 [m, ldy] = x W~^T (+bias) */
+  SQ_EPI_F16_RELU = 1,  /* y fp16 = relu(x W~^T + bias)        (OPT fc1, R11) */
+  SQ_EPI_F16_GELU = 2,  /* y fp16 = gelu_tanh(x W~^T + bias)   (BLOOM fc1, R11) */
+  SQ_EPI_F32_ACCUM = 3  /* y fp32 [m, ldy] += x W~^T (+bias)  (fused residual add, R9) */
+} sq_epilogue;
+
+/* ------------------------------------------------------------------------
+ * a4 — decode linear (P:57 decode phase, memory-bound per P:106/P:164):
+ *   y = epi(x . W~^T), m in [1, 32] tokens (one per sequence of the decode
+ *   micro-batch xi).  Streams the packed weights once with 128-bit loads,
+ *   unpacks in registers, fp32 accumulation (CUDA-core unpack + mma.sync
+ *   dot products, K2).
+ *   x_dev fp16 [m, ldx] (ldx % 8 == 0, 16-B aligned).  y_dev per epi.
+ *   xsum_dev: optional float2 [k/128][32] group sums of x produced by
+ *     sq_xsum (NULL: computed internally into the workspace).
+ *   ws_dev/ws_bytes: >= sq_linear_workspace_bytes(w, m); must be ZEROED once
+ *     before first use (holds self-resetting counters); one workspace per
+ *     concurrently running call.
+ *   Deterministic: identical inputs give bit-identical outputs.
+ * ------------------------------------------------------------------------ */
+size_t sq_linear_workspace_bytes(const sq_qweight* w, int64_t m);
+sq_status sq_linear_decode(const sq_qweight* w, const void* x_dev, int64_t ldx, int64_t m,
+                           void* y_dev, int64_t ldy, int epi, const void* xsum_dev,
+                           void* ws_dev, size_t ws_bytes, sq_stream_t stream);
+
+/* Group sums used by sq_linear_decode: xsum[g][t] = (sum of x[t,k] over k%4<2 ; over k%4>=2)
+ * for the 128 k of group g, fp32, fixed summation order.  float2 [k/128][32]; slots t >= m
+ * are written as 0.  m <= 32. */
+sq_status sq_xsum(const void* x_dev, int64_t ldx, int64_t m, int64_t k, void* xsum_dev,
+                  sq_stream_t stream);
+
+/* ------------------------------------------------------------------------
+ * a3 — prefill linear (P:57 prefill phase, compute-bound per P:164): the same
+ *   function for m >= 1 prompt tokens (m = eta * s).  tcgen05 tensor cores:
+ *   packed weight tiles staged by TMA into shared memory, dequantized
+ *   (w~ = s*c + z in fp16) into tensor memory as the A operand, activation
+ *   tiles by TMA (128B swizzle) as the B operand, fp32 accumulation in TMEM.
+ *   x_dev fp16 [m, ldx] (ldx % 8 == 0).  n % 128 == 0.
+ * ------------------------------------------------------------------------ */
+sq_status sq_linear_prefill(const sq_qweight* w, const void* x_dev, int64_t ldx, int64_t m,
+                            void* y_dev, int64_t ldy, int epi, sq_stream_t stream);
+
+/* ------------------------------------------------------------------------
+ * a5 — stage forward (one pipeline stage = consecutive decoder layers, each
+ *   with its own bit-width, P:152/P:160/P:198; glue R11, attention stub R12):
+ *     a = LN(x); [q k v] = a Wqkv^T (+b); h = x + v Wo^T (+b);
+ *     u = act(LN(h) W1^T + b1); x = h + u W2^T (+b2)
+ *   phase SQ_PREFILL uses sq_linear_prefill kernels, SQ_DECODE (tokens <= 32)
+ *   the decode kernels.  x_in/x_out fp32 [tokens, h1] (may alias).
+ *   qkv_dbg_dev: optional fp16 [tokens, 3*h1] receiving the LAST layer's q,k,v.
+ *   ws: >= sq_stage_workspace_bytes(...), zeroed once before first use.
+ * ------------------------------------------------------------------------ */
+typedef struct {
+  int32_t bits;          /* this layer's precision (all four linears share it) */
+  int32_t act;           /* 0 = ReLU (OPT), 1 = tanh-GeLU (BLOOM) */
+  sq_qweight qkv;        /* [3*h1, h1] (q, k, v stacked along n) */
+  sq_qweight o;          /* [h1, h1] */
+  sq_qweight fc1;        /* [h2, h1] */
+  sq_qweight fc2;        /* [h1, h2] */
+} sq_layer;
+
+typedef enum { SQ_PREFILL = 0, SQ_DECODE = 1 } sq_phase;
+
+size_t sq_stage_workspace_bytes(const sq_layer* layers, int n_layers, int64_t max_tokens);
+sq_status sq_stage_forward(const sq_layer* layers, int n_layers, int phase, const float* x_in_dev,
+                           int64_t tokens, float* x_out_dev, void* qkv_dbg_dev, void* ws_dev,
+                           size_t ws_bytes, sq_stream_t stream);
+
+/* Loop-back glue (R14): out_row = x (fp32 copy) and e = LN(x) for the next decode step. */
+sq_status sq_layernorm_f32(const float* x_dev, int64_t rows, int64_t d, float* y_dev,
+                           sq_stream_t stream);
+
+/* ------------------------------------------------------------------------
+ * a6 — uneven layer-wise pipeline with phase-specific micro-batches
+ *   (eq. (4), eqs. (5)-(8), (15)-(16) P:210-232).
+ * ------------------------------------------------------------------------ */
+typedef struct sq_comm sq_comm;   /* owns NCCL link communicators + comm streams + events */
+
+size_t sq_comm_unique_id_bytes(void);                         /* 128 */
+sq_status sq_comm_get_unique_id(uint8_t* id_host);            /* rank 0; broadcast by caller */
+/* One process per GPU; id_host from sq_comm_get_unique_id on rank 0 (world comm),
+ * nranks = number of pipeline stages.  Collective over all ranks. */
+sq_status sq_comm_init(sq_comm** out, const uint8_t* id_host, int nranks, int rank);
+/* Single-process "virtual pipeline": every stage on the current device, transfers
+ * are device copies.  Bitwise reference for the multi-GPU run. */
+sq_status sq_comm_init_local(sq_comm** out, int nstages);
+sq_status sq_comm_destroy(sq_comm* comm);
+
+typedef struct {            /* host memory, identical on every rank */
+  int32_t n_layers, n_stages;
+  int32_t hidden, ffn;      /* h1, h2 */
+  int32_t group;            /* 128 */
+  const int32_t* bits;            /* [n_layers], in {3,4,8,16}            (y_{i,b}) */
+  const int32_t* stage_of_layer;  /* [n_layers] non-decreasing 0..n_stages-1, every stage
+                                     non-empty (u_{i,j}, eqs. 15-16) */
+  int32_t B;                /* global batch (sequences) */
+  int32_t eta, xi;          /* prefill / decode micro-batch sizes (sequences) */
+  int32_t prompt_len;       /* s */
+  int32_t n_decode;         /* decode steps after the prefill token (R14) */
+} sq_plan;
+
+typedef struct {
+  double t_total_ms, t_prefill_ms, t_decode_ms;  /* device time (events) on this rank */
+  double tokens_per_s;      /* B*(1+n_decode) / t_total */
+  int64_t bytes_sent;       /* inter-stage bytes sent by this rank */
+  int64_t gpu_launches;     /* kernels launched by this rank */
+} sq_run_stats;
+
+size_t sq_pipeline_workspace_bytes(const sq_plan* plan, const sq_layer* layers, int rank);
+/* rank >= 0: this process's stage (layers = its layers, in order); rank == -1 with a
+ * local comm: all stages (layers = all n_layers).  x0_dev: embeddings fp32 [B, s, h1]
+ * (needed on stage 0); out_dev: fp32 [B, 1+n_decode, h1] (written on the last stage).
+ * Blocking: returns after the run completed on this rank. */
+sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers, int n_layers,
+                          sq_comm* comm, const float* x0_dev, float* out_dev, void* ws_dev,
+                          size_t ws_bytes, sq_run_stats* stats, sq_stream_t stream);
+
+/* Validate a plan (contiguity eqs. 15-16, non-empty stages, bits set, micro-batches). */
+sq_status sq_plan_check(const sq_plan* plan);
+
+/* ------------------------------------------------------------------------
+ * Measurement hooks (bench.py): per-kernel-class CUDA-event timing of every
+ * launch made by the library while enabled, on the launching stream.
+ * class 0 = decode GEMV, 1 = prefill GEMM, 2 = glue (LN/xsum), 3 = quantize/pack.
+ * ------------------------------------------------------------------------ */
+typedef struct {
+  int64_t launches[4];
+  double ms[4];             /* summed event durations */
+  double bytes[4];          /* algorithmic bytes */
+  double flops[4];          /* algorithmic flops */
+} sq_profile;
+sq_status sq_profile_enable(int on);
+sq_status sq_profile_read(sq_profile* out);   /* synchronizes the device */
+int64_t sq_launch_count(void);                /* kernels launched by the library so far */
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SQ_H_ */

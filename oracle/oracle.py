@@ -72,11 +72,14 @@ def quantize_groups(w: np.ndarray, bits: int, group: int = 128):
 
 
 def pack(codes: np.ndarray, scales: np.ndarray, zeros: np.ndarray, bits: int, group: int = 128):
-    """O2 (DESIGN.md layouts).  -> (packed u8 [n, k*bits/8], meta u32 [k/g, n])."""
+    """O2 (DESIGN.md layouts L8/L4/L3 + tiling T16).
+
+    -> (packed u8 [n/16, k/128, 16, 128*bits/8] flattened to [n, k*bits/8] bytes,
+        meta u32 [n/16, k/128, 16] flattened)."""
     codes = np.ascontiguousarray(codes, np.uint8)
     n, k = codes.shape
     packed = np.empty((n, k * bits // 8), np.uint8)
-    meta = np.empty((k // group, n), np.uint32)
+    meta = np.empty((n // 16, k // 128, 16), np.uint32)
     _check(_lib().oq_pack(_p(codes), _p(np.ascontiguousarray(scales, np.float16)),
                           _p(np.ascontiguousarray(zeros, np.float16)), n, k, bits, group,
                           _p(packed), _p(meta)), "pack")

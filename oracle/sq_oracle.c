@@ -17,7 +17,7 @@
  *                       asymmetric S_W of P:184; readings R1-R6 of DESIGN.md.
  *                       Pinned by brute-force argmin, |w - w~| <= s/2, grid-aligned
  *                       recovery, constant groups, closed-form scale bound.
- *   oq_pack/oq_unpack   Layout L3/L4/L8 of DESIGN.md (paper silent).  Pinned by
+ *   oq_pack/oq_unpack   Layouts L3/L4/L8 + tiling T16 of DESIGN.md (paper silent).  Pinned by
  *                       hand-derived golden words (tests/golden/pack_words.txt),
  *                       round trip, and the P:160 byte count.
  *   oq_dequant_row      x~ = s_x x^ + q_x, exact in fp64.
@@ -94,81 +94,85 @@ int oq_quantize_groups(const uint16_t* w, int64_t n, int64_t k, int bits, int gr
   return 0;
 }
 
-/* ---------------- O2/O3: bit packing (DESIGN.md layouts L8, L4, L3) ----------------
- * Rows are contiguous, row pitch = k*bits/8 bytes, codes in k order within a row.
- * L8: byte k.
- * L4: 32-bit little-endian word k/8, nibble (k%8)/2 + 4*(k%2)   (even k in the low
- *     four nibbles, odd k in the high four).
- * L3: blocks of 32 codes = 3 words [L0, L1, H]; for k' = k%32: a = k'/16,
- *     i = (k'%16)/2, e = k'%2; low two bits at word La, bits 2i + 16e;
+/* ---------------- O2/O3: bit packing (DESIGN.md layouts L8, L4, L3 + tiling T16) ----------------
+ * Within one row and one group of 128 codes (GB = 128*bits/8 bytes):
+ * L8: byte j = c_j.
+ * L4: 32-bit little-endian word j/8, nibble (j%8)/2 + 4*(j%2)   (even j in the low
+ *     four nibbles, odd j in the high four).
+ * L3: blocks of 32 codes = 3 words [L0, L1, H]; for j' = j%32: a = j'/16,
+ *     i = (j'%16)/2, e = j'%2; low two bits at word La, bits 2i + 16e;
  *     high bit at word H, bit i + 8a + 16e.
- * meta: uint32 [k/group][n], low half = scale, high half = zero (group-major).
+ * T16 (placement): rows are grouped in tiles of 16; the 16 rows' bytes of group g of
+ *     tile t form one contiguous chunk ("unit") at byte ((t*kg + g)*16 + r%16)*GB,
+ *     kg = k/128, units ordered tile-major / group-minor.
+ * meta: uint32 at ((t*kg + g)*16 + r%16), low half = scale, high half = zero.
+ * Requires n % 16 == 0, k % 128 == 0, group == 128.
  */
 size_t oq_packed_bytes(int64_t n, int64_t k, int bits) { return (size_t)(n * k * bits / 8); }
 
+static int64_t unit_off(int64_t r, int64_t g, int64_t kg) { return ((r / 16) * kg + g) * 16 + r % 16; }
+
 int oq_pack(const uint8_t* codes, const uint16_t* scales, const uint16_t* zeros, int64_t n,
             int64_t k, int bits, int group, uint8_t* packed, uint32_t* meta) {
-  if (!(bits == 3 || bits == 4 || bits == 8) || k % 32 || k % group) return 1;
-  const int64_t pitch = k * bits / 8;
-  memset(packed, 0, (size_t)(n * pitch));
+  if (!(bits == 3 || bits == 4 || bits == 8) || k % 128 || group != 128 || n % 16) return 1;
+  const int64_t kg = k / 128, GB = 128 * bits / 8;
+  memset(packed, 0, (size_t)(n * k * bits / 8));
   for (int64_t r = 0; r < n; ++r) {
-    uint8_t* row = packed + r * pitch;
     for (int64_t kk = 0; kk < k; ++kk) {
       uint32_t c = codes[r * k + kk];
+      const int64_t g = kk / 128, j = kk % 128;
+      uint8_t* grp = packed + unit_off(r, g, kg) * GB;
       if (bits == 8) {
-        row[kk] = (uint8_t)c;
+        grp[j] = (uint8_t)c;
       } else if (bits == 4) {
         uint32_t word;
-        int64_t wi = kk / 8;
-        int nib = (int)((kk % 8) / 2 + 4 * (kk % 2));
-        memcpy(&word, row + 4 * wi, 4);
+        int64_t wi = j / 8;
+        int nib = (int)((j % 8) / 2 + 4 * (j % 2));
+        memcpy(&word, grp + 4 * wi, 4);
         word |= (c & 0xF) << (4 * nib);
-        memcpy(row + 4 * wi, &word, 4);
+        memcpy(grp + 4 * wi, &word, 4);
       } else {
-        int64_t blk = kk / 32;
-        int kp = (int)(kk % 32), a = kp / 16, i = (kp % 16) / 2, e = kp % 2;
+        int64_t blk = j / 32;
+        int kp = (int)(j % 32), a = kp / 16, i = (kp % 16) / 2, e = kp % 2;
         uint32_t lw, hw;
-        memcpy(&lw, row + 4 * (3 * blk + a), 4);
-        memcpy(&hw, row + 4 * (3 * blk + 2), 4);
+        memcpy(&lw, grp + 4 * (3 * blk + a), 4);
+        memcpy(&hw, grp + 4 * (3 * blk + 2), 4);
         lw |= (c & 3u) << (2 * i + 16 * e);
         hw |= ((c >> 2) & 1u) << (i + 8 * a + 16 * e);
-        memcpy(row + 4 * (3 * blk + a), &lw, 4);
-        memcpy(row + 4 * (3 * blk + 2), &hw, 4);
+        memcpy(grp + 4 * (3 * blk + a), &lw, 4);
+        memcpy(grp + 4 * (3 * blk + 2), &hw, 4);
       }
     }
   }
-  const int64_t ng = k / group;
-  for (int64_t g = 0; g < ng; ++g)
-    for (int64_t r = 0; r < n; ++r)
-      meta[g * n + r] = (uint32_t)scales[r * ng + g] | ((uint32_t)zeros[r * ng + g] << 16);
+  for (int64_t r = 0; r < n; ++r)
+    for (int64_t g = 0; g < kg; ++g)
+      meta[unit_off(r, g, kg)] = (uint32_t)scales[r * kg + g] | ((uint32_t)zeros[r * kg + g] << 16);
   return 0;
 }
 
-int oq_unpack(const uint8_t* packed, int64_t n, int64_t k, int bits, uint8_t* codes) {
-  if (!(bits == 3 || bits == 4 || bits == 8) || k % 32) return 1;
-  const int64_t pitch = k * bits / 8;
-  for (int64_t r = 0; r < n; ++r) {
-    const uint8_t* row = packed + r * pitch;
-    for (int64_t kk = 0; kk < k; ++kk) {
-      uint32_t c;
-      if (bits == 8) {
-        c = row[kk];
-      } else if (bits == 4) {
-        uint32_t word;
-        memcpy(&word, row + 4 * (kk / 8), 4);
-        int nib = (int)((kk % 8) / 2 + 4 * (kk % 2));
-        c = (word >> (4 * nib)) & 0xF;
-      } else {
-        int64_t blk = kk / 32;
-        int kp = (int)(kk % 32), a = kp / 16, i = (kp % 16) / 2, e = kp % 2;
-        uint32_t lw, hw;
-        memcpy(&lw, row + 4 * (3 * blk + a), 4);
-        memcpy(&hw, row + 4 * (3 * blk + 2), 4);
-        c = ((lw >> (2 * i + 16 * e)) & 3u) | (((hw >> (i + 8 * a + 16 * e)) & 1u) << 2);
-      }
-      codes[r * k + kk] = (uint8_t)c;
-    }
+/* O3: code of row r, column kk (inverse of oq_pack's placement and bit layout) */
+static uint32_t code_at(const uint8_t* packed, int64_t r, int64_t kk, int64_t kg, int bits) {
+  const int64_t GB = 128 * bits / 8, g = kk / 128, j = kk % 128;
+  const uint8_t* grp = packed + unit_off(r, g, kg) * GB;
+  if (bits == 8) return grp[j];
+  if (bits == 4) {
+    uint32_t word;
+    memcpy(&word, grp + 4 * (j / 8), 4);
+    int nib = (int)((j % 8) / 2 + 4 * (j % 2));
+    return (word >> (4 * nib)) & 0xF;
   }
+  int64_t blk = j / 32;
+  int kp = (int)(j % 32), a = kp / 16, i = (kp % 16) / 2, e = kp % 2;
+  uint32_t lw, hw;
+  memcpy(&lw, grp + 4 * (3 * blk + a), 4);
+  memcpy(&hw, grp + 4 * (3 * blk + 2), 4);
+  return ((lw >> (2 * i + 16 * e)) & 3u) | (((hw >> (i + 8 * a + 16 * e)) & 1u) << 2);
+}
+
+int oq_unpack(const uint8_t* packed, int64_t n, int64_t k, int bits, uint8_t* codes) {
+  if (!(bits == 3 || bits == 4 || bits == 8) || k % 128 || n % 16) return 1;
+  for (int64_t r = 0; r < n; ++r)
+    for (int64_t kk = 0; kk < k; ++kk) codes[r * k + kk] = (uint8_t)code_at(packed, r, kk, k / 128, bits);
   return 0;
 }
 
@@ -178,18 +182,18 @@ int oq_unpack(const uint8_t* packed, int64_t n, int64_t k, int bits, uint8_t* co
  */
 static void dequant_row(const uint8_t* packed, const uint32_t* meta, int64_t n, int64_t k,
                         int bits, int group, int64_t r, double* out, uint8_t* tmp_codes) {
+  (void)group; (void)n; (void)tmp_codes;
   if (bits == 16) {
     const uint16_t* wrow = (const uint16_t*)packed + r * k;
     for (int64_t kk = 0; kk < k; ++kk) out[kk] = (double)h2f(wrow[kk]);
     return;
   }
-  const int64_t pitch = k * bits / 8;
-  oq_unpack(packed + r * pitch, 1, k, bits, tmp_codes);
+  const int64_t kg = k / 128;
   for (int64_t kk = 0; kk < k; ++kk) {
-    uint32_t m = meta[(kk / group) * n + r];
+    uint32_t m = meta[unit_off(r, kk / 128, kg)];
     double s = (double)h2f((uint16_t)(m & 0xFFFF));
     double z = (double)h2f((uint16_t)(m >> 16));
-    out[kk] = s * (double)tmp_codes[kk] + z;
+    out[kk] = s * (double)code_at(packed, r, kk, kg, bits) + z;
   }
 }
 

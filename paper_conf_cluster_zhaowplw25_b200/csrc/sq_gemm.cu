@@ -1,0 +1,432 @@
+// K3 — prefill dequant-GEMM on tcgen05 (P:57 prefill phase; compute-bound,
+// arithmetic intensity 6354-9553 on V100; dequant overhead made FP16
+// faster than 3/4-bit in prefill on the paper's GPUs, P:108 — here it is
+// hidden behind the tensor cores).
+//
+// Y^T tile [128 weight rows x 256 tokens] = W~[128 x K] . X[256 x K]^T
+//
+//  * A operand = dequantized weights in TENSOR MEMORY (tcgen05.mma ... [a_tmem]):
+//    packed codes + meta of a 128-row x 128-k group are staged into shared memory
+//    by TMA (swizzled so each thread's row is bank-conflict free), four "dequant"
+//    warps (one per TMEM sub-partition, one thread per weight row) turn them into
+//    fp16 w~ = s*c + z (magic-number unpack, HSUB2 + HFMA2) and tcgen05.st them
+//    into a 2-slot TMEM ring.  Keeping A out of shared memory leaves the SMEM
+//    port to the activation stream (K3).
+//  * B operand = activation tile [256 tokens x 64 k] fp16 by TMA, 128B swizzle,
+//    K-major; 4-stage ring.
+//  * D = fp32 accumulator in TMEM (256 columns); one thread issues
+//    tcgen05.mma.cta_group::1.kind::f16 (M=128, N=256, K=16).
+//  * Epilogue: the dequant warps tcgen05.ld the accumulator (lane = weight row,
+//    column = token), add bias / activation / residual, store y.
+// Warp roles: 0 = TMA producer, 1 = MMA issuer (+TMEM alloc), 2..5 = dequant+epilogue.
+#include <cuda.h>
+
+#include <cstring>
+#include <mutex>
+
+#include "sq_common.cuh"
+
+namespace sq {
+namespace {
+
+constexpr int BN = 128;   // weight rows per tile (TMEM lanes, MMA M)
+constexpr int BT = 256;   // tokens per tile (MMA N)
+constexpr int XK = 64;    // k per activation stage (one 128-B swizzle row)
+constexpr int S_X = 4;
+constexpr int S_A = 2;
+constexpr int X_STAGE_BYTES = BT * XK * 2;  // 32 KB
+constexpr int TMEM_COLS = 512;
+constexpr int D_COL = 0;
+constexpr int A_COL = 256;
+constexpr int NUM_THREADS = 192;
+
+template <int BITS>
+struct GCfg;
+template <>
+struct GCfg<3> { static constexpr int GB = 48; static constexpr int S_W = 4; };
+template <>
+struct GCfg<4> { static constexpr int GB = 64; static constexpr int S_W = 4; };
+template <>
+struct GCfg<8> { static constexpr int GB = 128; static constexpr int S_W = 3; };
+template <>
+struct GCfg<16> { static constexpr int GB = 256; static constexpr int S_W = 2; };
+
+template <int BITS>
+struct Smem {
+  static constexpr int W_STAGE = ((BN * GCfg<BITS>::GB + 1023) / 1024) * 1024;
+  static constexpr int OFF_X = 0;
+  static constexpr int OFF_W = OFF_X + S_X * X_STAGE_BYTES;
+  static constexpr int OFF_META = OFF_W + GCfg<BITS>::S_W * W_STAGE;
+  static constexpr int OFF_BAR = OFF_META + GCfg<BITS>::S_W * BN * 4;
+  static constexpr int NUM_BARS = 2 * S_X + 2 * GCfg<BITS>::S_W + 2 * S_A + 1;
+  static constexpr int OFF_TMEM = OFF_BAR + NUM_BARS * 8;
+  static constexpr int BYTES = OFF_TMEM + 16 + 1024;  // + alignment slack
+};
+
+struct GemmP {
+  const uint32_t* meta;   // [K/128][N]
+  const __half* bias;
+  void* y;
+  int64_t ldy;
+  int64_t m;
+  int64_t n;
+  int kg;
+};
+
+__device__ __forceinline__ uint64_t make_sw128_desc(uint32_t saddr) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFF);
+  d |= (uint64_t)1 << 16;              // LBO (ignored for swizzled K-major)
+  d |= (uint64_t)(1024 >> 4) << 32;    // SBO: 8 rows x 128 B
+  d |= (uint64_t)1 << 46;              // descriptor version (sm_100)
+  d |= (uint64_t)2 << 61;              // SWIZZLE_128B
+  return d;
+}
+
+// instruction descriptor: kind::f16, A=B=f16 K-major, D=f32, M=128, N=256
+constexpr uint32_t kIdesc = (1u << 4) | ((uint32_t)(BT >> 3) << 17) | ((uint32_t)(BN >> 4) << 24);
+
+__device__ __forceinline__ uint32_t hsub_fma(uint32_t h, uint32_t off2, uint32_t s2, uint32_t z2) {
+  __half2 c = __hsub2(*reinterpret_cast<__half2*>(&h), *reinterpret_cast<__half2*>(&off2));
+  __half2 r = __hfma2(c, *reinterpret_cast<__half2*>(&s2), *reinterpret_cast<__half2*>(&z2));
+  return *reinterpret_cast<uint32_t*>(&r);
+}
+
+// Dequantize this thread's row (r) of one 128-k group into 64 half2 columns,
+// written to TMEM in 4 batches of 16 columns.
+template <int BITS>
+__device__ __forceinline__ void dequant_row_to_tmem(const uint8_t* wst, uint32_t meta, int r, uint32_t taddr) {
+  const uint32_t s2 = (meta & 0xFFFFu) * 0x10001u;
+  const uint32_t z2 = (meta >> 16) * 0x10001u;
+  constexpr uint32_t K1024 = 0x64006400u, K64 = 0x54005400u;
+  if constexpr (BITS == 4) {
+    const uint8_t* row = wst + r * 64;
+#pragma unroll
+    for (int b = 0; b < 4; ++b) {
+      const int pc = b ^ ((r >> 1) & 3);  // SWIZZLE_64B
+      uint4 v = *reinterpret_cast<const uint4*>(row + pc * 16);
+      const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
+      uint32_t o[16];
+#pragma unroll
+      for (int w = 0; w < 4; ++w) {
+        const uint32_t x = wv[w], x8 = x >> 8;
+        o[4 * w + 0] = hsub_fma(lop3_and_or(x, 0x000F000Fu, K1024), K1024, s2, z2);
+        o[4 * w + 1] = hsub_fma(lop3_and_or(x, 0x00F000F0u, K64), K64, s2, z2);
+        o[4 * w + 2] = hsub_fma(lop3_and_or(x8, 0x000F000Fu, K1024), K1024, s2, z2);
+        o[4 * w + 3] = hsub_fma(lop3_and_or(x8, 0x00F000F0u, K64), K64, s2, z2);
+      }
+      tmem_st16(taddr + 16 * b, o);
+    }
+  } else if constexpr (BITS == 8) {
+    const uint8_t* row = wst + r * 128;
+#pragma unroll
+    for (int b = 0; b < 4; ++b) {
+      uint32_t o[16];
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int c = 2 * b + h, pc = c ^ (r & 7);  // SWIZZLE_128B
+        uint4 v = *reinterpret_cast<const uint4*>(row + pc * 16);
+        const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+          o[8 * h + 2 * t] = hsub_fma(prmt(wv[t], 0x64646464u, 0x4140u), K1024, s2, z2);
+          o[8 * h + 2 * t + 1] = hsub_fma(prmt(wv[t], 0x64646464u, 0x4342u), K1024, s2, z2);
+        }
+      }
+      tmem_st16(taddr + 16 * b, o);
+    }
+  } else if constexpr (BITS == 3) {
+    const uint32_t* row = reinterpret_cast<const uint32_t*>(wst + r * 48);
+#pragma unroll
+    for (int bl = 0; bl < 4; ++bl) {
+      const uint32_t L0 = row[3 * bl], L1 = row[3 * bl + 1], H = row[3 * bl + 2];
+      uint32_t o[16];
+#pragma unroll
+      for (int a = 0; a < 2; ++a) {
+        const uint32_t La = a ? L1 : L0;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const uint32_t lo = La >> (2 * i);
+          const int sh = i + 8 * a - 2;
+          const uint32_t hs = sh >= 0 ? (H >> sh) : (H << (-sh));
+          uint32_t t;
+          asm("lop3.b32 %0, %1, %2, %3, 0xD8;" : "=r"(t) : "r"(hs), "r"(lo), "r"(0x00030003u));  // mask ? lo : hs
+          o[8 * a + i] = hsub_fma(lop3_and_or(t, 0x00070007u, K1024), K1024, s2, z2);
+        }
+      }
+      tmem_st16(taddr + 16 * bl, o);
+    }
+  } else {
+    // fp16: two SW128 regions (k 0..63, 64..127) of [128 rows x 128 B]
+#pragma unroll
+    for (int b = 0; b < 4; ++b) {
+      const uint8_t* region = wst + (b >> 1) * (BN * 128) + r * 128;
+      uint32_t o[16];
+#pragma unroll
+      for (int h = 0; h < 4; ++h) {
+        const int c = 4 * (b & 1) + h, pc = c ^ (r & 7);
+        uint4 v = *reinterpret_cast<const uint4*>(region + pc * 16);
+        o[4 * h] = v.x; o[4 * h + 1] = v.y; o[4 * h + 2] = v.z; o[4 * h + 3] = v.w;
+      }
+      tmem_st16(taddr + 16 * b, o);
+    }
+  }
+}
+
+template <int BITS, int EPI>
+__global__ void __launch_bounds__(NUM_THREADS, 1)
+    k_gemm(const __grid_constant__ CUtensorMap tm_x, const __grid_constant__ CUtensorMap tm_w,
+           const __grid_constant__ CUtensorMap tm_m, const GemmP p) {
+  using SM = Smem<BITS>;
+  constexpr int S_W = GCfg<BITS>::S_W;
+  constexpr int GB = GCfg<BITS>::GB;
+  constexpr uint32_t W_BYTES = BN * GB;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + SM::OFF_BAR);
+  uint64_t* full_x = bars;
+  uint64_t* empty_x = full_x + S_X;
+  uint64_t* full_w = empty_x + S_X;
+  uint64_t* empty_w = full_w + S_W;
+  uint64_t* full_a = empty_w + S_W;
+  uint64_t* empty_a = full_a + S_A;
+  uint64_t* d_full = empty_a + S_A;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(smem + SM::OFF_TMEM);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t n0 = (int64_t)blockIdx.y * BN;   // weight-row tile
+  const int64_t t0 = (int64_t)blockIdx.x * BT;   // token tile
+  const int kg = p.kg;
+
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < S_X; ++i) { mbar_init(&full_x[i], 1); mbar_init(&empty_x[i], 1); }
+    for (int i = 0; i < S_W; ++i) { mbar_init(&full_w[i], 1); mbar_init(&empty_w[i], 4); }
+    for (int i = 0; i < S_A; ++i) { mbar_init(&full_a[i], 4); mbar_init(&empty_a[i], 1); }
+    mbar_init(d_full, 1);
+    fence_barrier_init();
+    prefetch_tmap(&tm_x);
+    prefetch_tmap(&tm_w);
+    if constexpr (BITS != 16) prefetch_tmap(&tm_m);
+  }
+  if (warp == 1) tmem_alloc(tmem_slot, TMEM_COLS);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    // ---------------- TMA producer
+    if (lane == 0) {
+      int it_x = 0;
+      for (int g = 0; g < kg; ++g) {
+        const int sw = g % S_W, rw = g / S_W;
+        mbar_wait(&empty_w[sw], (rw & 1) ^ 1);
+        uint8_t* wdst = smem + SM::OFF_W + sw * SM::W_STAGE;
+        mbar_arrive_expect_tx(&full_w[sw], W_BYTES + (BITS != 16 ? BN * 4 : 0));
+        if constexpr (BITS == 16) {
+          tma_load_2d(wdst, &tm_w, &full_w[sw], g * 128, (int32_t)n0);
+          tma_load_2d(wdst + BN * 128, &tm_w, &full_w[sw], g * 128 + 64, (int32_t)n0);
+        } else {
+          // placement T16: 4-D box {GB bytes, 16 rows, 1 group, 8 row tiles} -> [128 rows][GB]
+          tma_load_4d(wdst, &tm_w, &full_w[sw], 0, 0, g, (int32_t)(n0 / 16));
+          tma_load_3d(smem + SM::OFF_META + sw * BN * 4, &tm_m, &full_w[sw], 0, g, (int32_t)(n0 / 16));
+        }
+        for (int h = 0; h < 2; ++h, ++it_x) {
+          const int sx = it_x % S_X, rx = it_x / S_X;
+          mbar_wait(&empty_x[sx], (rx & 1) ^ 1);
+          mbar_arrive_expect_tx(&full_x[sx], X_STAGE_BYTES);
+          tma_load_2d(smem + SM::OFF_X + sx * X_STAGE_BYTES, &tm_x, &full_x[sx], g * 128 + h * XK, (int32_t)t0);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ---------------- MMA issuer (single thread)
+    if (lane == 0) {
+      int it_x = 0;
+      for (int g = 0; g < kg; ++g) {
+        const int sa = g % S_A, ra = g / S_A;
+        mbar_wait(&full_a[sa], ra & 1);
+        tc_fence_after();
+        for (int h = 0; h < 2; ++h, ++it_x) {
+          const int sx = it_x % S_X, rx = it_x / S_X;
+          mbar_wait(&full_x[sx], rx & 1);
+          tc_fence_after();
+          const uint32_t xs = smem_u32(smem + SM::OFF_X + sx * X_STAGE_BYTES);
+#pragma unroll
+          for (int kk = 0; kk < XK / 16; ++kk) {
+            const uint64_t bdesc = make_sw128_desc(xs + kk * 32);
+            const uint32_t a_tm = tmem + A_COL + sa * 64 + h * 32 + kk * 8;
+            tc_mma_ts(tmem + D_COL, a_tm, bdesc, kIdesc, (g | h | kk) != 0);
+          }
+          tc_commit(&empty_x[sx]);
+        }
+        tc_commit(&empty_a[sa]);
+      }
+      tc_commit(d_full);
+    }
+  } else {
+    // ---------------- dequant warps (one thread per weight row), then epilogue
+    const int sp = warp & 3;            // TMEM sub-partition this warp may access
+    const int r = sp * 32 + lane;       // row within the tile
+    const uint32_t lane_base = (uint32_t)(sp * 32) << 16;
+    for (int g = 0; g < kg; ++g) {
+      const int sw = g % S_W, rw = g / S_W;
+      const int sa = g % S_A, ra = g / S_A;
+      mbar_wait(&full_w[sw], rw & 1);
+      mbar_wait(&empty_a[sa], (ra & 1) ^ 1);
+      tc_fence_after();
+      const uint32_t meta = reinterpret_cast<const uint32_t*>(smem + SM::OFF_META + sw * BN * 4)[r];
+      dequant_row_to_tmem<BITS>(smem + SM::OFF_W + sw * SM::W_STAGE, meta, r, tmem + lane_base + A_COL + sa * 64);
+      tc_wait_st();
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) {
+        mbar_arrive(&empty_w[sw]);
+        mbar_arrive(&full_a[sa]);
+      }
+    }
+    // ---------------- epilogue
+    mbar_wait(d_full, 0);
+    tc_fence_after();
+    const int64_t nrow = n0 + r;
+    float bias = 0.f;
+    if (p.bias) bias = __half2float(p.bias[nrow]);
+#pragma unroll 1
+    for (int c = 0; c < BT / 16; ++c) {
+      uint32_t v[16];
+      tmem_ld16(tmem + lane_base + D_COL + c * 16, v);
+      tc_wait_ld();
+#pragma unroll
+      for (int i = 0; i < 16; ++i) {
+        const int64_t tok = t0 + c * 16 + i;
+        if (tok < p.m) {
+          const float o = __uint_as_float(v[i]) + bias;
+          if constexpr (EPI == SQ_EPI_F32_ACCUM) {
+            float* yp = static_cast<float*>(p.y) + tok * p.ldy + nrow;
+            *yp += o;
+          } else {
+            static_cast<__half*>(p.y)[tok * p.ldy + nrow] = __float2half_rn(apply_act<EPI>(o));
+          }
+        }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc(tmem, TMEM_COLS);
+  }
+}
+
+// ---------------------------------------------------------------- host side
+typedef CUresult (*EncodeFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                             const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                             CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeFn get_encode() {
+  static EncodeFn fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<EncodeFn>(f);
+  });
+  return fn;
+}
+
+cudaError_t encode_nd(CUtensorMap* m, CUtensorMapDataType dt, const void* ptr, int rank, const uint64_t* dims,
+                      const uint64_t* strides_bytes, const uint32_t* box, CUtensorMapSwizzle sw) {
+  EncodeFn fn = get_encode();
+  if (!fn) return cudaErrorNotSupported;
+  cuuint64_t d[5], st[4];
+  cuuint32_t b[5], es[5];
+  for (int i = 0; i < rank; ++i) { d[i] = dims[i]; b[i] = box[i]; es[i] = 1; }
+  for (int i = 0; i + 1 < rank; ++i) st[i] = strides_bytes[i];
+  CUresult r = fn(m, dt, (cuuint32_t)rank, const_cast<void*>(ptr), d, st, b, es, CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
+                  CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
+}
+
+cudaError_t encode_2d(CUtensorMap* m, CUtensorMapDataType dt, const void* ptr, uint64_t inner, uint64_t outer,
+                      uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer, CUtensorMapSwizzle sw) {
+  const uint64_t dims[2] = {inner, outer}, st[1] = {row_bytes};
+  const uint32_t box[2] = {box_inner, box_outer};
+  return encode_nd(m, dt, ptr, 2, dims, st, box, sw);
+}
+
+template <int BITS, int EPI>
+cudaError_t launch_be(const CUtensorMap& tx, const CUtensorMap& tw, const CUtensorMap& tm, const GemmP& p, cudaStream_t s) {
+  auto kern = k_gemm<BITS, EPI>;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Smem<BITS>::BYTES);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  dim3 grid((unsigned)((p.m + BT - 1) / BT), (unsigned)(p.n / BN));
+  kern<<<grid, NUM_THREADS, Smem<BITS>::BYTES, s>>>(tx, tw, tm, p);
+  return cudaGetLastError();
+}
+
+template <int BITS>
+cudaError_t launch_b(const CUtensorMap& tx, const CUtensorMap& tw, const CUtensorMap& tm, const GemmP& p, int epi,
+                     cudaStream_t s) {
+  switch (epi) {
+    case SQ_EPI_F16: return launch_be<BITS, SQ_EPI_F16>(tx, tw, tm, p, s);
+    case SQ_EPI_F16_RELU: return launch_be<BITS, SQ_EPI_F16_RELU>(tx, tw, tm, p, s);
+    case SQ_EPI_F16_GELU: return launch_be<BITS, SQ_EPI_F16_GELU>(tx, tw, tm, p, s);
+    default: return launch_be<BITS, SQ_EPI_F32_ACCUM>(tx, tw, tm, p, s);
+  }
+}
+
+}  // namespace
+
+cudaError_t launch_gemm(const sq_qweight& w, const __half* x, int64_t ldx, int64_t m, void* y, int64_t ldy, int epi,
+                        cudaStream_t s) {
+  CUtensorMap tx, tw, tm;
+  memset(&tm, 0, sizeof(tm));
+  cudaError_t e = encode_2d(&tx, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, x, (uint64_t)w.k, (uint64_t)m, (uint64_t)ldx * 2,
+                            XK, BT, CU_TENSOR_MAP_SWIZZLE_128B);
+  if (e != cudaSuccess) return e;
+  if (w.bits == 16) {
+    e = encode_2d(&tw, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, w.packed, (uint64_t)w.k, (uint64_t)w.n, (uint64_t)w.k * 2, 64,
+                  BN, CU_TENSOR_MAP_SWIZZLE_128B);
+  } else {
+    // placement T16: [n/16 tiles][kg groups][16 rows][GB bytes]
+    const uint64_t gb = 128 * w.bits / 8, kg = (uint64_t)w.k / 128, nt = (uint64_t)w.n / 16;
+    CUtensorMapSwizzle sw = w.bits == 8 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                        : (w.bits == 4 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_NONE);
+    const uint64_t dw[4] = {gb, 16, kg, nt}, sw_[3] = {gb, 16 * gb, kg * 16 * gb};
+    const uint32_t bw[4] = {(uint32_t)gb, 16, 1, BN / 16};
+    e = encode_nd(&tw, CU_TENSOR_MAP_DATA_TYPE_UINT8, w.packed, 4, dw, sw_, bw, sw);
+    if (e == cudaSuccess) {
+      const uint64_t dm[3] = {16, kg, nt}, sm_[2] = {64, kg * 64};
+      const uint32_t bm[3] = {16, 1, BN / 16};
+      e = encode_nd(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, w.meta, 3, dm, sm_, bm, CU_TENSOR_MAP_SWIZZLE_NONE);
+    }
+  }
+  if (e != cudaSuccess) return e;
+  GemmP p{};
+  p.meta = static_cast<const uint32_t*>(w.meta);
+  p.bias = static_cast<const __half*>(w.bias);
+  p.y = y;
+  p.ldy = ldy;
+  p.m = m;
+  p.n = w.n;
+  p.kg = (int)(w.k / 128);
+  auto t = prof_begin(KC_GEMM, (double)w.n * w.k * w.bits / 8.0 + 2.0 * m * w.k, 2.0 * m * w.n * w.k, s);
+  switch (w.bits) {
+    case 3: e = launch_b<3>(tx, tw, tm, p, epi, s); break;
+    case 4: e = launch_b<4>(tx, tw, tm, p, epi, s); break;
+    case 8: e = launch_b<8>(tx, tw, tm, p, epi, s); break;
+    default: e = launch_b<16>(tx, tw, tm, p, epi, s); break;
+  }
+  prof_end(t, s);
+  count_launch();
+  return e;
+}
+
+}  // namespace sq

@@ -1,0 +1,537 @@
+// K2 — decode dequant-GEMV (P:57 decode phase; "predominantly memory-bound",
+// P:106; decode arithmetic intensity 43-48 on V100).
+//
+// y[m, n] = epi( sum_k x[m, k] * (s[n,g] * c[n,k] + z[n,g]) ),  m <= 32.
+//
+// Design (K2):
+//  * Work unit = 16 output rows x one group (128 k).  The U units are flattened
+//    row-tile-major / group-minor and split evenly over one 16-warp CTA per SM
+//    (and evenly over the CTA's warps): every SM streams the same number of
+//    bytes whatever the shape.
+//  * A lane streams 32 consecutive codes of two rows (g, g+8) per unit with
+//    128-bit loads (INT4 2x16 B, INT8 2x32 B, INT3 2x12 B) from a D-deep
+//    register ring, plus the group metadata; the activation fragment comes
+//    from L1 (re-read by all warps), its group sums from shared memory.
+//  * Unpack in registers with the fp16 "magic number" trick: one LOP3 (PRMT
+//    for INT8) turns a pair of codes into half2(off + c) exactly (off = 1024,
+//    or 64 for the second nibble of each byte in L4) — no per-weight multiply.
+//  * Dot products on mma.sync.m16n8k16 with fp32 accumulation (16 weight rows
+//    = A operand, up to 8 tokens per n8 tile = B operand).  Per group:
+//       sum_k x (off_k + c_k) = sum_k x c_k + xoff   =>
+//       y += s * (D - xoff) + z * xs,   xs = sum x,  xoff = sum off_k x
+//    with (xs, xoff) from sq_xsum (per-group factorised scale/zero).
+//  * Split tiles are reduced in shared memory in fixed warp order; a tile that
+//    straddles two CTAs is finished by the last CTA (atomic counter, fixed CTA
+//    order).  Deterministic; counters self-reset.
+#include "sq_common.cuh"
+
+namespace sq {
+namespace {
+
+constexpr int kWarps = 16;  // one 512-thread CTA per SM
+constexpr int kThreads = kWarps * 32;
+constexpr int kRows = 16;   // rows per unit (mma M)
+constexpr int kXsTok = 32;  // token slots per group in the xsum buffer
+
+struct GemvP {
+  const uint8_t* packed;
+  const uint32_t* meta;
+  const __half* bias;
+  const __half* x;
+  int ldx;
+  int m;
+  int n;
+  int kg;              // groups per row (k / 128)
+  const float2* xsum;  // [kg][32]
+  void* y;
+  int ldy;
+  float* part;  // [CTAs][2][TOK][16] cross-CTA partials
+  int* cnt;     // [n / 16]
+  int U;        // units
+  int W;        // CTAs
+};
+
+template <int BITS>
+struct Cfg;
+template <>
+struct Cfg<3> { static constexpr int LU = 3; static constexpr int GB = 48; static constexpr int D = 4; };
+template <>
+struct Cfg<4> { static constexpr int LU = 4; static constexpr int GB = 64; static constexpr int D = 4; };
+template <>
+struct Cfg<8> { static constexpr int LU = 8; static constexpr int GB = 128; static constexpr int D = 2; };
+template <>
+struct Cfg<16> { static constexpr int LU = 16; static constexpr int GB = 256; static constexpr int D = 1; };
+
+// bytes of one row's 32 codes held by a lane (k in [32q, 32q+32) of the group)
+template <int BITS>
+constexpr int lane_bytes() { return 32 * BITS / 8; }
+
+// this lane's 32 consecutive codes of one row of the current group; p already points at them
+template <int BITS>
+__device__ __forceinline__ void load_codes(const uint8_t* __restrict__ p, uint32_t* c) {
+  if constexpr (BITS == 4) {
+    uint4 v = ldg_nc_v4(p);
+    c[0] = v.x; c[1] = v.y; c[2] = v.z; c[3] = v.w;
+  } else if constexpr (BITS == 8) {
+    uint4 v0 = ldg_nc_v4(p), v1 = ldg_nc_v4(p + 16);
+    c[0] = v0.x; c[1] = v0.y; c[2] = v0.z; c[3] = v0.w;
+    c[4] = v1.x; c[5] = v1.y; c[6] = v1.z; c[7] = v1.w;
+  } else if constexpr (BITS == 3) {
+    c[0] = ldg_nc_u32(p);
+    c[1] = ldg_nc_u32(p + 4);
+    c[2] = ldg_nc_u32(p + 8);
+  } else {
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      uint4 v = ldg_nc_v4(p + 16 * j);
+      c[4 * j] = v.x; c[4 * j + 1] = v.y; c[4 * j + 2] = v.z; c[4 * j + 3] = v.w;
+    }
+  }
+}
+
+// Fragment registers of chunk t (k0 = 32q + 4t): lo = codes (k0, k0+1), hi = (k0+2, k0+3), as half2(off + c).
+template <int BITS>
+__device__ __forceinline__ void frag(const uint32_t* c, int t, uint32_t& lo, uint32_t& hi) {
+  if constexpr (BITS == 4) {
+    // L4: word w holds k = 8w..8w+7, even k in nibbles 0-3, odd k in nibbles 4-7.
+    const uint32_t v = (t & 1) ? (c[t >> 1] >> 8) : c[t >> 1];
+    lo = lop3_and_or(v, 0x000F000Fu, 0x64006400u);  // 1024 + c
+    hi = lop3_and_or(v, 0x00F000F0u, 0x54005400u);  //   64 + c
+  } else if constexpr (BITS == 8) {
+    lo = prmt(c[t], 0x64646464u, 0x4140u);
+    hi = prmt(c[t], 0x64646464u, 0x4342u);
+  } else if constexpr (BITS == 3) {
+    // L3: pair (a, i) = k' 16a + 2i (+1): low bits La >> 2i, high bit H >> (i + 8a).
+    const int a = t >> 2;
+    const uint32_t La = c[a], H = c[2];
+#pragma unroll
+    for (int e = 0; e < 2; ++e) {
+      const int i = 2 * (t & 3) + e;
+      const uint32_t l = La >> (2 * i);
+      const int sh = i + 8 * a - 2;
+      const uint32_t hs = sh >= 0 ? (H >> sh) : (H << (-sh));
+      uint32_t s;
+      asm("lop3.b32 %0, %1, %2, %3, 0xD8;" : "=r"(s) : "r"(hs), "r"(l), "r"(0x00030003u));  // mask ? l : hs
+      const uint32_t r = lop3_and_or(s, 0x00070007u, 0x64006400u);
+      if (e == 0) lo = r; else hi = r;
+    }
+  } else {
+    lo = c[2 * t];
+    hi = c[2 * t + 1];
+  }
+}
+
+// predicated 16-B load (no divergent branch): dst unchanged when !pred
+__device__ __forceinline__ void ldg_v4_pred(uint32_t* d, const void* p, bool pred) {
+  asm volatile(
+      "{\n\t.reg .pred pp;\n\tsetp.ne.b32 pp, %5, 0;\n\t"
+      "@pp ld.global.nc.v4.u32 {%0,%1,%2,%3}, [%4];\n\t}"
+      : "+r"(d[0]), "+r"(d[1]), "+r"(d[2]), "+r"(d[3])
+      : "l"(p), "r"((int)pred));
+}
+
+template <int TOK>
+struct NT { static constexpr int v = TOK / 8; };  // token n8 tiles
+
+template <int TOK, int EPI>
+__device__ __forceinline__ void store_out(const GemvP& p, int tile, int g, int q, const float (&v)[NT<TOK>::v][4]) {
+  const int r0 = tile * kRows + g, r1 = r0 + 8;
+  float b0 = 0.f, b1 = 0.f;
+  if (p.bias) { b0 = __half2float(p.bias[r0]); b1 = __half2float(p.bias[r1]); }
+#pragma unroll
+  for (int j = 0; j < NT<TOK>::v; ++j) {
+#pragma unroll
+    for (int e = 0; e < 2; ++e) {
+      const int tok = 8 * j + 2 * q + e;
+      if (tok >= p.m) continue;
+      const float o0 = v[j][e] + b0, o1 = v[j][2 + e] + b1;
+      if constexpr (EPI == SQ_EPI_F32_ACCUM) {
+        float* yp = static_cast<float*>(p.y) + (int64_t)tok * p.ldy;
+        yp[r0] += o0;
+        yp[r1] += o1;
+      } else {
+        __half* yp = static_cast<__half*>(p.y) + (int64_t)tok * p.ldy;
+        yp[r0] = __float2half_rn(apply_act<EPI>(o0));
+        yp[r1] = __float2half_rn(apply_act<EPI>(o1));
+      }
+    }
+  }
+}
+
+__device__ __forceinline__ int range_lo(int i, int total, int parts) {
+  return (int)(((long long)i * total) / parts);
+}
+
+template <int BITS, int TOK, int EPI>
+__global__ void __launch_bounds__(kThreads, 1) k_gemv(const GemvP p) {
+  constexpr int LU = Cfg<BITS>::LU;
+  constexpr int GB = Cfg<BITS>::GB;
+  constexpr int D = Cfg<BITS>::D;
+  constexpr int NJ = NT<TOK>::v;
+  constexpr bool Q = BITS != 16;
+  extern __shared__ float4 smem4[];
+  float* part_s = reinterpret_cast<float*>(smem4);  // [16 warps][2][TOK][16]
+  float2* xs_s = reinterpret_cast<float2*>(part_s + kWarps * 2 * TOK * kRows);  // [kg][32]
+
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31, g = lane >> 2, q = lane & 3;
+  const int kg = p.kg, m = p.m;
+  const int C0 = range_lo(blockIdx.x, p.U, gridDim.x), C1 = range_lo(blockIdx.x + 1, p.U, gridDim.x);
+  const int R = C1 - C0;
+  const int u0 = C0 + range_lo(warp, R, kWarps), u1 = C0 + range_lo(warp + 1, R, kWarps);
+  const int nunits = u1 - u0;
+  const int head_tile = u0 / kg;
+  const int grp0 = u0 - head_tile * kg;
+  const int64_t pitch = (int64_t)kg * GB;
+
+  // ---- fetch cursor: codes of rows g, g+8 and their meta, D units ahead.
+  // Quantized weights use placement T16: unit u is 16 x GB contiguous bytes at u * 16 * GB,
+  // row r of the unit at r * GB, so the stream is one pointer bumped by a constant.
+  constexpr int UB = 16 * GB;
+  const uint8_t* fcp;
+  const uint32_t* fmp = nullptr;
+  int fgrp = grp0;
+  const int64_t cp_wrap = 15 * pitch;  // (fp16 only) end of row g -> start of row g+16
+  if constexpr (Q) {
+    fcp = p.packed + (int64_t)u0 * UB + g * GB + q * lane_bytes<BITS>();
+    fmp = p.meta + (int64_t)u0 * 16 + g;
+  } else {
+    fcp = p.packed + ((int64_t)head_tile * kRows + g) * pitch + (int64_t)grp0 * GB + q * 64;
+  }
+  uint32_t cb[D][2][LU];
+  uint32_t mb[D][2];
+  auto issue = [&](int slot) {
+    if constexpr (Q) {
+      load_codes<BITS>(fcp, cb[slot][0]);
+      load_codes<BITS>(fcp + 8 * GB, cb[slot][1]);
+      mb[slot][0] = ldg_nc_u32(fmp);
+      mb[slot][1] = ldg_nc_u32(fmp + 8);
+      fcp += UB;
+      fmp += 16;
+    } else {
+      load_codes<BITS>(fcp, cb[slot][0]);
+      load_codes<BITS>(fcp + 8 * pitch, cb[slot][1]);
+      fcp += GB;
+      if (++fgrp == kg) { fgrp = 0; fcp += cp_wrap; }
+    }
+  };
+#pragma unroll
+  for (int j = 0; j < D; ++j)
+    if (j < nunits) issue(j);
+
+  // ---- stage (xs, xoff) per (group, token) in shared memory (overlaps the weight loads):
+  //      xs = sum x, xoff = sum off_k x  (off = 1024, or 1024 / 64 for the two nibble slots of L4)
+  if constexpr (Q) {
+    for (int i = threadIdx.x; i < kg * kXsTok; i += kThreads) {
+      const float2 v = __ldg(p.xsum + i);
+      const float xsv = v.x + v.y;
+      const float xov = BITS == 4 ? fmaf(1024.f, v.x, 64.f * v.y) : 1024.f * xsv;
+      xs_s[i] = make_float2(xsv, xov);
+    }
+  }
+  __syncthreads();
+
+  // activation fragment pointers for token n8-tile j: row 8j + g (predicated off beyond m)
+  const __half* xrow[NJ];
+  bool xon[NJ];
+#pragma unroll
+  for (int j = 0; j < NJ; ++j) {
+    xon[j] = (8 * j + g) < m;
+    xrow[j] = p.x + (int64_t)(xon[j] ? 8 * j + g : 0) * p.ldx + q * 32;
+  }
+
+  // activation fragment (NJ == 1: persistent, lanes beyond m keep zeros under predicated loads)
+  uint32_t xt1[16];
+#pragma unroll
+  for (int i = 0; i < 16; ++i) xt1[i] = 0u;
+
+  int tile = head_tile, grp = grp0;
+  bool seg_from_start = (grp0 == 0);
+  float acc[NJ][4];
+#pragma unroll
+  for (int j = 0; j < NJ; ++j)
+#pragma unroll
+    for (int i = 0; i < 4; ++i) acc[j][i] = 0.f;
+
+  for (int base = 0; base < nunits; base += D) {
+#pragma unroll
+    for (int s = 0; s < D; ++s) {
+      const int ui = base + s;
+      if (ui >= nunits) break;
+#pragma unroll
+      for (int j = 0; j < NJ; ++j) {
+        const __half* xp = xrow[j] + grp * 128;
+        uint32_t xloc[16];
+        uint32_t* xtj = NJ == 1 ? xt1 : xloc;
+        if (NJ > 1) {
+#pragma unroll
+          for (int i = 0; i < 16; ++i) xloc[i] = 0u;
+        }
+#pragma unroll
+        for (int i = 0; i < 4; ++i) ldg_v4_pred(xtj + 4 * i, xp + 8 * i, xon[j]);
+        if constexpr (!Q) {
+#pragma unroll
+          for (int t = 0; t < 8; ++t) {
+            uint32_t a[4];
+            frag<BITS>(cb[s][0], t, a[0], a[2]);
+            frag<BITS>(cb[s][1], t, a[1], a[3]);
+            mma_16816(acc[j], a, xtj[2 * t], xtj[2 * t + 1], acc[j]);
+          }
+        } else {
+          float d[4];
+          {
+            uint32_t a[4];
+            frag<BITS>(cb[s][0], 0, a[0], a[2]);
+            frag<BITS>(cb[s][1], 0, a[1], a[3]);
+            mma_16816_zc(d, a, xtj[0], xtj[1]);
+          }
+#pragma unroll
+          for (int t = 1; t < 8; ++t) {
+            uint32_t a[4];
+            frag<BITS>(cb[s][0], t, a[0], a[2]);
+            frag<BITS>(cb[s][1], t, a[1], a[3]);
+            mma_16816(d, a, xtj[2 * t], xtj[2 * t + 1], d);
+          }
+          const float2 f0 = __half22float2(*reinterpret_cast<const __half2*>(&mb[s][0]));  // (s, z) row g
+          const float2 f1 = __half22float2(*reinterpret_cast<const __half2*>(&mb[s][1]));  // row g+8
+          const float4 xv = *reinterpret_cast<const float4*>(xs_s + grp * kXsTok + 8 * j + 2 * q);
+          // y += s * (D - xoff) + z * xs   (tokens 2q: xv.x/xv.y, 2q+1: xv.z/xv.w)
+          acc[j][0] = fmaf(-f0.x, xv.y, fmaf(f0.y, xv.x, fmaf(f0.x, d[0], acc[j][0])));
+          acc[j][1] = fmaf(-f0.x, xv.w, fmaf(f0.y, xv.z, fmaf(f0.x, d[1], acc[j][1])));
+          acc[j][2] = fmaf(-f1.x, xv.y, fmaf(f1.y, xv.x, fmaf(f1.x, d[2], acc[j][2])));
+          acc[j][3] = fmaf(-f1.x, xv.w, fmaf(f1.y, xv.z, fmaf(f1.x, d[3], acc[j][3])));
+        }
+      }
+      if (ui + D < nunits) issue(s);
+
+      // ---- segment end: row tile finished or this warp's run finished
+      const bool tile_end = (grp == kg - 1);
+      if (tile_end || ui == nunits - 1) {
+        if (seg_from_start && tile_end) {
+          store_out<TOK, EPI>(p, tile, g, q, acc);
+        } else {
+          const int slot = (tile == head_tile) ? 0 : 1;  // head / tail tile of this warp
+          float* pp = part_s + ((warp * 2 + slot) * TOK) * kRows;
+#pragma unroll
+          for (int j = 0; j < NJ; ++j)
+#pragma unroll
+            for (int e = 0; e < 2; ++e) {
+              const int tok = 8 * j + 2 * q + e;
+              pp[tok * kRows + g] = acc[j][e];
+              pp[tok * kRows + g + 8] = acc[j][2 + e];
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < NJ; ++j)
+#pragma unroll
+          for (int i = 0; i < 4; ++i) acc[j][i] = 0.f;
+        seg_from_start = true;
+      }
+      if (++grp == kg) { grp = 0; ++tile; }
+    }
+  }
+  __syncthreads();
+
+  // ---- CTA-level reduction of split tiles (fixed warp order), then cross-CTA fix-up
+  if (R <= 0) return;
+  const int t_first = C0 / kg, t_last = (C1 - 1) / kg;
+  for (int t = t_first + warp; t <= t_last; t += kWarps) {
+    const int lo = t * kg > C0 ? t * kg : C0;
+    const int hi = (t + 1) * kg < C1 ? (t + 1) * kg : C1;  // exclusive
+    const int wa = (int)(((long long)(lo - C0 + 1) * kWarps - 1) / R);
+    const int wb = (int)(((long long)(hi - C0) * kWarps - 1) / R);
+    if (wa == wb && lo == t * kg && hi == (t + 1) * kg) continue;  // one warp stored it directly
+    float v[NJ][4];
+#pragma unroll
+    for (int j = 0; j < NJ; ++j)
+#pragma unroll
+      for (int i = 0; i < 4; ++i) v[j][i] = 0.f;
+    for (int wi = wa; wi <= wb; ++wi) {
+      const int wlo = C0 + range_lo(wi, R, kWarps), whi = C0 + range_lo(wi + 1, R, kWarps);
+      if (whi <= wlo) continue;  // empty warp range
+      const int sl = (wlo < t * kg) ? 1 : 0;
+      const float* qp = part_s + ((wi * 2 + sl) * TOK) * kRows;
+#pragma unroll
+      for (int j = 0; j < NJ; ++j)
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+          const int tok = 8 * j + 2 * q + e;
+          v[j][e] += qp[tok * kRows + g];
+          v[j][2 + e] += qp[tok * kRows + g + 8];
+        }
+    }
+    if (lo == t * kg && hi == (t + 1) * kg) {  // tile entirely inside this CTA
+      store_out<TOK, EPI>(p, t, g, q, v);
+      continue;
+    }
+    // straddles a CTA boundary: publish this CTA's partial, the last CTA reduces
+    const int cslot = (C0 < t * kg) ? 1 : 0;
+    float* gp = p.part + (((int64_t)blockIdx.x * 2 + cslot) * TOK) * kRows;
+#pragma unroll
+    for (int j = 0; j < NJ; ++j)
+#pragma unroll
+      for (int e = 0; e < 2; ++e) {
+        const int tok = 8 * j + 2 * q + e;
+        __stcg(gp + tok * kRows + g, v[j][e]);
+        __stcg(gp + tok * kRows + g + 8, v[j][2 + e]);
+      }
+    __threadfence();
+    __syncwarp();
+    const int NC = gridDim.x;
+    const int ca = (int)(((long long)(t * kg + 1) * NC - 1) / p.U);
+    const int cb2 = (int)(((long long)((t + 1) * kg) * NC - 1) / p.U);
+    int old = 0;
+    if (lane == 0) old = atomicAdd(p.cnt + t, 1);
+    old = __shfl_sync(0xffffffff, old, 0);
+    if (old != cb2 - ca) continue;
+    __threadfence();
+#pragma unroll
+    for (int j = 0; j < NJ; ++j)
+#pragma unroll
+      for (int i = 0; i < 4; ++i) v[j][i] = 0.f;
+    for (int c = ca; c <= cb2; ++c) {
+      const int sl = (range_lo(c, p.U, NC) < t * kg) ? 1 : 0;
+      const float* qp = p.part + (((int64_t)c * 2 + sl) * TOK) * kRows;
+#pragma unroll
+      for (int j = 0; j < NJ; ++j)
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+          const int tok = 8 * j + 2 * q + e;
+          v[j][e] += __ldcg(qp + tok * kRows + g);
+          v[j][2 + e] += __ldcg(qp + tok * kRows + g + 8);
+        }
+    }
+    store_out<TOK, EPI>(p, t, g, q, v);
+    if (lane == 0) p.cnt[t] = 0;
+  }
+}
+
+// xsum[g][t] = (sum_{k%4<2} x[t,k], sum_{k%4>=2} x[t,k]) over group g, t < 32 (0 for t >= m);
+// one warp per (g, t), fixed summation order.
+__global__ void k_xsum(const __half* __restrict__ x, int64_t ldx, int64_t m, int kg, float2* __restrict__ out) {
+  const int64_t id = (int64_t)blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5);
+  if (id >= (int64_t)kg * kXsTok) return;
+  const int lane = threadIdx.x & 31;
+  const int64_t g = id / kXsTok, t = id % kXsTok;
+  float a = 0.f, b = 0.f;
+  if (t < m) {
+    const uint2 raw = *reinterpret_cast<const uint2*>(x + t * ldx + g * 128 + lane * 4);
+    const __half2 lo = *reinterpret_cast<const __half2*>(&raw.x), hi = *reinterpret_cast<const __half2*>(&raw.y);
+    a = __low2float(lo) + __high2float(lo);  // k%4 in {0,1}
+    b = __low2float(hi) + __high2float(hi);  // k%4 in {2,3}
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    a += __shfl_xor_sync(0xffffffff, a, o);
+    b += __shfl_xor_sync(0xffffffff, b, o);
+  }
+  if (lane == 0) out[id] = make_float2(a, b);
+}
+
+size_t gemv_smem(int tok, int kg) { return (size_t)kWarps * 2 * tok * kRows * 4 + (size_t)kg * kXsTok * 8; }
+
+template <int BITS, int TOK, int EPI>
+cudaError_t launch_e(const GemvP& p, cudaStream_t s) {
+  auto kern = k_gemv<BITS, TOK, EPI>;
+  const size_t smem = gemv_smem(TOK, p.kg);
+  static size_t attr = 0;
+  if (smem > attr) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    attr = smem;
+  }
+  kern<<<(unsigned)p.W, kThreads, smem, s>>>(p);
+  return cudaGetLastError();
+}
+
+template <int BITS, int TOK>
+cudaError_t launch_t(const GemvP& p, int epi, cudaStream_t s) {
+  switch (epi) {
+    case SQ_EPI_F16: return launch_e<BITS, TOK, SQ_EPI_F16>(p, s);
+    case SQ_EPI_F16_RELU: return launch_e<BITS, TOK, SQ_EPI_F16_RELU>(p, s);
+    case SQ_EPI_F16_GELU: return launch_e<BITS, TOK, SQ_EPI_F16_GELU>(p, s);
+    default: return launch_e<BITS, TOK, SQ_EPI_F32_ACCUM>(p, s);
+  }
+}
+
+template <int BITS>
+cudaError_t launch_b(const GemvP& p, int epi, cudaStream_t s) {
+  if (p.m <= 8) return launch_t<BITS, 8>(p, epi, s);
+  if (p.m <= 16) return launch_t<BITS, 16>(p, epi, s);
+  return launch_t<BITS, 32>(p, epi, s);
+}
+
+// number of CTAs: one per SM (fewer for tiny problems so every warp gets >= 1 unit)
+int64_t gemv_ctas(int64_t U) {
+  const int64_t full = (int64_t)num_sms();
+  const int64_t need = (U + kWarps - 1) / kWarps;
+  return need < full ? need : full;
+}
+
+int tok_pad(int64_t m) { return m <= 8 ? 8 : (m <= 16 ? 16 : 32); }
+
+// fixed-size counter region (n <= 65536) so linears of different n can share one workspace
+constexpr int64_t kMaxN = 65536;
+size_t cnt_bytes(int64_t) { return (size_t)(kMaxN / kRows) * sizeof(int); }
+
+}  // namespace
+
+size_t xsum_bytes(int64_t k) { return (size_t)(k / 128) * kXsTok * sizeof(float2); }
+
+size_t gemv_workspace_bytes(int64_t n, int64_t k, int64_t m) {
+  const int64_t U = (n / kRows) * (k / 128);
+  const int64_t W = gemv_ctas(U);
+  size_t part = (size_t)W * 2 * tok_pad(m) * kRows * sizeof(float);  // per-CTA boundary partials
+  return cnt_bytes(n) + part + xsum_bytes(k) + 256;
+}
+
+cudaError_t launch_xsum(const __half* x, int64_t ldx, int64_t m, int64_t k, float2* xsum, cudaStream_t s) {
+  const int64_t items = (k / 128) * kXsTok;
+  auto t = prof_begin(KC_GLUE, (double)m * k * 2 + items * 8.0, 0, s);
+  k_xsum<<<(unsigned)((items + 7) / 8), 256, 0, s>>>(x, ldx, m, (int)(k / 128), xsum);
+  prof_end(t, s);
+  count_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t launch_gemv(const sq_qweight& w, const __half* x, int64_t ldx, int m, void* y, int64_t ldy, int epi,
+                        const float2* xsum, void* ws, cudaStream_t s) {
+  if (w.n > kMaxN || w.n / kRows * (w.k / 128) >= (1ll << 31) / 256) return cudaErrorInvalidValue;  // 32-bit index math
+  GemvP p{};
+  p.packed = static_cast<const uint8_t*>(w.packed);
+  p.meta = static_cast<const uint32_t*>(w.meta);
+  p.bias = static_cast<const __half*>(w.bias);
+  p.x = x;
+  p.ldx = (int)ldx;
+  p.m = m;
+  p.n = (int)w.n;
+  p.kg = (int)(w.k / 128);
+  p.y = y;
+  p.ldy = (int)ldy;
+  p.U = (int)((w.n / kRows) * p.kg);
+  p.W = (int)gemv_ctas(p.U);
+  uint8_t* base = static_cast<uint8_t*>(ws);
+  p.cnt = reinterpret_cast<int*>(base);
+  p.part = reinterpret_cast<float*>(base + cnt_bytes(w.n));
+  float2* xs_ws = reinterpret_cast<float2*>(base + cnt_bytes(w.n) + (size_t)p.W * 2 * tok_pad(m) * kRows * sizeof(float));
+  if (w.bits != 16 && xsum == nullptr) {
+    cudaError_t e = launch_xsum(x, ldx, m, w.k, xs_ws, s);
+    if (e != cudaSuccess) return e;
+    xsum = xs_ws;
+  }
+  p.xsum = xsum;
+  const double bytes = (double)w.n * w.k * w.bits / 8.0 + (w.bits != 16 ? (double)w.n * (w.k / 128) * 4.0 : 0.0);
+  auto t = prof_begin(KC_GEMV, bytes, 2.0 * m * w.n * w.k, s);
+  cudaError_t e;
+  switch (w.bits) {
+    case 3: e = launch_b<3>(p, epi, s); break;
+    case 4: e = launch_b<4>(p, epi, s); break;
+    case 8: e = launch_b<8>(p, epi, s); break;
+    default: e = launch_b<16>(p, epi, s); break;
+  }
+  prof_end(t, s);
+  count_launch();
+  return e;
+}
+
+}  // namespace sq

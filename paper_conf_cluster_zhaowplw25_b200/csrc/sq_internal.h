@@ -1,0 +1,54 @@
+// Internal declarations shared by the libsq translation units (not installed).
+#pragma once
+#include <cstdarg>
+#include <cstdint>
+#include <cuda_fp16.h>
+#include <cuda_runtime.h>
+
+#include "sq.h"
+
+namespace sq {
+
+// ---- error state (thread-local message, sq_last_error) ----
+sq_status fail(sq_status st, const char* fmt, ...);
+sq_status cuda_check(cudaError_t e, const char* what);
+
+// ---- launch accounting / profiling (sq_profile_*) ----
+enum KClass { KC_GEMV = 0, KC_GEMM = 1, KC_GLUE = 2, KC_QUANT = 3 };
+struct ProfTicket {
+  int slot = -1;
+};
+ProfTicket prof_begin(int kclass, double bytes, double flops, cudaStream_t s);
+void prof_end(ProfTicket t, cudaStream_t s);
+void count_launch(int n = 1);
+
+// ---- kernel launchers (validated arguments) ----
+cudaError_t launch_quantize(const __half* w, int64_t n, int64_t k, int bits, int group, uint8_t* codes,
+                            __half* scales, __half* zeros, cudaStream_t s);
+cudaError_t launch_pack(const uint8_t* codes, const __half* scales, const __half* zeros, int64_t n, int64_t k,
+                        int bits, int group, void* packed, uint32_t* meta, cudaStream_t s);
+cudaError_t launch_xsum(const __half* x, int64_t ldx, int64_t m, int64_t k, float2* xsum, cudaStream_t s);
+
+size_t gemv_workspace_bytes(int64_t n, int64_t k, int64_t m);
+size_t xsum_bytes(int64_t k);
+cudaError_t launch_gemv(const sq_qweight& w, const __half* x, int64_t ldx, int m, void* y, int64_t ldy, int epi,
+                        const float2* xsum, void* ws, cudaStream_t s);
+
+cudaError_t launch_gemm(const sq_qweight& w, const __half* x, int64_t ldx, int64_t m, void* y, int64_t ldy,
+                        int epi, cudaStream_t s);
+
+cudaError_t launch_layernorm_f16(const float* x, int64_t rows, int64_t d, __half* y, float2* xsum,
+                                 const float* copy_src, float* copy_dst, cudaStream_t s);
+cudaError_t launch_layernorm_f32(const float* x, int64_t rows, int64_t d, float* y, cudaStream_t s);
+cudaError_t launch_copy_rows(const float* src, int64_t sstride, int64_t rows, int64_t d, float* dst, int64_t dstride,
+                             cudaStream_t s);
+
+// ---- stage forward (sq_stage.cu), used by the pipeline runner ----
+size_t stage_workspace_bytes(const sq_layer* layers, int n_layers, int64_t max_tokens);
+sq_status stage_forward(const sq_layer* layers, int n_layers, int phase, const float* x_in, int64_t tokens,
+                        float* x_out, void* qkv_dbg, void* ws, size_t ws_bytes, cudaStream_t s);
+sq_status check_layers(const sq_layer* layers, int n_layers, const char* who);
+
+int num_sms();
+
+}  // namespace sq

@@ -1,0 +1,393 @@
+// a6 — uneven layer-wise pipeline with phase-specific micro-batch sizes
+// ("the slowest stage limits the overall pipeline throughput"; P:152 one
+// worker per stage, master re-batches between phases; eq. (4) P:202-204:
+// latency = all stages + (mu - 1) x slowest, mu_pre = ceil(B/eta),
+// mu_dec = ceil(B/xi); eq. (7) P:214 asynchronous transfers; eqs. (15)-(16)
+// contiguous partition).
+//
+// One process per GPU.  Stage r holds layers {l : stage_of_layer[l] == r}.
+// Transfers are NCCL point-to-point over NVLink on two dedicated streams
+// (send / recv), each on its own 2-rank "link" communicator (r -> r+1 mod P),
+// so every communicator is driven by exactly one stream in one order and the
+// ring (forward activations + last->first loop-back) cannot deadlock.
+// Compute of micro-batch m+1 overlaps the transfer of micro-batch m
+// (double-buffered activations, CUDA events for the dependencies).
+//
+// Items (identical order on every rank): prefill m = 0..mu_pre-1, then decode
+// t = 1..n_decode, m = 0..mu_dec-1.  The last stage writes out[b, 0] (hidden at
+// the last prompt position) / out[b, t] and loops LN(hidden) back to stage 0
+// as the next decode input (R13/R14).
+#include <nccl.h>
+
+#include <algorithm>
+#include <cstring>
+#include <vector>
+
+#include "sq_common.cuh"
+
+struct sq_comm {
+  int nranks = 1, rank = 0;
+  bool local = false;
+  ncclComm_t world = nullptr, send_comm = nullptr, recv_comm = nullptr;
+  cudaStream_t s_send = nullptr, s_recv = nullptr;
+};
+
+namespace sq {
+namespace {
+
+sq_status nccl_check(ncclResult_t r, const char* what) {
+  if (r == ncclSuccess) return SQ_OK;
+  return fail(SQ_ENCCL, "%s: %s", what, ncclGetErrorString(r));
+}
+
+struct PlanView {
+  int L, P, h1, h2, B, eta, xi, s, n_dec;
+  int mu_pre, mu_dec;
+  std::vector<int> first_layer;  // [P+1]
+};
+
+PlanView view(const sq_plan& pl) {
+  PlanView v{};
+  v.L = pl.n_layers; v.P = pl.n_stages; v.h1 = pl.hidden; v.h2 = pl.ffn; v.B = pl.B;
+  v.eta = pl.eta; v.xi = pl.xi; v.s = pl.prompt_len; v.n_dec = pl.n_decode;
+  v.mu_pre = (pl.B + pl.eta - 1) / pl.eta;
+  v.mu_dec = (pl.B + pl.xi - 1) / pl.xi;
+  v.first_layer.assign(v.P + 1, v.L);
+  for (int l = v.L - 1; l >= 0; --l) v.first_layer[pl.stage_of_layer[l]] = l;
+  v.first_layer[v.P] = v.L;
+  return v;
+}
+
+struct Ws {
+  size_t stage, act, decin, lb, total;
+};
+
+Ws ws_layout(const PlanView& v, const sq_layer* layers, int n_layers, int rank) {
+  Ws w{};
+  size_t off = 0;
+  auto al = [](size_t x) { return (x + 255) / 256 * 256; };
+  const int64_t tmax = std::max<int64_t>((int64_t)v.eta * v.s, v.xi);
+  w.stage = off; off += al(stage_workspace_bytes(layers, n_layers, tmax));
+  w.act = off;   off += 2 * al((size_t)tmax * v.h1 * 4);
+  const bool first = rank <= 0, last = rank < 0 || rank == v.P - 1;
+  w.decin = off; if (first) off += al((size_t)v.B * v.h1 * 4);
+  w.lb = off;    if (last) off += 2 * al((size_t)std::max(v.eta, v.xi) * v.h1 * 4);
+  w.total = off;
+  return w;
+}
+
+}  // namespace
+}  // namespace sq
+
+using namespace sq;
+
+extern "C" {
+
+sq_status sq_plan_check(const sq_plan* p) {
+  if (!p) return fail(SQ_EINVAL, "sq_plan_check: null plan");
+  if (p->n_layers < 1 || p->n_stages < 1 || p->n_stages > p->n_layers)
+    return fail(SQ_EINVAL, "sq_plan_check: need 1 <= n_stages <= n_layers");
+  if (p->hidden <= 0 || p->hidden % 128 || p->ffn <= 0 || p->ffn % 128 || p->group != 128)
+    return fail(SQ_EINVAL, "sq_plan_check: hidden/ffn multiples of 128, group 128");
+  if (!p->bits || !p->stage_of_layer) return fail(SQ_EINVAL, "sq_plan_check: null bits/stage_of_layer");
+  if (p->B < 1 || p->eta < 1 || p->xi < 1 || p->xi > 32 || p->prompt_len < 1 || p->n_decode < 0)
+    return fail(SQ_EINVAL, "sq_plan_check: need B,eta,s >= 1, 1 <= xi <= 32, n_decode >= 0");
+  // eqs. (15)-(16): u_{1,1} = 1, u_{L,N} = 1, adjacent layers on the same or next stage
+  if (p->stage_of_layer[0] != 0 || p->stage_of_layer[p->n_layers - 1] != p->n_stages - 1)
+    return fail(SQ_EINVAL, "sq_plan_check: first layer must be on stage 0 and last on stage n_stages-1");
+  for (int l = 0; l < p->n_layers; ++l) {
+    const int b = p->bits[l];
+    if (b != 3 && b != 4 && b != 8 && b != 16) return fail(SQ_EINVAL, "sq_plan_check: layer %d bits %d", l, b);
+    if (l > 0) {
+      const int d = p->stage_of_layer[l] - p->stage_of_layer[l - 1];
+      if (d != 0 && d != 1) return fail(SQ_EINVAL, "sq_plan_check: partition not contiguous at layer %d", l);
+    }
+  }
+  return SQ_OK;
+}
+
+size_t sq_comm_unique_id_bytes(void) { return sizeof(ncclUniqueId); }
+
+sq_status sq_comm_get_unique_id(uint8_t* id_host) {
+  if (!id_host) return fail(SQ_EINVAL, "sq_comm_get_unique_id: null");
+  ncclUniqueId id;
+  sq_status st = nccl_check(ncclGetUniqueId(&id), "ncclGetUniqueId");
+  if (st) return st;
+  memcpy(id_host, &id, sizeof(id));
+  return SQ_OK;
+}
+
+sq_status sq_comm_init(sq_comm** out, const uint8_t* id_host, int nranks, int rank) {
+  if (!out || !id_host || nranks < 1 || rank < 0 || rank >= nranks)
+    return fail(SQ_EINVAL, "sq_comm_init: bad arguments");
+  if (nranks > 1 && nranks % 2) return fail(SQ_ENOTSUP, "sq_comm_init: odd stage counts > 1 not implemented");
+  sq_comm* c = new sq_comm();
+  c->nranks = nranks;
+  c->rank = rank;
+  if (nranks > 1) {
+    ncclUniqueId id;
+    memcpy(&id, id_host, sizeof(id));
+    sq_status st = nccl_check(ncclCommInitRank(&c->world, nranks, id, rank), "ncclCommInitRank");
+    if (st) { delete c; return st; }
+    // links L_j = (j -> j+1 mod P).  Split A holds the even links, split B the odd ones;
+    // inside a link the sender is comm-rank 0 (key 0), the receiver comm-rank 1.
+    const int P = nranks, r = rank;
+    ncclComm_t a = nullptr, b = nullptr;
+    const int colorA = r / 2, keyA = r % 2;                       // even r: sender of L_r; odd r: receiver of L_{r-1}
+    const int colorB = (r % 2) ? r / 2 : ((r - 1 + P) % P) / 2;   // odd r: sender of L_r; even r: receiver of L_{r-1}
+    const int keyB = (r % 2) ? 0 : 1;
+    if ((st = nccl_check(ncclCommSplit(c->world, colorA, keyA, &a, nullptr), "ncclCommSplit(A)"))) { delete c; return st; }
+    if ((st = nccl_check(ncclCommSplit(c->world, colorB, keyB, &b, nullptr), "ncclCommSplit(B)"))) { delete c; return st; }
+    c->send_comm = (r % 2 == 0) ? a : b;
+    c->recv_comm = (r % 2 == 0) ? b : a;
+  }
+  cudaStreamCreateWithFlags(&c->s_send, cudaStreamNonBlocking);
+  cudaStreamCreateWithFlags(&c->s_recv, cudaStreamNonBlocking);
+  *out = c;
+  return SQ_OK;
+}
+
+sq_status sq_comm_init_local(sq_comm** out, int nstages) {
+  if (!out || nstages < 1) return fail(SQ_EINVAL, "sq_comm_init_local: bad arguments");
+  sq_comm* c = new sq_comm();
+  c->nranks = nstages;
+  c->rank = -1;
+  c->local = true;
+  *out = c;
+  return SQ_OK;
+}
+
+sq_status sq_comm_destroy(sq_comm* c) {
+  if (!c) return SQ_OK;
+  if (c->send_comm) ncclCommDestroy(c->send_comm);
+  if (c->recv_comm) ncclCommDestroy(c->recv_comm);
+  if (c->world) ncclCommDestroy(c->world);
+  if (c->s_send) cudaStreamDestroy(c->s_send);
+  if (c->s_recv) cudaStreamDestroy(c->s_recv);
+  delete c;
+  return SQ_OK;
+}
+
+size_t sq_pipeline_workspace_bytes(const sq_plan* plan, const sq_layer* layers, int rank) {
+  if (sq_plan_check(plan) != SQ_OK || !layers) return 0;
+  PlanView v = view(*plan);
+  const int n = rank < 0 ? v.L : v.first_layer[rank + 1] - v.first_layer[rank];
+  return ws_layout(v, layers, n, rank).total;
+}
+
+sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers, int n_layers, sq_comm* comm,
+                          const float* x0, float* out, void* ws_dev, size_t ws_bytes, sq_run_stats* stats,
+                          sq_stream_t stream_) {
+  sq_status st = sq_plan_check(plan);
+  if (st) return st;
+  const PlanView v = view(*plan);
+  const bool local = (rank < 0);
+  if (local && comm && !comm->local) return fail(SQ_EINVAL, "sq_pipeline_run: rank -1 needs a local comm (or NULL)");
+  if (!local) {
+    if (rank >= v.P) return fail(SQ_EINVAL, "sq_pipeline_run: rank %d >= n_stages %d", rank, v.P);
+    if (v.P > 1 && (!comm || comm->local || comm->nranks != v.P || comm->rank != rank))
+      return fail(SQ_EINVAL, "sq_pipeline_run: comm does not match (nranks %d, rank %d)", comm ? comm->nranks : -1,
+                  comm ? comm->rank : -1);
+  }
+  const int my_first = local ? 0 : v.first_layer[rank];
+  const int my_n = local ? v.L : v.first_layer[rank + 1] - v.first_layer[rank];
+  if (n_layers != my_n) return fail(SQ_EINVAL, "sq_pipeline_run: got %d layers, plan assigns %d to rank %d", n_layers, my_n, rank);
+  if ((st = check_layers(layers, n_layers, "sq_pipeline_run"))) return st;
+  for (int i = 0; i < n_layers; ++i) {
+    if (layers[i].bits != plan->bits[my_first + i]) return fail(SQ_EINVAL, "sq_pipeline_run: layer %d bits differ from plan", my_first + i);
+    if (layers[i].o.n != v.h1 || layers[i].fc1.n != v.h2) return fail(SQ_EINVAL, "sq_pipeline_run: layer shapes differ from plan");
+  }
+  const bool is_first = local || rank == 0, is_last = local || rank == v.P - 1;
+  if (is_first && !x0) return fail(SQ_EINVAL, "sq_pipeline_run: stage 0 needs x0");
+  if (is_last && !out) return fail(SQ_EINVAL, "sq_pipeline_run: last stage needs out");
+  const Ws W = ws_layout(v, layers, n_layers, rank);
+  if (!ws_dev || ws_bytes < W.total || (reinterpret_cast<uintptr_t>(ws_dev) & 255u))
+    return fail(SQ_ENOMEM, "sq_pipeline_run: workspace %zu < %zu (or null / not 256-B aligned)", ws_bytes, W.total);
+
+  cudaStream_t S = (cudaStream_t)stream_;
+  uint8_t* base = static_cast<uint8_t*>(ws_dev);
+  void* stage_ws = base + W.stage;
+  const int64_t tmax = std::max<int64_t>((int64_t)v.eta * v.s, v.xi);
+  const size_t act_slot = ((size_t)tmax * v.h1 * 4 + 255) / 256 * 256;
+  float* act[2] = {reinterpret_cast<float*>(base + W.act), reinterpret_cast<float*>(base + W.act + act_slot)};
+  float* dec_in = reinterpret_cast<float*>(base + W.decin);
+  const size_t lb_slot = ((size_t)std::max(v.eta, v.xi) * v.h1 * 4 + 255) / 256 * 256;
+  float* lb[2] = {reinterpret_cast<float*>(base + W.lb), reinterpret_cast<float*>(base + W.lb + lb_slot)};
+  const int64_t out_rows = 1 + v.n_dec;
+  const int64_t h1 = v.h1;
+  const size_t stage_ws_bytes = W.act - W.stage;
+  const bool dist = !local && v.P > 1;
+
+  const int64_t launches0 = sq_launch_count();
+  cudaEvent_t ev_start, ev_pre, ev_end;
+  cudaEventCreate(&ev_start); cudaEventCreate(&ev_pre); cudaEventCreate(&ev_end);
+  cudaEvent_t ev_free[2], ev_lbfree[2], ev_recv[2], ev_ready, ev_lbready[2], ev_consumed, ev_dec_read;
+  for (int i = 0; i < 2; ++i) {
+    cudaEventCreateWithFlags(&ev_free[i], cudaEventDisableTiming);
+    cudaEventCreateWithFlags(&ev_lbfree[i], cudaEventDisableTiming);
+    cudaEventCreateWithFlags(&ev_recv[i], cudaEventDisableTiming);
+    cudaEventCreateWithFlags(&ev_lbready[i], cudaEventDisableTiming);
+  }
+  cudaEventCreateWithFlags(&ev_ready, cudaEventDisableTiming);
+  cudaEventCreateWithFlags(&ev_consumed, cudaEventDisableTiming);
+  cudaEventCreateWithFlags(&ev_dec_read, cudaEventDisableTiming);
+  cudaEventRecord(ev_start, S);
+  if (dist) {
+    cudaStreamWaitEvent(comm->s_send, ev_start, 0);
+    cudaStreamWaitEvent(comm->s_recv, ev_start, 0);
+  }
+  int64_t bytes_sent = 0;
+  cudaError_t ce = cudaSuccess;
+  sq_status rs = SQ_OK;
+
+  // loop-back bookkeeping at stage 0 (distributed): LB index i -> rows of dec_in
+  // order: prefill mb 0..mu_pre-1, then decode (t, m) for t = 1..n_dec-1
+  const int n_lb = v.mu_pre + std::max(0, v.n_dec - 1) * v.mu_dec;
+  auto lb_rows = [&](int i, int64_t& row0, int64_t& nrows) {
+    if (i < v.mu_pre) {
+      row0 = (int64_t)i * v.eta;
+      nrows = std::min<int64_t>(v.eta, v.B - row0);
+    } else {
+      const int m = (i - v.mu_pre) % v.mu_dec;
+      row0 = (int64_t)m * v.xi;
+      nrows = std::min<int64_t>(v.xi, v.B - row0);
+    }
+  };
+  int lb_posted = 0;
+  auto post_lb_recvs = [&](int upto) {  // stage 0: post loop-back recvs [lb_posted, upto]
+    for (; lb_posted <= upto && lb_posted < n_lb; ++lb_posted) {
+      int64_t r0, nr;
+      lb_rows(lb_posted, r0, nr);
+      // WAR: a decode loop-back overwrites dec_in rows that earlier decode items read
+      if (lb_posted >= v.mu_pre) cudaStreamWaitEvent(comm->s_recv, ev_dec_read, 0);
+      ncclResult_t nr_ = ncclRecv(dec_in + r0 * h1, (size_t)(nr * h1), ncclFloat32, 0, comm->recv_comm, comm->s_recv);
+      if (nr_ != ncclSuccess) { rs = nccl_check(nr_, "ncclRecv(loop-back)"); return; }
+    }
+    cudaEventRecord(ev_recv[0], comm->s_recv);
+    cudaStreamWaitEvent(S, ev_recv[0], 0);
+  };
+
+  const int total_items = v.mu_pre + v.n_dec * v.mu_dec;
+  int slot = 0, lbslot = 0;
+  for (int it = 0; it < total_items && rs == SQ_OK && ce == cudaSuccess; ++it) {
+    const bool pre = it < v.mu_pre;
+    const int m = pre ? it : (it - v.mu_pre) % v.mu_dec;
+    const int t = pre ? 0 : 1 + (it - v.mu_pre) / v.mu_dec;
+    const int64_t seq0 = pre ? (int64_t)m * v.eta : (int64_t)m * v.xi;
+    const int64_t nseq = std::min<int64_t>(pre ? v.eta : v.xi, v.B - seq0);
+    const int64_t T = pre ? nseq * v.s : nseq;
+    const int phase = pre ? SQ_PREFILL : SQ_DECODE;
+    if (pre == false && it == v.mu_pre) cudaEventRecord(ev_pre, S);
+    float* buf = act[slot];
+
+    // ---------------- input
+    const float* x_in;
+    if (is_first) {
+      if (pre) {
+        x_in = x0 + seq0 * v.s * h1;
+      } else {
+        if (dist) {
+          int need;
+          if (t == 1) need = (int)((seq0 + nseq - 1) / v.eta);
+          else need = v.mu_pre + (t - 2) * v.mu_dec + m;
+          post_lb_recvs(need);
+          if (rs) break;
+        }
+        x_in = dec_in + seq0 * h1;
+      }
+      if (dist) cudaStreamWaitEvent(S, ev_free[slot], 0);  // previous send from this buffer done
+    } else {
+      // recv into buf (after its previous send completed)
+      cudaStreamWaitEvent(comm->s_recv, ev_free[slot], 0);
+      ncclResult_t r = ncclRecv(buf, (size_t)(T * h1), ncclFloat32, 0, comm->recv_comm, comm->s_recv);
+      if (r != ncclSuccess) { rs = nccl_check(r, "ncclRecv"); break; }
+      cudaEventRecord(ev_recv[slot], comm->s_recv);
+      cudaStreamWaitEvent(S, ev_recv[slot], 0);
+      x_in = buf;
+    }
+
+    // ---------------- compute: this rank's layers (local mode: every stage in order)
+    if (local) {
+      const float* xi = x_in;
+      for (int r = 0; r < v.P && rs == SQ_OK; ++r) {
+        const int f = v.first_layer[r], nl = v.first_layer[r + 1] - f;
+        rs = stage_forward(layers + f, nl, phase, xi, T, buf, nullptr, stage_ws, stage_ws_bytes, S);
+        xi = buf;  // the "transfer" to the next stage is the buffer itself
+      }
+    } else {
+      rs = stage_forward(layers, n_layers, phase, x_in, T, buf, nullptr, stage_ws, stage_ws_bytes, S);
+    }
+    if (rs) break;
+    if (is_first && !pre && dist) cudaEventRecord(ev_dec_read, S);
+
+    // ---------------- output
+    if (!is_last) {
+      cudaEventRecord(ev_ready, S);
+      cudaStreamWaitEvent(comm->s_send, ev_ready, 0);
+      ncclResult_t r = ncclSend(buf, (size_t)(T * h1), ncclFloat32, 1, comm->send_comm, comm->s_send);
+      if (r != ncclSuccess) { rs = nccl_check(r, "ncclSend"); break; }
+      bytes_sent += T * h1 * 4;
+      cudaEventRecord(ev_free[slot], comm->s_send);
+    } else {
+      // out rows and LN loop-back
+      const float* src = pre ? buf + (int64_t)(v.s - 1) * h1 : buf;
+      const int64_t sstride = pre ? (int64_t)v.s * h1 : h1;
+      ce = launch_copy_rows(src, sstride, nseq, h1, out + (seq0 * out_rows + t) * h1, out_rows * h1, S);
+      if (ce) break;
+      const bool need_lb = t < v.n_dec;  // the last step's successor input is never consumed
+      if (need_lb) {
+        if (!dist) {
+          // single-GPU (or virtual) pipeline: e = LN(hidden) straight into dec_in
+          ce = launch_copy_rows(src, sstride, nseq, h1, lb[0], h1, S);
+          if (!ce) ce = launch_layernorm_f32(lb[0], nseq, h1, dec_in + seq0 * h1, S);
+        } else {
+          cudaStreamWaitEvent(S, ev_lbfree[lbslot], 0);
+          ce = launch_copy_rows(src, sstride, nseq, h1, lb[lbslot], h1, S);
+          if (!ce) ce = launch_layernorm_f32(lb[lbslot], nseq, h1, lb[lbslot], S);
+          if (ce) break;
+          cudaEventRecord(ev_lbready[lbslot], S);
+          cudaStreamWaitEvent(comm->s_send, ev_lbready[lbslot], 0);
+          ncclResult_t r = ncclSend(lb[lbslot], (size_t)(nseq * h1), ncclFloat32, 1, comm->send_comm, comm->s_send);
+          if (r != ncclSuccess) { rs = nccl_check(r, "ncclSend(loop-back)"); break; }
+          bytes_sent += nseq * h1 * 4;
+          cudaEventRecord(ev_lbfree[lbslot], comm->s_send);
+          lbslot ^= 1;
+        }
+        if (ce) break;
+      }
+      if (dist) cudaEventRecord(ev_free[slot], S);
+    }
+    slot ^= 1;
+  }
+  if (v.mu_dec == 0 || v.n_dec == 0) cudaEventRecord(ev_pre, S);
+  if (dist && rs == SQ_OK) {
+    cudaEventRecord(ev_ready, comm->s_send);
+    cudaStreamWaitEvent(S, ev_ready, 0);
+    cudaEventRecord(ev_consumed, comm->s_recv);
+    cudaStreamWaitEvent(S, ev_consumed, 0);
+  }
+  cudaEventRecord(ev_end, S);
+  cudaError_t se = cudaEventSynchronize(ev_end);
+  if (ce == cudaSuccess) ce = se;
+  if (ce == cudaSuccess) ce = cudaGetLastError();
+  if (stats && rs == SQ_OK && ce == cudaSuccess) {
+    float tt = 0.f, tp = 0.f;
+    cudaEventElapsedTime(&tt, ev_start, ev_end);
+    cudaEventElapsedTime(&tp, ev_start, ev_pre);
+    stats->t_total_ms = tt;
+    stats->t_prefill_ms = tp;
+    stats->t_decode_ms = tt - tp;
+    stats->tokens_per_s = tt > 0 ? (double)v.B * (1 + v.n_dec) / (tt * 1e-3) : 0.0;
+    stats->bytes_sent = bytes_sent;
+    stats->gpu_launches = sq_launch_count() - launches0;
+  }
+  cudaEventDestroy(ev_start); cudaEventDestroy(ev_pre); cudaEventDestroy(ev_end);
+  for (int i = 0; i < 2; ++i) {
+    cudaEventDestroy(ev_free[i]); cudaEventDestroy(ev_lbfree[i]); cudaEventDestroy(ev_recv[i]); cudaEventDestroy(ev_lbready[i]);
+  }
+  cudaEventDestroy(ev_ready); cudaEventDestroy(ev_consumed); cudaEventDestroy(ev_dec_read);
+  if (rs) return rs;
+  return cuda_check(ce, "sq_pipeline_run");
+}
+
+}  // extern "C"

@@ -1,0 +1,167 @@
+// a5 — stage forward: the consecutive decoder layers of one pipeline stage, each
+// with its own bit-width from the plan.  Per layer
+// (R11/R12, pre-LN block, attention stub = V):
+//   a = LN(x) -> fp16 (+ group sums)     [K5]
+//   qkv = a Wqkv^T (+b)                  [K2 decode | K3 prefill]   fp16
+//   x  += v Wo^T (+b)                    [K2 | K3, fused fp32 residual add]
+//   a = LN(x)                            [K5]
+//   u = act(a W1^T + b1)                 [K2 | K3, fused activation] fp16
+//   x += u W2^T (+b2)                    [K2 | K3, fused fp32 residual add]
+// The residual stream stays fp32 in HBM (R9); every linear reads fp16.
+#include <cstring>
+
+#include "sq_common.cuh"
+
+namespace sq {
+namespace {
+
+struct WsLayout {
+  size_t a16, qkv16, u16, xs, gemv, total;
+};
+
+int64_t align_up(int64_t v, int64_t a) { return (v + a - 1) / a * a; }
+
+WsLayout layout(const sq_layer* layers, int n_layers, int64_t T) {
+  // The decode GEMV region (self-resetting counters first) sits at a FIXED offset 0 and is
+  // sized for the largest decode micro-batch (32 tokens), so its zero-initialised counters
+  // are never overwritten by activations when the token count changes between calls.
+  const int64_t h1 = layers[0].o.n, h2 = layers[0].fc1.n;
+  WsLayout L{};
+  size_t g = 0;
+  for (int l = 0; l < n_layers; ++l) {
+    const sq_qweight* ws[4] = {&layers[l].qkv, &layers[l].o, &layers[l].fc1, &layers[l].fc2};
+    for (auto* w : ws) {
+      size_t b = gemv_workspace_bytes(w->n, w->k, 32);
+      if (b > g) g = b;
+    }
+  }
+  size_t off = 0;
+  L.gemv = off;  off += align_up((int64_t)g, 256);
+  L.a16 = off;   off += align_up(T * h1 * 2, 256);
+  L.qkv16 = off; off += align_up(T * 3 * h1 * 2, 256);
+  L.u16 = off;   off += align_up(T * h2 * 2, 256);
+  L.xs = off;    off += align_up((int64_t)xsum_bytes(h2 > h1 ? h2 : h1), 256);
+  L.total = off;
+  return L;
+}
+
+sq_status check_w(const sq_qweight& w, int64_t n, int64_t k, int bits, const char* who, int l, const char* name) {
+  if (w.n != n || w.k != k) return fail(SQ_EINVAL, "%s: layer %d %s shape [%lld,%lld] != [%lld,%lld]", who, l, name, (long long)w.n, (long long)w.k, (long long)n, (long long)k);
+  if (w.bits != bits) return fail(SQ_EINVAL, "%s: layer %d %s bits %d != layer bits %d", who, l, name, w.bits, bits);
+  if (w.bits != 3 && w.bits != 4 && w.bits != 8 && w.bits != 16) return fail(SQ_EINVAL, "%s: bad bits", who);
+  if (w.bits != 16 && (w.group != 128 || !w.meta)) return fail(SQ_ENOTSUP, "%s: layer %d %s needs group 128 + meta", who, l, name);
+  if (!w.packed) return fail(SQ_EINVAL, "%s: layer %d %s null packed", who, l, name);
+  return SQ_OK;
+}
+
+}  // namespace
+
+sq_status check_layers(const sq_layer* layers, int n_layers, const char* who) {
+  if (!layers || n_layers <= 0) return fail(SQ_EINVAL, "%s: no layers", who);
+  const int64_t h1 = layers[0].o.n, h2 = layers[0].fc1.n;
+  if (h1 <= 0 || h1 % 128 || h1 > 14336 || h2 <= 0 || h2 % 128)
+    return fail(SQ_EINVAL, "%s: hidden %lld must be a multiple of 128 <= 14336; ffn %lld multiple of 128", who, (long long)h1, (long long)h2);
+  for (int l = 0; l < n_layers; ++l) {
+    const sq_layer& L = layers[l];
+    if (L.act != 0 && L.act != 1) return fail(SQ_EINVAL, "%s: layer %d act %d", who, l, L.act);
+    sq_status st;
+    if ((st = check_w(L.qkv, 3 * h1, h1, L.bits, who, l, "qkv"))) return st;
+    if ((st = check_w(L.o, h1, h1, L.bits, who, l, "o"))) return st;
+    if ((st = check_w(L.fc1, h2, h1, L.bits, who, l, "fc1"))) return st;
+    if ((st = check_w(L.fc2, h1, h2, L.bits, who, l, "fc2"))) return st;
+  }
+  return SQ_OK;
+}
+
+size_t stage_workspace_bytes(const sq_layer* layers, int n_layers, int64_t max_tokens) {
+  return layout(layers, n_layers, max_tokens).total;
+}
+
+sq_status stage_forward(const sq_layer* layers, int n_layers, int phase, const float* x_in, int64_t T, float* x_out,
+                        void* qkv_dbg, void* ws, size_t ws_bytes, cudaStream_t s) {
+  const int64_t h1 = layers[0].o.n, h2 = layers[0].fc1.n;
+  const WsLayout W = layout(layers, n_layers, T);
+  uint8_t* base = static_cast<uint8_t*>(ws);
+  __half* a16 = reinterpret_cast<__half*>(base + W.a16);
+  __half* qkv16 = reinterpret_cast<__half*>(base + W.qkv16);
+  __half* u16 = reinterpret_cast<__half*>(base + W.u16);
+  float2* xs = reinterpret_cast<float2*>(base + W.xs);
+  void* gws = base + W.gemv;
+  const bool dec = phase == SQ_DECODE;
+  auto lin = [&](const sq_qweight& w, const __half* x, int64_t ldx, void* y, int64_t ldy, int epi,
+                 const float2* xsum) -> cudaError_t {
+    if (dec) return launch_gemv(w, x, ldx, (int)T, y, ldy, epi, xsum, gws, s);
+    return launch_gemm(w, x, ldx, T, y, ldy, epi, s);
+  };
+  cudaError_t e = cudaSuccess;
+  for (int l = 0; l < n_layers && e == cudaSuccess; ++l) {
+    const sq_layer& L = layers[l];
+    const bool q = L.bits != 16;
+    const float* xr = (l == 0) ? x_in : x_out;
+    const bool copy = (l == 0 && x_in != x_out);
+    // a = LN(x) (layer 0 also initialises the residual buffer x_out = x_in)
+    e = launch_layernorm_f16(xr, T, h1, a16, (dec && q) ? xs : nullptr, copy ? x_in : nullptr, copy ? x_out : nullptr, s);
+    if (e) break;
+    e = lin(L.qkv, a16, h1, qkv16, 3 * h1, SQ_EPI_F16, (dec && q) ? xs : nullptr);
+    if (e) break;
+    // attention stub: attn = v = qkv[:, 2h1:3h1] (R12)
+    const __half* v = qkv16 + 2 * h1;
+    if (dec && q) {
+      e = launch_xsum(v, 3 * h1, T, h1, xs, s);
+      if (e) break;
+    }
+    e = lin(L.o, v, 3 * h1, x_out, h1, SQ_EPI_F32_ACCUM, (dec && q) ? xs : nullptr);
+    if (e) break;
+    e = launch_layernorm_f16(x_out, T, h1, a16, (dec && q) ? xs : nullptr, nullptr, nullptr, s);
+    if (e) break;
+    e = lin(L.fc1, a16, h1, u16, h2, L.act == 0 ? SQ_EPI_F16_RELU : SQ_EPI_F16_GELU, (dec && q) ? xs : nullptr);
+    if (e) break;
+    if (dec && q) {
+      e = launch_xsum(u16, h2, T, h2, xs, s);
+      if (e) break;
+    }
+    e = lin(L.fc2, u16, h2, x_out, h1, SQ_EPI_F32_ACCUM, (dec && q) ? xs : nullptr);
+    if (e) break;
+    if (qkv_dbg && l == n_layers - 1)
+      e = cudaMemcpyAsync(qkv_dbg, qkv16, (size_t)T * 3 * h1 * 2, cudaMemcpyDeviceToDevice, s);
+  }
+  return cuda_check(e, "sq_stage_forward");
+}
+
+}  // namespace sq
+
+using namespace sq;
+
+extern "C" {
+
+size_t sq_stage_workspace_bytes(const sq_layer* layers, int n_layers, int64_t max_tokens) {
+  if (!layers || n_layers <= 0 || max_tokens <= 0) return 0;
+  return stage_workspace_bytes(layers, n_layers, max_tokens);
+}
+
+sq_status sq_stage_forward(const sq_layer* layers, int n_layers, int phase, const float* x_in_dev, int64_t tokens,
+                           float* x_out_dev, void* qkv_dbg_dev, void* ws_dev, size_t ws_bytes, sq_stream_t stream) {
+  sq_status st = check_layers(layers, n_layers, "sq_stage_forward");
+  if (st) return st;
+  if (phase != SQ_PREFILL && phase != SQ_DECODE) return fail(SQ_EINVAL, "sq_stage_forward: bad phase %d", phase);
+  if (tokens < 1 || (phase == SQ_DECODE && tokens > 32))
+    return fail(SQ_EINVAL, "sq_stage_forward: tokens=%lld (decode needs 1..32)", (long long)tokens);
+  if (phase == SQ_PREFILL) {
+    for (int l = 0; l < n_layers; ++l)
+      if (layers[l].o.n % 128 || layers[l].fc1.n % 128) return fail(SQ_EINVAL, "sq_stage_forward: prefill needs n%%128==0");
+  }
+  if (!x_in_dev || !x_out_dev || (reinterpret_cast<uintptr_t>(x_in_dev) & 15u) || (reinterpret_cast<uintptr_t>(x_out_dev) & 15u))
+    return fail(SQ_EINVAL, "sq_stage_forward: x_in/x_out null or not 16-B aligned");
+  const size_t need = stage_workspace_bytes(layers, n_layers, tokens);
+  if (!ws_dev || ws_bytes < need || (reinterpret_cast<uintptr_t>(ws_dev) & 255u))
+    return fail(SQ_ENOMEM, "sq_stage_forward: workspace %zu < %zu (or null / not 256-B aligned)", ws_bytes, need);
+  return stage_forward(layers, n_layers, phase, x_in_dev, tokens, x_out_dev, qkv_dbg_dev, ws_dev, ws_bytes,
+                       (cudaStream_t)stream);
+}
+
+sq_status sq_layernorm_f32(const float* x_dev, int64_t rows, int64_t d, float* y_dev, sq_stream_t stream) {
+  if (!x_dev || !y_dev || rows <= 0 || d <= 0 || d % 128 || d > 14336) return fail(SQ_EINVAL, "sq_layernorm_f32: bad args");
+  return cuda_check(launch_layernorm_f32(x_dev, rows, d, y_dev, (cudaStream_t)stream), "sq_layernorm_f32");
+}
+
+}  // extern "C"

@@ -1,0 +1,166 @@
+"""Stage / pipeline bindings over libsq (marshalling only) + device-resident model builder.
+
+``Layer`` owns the four quantized linears of one decoder layer (P:160 linear
+set; R11).  ``build_layers`` creates synthetic OPT/BLOOM-shaped
+layers directly in HBM with the seeded counter generator (synth/), quantizing
+and packing them with the library's own kernels (load-time path).
+"""
+from __future__ import annotations
+
+import ctypes
+
+import torch
+
+from . import (P, QLinear, SQ_DECODE, SQ_PREFILL, _L, _check, _ptr, _stream, sq_layer, sq_plan,
+               sq_run_stats)
+
+
+class Layer:
+    def __init__(self, bits: int, act: int, qkv: QLinear, o: QLinear, fc1: QLinear, fc2: QLinear):
+        self.bits, self.act = bits, act
+        self.qkv, self.o, self.fc1, self.fc2 = qkv, o, fc1, fc2
+
+    def c_struct(self) -> sq_layer:
+        return sq_layer(self.bits, self.act, self.qkv.c, self.o.c, self.fc1.c, self.fc2.c)
+
+    def nbytes(self) -> int:
+        return sum(l.nbytes() for l in (self.qkv, self.o, self.fc1, self.fc2))
+
+
+def layer_array(layers: list[Layer]):
+    return (sq_layer * len(layers))(*[l.c_struct() for l in layers])
+
+
+def build_layers(n_layers: int, h1: int, h2: int, bits: list[int], act: int = 0, bias: bool = True,
+                 layer_offset: int = 0, device: str = "cuda", stream=None) -> list[Layer]:
+    """Synthetic layers (W ~ N(0, 1/K) + 0.1 % outliers) built in HBM."""
+    import synth
+    layers = []
+    dims = {"qkv": (3 * h1, h1), "o": (h1, h1), "fc1": (h2, h1), "fc2": (h1, h2)}
+    scratch = torch.empty(max(n * k for n, k in dims.values()), dtype=torch.float16, device=device)
+    s = torch.cuda.current_stream() if stream is None else stream
+    for i in range(n_layers):
+        l = layer_offset + i
+        b = int(bits[i])
+        lins = {}
+        for name, (n, k) in dims.items():
+            seed = synth.weight_seed(l, name)
+            if b == 16:
+                w = torch.empty((n, k), dtype=torch.float16, device=device)
+                synth.device_weight_f16(w.data_ptr(), seed, n, k, s.cuda_stream)
+            else:
+                w = scratch[: n * k].view(n, k)
+                synth.device_weight_f16(w.data_ptr(), seed, n, k, s.cuda_stream)
+            bvec = None
+            if bias:
+                bvec = torch.from_numpy(synth.bias_f16(seed, n)).to(device)
+            lins[name] = QLinear.from_fp16(w, b, bvec, stream=s)
+        layers.append(Layer(b, act, lins["qkv"], lins["o"], lins["fc1"], lins["fc2"]))
+    torch.cuda.synchronize()
+    return layers
+
+
+# ---------------------------------------------------------------- a5
+def sq_stage_workspace_bytes(layers: list[Layer], max_tokens: int) -> int:
+    arr = layer_array(layers)
+    return int(_L.sq_stage_workspace_bytes(arr, len(layers), max_tokens))
+
+
+class StageWorkspace:
+    def __init__(self, layers: list[Layer], max_tokens: int, device="cuda"):
+        self.buf = torch.zeros(sq_stage_workspace_bytes(layers, max_tokens) + 256, dtype=torch.uint8, device=device)
+        off = (-self.buf.data_ptr()) % 256
+        self.ptr = self.buf.data_ptr() + off
+        self.nbytes = self.buf.numel() - off
+
+
+def sq_stage_forward(layers: list[Layer], phase: int, x_in: torch.Tensor, x_out: torch.Tensor,
+                     ws: StageWorkspace, qkv_dbg: torch.Tensor | None = None, stream=None, arr=None) -> torch.Tensor:
+    """a5: run this stage's layers on x fp32 [tokens, h1] (x_in and x_out may alias)."""
+    arr = layer_array(layers) if arr is None else arr
+    _check(_L.sq_stage_forward(arr, len(layers), phase, _ptr(x_in), x_in.shape[0], _ptr(x_out), _ptr(qkv_dbg),
+                               ctypes.c_void_p(ws.ptr), ws.nbytes, _stream(stream)))
+    return x_out
+
+
+def sq_layernorm_f32(x: torch.Tensor, y: torch.Tensor, stream=None) -> torch.Tensor:
+    _check(_L.sq_layernorm_f32(_ptr(x), x.shape[0], x.shape[1], _ptr(y), _stream(stream)))
+    return y
+
+
+# ---------------------------------------------------------------- a6
+class Plan:
+    """Host-side plan (per-layer bits, layer->stage partition, micro-batch sizes)."""
+
+    def __init__(self, bits: list[int], stage_of_layer: list[int], hidden: int, ffn: int, B: int, eta: int,
+                 xi: int, prompt_len: int, n_decode: int, group: int = 128):
+        self.bits = [int(b) for b in bits]
+        self.stage_of_layer = [int(s) for s in stage_of_layer]
+        self.n_layers = len(bits)
+        self.n_stages = max(self.stage_of_layer) + 1
+        self.hidden, self.ffn, self.B, self.eta, self.xi = hidden, ffn, B, eta, xi
+        self.prompt_len, self.n_decode, self.group = prompt_len, n_decode, group
+        self._bits = (ctypes.c_int32 * self.n_layers)(*self.bits)
+        self._sol = (ctypes.c_int32 * self.n_layers)(*self.stage_of_layer)
+        self.c = sq_plan(self.n_layers, self.n_stages, hidden, ffn, group, self._bits, self._sol, B, eta, xi,
+                         prompt_len, n_decode)
+
+    def layers_of(self, rank: int) -> list[int]:
+        return [l for l, s in enumerate(self.stage_of_layer) if s == rank]
+
+
+def sq_plan_check(plan: Plan) -> None:
+    _check(_L.sq_plan_check(ctypes.byref(plan.c)))
+
+
+class Comm:
+    def __init__(self, handle: int):
+        self.h = ctypes.c_void_p(handle)
+
+    @classmethod
+    def local(cls, nstages: int) -> "Comm":
+        h = ctypes.c_void_p()
+        _check(_L.sq_comm_init_local(ctypes.byref(h), nstages))
+        return cls(h.value)
+
+    @classmethod
+    def nccl(cls, uid: bytes, nranks: int, rank: int) -> "Comm":
+        h = ctypes.c_void_p()
+        buf = (ctypes.c_uint8 * len(uid)).from_buffer_copy(uid)
+        _check(_L.sq_comm_init(ctypes.byref(h), buf, nranks, rank))
+        return cls(h.value)
+
+    def destroy(self) -> None:
+        if self.h:
+            _L.sq_comm_destroy(self.h)
+            self.h = ctypes.c_void_p()
+
+
+def sq_comm_get_unique_id() -> bytes:
+    n = int(_L.sq_comm_unique_id_bytes())
+    buf = (ctypes.c_uint8 * n)()
+    _check(_L.sq_comm_get_unique_id(buf))
+    return bytes(buf)
+
+
+class PipelineWorkspace:
+    def __init__(self, plan: Plan, layers: list[Layer], rank: int, device="cuda"):
+        arr = layer_array(layers)
+        n = int(_L.sq_pipeline_workspace_bytes(ctypes.byref(plan.c), arr, rank))
+        if n == 0:
+            raise ValueError("invalid plan/layers for workspace query")
+        self.buf = torch.zeros(n + 256, dtype=torch.uint8, device=device)
+        off = (-self.buf.data_ptr()) % 256
+        self.ptr = self.buf.data_ptr() + off
+        self.nbytes = n
+
+
+def sq_pipeline_run(plan: Plan, rank: int, layers: list[Layer], comm: Comm | None, x0: torch.Tensor | None,
+                    out: torch.Tensor | None, ws: PipelineWorkspace, stream=None, arr=None) -> dict:
+    """a6: run the whole generation (prefill + n_decode steps) for this rank (rank -1: all stages)."""
+    arr = layer_array(layers) if arr is None else arr
+    st = sq_run_stats()
+    _check(_L.sq_pipeline_run(ctypes.byref(plan.c), rank, arr, len(layers), comm.h if comm else None, _ptr(x0),
+                              _ptr(out), ctypes.c_void_p(ws.ptr), ws.nbytes, ctypes.byref(st), _stream(stream)))
+    return {"t_total_ms": st.t_total_ms, "t_prefill_ms": st.t_prefill_ms, "t_decode_ms": st.t_decode_ms,
+            "tokens_per_s": st.tokens_per_s, "bytes_sent": st.bytes_sent, "gpu_launches": st.gpu_launches}

@@ -1,0 +1,213 @@
+"""GPU parity: quantize/pack bit-exact and decode/prefill linears vs the CPU oracle.
+
+Tolerance for floating point (R10, BASELINE.json north_star):
+normwise max|y - y_ref| / max|y_ref| <= 2e-3 against the fp64 oracle.
+Codes, scales, zeros, packed words and meta must match bit-exactly.
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+import torch
+
+import synth
+from oracle import oracle as O
+
+pytestmark = pytest.mark.gpu
+TOL = 2e-3
+
+
+def sqm():
+    import paper_conf_cluster_zhaowplw25_b200 as sq
+    return sq
+
+
+def normwise(y, ref):
+    y = np.asarray(y, np.float64)
+    ref = np.asarray(ref, np.float64)
+    return float(np.abs(y - ref).max() / max(np.abs(ref).max(), 1e-30))
+
+
+def adversarial_weight(n=64, k=512, seed=3):
+    w = synth.weight_f16(seed, n, k).copy()
+    w[0, :128] = np.float16(0.5)                      # constant group
+    w[1, 128:256] = np.float16(-0.0)                  # -0 group
+    w[1, 130] = np.float16(0.0)
+    w[2, :128] = np.float16(6e-8)                     # subnormal range
+    w[2, 5] = np.float16(-6e-8)
+    w[3, 0], w[3, 1] = np.float16(65504.0), np.float16(-65504.0)  # extremes
+    w[4, :128] = (np.arange(128) % 16).astype(np.float16) * np.float16(0.25)  # exact ties for b=3
+    w[5, 128:256] = np.linspace(-1, 1, 128).astype(np.float16)
+    w[6, 7] = np.float16(30.0)                        # outlier
+    return w
+
+
+@pytest.mark.parametrize("bits", [3, 4, 8])
+@pytest.mark.parametrize("group", [128, 64, 32])
+def test_quantize_bit_exact_adversarial(bits, group):
+    sq = sqm()
+    w = adversarial_weight()
+    codes, s, z = O.quantize_groups(w, bits, group)
+    gc, gs, gz = sq.sq_quantize_groups(torch.from_numpy(w).cuda(), bits, group)
+    assert np.array_equal(gc.cpu().numpy(), codes)
+    assert np.array_equal(gs.cpu().numpy().view(np.uint16), s.view(np.uint16))
+    assert np.array_equal(gz.cpu().numpy().view(np.uint16), z.view(np.uint16))
+
+
+@pytest.mark.parametrize("bits", [3, 4, 8])
+def test_pack_bit_exact(bits):
+    sq = sqm()
+    w = adversarial_weight(n=48, k=640, seed=bits)
+    codes, s, z = O.quantize_groups(w, bits)
+    packed, meta = O.pack(codes, s, z, bits)
+    gp, gm = sq.sq_pack(torch.from_numpy(codes).cuda(), torch.from_numpy(s).cuda(), torch.from_numpy(z).cuda(), bits)
+    assert np.array_equal(gp.cpu().numpy(), packed)
+    assert np.array_equal(gm.cpu().numpy().view(np.uint32).reshape(-1), meta.reshape(-1))
+
+
+@pytest.mark.parametrize("bits", [3, 4, 8])
+def test_quantize_pack_bit_exact_opt13b_linear(bits):
+    # full OPT-13B q/k/v/o shape (5120 x 5120), device-generated weights (same generator)
+    sq = sqm()
+    n = k = 5120
+    seed = synth.weight_seed(0, "o")
+    wd = torch.empty((n, k), dtype=torch.float16, device="cuda")
+    synth.device_weight_f16(wd.data_ptr(), seed, n, k)
+    w = synth.weight_f16(seed, n, k)
+    assert np.array_equal(wd.cpu().numpy().view(np.uint16), w.view(np.uint16))
+    codes, s, z = O.quantize_groups(w, bits)
+    packed, meta = O.pack(codes, s, z, bits)
+    q = sq.QLinear.from_fp16(wd, bits)
+    assert np.array_equal(q.packed.cpu().numpy(), packed)
+    assert np.array_equal(q.meta.cpu().numpy().view(np.uint32).reshape(-1), meta.reshape(-1))
+
+
+def _make(bits, n, k, seed, bias=True):
+    sq = sqm()
+    w = synth.weight_f16(seed, n, k)
+    b = synth.bias_f16(seed, n) if bias else None
+    qo = O.QWeight(w, bits, bias=b)
+    qg = sq.QLinear.from_fp16(torch.from_numpy(w).cuda(), bits, torch.from_numpy(b).cuda() if bias else None)
+    return qo, qg
+
+
+def _ref_epi(y, epi):
+    if epi == 1:
+        return np.maximum(y, 0)
+    if epi == 2:
+        return 0.5 * y * (1 + np.tanh(np.sqrt(2 / np.pi) * (y + 0.044715 * y ** 3)))
+    return y
+
+
+def _run_linear(kind, qg, x, epi, y0=None):
+    sq = sqm()
+    m = x.shape[0]
+    xt = torch.from_numpy(x).cuda()
+    if epi == sq.SQ_EPI_F32_ACCUM:
+        y = torch.from_numpy(y0.copy()).cuda()
+    else:
+        y = torch.empty((m, qg.n), dtype=torch.float16, device="cuda")
+    if kind == "decode":
+        sq.sq_linear_decode(qg, xt, y, epi)
+    else:
+        sq.sq_linear_prefill(qg, xt, y, epi)
+    torch.cuda.synchronize()
+    return y.float().cpu().numpy().astype(np.float64)
+
+
+SHAPES = [(256, 512), (144, 384), (768, 768), (1024, 128), (528, 1280)]
+
+
+@pytest.mark.parametrize("bits", [3, 4, 8, 16])
+@pytest.mark.parametrize("m", [1, 2, 5, 8, 9, 16, 17, 32])
+def test_decode_parity(bits, m):
+    for si, (n, k) in enumerate(SHAPES):
+        qo, qg = _make(bits, n, k, seed=100 + si)
+        x = synth.act_f16(200 + m, m, k)
+        ref = O.linear(x, qo)
+        y = _run_linear("decode", qg, x, 0)
+        assert normwise(y, ref) <= TOL, (n, k, normwise(y, ref))
+
+
+@pytest.mark.parametrize("bits", [3, 4, 8, 16])
+@pytest.mark.parametrize("epi", [1, 2, 3])
+def test_decode_epilogues(bits, epi):
+    n, k, m = 272, 640, 3
+    qo, qg = _make(bits, n, k, seed=300)
+    x = synth.act_f16(301, m, k)
+    lin = O.linear(x, qo)
+    if epi == 3:
+        y0 = synth.hidden_f32(302, m, n)
+        y = _run_linear("decode", qg, x, epi, y0)
+        assert normwise(y - y0, lin) <= TOL
+    else:
+        y = _run_linear("decode", qg, x, epi)
+        assert normwise(y, _ref_epi(lin, epi)) <= TOL
+
+
+@pytest.mark.parametrize("bits", [3, 4, 8, 16])
+def test_decode_deterministic(bits):
+    n, k, m = 2048, 1536, 7
+    qo, qg = _make(bits, n, k, seed=400)
+    x = synth.act_f16(401, m, k)
+    a = _run_linear("decode", qg, x, 0)
+    b = _run_linear("decode", qg, x, 0)
+    assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("bits", [3, 4, 8])
+@pytest.mark.parametrize("shape", [(20480, 5120), (5120, 20480)])
+def test_decode_full_size_sampled(bits, shape):
+    # OPT-13B fc1 / fc2 at micro-batch 32 (configs[1]); oracle on 48 sampled output rows
+    sq = sqm()
+    n, k = shape
+    seed = synth.weight_seed(1, "fc1" if n > k else "fc2")
+    wd = torch.empty((n, k), dtype=torch.float16, device="cuda")
+    synth.device_weight_f16(wd.data_ptr(), seed, n, k)
+    qg = sq.QLinear.from_fp16(wd, bits)
+    del wd
+    m = 32
+    x = synth.act_f16(7, m, k)
+    y = _run_linear("decode", qg, x, 0)
+    rows = np.random.default_rng(bits).choice(n, 48, replace=False)
+    rows[0], rows[1] = 0, n - 1
+    wr = synth.weight_f16(seed, n, k, rows=rows)
+    ref = O.linear(x, O.QWeight(wr, bits))
+    assert normwise(y[:, rows], ref) <= TOL
+
+
+@pytest.mark.parametrize("bits", [3, 4, 8, 16])
+@pytest.mark.parametrize("m", [1, 37, 128, 300, 513])
+def test_prefill_parity(bits, m):
+    for si, (n, k) in enumerate([(256, 512), (384, 1280), (128, 128)]):
+        qo, qg = _make(bits, n, k, seed=500 + si)
+        x = synth.act_f16(600 + m, m, k)
+        ref = O.linear(x, qo)
+        y = _run_linear("prefill", qg, x, 0)
+        assert normwise(y, ref) <= TOL, (n, k, m, normwise(y, ref))
+
+
+@pytest.mark.parametrize("bits", [4, 16])
+@pytest.mark.parametrize("epi", [1, 2, 3])
+def test_prefill_epilogues(bits, epi):
+    n, k, m = 384, 512, 77
+    qo, qg = _make(bits, n, k, seed=700)
+    x = synth.act_f16(701, m, k)
+    lin = O.linear(x, qo)
+    if epi == 3:
+        y0 = synth.hidden_f32(702, m, n)
+        y = _run_linear("prefill", qg, x, epi, y0)
+        assert normwise(y - y0, lin) <= TOL
+    else:
+        y = _run_linear("prefill", qg, x, epi)
+        assert normwise(y, _ref_epi(lin, epi)) <= TOL
+
+
+def test_one_token_prefill_equals_decode_function():
+    # S8c: a 1-token prefill computes the same function as a decode step
+    qo, qg = _make(4, 512, 1024, seed=800)
+    x = synth.act_f16(801, 1, 1024)
+    a = _run_linear("prefill", qg, x, 0)
+    b = _run_linear("decode", qg, x, 0)
+    ref = O.linear(x, qo)
+    assert normwise(a, ref) <= TOL and normwise(b, ref) <= TOL

@@ -90,7 +90,7 @@ def test_half_step_bound_with_outliers(bits):
 @pytest.mark.parametrize("bits", [3, 4, 8])
 def test_grid_aligned_weights_recovered_exactly(bits):
     # Special case: W on a quantization grid with codes spanning 0..2^b-1 -> lossless.
-    w, c, s, z = synth.grid_aligned_weight_f16(5, 8, 256, bits)
+    w, c, s, z = synth.grid_aligned_weight_f16(5, 16, 256, bits)
     codes, s2, z2 = O.quantize_groups(w, bits, 128)
     assert np.array_equal(codes, c)
     assert np.array_equal(s2, s) and np.array_equal(z2, z)
@@ -122,7 +122,7 @@ def _golden():
 
 
 def _example_codes(bits, name):
-    c = np.zeros((1, 128), np.uint8)
+    c = np.zeros((16, 128), np.uint8)  # one 16-row tile (T16); the example lives in row 0
     if name == "ramp":
         c[0] = np.arange(128) % (1 << bits)
     elif name == "single13":
@@ -138,9 +138,11 @@ def _example_codes(bits, name):
 def test_pack_hand_derived_words(row):
     bits, name, words = row
     c = _example_codes(bits, name)
-    s = np.zeros((1, 1), np.float16)
+    s = np.zeros((16, 1), np.float16)
     packed, meta = O.pack(c, s, s, bits)
-    got = packed.view("<u4")[0]
+    gb = 128 * bits // 8
+    got = packed.reshape(-1)[:gb].view("<u4")  # row 0's chunk of unit (tile 0, group 0)
+    assert not packed.reshape(-1)[gb:].any()
     for i, wv in words.items():
         assert got[i] == wv, (i, hex(got[i]), hex(wv))
     if name.startswith("single"):
@@ -149,7 +151,7 @@ def test_pack_hand_derived_words(row):
 
 
 @pytest.mark.parametrize("bits", [3, 4, 8])
-@pytest.mark.parametrize("shape", [(1, 128), (5, 384), (16, 1024)])
+@pytest.mark.parametrize("shape", [(16, 128), (32, 384), (48, 1024)])
 def test_pack_unpack_round_trip(bits, shape):
     rng = np.random.default_rng(bits * 100 + shape[1])
     c = rng.integers(0, 1 << bits, size=shape).astype(np.uint8)
@@ -159,14 +161,21 @@ def test_pack_unpack_round_trip(bits, shape):
     assert np.array_equal(O.unpack(packed, *shape, bits), c)
 
 
-def test_meta_layout_group_major():
+def test_tile_placement_t16():
+    # T16: unit (tile t, group g) = rows 16t..16t+15 of group g, contiguous, tile-major/group-minor;
+    # meta[(t*kg + g)*16 + r%16] = scale | zero << 16
     rng = np.random.default_rng(3)
-    s = rng.standard_normal((4, 3)).astype(np.float16)
-    z = rng.standard_normal((4, 3)).astype(np.float16)
-    _, meta = O.pack(np.zeros((4, 384), np.uint8), s, z, 4)
-    assert meta.shape == (3, 4)
-    assert np.array_equal((meta & 0xFFFF).astype(np.uint16), s.view(np.uint16).T)
-    assert np.array_equal((meta >> 16).astype(np.uint16), z.view(np.uint16).T)
+    n, k, bits = 32, 384, 8
+    c = rng.integers(0, 256, size=(n, k)).astype(np.uint8)
+    s = rng.standard_normal((n, 3)).astype(np.float16)
+    z = rng.standard_normal((n, 3)).astype(np.float16)
+    packed, meta = O.pack(c, s, z, bits)
+    flat = packed.reshape(-1)
+    for r in (0, 7, 16, 31):
+        for g in range(3):
+            off = ((r // 16) * 3 + g) * 16 + r % 16
+            assert np.array_equal(flat[off * 128:(off + 1) * 128], c[r, 128 * g:128 * (g + 1)])
+            assert meta.reshape(-1)[off] == (int(s[r, g].view(np.uint16)) | (int(z[r, g].view(np.uint16)) << 16))
 
 
 @pytest.mark.parametrize("h1", [768, 5120, 7168, 9216, 14336])
@@ -193,7 +202,7 @@ def test_linear_fp16_equals_numpy_matmul():
 
 @pytest.mark.parametrize("bits", [3, 4, 8])
 def test_linear_grid_aligned_equals_unquantized(bits):
-    w, *_ = synth.grid_aligned_weight_f16(9, 40, 256, bits)
+    w, *_ = synth.grid_aligned_weight_f16(9, 48, 256, bits)
     x = synth.act_f16(10, 5, 256)
     yq = O.linear(x, O.QWeight(w, bits))
     y16 = x.astype(np.float64) @ w.astype(np.float64).T
