@@ -216,6 +216,29 @@ sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers,
 /* Validate a plan (contiguity eqs. 15-16, non-empty stages, bits set, micro-batches). */
 sq_status sq_plan_check(const sq_plan* plan);
 
+/* Host-only: the exact op sequence `rank` executes inside sq_pipeline_run (rank -1, or a
+ * 1-stage plan: the single-process order).  Items: prefill m = 0..mu_pre-1, then decode
+ * t = 1..n_decode, m = 0..mu_dec-1 (R13/R14).  Send/recv ops name the peer's global rank;
+ * the sequence of SEND ops of rank j to j+1 equals, op for op and size for size, the
+ * sequence of RECV ops of rank j+1 from j (tests/test_pipeline_schedule.py).  Returns the
+ * number of ops (writes at most max_ops; ops may be NULL to query), or -1 on a bad plan. */
+typedef enum {
+  SQ_OP_RECV_LB = 0,       /* stage 0: loop-back rows LN(hidden) from the last stage -> decode input */
+  SQ_OP_RECV_ACT = 1,      /* hidden [rows, h1] fp32 from the previous stage */
+  SQ_OP_COMPUTE = 2,       /* this stage's layers on the item (phase, rows tokens) */
+  SQ_OP_SEND_ACT = 3,      /* hidden to the next stage */
+  SQ_OP_OUT = 4,           /* last stage: write out[b, t] (prefill: last prompt position) */
+  SQ_OP_SEND_LB = 5,       /* last stage: LN(out rows) to stage 0 */
+  SQ_OP_LOOPBACK_LOCAL = 6 /* single process: LN(out rows) -> decode input in place */
+} sq_op_kind;
+typedef struct {
+  int32_t kind, item, phase, t;   /* t: decode step (0 = prefill) */
+  int32_t slot, peer;             /* activation buffer slot; peer global rank (-1 none) */
+  int64_t seq0, nseq;             /* sequences of the item / loop-back rows */
+  int64_t rows;                   /* tokens moved or computed */
+} sq_sched_op;
+int64_t sq_pipeline_schedule(const sq_plan* plan, int rank, sq_sched_op* ops, int64_t max_ops);
+
 /* ------------------------------------------------------------------------
  * Measurement hooks (bench.py): per-kernel-class CUDA-event timing of every
  * launch made by the library while enabled, on the launching stream.

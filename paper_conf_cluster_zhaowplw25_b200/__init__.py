@@ -56,6 +56,14 @@ class sq_run_stats(ctypes.Structure):
                 ("tokens_per_s", ctypes.c_double), ("bytes_sent", I64), ("gpu_launches", I64)]
 
 
+class sq_sched_op(ctypes.Structure):
+    _fields_ = [("kind", I32), ("item", I32), ("phase", I32), ("t", I32), ("slot", I32), ("peer", I32),
+                ("seq0", I64), ("nseq", I64), ("rows", I64)]
+
+
+SQ_OP_NAMES = ["RECV_LB", "RECV_ACT", "COMPUTE", "SEND_ACT", "OUT", "SEND_LB", "LOOPBACK_LOCAL"]
+
+
 class sq_profile(ctypes.Structure):
     _fields_ = [("launches", I64 * 4), ("ms", ctypes.c_double * 4), ("bytes", ctypes.c_double * 4),
                 ("flops", ctypes.c_double * 4)]
@@ -90,7 +98,7 @@ EXPORTED = [
     "sq_stage_workspace_bytes", "sq_stage_forward", "sq_layernorm_f32", "sq_comm_unique_id_bytes",
     "sq_comm_get_unique_id", "sq_comm_init", "sq_comm_init_local", "sq_comm_destroy",
     "sq_pipeline_workspace_bytes", "sq_pipeline_run", "sq_plan_check", "sq_profile_enable", "sq_profile_read",
-    "sq_launch_count",
+    "sq_launch_count", "sq_pipeline_schedule",
 ]
 
 
@@ -112,6 +120,7 @@ _opt("sq_pipeline_workspace_bytes", ctypes.c_size_t, ctypes.POINTER(sq_plan), ct
 _opt("sq_pipeline_run", ctypes.c_int, ctypes.POINTER(sq_plan), ctypes.c_int, ctypes.POINTER(sq_layer), ctypes.c_int,
      P, P, P, P, ctypes.c_size_t, ctypes.POINTER(sq_run_stats), P)
 _opt("sq_plan_check", ctypes.c_int, ctypes.POINTER(sq_plan))
+_opt("sq_pipeline_schedule", I64, ctypes.POINTER(sq_plan), ctypes.c_int, ctypes.POINTER(sq_sched_op), I64)
 
 
 def _check(st: int) -> None:

@@ -18,38 +18,29 @@
 //    tcgen05.mma.cta_group::1.kind::f16 (M=128, N=256, K=16).
 //  * Epilogue: the dequant warps tcgen05.ld the accumulator (lane = weight row,
 //    column = token), add bias / activation / residual, store y.
-// Warp roles: 0 = TMA producer, 1 = MMA issuer (+TMEM alloc), 2..5 = dequant+epilogue.
+// Warp roles: 0 = TMA producer, 1 = MMA issuer (+TMEM alloc), 2..9 = dequant (2 groups) + epilogue.
 #include <cuda.h>
 
 #include <cstring>
 #include <mutex>
 
-#include "sq_common.cuh"
+#include "sq_tc.cuh"
 
 namespace sq {
 namespace {
+using namespace tc;
 
 constexpr int BN = 128;   // weight rows per tile (TMEM lanes, MMA M)
 constexpr int BT = 256;   // tokens per tile (MMA N)
 constexpr int XK = 64;    // k per activation stage (one 128-B swizzle row)
 constexpr int S_X = 4;
-constexpr int S_A = 2;
+constexpr int S_A = 3;
+constexpr int DQ_GROUPS = 2;  // dequant warp-groups on alternating groups of k
 constexpr int X_STAGE_BYTES = BT * XK * 2;  // 32 KB
 constexpr int TMEM_COLS = 512;
 constexpr int D_COL = 0;
 constexpr int A_COL = 256;
-constexpr int NUM_THREADS = 192;
-
-template <int BITS>
-struct GCfg;
-template <>
-struct GCfg<3> { static constexpr int GB = 48; static constexpr int S_W = 4; };
-template <>
-struct GCfg<4> { static constexpr int GB = 64; static constexpr int S_W = 4; };
-template <>
-struct GCfg<8> { static constexpr int GB = 128; static constexpr int S_W = 3; };
-template <>
-struct GCfg<16> { static constexpr int GB = 256; static constexpr int S_W = 2; };
+constexpr int NUM_THREADS = 32 * (2 + 4 * DQ_GROUPS);
 
 template <int BITS>
 struct Smem {
@@ -64,7 +55,8 @@ struct Smem {
 };
 
 struct GemmP {
-  const uint32_t* meta;   // [K/128][N]
+  const uint8_t* packed;
+  const uint32_t* meta;   // T16 [N/16][K/128][16]
   const __half* bias;
   void* y;
   int64_t ldy;
@@ -73,105 +65,8 @@ struct GemmP {
   int kg;
 };
 
-__device__ __forceinline__ uint64_t make_sw128_desc(uint32_t saddr) {
-  uint64_t d = 0;
-  d |= (uint64_t)((saddr >> 4) & 0x3FFF);
-  d |= (uint64_t)1 << 16;              // LBO (ignored for swizzled K-major)
-  d |= (uint64_t)(1024 >> 4) << 32;    // SBO: 8 rows x 128 B
-  d |= (uint64_t)1 << 46;              // descriptor version (sm_100)
-  d |= (uint64_t)2 << 61;              // SWIZZLE_128B
-  return d;
-}
-
 // instruction descriptor: kind::f16, A=B=f16 K-major, D=f32, M=128, N=256
-constexpr uint32_t kIdesc = (1u << 4) | ((uint32_t)(BT >> 3) << 17) | ((uint32_t)(BN >> 4) << 24);
-
-__device__ __forceinline__ uint32_t hsub_fma(uint32_t h, uint32_t off2, uint32_t s2, uint32_t z2) {
-  __half2 c = __hsub2(*reinterpret_cast<__half2*>(&h), *reinterpret_cast<__half2*>(&off2));
-  __half2 r = __hfma2(c, *reinterpret_cast<__half2*>(&s2), *reinterpret_cast<__half2*>(&z2));
-  return *reinterpret_cast<uint32_t*>(&r);
-}
-
-// Dequantize this thread's row (r) of one 128-k group into 64 half2 columns,
-// written to TMEM in 4 batches of 16 columns.
-template <int BITS>
-__device__ __forceinline__ void dequant_row_to_tmem(const uint8_t* wst, uint32_t meta, int r, uint32_t taddr) {
-  const uint32_t s2 = (meta & 0xFFFFu) * 0x10001u;
-  const uint32_t z2 = (meta >> 16) * 0x10001u;
-  constexpr uint32_t K1024 = 0x64006400u, K64 = 0x54005400u;
-  if constexpr (BITS == 4) {
-    const uint8_t* row = wst + r * 64;
-#pragma unroll
-    for (int b = 0; b < 4; ++b) {
-      const int pc = b ^ ((r >> 1) & 3);  // SWIZZLE_64B
-      uint4 v = *reinterpret_cast<const uint4*>(row + pc * 16);
-      const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
-      uint32_t o[16];
-#pragma unroll
-      for (int w = 0; w < 4; ++w) {
-        const uint32_t x = wv[w], x8 = x >> 8;
-        o[4 * w + 0] = hsub_fma(lop3_and_or(x, 0x000F000Fu, K1024), K1024, s2, z2);
-        o[4 * w + 1] = hsub_fma(lop3_and_or(x, 0x00F000F0u, K64), K64, s2, z2);
-        o[4 * w + 2] = hsub_fma(lop3_and_or(x8, 0x000F000Fu, K1024), K1024, s2, z2);
-        o[4 * w + 3] = hsub_fma(lop3_and_or(x8, 0x00F000F0u, K64), K64, s2, z2);
-      }
-      tmem_st16(taddr + 16 * b, o);
-    }
-  } else if constexpr (BITS == 8) {
-    const uint8_t* row = wst + r * 128;
-#pragma unroll
-    for (int b = 0; b < 4; ++b) {
-      uint32_t o[16];
-#pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        const int c = 2 * b + h, pc = c ^ (r & 7);  // SWIZZLE_128B
-        uint4 v = *reinterpret_cast<const uint4*>(row + pc * 16);
-        const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
-#pragma unroll
-        for (int t = 0; t < 4; ++t) {
-          o[8 * h + 2 * t] = hsub_fma(prmt(wv[t], 0x64646464u, 0x4140u), K1024, s2, z2);
-          o[8 * h + 2 * t + 1] = hsub_fma(prmt(wv[t], 0x64646464u, 0x4342u), K1024, s2, z2);
-        }
-      }
-      tmem_st16(taddr + 16 * b, o);
-    }
-  } else if constexpr (BITS == 3) {
-    const uint32_t* row = reinterpret_cast<const uint32_t*>(wst + r * 48);
-#pragma unroll
-    for (int bl = 0; bl < 4; ++bl) {
-      const uint32_t L0 = row[3 * bl], L1 = row[3 * bl + 1], H = row[3 * bl + 2];
-      uint32_t o[16];
-#pragma unroll
-      for (int a = 0; a < 2; ++a) {
-        const uint32_t La = a ? L1 : L0;
-#pragma unroll
-        for (int i = 0; i < 8; ++i) {
-          const uint32_t lo = La >> (2 * i);
-          const int sh = i + 8 * a - 2;
-          const uint32_t hs = sh >= 0 ? (H >> sh) : (H << (-sh));
-          uint32_t t;
-          asm("lop3.b32 %0, %1, %2, %3, 0xD8;" : "=r"(t) : "r"(hs), "r"(lo), "r"(0x00030003u));  // mask ? lo : hs
-          o[8 * a + i] = hsub_fma(lop3_and_or(t, 0x00070007u, K1024), K1024, s2, z2);
-        }
-      }
-      tmem_st16(taddr + 16 * bl, o);
-    }
-  } else {
-    // fp16: two SW128 regions (k 0..63, 64..127) of [128 rows x 128 B]
-#pragma unroll
-    for (int b = 0; b < 4; ++b) {
-      const uint8_t* region = wst + (b >> 1) * (BN * 128) + r * 128;
-      uint32_t o[16];
-#pragma unroll
-      for (int h = 0; h < 4; ++h) {
-        const int c = 4 * (b & 1) + h, pc = c ^ (r & 7);
-        uint4 v = *reinterpret_cast<const uint4*>(region + pc * 16);
-        o[4 * h] = v.x; o[4 * h + 1] = v.y; o[4 * h + 2] = v.z; o[4 * h + 3] = v.w;
-      }
-      tmem_st16(taddr + 16 * b, o);
-    }
-  }
-}
+constexpr uint32_t kIdesc = make_idesc(BN, BT);
 
 template <int BITS, int EPI>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
@@ -227,9 +122,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           tma_load_2d(wdst, &tm_w, &full_w[sw], g * 128, (int32_t)n0);
           tma_load_2d(wdst + BN * 128, &tm_w, &full_w[sw], g * 128 + 64, (int32_t)n0);
         } else {
-          // placement T16: 4-D box {GB bytes, 16 rows, 1 group, 8 row tiles} -> [128 rows][GB]
-          tma_load_4d(wdst, &tm_w, &full_w[sw], 0, 0, g, (int32_t)(n0 / 16));
-          tma_load_3d(smem + SM::OFF_META + sw * BN * 4, &tm_m, &full_w[sw], 0, g, (int32_t)(n0 / 16));
+          // placement T16: 8 contiguous units of 16 rows -> [128 rows][GB] (bulk copies)
+          load_w_tile<BITS>(wdst, smem + SM::OFF_META + sw * BN * 4, p.packed, p.meta, n0 / 16, g, kg, &full_w[sw]);
         }
         for (int h = 0; h < 2; ++h, ++it_x) {
           const int sx = it_x % S_X, rx = it_x / S_X;
@@ -265,11 +159,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       tc_commit(d_full);
     }
   } else {
-    // ---------------- dequant warps (one thread per weight row), then epilogue
+    // ---------------- dequant warps (one thread per weight row; group gi takes k-groups
+    // g = gi (mod 2) so one group's tcgen05.st latency overlaps the other's unpack), then epilogue
     const int sp = warp & 3;            // TMEM sub-partition this warp may access
+    const int gi = (warp - 2) >> 2;
     const int r = sp * 32 + lane;       // row within the tile
     const uint32_t lane_base = (uint32_t)(sp * 32) << 16;
-    for (int g = 0; g < kg; ++g) {
+    for (int g = gi; g < kg; g += DQ_GROUPS) {
       const int sw = g % S_W, rw = g / S_W;
       const int sa = g % S_A, ra = g / S_A;
       mbar_wait(&full_w[sw], rw & 1);
@@ -285,14 +181,14 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         mbar_arrive(&full_a[sa]);
       }
     }
-    // ---------------- epilogue
-    mbar_wait(d_full, 0);
+    // ---------------- epilogue (each dequant group drains half of the 256 token columns)
+    mbar_wait_sleepy(d_full, 0);
     tc_fence_after();
     const int64_t nrow = n0 + r;
     float bias = 0.f;
     if (p.bias) bias = __half2float(p.bias[nrow]);
 #pragma unroll 1
-    for (int c = 0; c < BT / 16; ++c) {
+    for (int c = gi * (BT / 32); c < (gi + 1) * (BT / 32); ++c) {
       uint32_t v[16];
       tmem_ld16(tmem + lane_base + D_COL + c * 16, v);
       tc_wait_ld();
@@ -410,6 +306,7 @@ cudaError_t launch_gemm(const sq_qweight& w, const __half* x, int64_t ldx, int64
   }
   if (e != cudaSuccess) return e;
   GemmP p{};
+  p.packed = static_cast<const uint8_t*>(w.packed);
   p.meta = static_cast<const uint32_t*>(w.meta);
   p.bias = static_cast<const __half*>(w.bias);
   p.y = y;

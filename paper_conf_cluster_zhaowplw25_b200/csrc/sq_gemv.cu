@@ -23,6 +23,8 @@
 //  * Split tiles are reduced in shared memory in fixed warp order; a tile that
 //    straddles two CTAs is finished by the last CTA (atomic counter, fixed CTA
 //    order).  Deterministic; counters self-reset.
+#include <cstdlib>
+
 #include "sq_common.cuh"
 
 namespace sq {
@@ -101,18 +103,21 @@ __device__ __forceinline__ void frag(const uint32_t* c, int t, uint32_t& lo, uin
     lo = prmt(c[t], 0x64646464u, 0x4140u);
     hi = prmt(c[t], 0x64646464u, 0x4342u);
   } else if constexpr (BITS == 3) {
-    // L3: pair (a, i) = k' 16a + 2i (+1): low bits La >> 2i, high bit H >> (i + 8a).
+    // L3: pair (a, i) = k' 16a + 2i (+1): low bits at La bits 2i(+16), high bit at H bit i+8a(+16).
+    // The code is assembled at mantissa bits 7..9 under exponent 2^3: half2(8 + c), exact, and
+    // the offset 8 (not 1024) keeps the per-group correction D - xoff free of cancellation.
     const int a = t >> 2;
     const uint32_t La = c[a], H = c[2];
 #pragma unroll
     for (int e = 0; e < 2; ++e) {
       const int i = 2 * (t & 3) + e;
-      const uint32_t l = La >> (2 * i);
-      const int sh = i + 8 * a - 2;
+      const int sl = 7 - 2 * i;              // low two bits -> bits 7..8
+      const uint32_t l = sl >= 0 ? (La << sl) : (La >> (-sl));
+      const int sh = i + 8 * a - 9;          // high bit -> bit 9
       const uint32_t hs = sh >= 0 ? (H >> sh) : (H << (-sh));
       uint32_t s;
-      asm("lop3.b32 %0, %1, %2, %3, 0xD8;" : "=r"(s) : "r"(hs), "r"(l), "r"(0x00030003u));  // mask ? l : hs
-      const uint32_t r = lop3_and_or(s, 0x00070007u, 0x64006400u);
+      asm("lop3.b32 %0, %1, %2, %3, 0xD8;" : "=r"(s) : "r"(hs), "r"(l), "r"(0x01800180u));  // mask ? l : hs
+      const uint32_t r = lop3_and_or(s, 0x03800380u, 0x48004800u);
       if (e == 0) lo = r; else hi = r;
     }
   } else {
@@ -220,12 +225,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemv(const GemvP p) {
     if (j < nunits) issue(j);
 
   // ---- stage (xs, xoff) per (group, token) in shared memory (overlaps the weight loads):
-  //      xs = sum x, xoff = sum off_k x  (off = 1024, or 1024 / 64 for the two nibble slots of L4)
+  //      xs = sum x, xoff = sum off_k x  (off = 1024 INT8, 1024 / 64 for the two nibble slots of L4, 8 INT3)
   if constexpr (Q) {
     for (int i = threadIdx.x; i < kg * kXsTok; i += kThreads) {
       const float2 v = __ldg(p.xsum + i);
       const float xsv = v.x + v.y;
-      const float xov = BITS == 4 ? fmaf(1024.f, v.x, 64.f * v.y) : 1024.f * xsv;
+      const float xov = BITS == 4 ? fmaf(1024.f, v.x, 64.f * v.y) : (BITS == 3 ? 8.f * xsv : 1024.f * xsv);
       xs_s[i] = make_float2(xsv, xov);
     }
   }
@@ -278,20 +283,27 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemv(const GemvP p) {
             mma_16816(acc[j], a, xtj[2 * t], xtj[2 * t + 1], acc[j]);
           }
         } else {
-          float d[4];
+          float d0[4], d1[4];  // two independent HMMA chains (even / odd chunks)
           {
-            uint32_t a[4];
+            uint32_t a[4], b[4];
             frag<BITS>(cb[s][0], 0, a[0], a[2]);
             frag<BITS>(cb[s][1], 0, a[1], a[3]);
-            mma_16816_zc(d, a, xtj[0], xtj[1]);
+            frag<BITS>(cb[s][0], 1, b[0], b[2]);
+            frag<BITS>(cb[s][1], 1, b[1], b[3]);
+            mma_16816_zc(d0, a, xtj[0], xtj[1]);
+            mma_16816_zc(d1, b, xtj[2], xtj[3]);
           }
 #pragma unroll
-          for (int t = 1; t < 8; ++t) {
-            uint32_t a[4];
+          for (int t = 2; t < 8; t += 2) {
+            uint32_t a[4], b[4];
             frag<BITS>(cb[s][0], t, a[0], a[2]);
             frag<BITS>(cb[s][1], t, a[1], a[3]);
-            mma_16816(d, a, xtj[2 * t], xtj[2 * t + 1], d);
+            frag<BITS>(cb[s][0], t + 1, b[0], b[2]);
+            frag<BITS>(cb[s][1], t + 1, b[1], b[3]);
+            mma_16816(d0, a, xtj[2 * t], xtj[2 * t + 1], d0);
+            mma_16816(d1, b, xtj[2 * t + 2], xtj[2 * t + 3], d1);
           }
+          const float d[4] = {d0[0] + d1[0], d0[1] + d1[1], d0[2] + d1[2], d0[3] + d1[3]};
           const float2 f0 = __half22float2(*reinterpret_cast<const __half2*>(&mb[s][0]));  // (s, z) row g
           const float2 f1 = __half22float2(*reinterpret_cast<const __half2*>(&mb[s][1]));  // row g+8
           const float4 xv = *reinterpret_cast<const float4*>(xs_s + grp * kXsTok + 8 * j + 2 * q);
@@ -482,7 +494,22 @@ size_t gemv_workspace_bytes(int64_t n, int64_t k, int64_t m) {
   const int64_t U = (n / kRows) * (k / 128);
   const int64_t W = gemv_ctas(U);
   size_t part = (size_t)W * 2 * tok_pad(m) * kRows * sizeof(float);  // per-CTA boundary partials
-  return cnt_bytes(n) + part + xsum_bytes(k) + 256;
+  size_t a = cnt_bytes(n) + part + xsum_bytes(k) + 256;
+  size_t b = n % 128 == 0 ? gemv_tc_workspace_bytes(n, k) : 0;
+  return a > b ? a : b;
+}
+
+// K2 (mma.sync, register unpack) for m <= 8; K2c (tcgen05, TMEM dequant) for 8 < m <= 32.
+// SQ_GEMV_PATH=mma|tc overrides (benchmarking).
+int gemv_path(int64_t n, int m, int bits) {
+  static int forced = -2;
+  if (forced == -2) {
+    const char* e = getenv("SQ_GEMV_PATH");
+    forced = !e ? -1 : (e[0] == 't' ? 1 : (e[0] == 'm' ? 0 : -1));
+  }
+  if (n % 128 || bits == 16) return 0;  // fp16 weights: 2 B/weight keeps even m = 32 HBM-bound on mma.sync
+  if (forced >= 0) return forced;
+  return m > 8 ? 1 : 0;
 }
 
 cudaError_t launch_xsum(const __half* x, int64_t ldx, int64_t m, int64_t k, float2* xsum, cudaStream_t s) {
@@ -496,6 +523,7 @@ cudaError_t launch_xsum(const __half* x, int64_t ldx, int64_t m, int64_t k, floa
 
 cudaError_t launch_gemv(const sq_qweight& w, const __half* x, int64_t ldx, int m, void* y, int64_t ldy, int epi,
                         const float2* xsum, void* ws, cudaStream_t s) {
+  if (gemv_path(w.n, m, w.bits) == 1) return launch_gemv_tc(w, x, ldx, m, y, ldy, epi, ws, s);
   if (w.n > kMaxN || w.n / kRows * (w.k / 128) >= (1ll << 31) / 256) return cudaErrorInvalidValue;  // 32-bit index math
   GemvP p{};
   p.packed = static_cast<const uint8_t*>(w.packed);

@@ -76,6 +76,59 @@ Ws ws_layout(const PlanView& v, const sq_layer* layers, int n_layers, int rank) 
   return w;
 }
 
+// ---- schedule: the op sequence of one rank (also exported as sq_pipeline_schedule)
+std::vector<sq_sched_op> make_schedule(const PlanView& v, int rank) {
+  const bool dist = rank >= 0 && v.P > 1;
+  const bool first = !dist || rank == 0, last = !dist || rank == v.P - 1;
+  std::vector<sq_sched_op> ops;
+  auto op = [&](int kind, int item, int phase, int t, int slot, int peer, int64_t seq0, int64_t nseq, int64_t rows) {
+    sq_sched_op o;
+    o.kind = kind; o.item = item; o.phase = phase; o.t = t; o.slot = slot; o.peer = peer;
+    o.seq0 = seq0; o.nseq = nseq; o.rows = rows;
+    ops.push_back(o);
+  };
+  // loop-back messages, in the order the last stage sends them: prefill mb 0..mu_pre-1,
+  // then decode (t, m) for t = 1..n_dec-1 (the last step's successor input is never used)
+  const int n_lb = v.mu_pre + std::max(0, v.n_dec - 1) * v.mu_dec;
+  int lb_posted = 0;
+  const int total = v.mu_pre + v.n_dec * v.mu_dec;
+  for (int it = 0; it < total; ++it) {
+    const bool pre = it < v.mu_pre;
+    const int m = pre ? it : (it - v.mu_pre) % v.mu_dec;
+    const int t = pre ? 0 : 1 + (it - v.mu_pre) / v.mu_dec;
+    const int64_t seq0 = pre ? (int64_t)m * v.eta : (int64_t)m * v.xi;
+    const int64_t nseq = std::min<int64_t>(pre ? v.eta : v.xi, v.B - seq0);
+    const int64_t T = pre ? nseq * v.s : nseq;
+    const int phase = pre ? SQ_PREFILL : SQ_DECODE;
+    const int slot = it & 1;
+    if (dist && first && !pre) {
+      // post the loop-back receives this item needs (and every earlier one, in order)
+      const int need = (t == 1) ? (int)((seq0 + nseq - 1) / v.eta) : v.mu_pre + (t - 2) * v.mu_dec + m;
+      for (; lb_posted <= need && lb_posted < n_lb; ++lb_posted) {
+        int64_t r0, nr;
+        if (lb_posted < v.mu_pre) {
+          r0 = (int64_t)lb_posted * v.eta;
+          nr = std::min<int64_t>(v.eta, v.B - r0);
+        } else {
+          const int mm = (lb_posted - v.mu_pre) % v.mu_dec;
+          r0 = (int64_t)mm * v.xi;
+          nr = std::min<int64_t>(v.xi, v.B - r0);
+        }
+        op(SQ_OP_RECV_LB, lb_posted, phase, t, 0, v.P - 1, r0, nr, nr);
+      }
+    }
+    if (dist && !first) op(SQ_OP_RECV_ACT, it, phase, t, slot, rank - 1, seq0, nseq, T);
+    op(SQ_OP_COMPUTE, it, phase, t, slot, -1, seq0, nseq, T);
+    if (!last) {
+      op(SQ_OP_SEND_ACT, it, phase, t, slot, rank + 1, seq0, nseq, T);
+    } else {
+      op(SQ_OP_OUT, it, phase, t, slot, -1, seq0, nseq, nseq);
+      if (t < v.n_dec) op(dist ? SQ_OP_SEND_LB : SQ_OP_LOOPBACK_LOCAL, it, phase, t, slot, dist ? 0 : -1, seq0, nseq, nseq);
+    }
+  }
+  return ops;
+}
+
 }  // namespace
 }  // namespace sq
 
@@ -104,6 +157,16 @@ sq_status sq_plan_check(const sq_plan* p) {
     }
   }
   return SQ_OK;
+}
+
+int64_t sq_pipeline_schedule(const sq_plan* plan, int rank, sq_sched_op* ops, int64_t max_ops) {
+  if (sq_plan_check(plan) != SQ_OK || rank >= plan->n_stages || rank < -1) return -1;
+  const std::vector<sq_sched_op> v = make_schedule(view(*plan), rank);
+  if (ops) {
+    const int64_t n = std::min<int64_t>(max_ops, (int64_t)v.size());
+    for (int64_t i = 0; i < n; ++i) ops[i] = v[i];
+  }
+  return (int64_t)v.size();
 }
 
 size_t sq_comm_unique_id_bytes(void) { return sizeof(ncclUniqueId); }
@@ -240,126 +303,106 @@ sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers,
   cudaError_t ce = cudaSuccess;
   sq_status rs = SQ_OK;
 
-  // loop-back bookkeeping at stage 0 (distributed): LB index i -> rows of dec_in
-  // order: prefill mb 0..mu_pre-1, then decode (t, m) for t = 1..n_dec-1
-  const int n_lb = v.mu_pre + std::max(0, v.n_dec - 1) * v.mu_dec;
-  auto lb_rows = [&](int i, int64_t& row0, int64_t& nrows) {
-    if (i < v.mu_pre) {
-      row0 = (int64_t)i * v.eta;
-      nrows = std::min<int64_t>(v.eta, v.B - row0);
-    } else {
-      const int m = (i - v.mu_pre) % v.mu_dec;
-      row0 = (int64_t)m * v.xi;
-      nrows = std::min<int64_t>(v.xi, v.B - row0);
+  // ---- execute this rank's schedule (sq_pipeline_schedule): one op at a time, compute on S,
+  // sends on s_send, receives on s_recv, CUDA events for every cross-stream dependency.
+  const std::vector<sq_sched_op> ops = make_schedule(v, rank);
+  int lbslot = 0;
+  bool lb_wait_pending = false;
+  bool pre_marked = false;
+  for (size_t oi = 0; oi < ops.size() && rs == SQ_OK && ce == cudaSuccess; ++oi) {
+    const sq_sched_op& o = ops[oi];
+    const bool pre = o.phase == SQ_PREFILL;
+    float* buf = act[o.slot];
+    if (!pre && !pre_marked) {
+      cudaEventRecord(ev_pre, S);
+      pre_marked = true;
     }
-  };
-  int lb_posted = 0;
-  auto post_lb_recvs = [&](int upto) {  // stage 0: post loop-back recvs [lb_posted, upto]
-    for (; lb_posted <= upto && lb_posted < n_lb; ++lb_posted) {
-      int64_t r0, nr;
-      lb_rows(lb_posted, r0, nr);
-      // WAR: a decode loop-back overwrites dec_in rows that earlier decode items read
-      if (lb_posted >= v.mu_pre) cudaStreamWaitEvent(comm->s_recv, ev_dec_read, 0);
-      ncclResult_t nr_ = ncclRecv(dec_in + r0 * h1, (size_t)(nr * h1), ncclFloat32, 0, comm->recv_comm, comm->s_recv);
-      if (nr_ != ncclSuccess) { rs = nccl_check(nr_, "ncclRecv(loop-back)"); return; }
-    }
-    cudaEventRecord(ev_recv[0], comm->s_recv);
-    cudaStreamWaitEvent(S, ev_recv[0], 0);
-  };
-
-  const int total_items = v.mu_pre + v.n_dec * v.mu_dec;
-  int slot = 0, lbslot = 0;
-  for (int it = 0; it < total_items && rs == SQ_OK && ce == cudaSuccess; ++it) {
-    const bool pre = it < v.mu_pre;
-    const int m = pre ? it : (it - v.mu_pre) % v.mu_dec;
-    const int t = pre ? 0 : 1 + (it - v.mu_pre) / v.mu_dec;
-    const int64_t seq0 = pre ? (int64_t)m * v.eta : (int64_t)m * v.xi;
-    const int64_t nseq = std::min<int64_t>(pre ? v.eta : v.xi, v.B - seq0);
-    const int64_t T = pre ? nseq * v.s : nseq;
-    const int phase = pre ? SQ_PREFILL : SQ_DECODE;
-    if (pre == false && it == v.mu_pre) cudaEventRecord(ev_pre, S);
-    float* buf = act[slot];
-
-    // ---------------- input
-    const float* x_in;
-    if (is_first) {
-      if (pre) {
-        x_in = x0 + seq0 * v.s * h1;
-      } else {
-        if (dist) {
-          int need;
-          if (t == 1) need = (int)((seq0 + nseq - 1) / v.eta);
-          else need = v.mu_pre + (t - 2) * v.mu_dec + m;
-          post_lb_recvs(need);
-          if (rs) break;
-        }
-        x_in = dec_in + seq0 * h1;
+    switch (o.kind) {
+      case SQ_OP_RECV_LB: {
+        // WAR: a decode loop-back overwrites dec_in rows that earlier decode items read
+        if (o.item >= v.mu_pre) cudaStreamWaitEvent(comm->s_recv, ev_dec_read, 0);
+        ncclResult_t r = ncclRecv(dec_in + o.seq0 * h1, (size_t)(o.nseq * h1), ncclFloat32, 0, comm->recv_comm, comm->s_recv);
+        if (r != ncclSuccess) rs = nccl_check(r, "ncclRecv(loop-back)");
+        lb_wait_pending = true;
+        break;
       }
-      if (dist) cudaStreamWaitEvent(S, ev_free[slot], 0);  // previous send from this buffer done
-    } else {
-      // recv into buf (after its previous send completed)
-      cudaStreamWaitEvent(comm->s_recv, ev_free[slot], 0);
-      ncclResult_t r = ncclRecv(buf, (size_t)(T * h1), ncclFloat32, 0, comm->recv_comm, comm->s_recv);
-      if (r != ncclSuccess) { rs = nccl_check(r, "ncclRecv"); break; }
-      cudaEventRecord(ev_recv[slot], comm->s_recv);
-      cudaStreamWaitEvent(S, ev_recv[slot], 0);
-      x_in = buf;
-    }
-
-    // ---------------- compute: this rank's layers (local mode: every stage in order)
-    if (local) {
-      const float* xi = x_in;
-      for (int r = 0; r < v.P && rs == SQ_OK; ++r) {
-        const int f = v.first_layer[r], nl = v.first_layer[r + 1] - f;
-        rs = stage_forward(layers + f, nl, phase, xi, T, buf, nullptr, stage_ws, stage_ws_bytes, S);
-        xi = buf;  // the "transfer" to the next stage is the buffer itself
+      case SQ_OP_RECV_ACT: {
+        cudaStreamWaitEvent(comm->s_recv, ev_free[o.slot], 0);  // previous use of the buffer finished
+        ncclResult_t r = ncclRecv(buf, (size_t)(o.rows * h1), ncclFloat32, 0, comm->recv_comm, comm->s_recv);
+        if (r != ncclSuccess) { rs = nccl_check(r, "ncclRecv"); break; }
+        cudaEventRecord(ev_recv[o.slot], comm->s_recv);
+        cudaStreamWaitEvent(S, ev_recv[o.slot], 0);
+        break;
       }
-    } else {
-      rs = stage_forward(layers, n_layers, phase, x_in, T, buf, nullptr, stage_ws, stage_ws_bytes, S);
-    }
-    if (rs) break;
-    if (is_first && !pre && dist) cudaEventRecord(ev_dec_read, S);
-
-    // ---------------- output
-    if (!is_last) {
-      cudaEventRecord(ev_ready, S);
-      cudaStreamWaitEvent(comm->s_send, ev_ready, 0);
-      ncclResult_t r = ncclSend(buf, (size_t)(T * h1), ncclFloat32, 1, comm->send_comm, comm->s_send);
-      if (r != ncclSuccess) { rs = nccl_check(r, "ncclSend"); break; }
-      bytes_sent += T * h1 * 4;
-      cudaEventRecord(ev_free[slot], comm->s_send);
-    } else {
-      // out rows and LN loop-back
-      const float* src = pre ? buf + (int64_t)(v.s - 1) * h1 : buf;
-      const int64_t sstride = pre ? (int64_t)v.s * h1 : h1;
-      ce = launch_copy_rows(src, sstride, nseq, h1, out + (seq0 * out_rows + t) * h1, out_rows * h1, S);
-      if (ce) break;
-      const bool need_lb = t < v.n_dec;  // the last step's successor input is never consumed
-      if (need_lb) {
-        if (!dist) {
-          // single-GPU (or virtual) pipeline: e = LN(hidden) straight into dec_in
-          ce = launch_copy_rows(src, sstride, nseq, h1, lb[0], h1, S);
-          if (!ce) ce = launch_layernorm_f32(lb[0], nseq, h1, dec_in + seq0 * h1, S);
+      case SQ_OP_COMPUTE: {
+        const float* x_in;
+        if (is_first) {
+          x_in = pre ? x0 + o.seq0 * v.s * h1 : dec_in + o.seq0 * h1;
+          if (lb_wait_pending) {
+            cudaEventRecord(ev_recv[0], comm->s_recv);
+            cudaStreamWaitEvent(S, ev_recv[0], 0);
+            lb_wait_pending = false;
+          }
+          if (dist) cudaStreamWaitEvent(S, ev_free[o.slot], 0);  // previous send from this buffer done
         } else {
-          cudaStreamWaitEvent(S, ev_lbfree[lbslot], 0);
-          ce = launch_copy_rows(src, sstride, nseq, h1, lb[lbslot], h1, S);
-          if (!ce) ce = launch_layernorm_f32(lb[lbslot], nseq, h1, lb[lbslot], S);
-          if (ce) break;
-          cudaEventRecord(ev_lbready[lbslot], S);
-          cudaStreamWaitEvent(comm->s_send, ev_lbready[lbslot], 0);
-          ncclResult_t r = ncclSend(lb[lbslot], (size_t)(nseq * h1), ncclFloat32, 1, comm->send_comm, comm->s_send);
-          if (r != ncclSuccess) { rs = nccl_check(r, "ncclSend(loop-back)"); break; }
-          bytes_sent += nseq * h1 * 4;
-          cudaEventRecord(ev_lbfree[lbslot], comm->s_send);
-          lbslot ^= 1;
+          x_in = buf;
         }
-        if (ce) break;
+        if (local) {
+          const float* xi = x_in;
+          for (int r = 0; r < v.P && rs == SQ_OK; ++r) {
+            const int f = v.first_layer[r], nl = v.first_layer[r + 1] - f;
+            rs = stage_forward(layers + f, nl, o.phase, xi, o.rows, buf, nullptr, stage_ws, stage_ws_bytes, S);
+            xi = buf;  // the "transfer" to the next stage is the buffer itself
+          }
+        } else {
+          rs = stage_forward(layers, n_layers, o.phase, x_in, o.rows, buf, nullptr, stage_ws, stage_ws_bytes, S);
+        }
+        if (is_first && !pre && dist) cudaEventRecord(ev_dec_read, S);
+        break;
       }
-      if (dist) cudaEventRecord(ev_free[slot], S);
+      case SQ_OP_SEND_ACT: {
+        cudaEventRecord(ev_ready, S);
+        cudaStreamWaitEvent(comm->s_send, ev_ready, 0);
+        ncclResult_t r = ncclSend(buf, (size_t)(o.rows * h1), ncclFloat32, 1, comm->send_comm, comm->s_send);
+        if (r != ncclSuccess) { rs = nccl_check(r, "ncclSend"); break; }
+        bytes_sent += o.rows * h1 * 4;
+        cudaEventRecord(ev_free[o.slot], comm->s_send);
+        break;
+      }
+      case SQ_OP_OUT: {
+        const float* src = pre ? buf + (int64_t)(v.s - 1) * h1 : buf;
+        const int64_t sstride = pre ? (int64_t)v.s * h1 : h1;
+        ce = launch_copy_rows(src, sstride, o.nseq, h1, out + (o.seq0 * out_rows + o.t) * h1, out_rows * h1, S);
+        if (dist) cudaEventRecord(ev_free[o.slot], S);
+        break;
+      }
+      case SQ_OP_LOOPBACK_LOCAL: {
+        const float* src = pre ? buf + (int64_t)(v.s - 1) * h1 : buf;
+        const int64_t sstride = pre ? (int64_t)v.s * h1 : h1;
+        ce = launch_copy_rows(src, sstride, o.nseq, h1, lb[0], h1, S);
+        if (!ce) ce = launch_layernorm_f32(lb[0], o.nseq, h1, dec_in + o.seq0 * h1, S);
+        break;
+      }
+      case SQ_OP_SEND_LB: {
+        const float* src = pre ? buf + (int64_t)(v.s - 1) * h1 : buf;
+        const int64_t sstride = pre ? (int64_t)v.s * h1 : h1;
+        cudaStreamWaitEvent(S, ev_lbfree[lbslot], 0);
+        ce = launch_copy_rows(src, sstride, o.nseq, h1, lb[lbslot], h1, S);
+        if (!ce) ce = launch_layernorm_f32(lb[lbslot], o.nseq, h1, lb[lbslot], S);
+        if (ce) break;
+        cudaEventRecord(ev_lbready[lbslot], S);
+        cudaStreamWaitEvent(comm->s_send, ev_lbready[lbslot], 0);
+        ncclResult_t r = ncclSend(lb[lbslot], (size_t)(o.nseq * h1), ncclFloat32, 1, comm->send_comm, comm->s_send);
+        if (r != ncclSuccess) { rs = nccl_check(r, "ncclSend(loop-back)"); break; }
+        bytes_sent += o.nseq * h1 * 4;
+        cudaEventRecord(ev_lbfree[lbslot], comm->s_send);
+        if (dist) cudaEventRecord(ev_free[o.slot], S);
+        lbslot ^= 1;
+        break;
+      }
     }
-    slot ^= 1;
   }
-  if (v.mu_dec == 0 || v.n_dec == 0) cudaEventRecord(ev_pre, S);
+  if (!pre_marked) cudaEventRecord(ev_pre, S);
   if (dist && rs == SQ_OK) {
     cudaEventRecord(ev_ready, comm->s_send);
     cudaStreamWaitEvent(S, ev_ready, 0);

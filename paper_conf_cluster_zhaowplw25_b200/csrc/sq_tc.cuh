@@ -1,0 +1,148 @@
+// tcgen05 building blocks shared by the prefill GEMM (K3) and the tensor-core
+// decode GEMV (K2c): SW128 smem descriptors, the instruction descriptor, and the
+// per-row dequantization of one 128-k group straight into tensor memory.
+//
+// Packed weight stages are UNSWIZZLED [128 rows][GB bytes] (8 contiguous T16 units of
+// 16 rows, fetched by cp.async.bulk); fp16 weight stages are two SW128 [128][128 B] tiles.
+#pragma once
+#include "sq_common.cuh"
+
+namespace sq {
+namespace tc {
+
+template <int BITS>
+struct GCfg;
+template <>
+struct GCfg<3> { static constexpr int GB = 48; static constexpr int S_W = 4; };
+template <>
+struct GCfg<4> { static constexpr int GB = 64; static constexpr int S_W = 4; };
+template <>
+struct GCfg<8> { static constexpr int GB = 128; static constexpr int S_W = 3; };
+template <>
+struct GCfg<16> { static constexpr int GB = 256; static constexpr int S_W = 2; };
+
+__device__ __forceinline__ uint64_t make_sw128_desc(uint32_t saddr) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFF);
+  d |= (uint64_t)1 << 16;              // LBO (ignored for swizzled K-major)
+  d |= (uint64_t)(1024 >> 4) << 32;    // SBO: 8 rows x 128 B
+  d |= (uint64_t)1 << 46;              // descriptor version (sm_100)
+  d |= (uint64_t)2 << 61;              // SWIZZLE_128B
+  return d;
+}
+
+// instruction descriptor: kind::f16, A=B=f16 K-major, D=f32, M x N
+constexpr uint32_t make_idesc(int M, int N) {
+  return (1u << 4) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+
+__device__ __forceinline__ uint32_t hsub_fma(uint32_t h, uint32_t off2, uint32_t s2, uint32_t z2) {
+  __half2 c = __hsub2(*reinterpret_cast<__half2*>(&h), *reinterpret_cast<__half2*>(&off2));
+  __half2 r = __hfma2(c, *reinterpret_cast<__half2*>(&s2), *reinterpret_cast<__half2*>(&z2));
+  return *reinterpret_cast<uint32_t*>(&r);
+}
+
+// Dequantize this thread's row (r) of one 128-k group into 64 half2 columns,
+// written to TMEM in 4 batches of 16 columns.
+template <int BITS>
+__device__ __forceinline__ void dequant_row_to_tmem(const uint8_t* wst, uint32_t meta, int r, uint32_t taddr) {
+  const uint32_t s2 = (meta & 0xFFFFu) * 0x10001u;
+  const uint32_t z2 = (meta >> 16) * 0x10001u;
+  constexpr uint32_t K1024 = 0x64006400u, K64 = 0x54005400u;
+  if constexpr (BITS == 4) {
+    // unswizzled [128 rows][64 B]: thread r visits its 16-B chunks in the order (j + r/2) % 4,
+    // so the 8 threads of each shared-memory phase hit 8 distinct 16-B bank groups
+    const uint8_t* row = wst + r * 64;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int b = (j + (r >> 1)) & 3;
+      uint4 v = *reinterpret_cast<const uint4*>(row + b * 16);
+      const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
+      uint32_t o[16];
+#pragma unroll
+      for (int w = 0; w < 4; ++w) {
+        const uint32_t x = wv[w], x8 = x >> 8;
+        o[4 * w + 0] = hsub_fma(lop3_and_or(x, 0x000F000Fu, K1024), K1024, s2, z2);
+        o[4 * w + 1] = hsub_fma(lop3_and_or(x, 0x00F000F0u, K64), K64, s2, z2);
+        o[4 * w + 2] = hsub_fma(lop3_and_or(x8, 0x000F000Fu, K1024), K1024, s2, z2);
+        o[4 * w + 3] = hsub_fma(lop3_and_or(x8, 0x00F000F0u, K64), K64, s2, z2);
+      }
+      tmem_st16(taddr + 16 * b, o);
+    }
+  } else if constexpr (BITS == 8) {
+    // unswizzled [128 rows][128 B]: batch (pair of 16-B chunks) (j + r) % 4, chunk order within the
+    // pair swapped for r%8 >= 4 -> 8 distinct bank groups per phase for every load instruction
+    const uint8_t* row = wst + r * 128;
+    const int sw = (r >> 2) & 1;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int b = (j + r) & 3;
+      uint32_t o[16];
+#pragma unroll
+      for (int hh = 0; hh < 2; ++hh) {
+        const int h = hh ^ sw, c = 2 * b + h;
+        uint4 v = *reinterpret_cast<const uint4*>(row + c * 16);
+        const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+          o[8 * h + 2 * t] = hsub_fma(prmt(wv[t], 0x64646464u, 0x4140u), K1024, s2, z2);
+          o[8 * h + 2 * t + 1] = hsub_fma(prmt(wv[t], 0x64646464u, 0x4342u), K1024, s2, z2);
+        }
+      }
+      tmem_st16(taddr + 16 * b, o);
+    }
+  } else if constexpr (BITS == 3) {
+    const uint32_t* row = reinterpret_cast<const uint32_t*>(wst + r * 48);
+#pragma unroll
+    for (int bl = 0; bl < 4; ++bl) {
+      const uint32_t L0 = row[3 * bl], L1 = row[3 * bl + 1], H = row[3 * bl + 2];
+      uint32_t o[16];
+#pragma unroll
+      for (int a = 0; a < 2; ++a) {
+        const uint32_t La = a ? L1 : L0;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const uint32_t lo = La >> (2 * i);
+          const int sh = i + 8 * a - 2;
+          const uint32_t hs = sh >= 0 ? (H >> sh) : (H << (-sh));
+          uint32_t t;
+          asm("lop3.b32 %0, %1, %2, %3, 0xD8;" : "=r"(t) : "r"(hs), "r"(lo), "r"(0x00030003u));  // mask ? lo : hs
+          o[8 * a + i] = hsub_fma(lop3_and_or(t, 0x00070007u, K1024), K1024, s2, z2);
+        }
+      }
+      tmem_st16(taddr + 16 * bl, o);
+    }
+  } else {
+    // fp16: two SW128 regions (k 0..63, 64..127) of [128 rows x 128 B]
+#pragma unroll
+    for (int b = 0; b < 4; ++b) {
+      const uint8_t* region = wst + (b >> 1) * (128 * 128) + r * 128;
+      uint32_t o[16];
+#pragma unroll
+      for (int h = 0; h < 4; ++h) {
+        const int c = 4 * (b & 1) + h, pc = c ^ (r & 7);
+        uint4 v = *reinterpret_cast<const uint4*>(region + pc * 16);
+        o[4 * h] = v.x; o[4 * h + 1] = v.y; o[4 * h + 2] = v.z; o[4 * h + 3] = v.w;
+      }
+      tmem_st16(taddr + 16 * b, o);
+    }
+  }
+}
+
+
+// Fetch the 128-row x 1-group weight tile (8 T16 units, each 16*GB contiguous bytes at unit
+// index t*kg + g) and its meta (8 x 64 B) with 16 bulk copies onto one mbarrier.
+template <int BITS>
+__device__ __forceinline__ void load_w_tile(uint8_t* wdst, uint8_t* mdst, const uint8_t* packed,
+                                            const uint32_t* meta, int64_t tile16, int g, int kg, uint64_t* bar) {
+  constexpr int UB = 16 * GCfg<BITS>::GB;
+#pragma unroll
+  for (int t = 0; t < 8; ++t) {
+    const int64_t u = (tile16 + t) * kg + g;
+    bulk_load(wdst + t * UB, packed + u * UB, UB, bar);
+    bulk_load(mdst + t * 64, meta + u * 16, 64, bar);
+  }
+}
+
+}  // namespace tc
+}  // namespace sq

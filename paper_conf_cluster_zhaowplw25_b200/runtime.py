@@ -113,6 +113,18 @@ def sq_plan_check(plan: Plan) -> None:
     _check(_L.sq_plan_check(ctypes.byref(plan.c)))
 
 
+def sq_pipeline_schedule(plan: Plan, rank: int) -> list[dict]:
+    """Host-only: the op sequence `rank` executes in sq_pipeline_run (see sq.h)."""
+    from . import SQ_OP_NAMES, sq_sched_op
+    n = int(_L.sq_pipeline_schedule(ctypes.byref(plan.c), rank, None, 0))
+    if n < 0:
+        raise ValueError("invalid plan")
+    arr = (sq_sched_op * max(n, 1))()
+    _L.sq_pipeline_schedule(ctypes.byref(plan.c), rank, arr, n)
+    return [{"kind": SQ_OP_NAMES[o.kind], "item": o.item, "phase": o.phase, "t": o.t, "slot": o.slot,
+             "peer": o.peer, "seq0": o.seq0, "nseq": o.nseq, "rows": o.rows} for o in arr[:n]]
+
+
 class Comm:
     def __init__(self, handle: int):
         self.h = ctypes.c_void_p(handle)
