@@ -111,31 +111,32 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 
   if (warp == 0) {
     // ---------------- TMA producer
-    if (lane == 0) {
+    {  // whole warp runs the loop (warp-uniform operands live in uniform registers); a leader issues
       int it_x = 0;
       for (int g = 0; g < kg; ++g) {
         const int sw = g % S_W, rw = g / S_W;
         mbar_wait(&empty_w[sw], (rw & 1) ^ 1);
         uint8_t* wdst = smem + SM::OFF_W + sw * SM::W_STAGE;
-        mbar_arrive_expect_tx(&full_w[sw], W_BYTES + (BITS != 16 ? BN * 4 : 0));
+        if (elect_one()) mbar_arrive_expect_tx(&full_w[sw], W_BYTES + (BITS != 16 ? BN * 4 : 0));
         if constexpr (BITS == 16) {
-          tma_load_2d(wdst, &tm_w, &full_w[sw], g * 128, (int32_t)n0);
-          tma_load_2d(wdst + BN * 128, &tm_w, &full_w[sw], g * 128 + 64, (int32_t)n0);
+          if (elect_one()) tma_load_2d(wdst, &tm_w, &full_w[sw], g * 128, (int32_t)n0);
+          if (elect_one()) tma_load_2d(wdst + BN * 128, &tm_w, &full_w[sw], g * 128 + 64, (int32_t)n0);
         } else {
-          // placement T16: 8 contiguous units of 16 rows -> [128 rows][GB] (bulk copies)
-          load_w_tile<BITS>(wdst, smem + SM::OFF_META + sw * BN * 4, p.packed, p.meta, n0 / 16, g, kg, &full_w[sw]);
+          // placement T16: 4-D box {GB bytes, 16 rows, 1 group, 8 row tiles} -> [128 rows][GB]
+          if (elect_one()) tma_load_4d(wdst, &tm_w, &full_w[sw], 0, 0, g, (int32_t)(n0 / 16));
+          if (elect_one()) tma_load_3d(smem + SM::OFF_META + sw * BN * 4, &tm_m, &full_w[sw], 0, g, (int32_t)(n0 / 16));
         }
         for (int h = 0; h < 2; ++h, ++it_x) {
           const int sx = it_x % S_X, rx = it_x / S_X;
           mbar_wait(&empty_x[sx], (rx & 1) ^ 1);
-          mbar_arrive_expect_tx(&full_x[sx], X_STAGE_BYTES);
-          tma_load_2d(smem + SM::OFF_X + sx * X_STAGE_BYTES, &tm_x, &full_x[sx], g * 128 + h * XK, (int32_t)t0);
+          if (elect_one()) mbar_arrive_expect_tx(&full_x[sx], X_STAGE_BYTES);
+          if (elect_one()) tma_load_2d(smem + SM::OFF_X + sx * X_STAGE_BYTES, &tm_x, &full_x[sx], g * 128 + h * XK, (int32_t)t0);
         }
       }
     }
   } else if (warp == 1) {
     // ---------------- MMA issuer (single thread)
-    if (lane == 0) {
+    {  // whole warp runs the loop; the elected leader issues tcgen05.mma / commit
       int it_x = 0;
       for (int g = 0; g < kg; ++g) {
         const int sa = g % S_A, ra = g / S_A;
@@ -150,13 +151,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           for (int kk = 0; kk < XK / 16; ++kk) {
             const uint64_t bdesc = make_sw128_desc(xs + kk * 32);
             const uint32_t a_tm = tmem + A_COL + sa * 64 + h * 32 + kk * 8;
-            tc_mma_ts(tmem + D_COL, a_tm, bdesc, kIdesc, (g | h | kk) != 0);
+            if (elect_one()) tc_mma_ts(tmem + D_COL, a_tm, bdesc, kIdesc, (g | h | kk) != 0);
           }
-          tc_commit(&empty_x[sx]);
+          if (elect_one()) tc_commit(&empty_x[sx]);
         }
-        tc_commit(&empty_a[sa]);
+        if (elect_one()) tc_commit(&empty_a[sa]);
       }
-      tc_commit(d_full);
+      if (elect_one()) tc_commit(d_full);
     }
   } else {
     // ---------------- dequant warps (one thread per weight row; group gi takes k-groups

@@ -73,7 +73,12 @@ struct TcP {
   int U;      // units = (n / 128) * kg
   float* part;  // [CTAs][2][32 tokens][128 rows]
   int* cnt;     // [n / 128]
+  unsigned long long* trace;  // debug: CTA 0 per-unit clock64 events (sq_debug_trace), or null
 };
+
+__device__ __forceinline__ void trace_ev(const TcP& p, int ev, int i) {
+  if (p.trace && blockIdx.x == 0 && i < 256) p.trace[ev * 256 + i] = clock64();
+}
 
 __device__ __forceinline__ int rlo(int i, int total, int parts) { return (int)(((long long)i * total) / parts); }
 
@@ -137,31 +142,35 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 
   if (warp == 0) {
     // ---------------- producer: weights (+meta) and the activation slice of every unit
-    if (lane == 0) {
+    {  // whole warp runs the loop (warp-uniform operands live in uniform registers); a leader issues
       for (int i = 0; i < nunits; ++i) {
         const int u = C0 + i, rt = u / kg, g = u - rt * kg;
         const int sw = i % S_W, rw = i / S_W;
         mbar_wait(&empty_w[sw], (rw & 1) ^ 1);
+        trace_ev(p, 0, i);
         uint8_t* wdst = smem + SM::OFF_W + sw * SM::W_STAGE;
-        mbar_arrive_expect_tx(&full_w[sw], W_BYTES + (BITS != 16 ? BN * 4 : 0));
+        if (elect_one()) mbar_arrive_expect_tx(&full_w[sw], W_BYTES + (BITS != 16 ? BN * 4 : 0));
         if constexpr (BITS == 16) {
-          tma_load_2d(wdst, &tm_w, &full_w[sw], g * 128, rt * BN);
-          tma_load_2d(wdst + BN * 128, &tm_w, &full_w[sw], g * 128 + 64, rt * BN);
+          if (elect_one()) tma_load_2d(wdst, &tm_w, &full_w[sw], g * 128, rt * BN);
+          if (elect_one()) tma_load_2d(wdst + BN * 128, &tm_w, &full_w[sw], g * 128 + 64, rt * BN);
         } else {
-          load_w_tile<BITS>(wdst, smem + SM::OFF_META + sw * BN * 4, p.packed, p.meta, (int64_t)rt * (BN / 16), g, kg,
-                            &full_w[sw]);
+          if (elect_one()) tma_load_4d(wdst, &tm_w, &full_w[sw], 0, 0, g, rt * (BN / 16));
+          trace_ev(p, 6, i);
+          if (elect_one()) tma_load_3d(smem + SM::OFF_META + sw * BN * 4, &tm_m, &full_w[sw], 0, g, rt * (BN / 16));
+          trace_ev(p, 7, i);
         }
         for (int h = 0; h < 2; ++h) {
           const int it = 2 * i + h, sx = it % S_X, rx = it / S_X;
           mbar_wait(&empty_x[sx], (rx & 1) ^ 1);
-          mbar_arrive_expect_tx(&full_x[sx], X_STAGE);
-          tma_load_2d(smem + SM::OFF_X + sx * X_STAGE, &tm_x, &full_x[sx], g * 128 + h * XK, 0);
+          if (elect_one()) mbar_arrive_expect_tx(&full_x[sx], X_STAGE);
+          if (elect_one()) tma_load_2d(smem + SM::OFF_X + sx * X_STAGE, &tm_x, &full_x[sx], g * 128 + h * XK, 0);
+          trace_ev(p, 8 + h, i);
         }
       }
     }
   } else if (warp == 1) {
     // ---------------- MMA issuer
-    if (lane == 0) {
+    {  // whole warp runs the loop; the elected leader issues tcgen05.mma / commit
       int seg = 0, dbuf = 0;
       for (int i = 0; i < nunits; ++i) {
         const int u = C0 + i, g = u % kg;
@@ -174,23 +183,27 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         }
         const int sa = i % S_A, ra = i / S_A;
         mbar_wait(&full_a[sa], ra & 1);
+        trace_ev(p, 3, i);
         tc_fence_after();
         for (int h = 0; h < 2; ++h) {
           const int it = 2 * i + h, sx = it % S_X, rx = it / S_X;
           mbar_wait(&full_x[sx], rx & 1);
+          trace_ev(p, 10 + 2 * h, i);
           tc_fence_after();
           const uint32_t xs = smem_u32(smem + SM::OFF_X + sx * X_STAGE);
 #pragma unroll
           for (int kk = 0; kk < XK / 16; ++kk) {
             const uint64_t bdesc = make_sw128_desc(xs + kk * 32);
             const uint32_t a_tm = tmem + A_COL + sa * 64 + h * 32 + kk * 8;
-            tc_mma_ts(tmem + D_COL + dbuf * BT, a_tm, bdesc, kIdescTc, (seg_first && h == 0 && kk == 0) ? 0u : 1u);
+            if (elect_one()) tc_mma_ts(tmem + D_COL + dbuf * BT, a_tm, bdesc, kIdescTc, (seg_first && h == 0 && kk == 0) ? 0u : 1u);
           }
-          tc_commit(&empty_x[sx]);
+          trace_ev(p, 11 + 2 * h, i);
+          if (elect_one()) tc_commit(&empty_x[sx]);
         }
-        tc_commit(&empty_a[sa]);
+        if (elect_one()) tc_commit(&empty_a[sa]);
+        trace_ev(p, 4, i);
         if (seg_last) {
-          tc_commit(&d_full[dbuf]);
+          if (elect_one()) tc_commit(&d_full[dbuf]);
           ++seg;
         }
       }
@@ -205,7 +218,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       const int sw = i % S_W, rw = i / S_W;
       const int sa = i % S_A, ra = i / S_A;
       mbar_wait(&full_w[sw], rw & 1);
+      if (threadIdx.x == 64) trace_ev(p, 1, i);
       mbar_wait(&empty_a[sa], (ra & 1) ^ 1);
+      if (threadIdx.x == 64) trace_ev(p, 5, i);
       tc_fence_after();
       const uint32_t meta = reinterpret_cast<const uint32_t*>(smem + SM::OFF_META + sw * BN * 4)[r];
       dequant_row_to_tmem<BITS>(smem + SM::OFF_W + sw * SM::W_STAGE, meta, r, tmem + lane_base + A_COL + sa * 64);
@@ -216,6 +231,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         mbar_arrive(&empty_w[sw]);
         mbar_arrive(&full_a[sa]);
       }
+      if (threadIdx.x == 64 || threadIdx.x == 64 + 128) trace_ev(p, 2, i);
     }
   } else {
     // ---------------- epilogue warps: drain finished segments
@@ -342,6 +358,8 @@ cudaError_t launch_tc_b(const CUtensorMap& tx, const CUtensorMap& tw, const CUte
   }
 }
 
+unsigned long long* g_trace = nullptr;
+
 int tc_ctas(int64_t U) {
   const int64_t full = num_sms();
   return (int)(U < full ? U : full);
@@ -399,6 +417,7 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
   uint8_t* base = static_cast<uint8_t*>(ws);
   p.cnt = reinterpret_cast<int*>(base);
   p.part = reinterpret_cast<float*>(base + kCntBytes);
+  p.trace = g_trace;
   const int nc = tc_ctas(p.U);
   const double bytes = (double)w.n * w.k * w.bits / 8.0 + (w.bits != 16 ? (double)w.n * (w.k / 128) * 4.0 : 0.0);
   auto t = prof_begin(KC_GEMV, bytes, 2.0 * m * w.n * w.k, s);
@@ -415,3 +434,7 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
 }
 
 }  // namespace sq
+
+// debug only (not part of include/sq.h): record CTA 0's per-unit clock64 events of the
+// tcgen05 decode kernel into a device buffer of 14 x 256 uint64 (tools/trace_tc.py)
+extern "C" void sq_debug_trace(void* dev_buf) { sq::g_trace = static_cast<unsigned long long*>(dev_buf); }

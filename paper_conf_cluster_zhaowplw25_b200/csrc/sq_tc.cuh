@@ -2,8 +2,11 @@
 // decode GEMV (K2c): SW128 smem descriptors, the instruction descriptor, and the
 // per-row dequantization of one 128-k group straight into tensor memory.
 //
-// Packed weight stages are UNSWIZZLED [128 rows][GB bytes] (8 contiguous T16 units of
-// 16 rows, fetched by cp.async.bulk); fp16 weight stages are two SW128 [128][128 B] tiles.
+// Packed weight stages are [128 rows][GB bytes] fetched by one 4-D TMA box (8 T16 units of
+// 16 rows) with SWIZZLE_64B (INT4) / SWIZZLE_128B (INT8) / none (INT3, 48-B rows are
+// conflict-free); fp16 weight stages are two SW128 [128][128 B] tiles.  tcgen05.st is
+// .sync.aligned: its TMEM column address must be warp-uniform, so the chunk order is static
+// and bank conflicts are avoided by the TMA swizzle, not by per-thread reordering.
 #pragma once
 #include "sq_common.cuh"
 
@@ -50,13 +53,11 @@ __device__ __forceinline__ void dequant_row_to_tmem(const uint8_t* wst, uint32_t
   const uint32_t z2 = (meta >> 16) * 0x10001u;
   constexpr uint32_t K1024 = 0x64006400u, K64 = 0x54005400u;
   if constexpr (BITS == 4) {
-    // unswizzled [128 rows][64 B]: thread r visits its 16-B chunks in the order (j + r/2) % 4,
-    // so the 8 threads of each shared-memory phase hit 8 distinct 16-B bank groups
     const uint8_t* row = wst + r * 64;
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int b = (j + (r >> 1)) & 3;
-      uint4 v = *reinterpret_cast<const uint4*>(row + b * 16);
+    for (int b = 0; b < 4; ++b) {
+      const int pc = b ^ ((r >> 1) & 3);  // SWIZZLE_64B
+      uint4 v = *reinterpret_cast<const uint4*>(row + pc * 16);
       const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
       uint32_t o[16];
 #pragma unroll
@@ -70,18 +71,14 @@ __device__ __forceinline__ void dequant_row_to_tmem(const uint8_t* wst, uint32_t
       tmem_st16(taddr + 16 * b, o);
     }
   } else if constexpr (BITS == 8) {
-    // unswizzled [128 rows][128 B]: batch (pair of 16-B chunks) (j + r) % 4, chunk order within the
-    // pair swapped for r%8 >= 4 -> 8 distinct bank groups per phase for every load instruction
     const uint8_t* row = wst + r * 128;
-    const int sw = (r >> 2) & 1;
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int b = (j + r) & 3;
+    for (int b = 0; b < 4; ++b) {
       uint32_t o[16];
 #pragma unroll
-      for (int hh = 0; hh < 2; ++hh) {
-        const int h = hh ^ sw, c = 2 * b + h;
-        uint4 v = *reinterpret_cast<const uint4*>(row + c * 16);
+      for (int h = 0; h < 2; ++h) {
+        const int c = 2 * b + h, pc = c ^ (r & 7);  // SWIZZLE_128B
+        uint4 v = *reinterpret_cast<const uint4*>(row + pc * 16);
         const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
         for (int t = 0; t < 4; ++t) {
