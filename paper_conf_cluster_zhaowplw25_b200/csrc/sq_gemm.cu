@@ -34,8 +34,10 @@ constexpr int BN = 128;   // weight rows per tile (TMEM lanes, MMA M)
 constexpr int BT = 256;   // tokens per tile (MMA N)
 constexpr int XK = 64;    // k per activation stage (one 128-B swizzle row)
 constexpr int S_X = 4;
-constexpr int S_A = 3;
+constexpr int S_A = 4;
 constexpr int DQ_GROUPS = 2;  // dequant warp-groups on alternating groups of k
+// ring depths S_A and S_W are multiples of DQ_GROUPS so that every slot belongs to one group
+// (consumed in order): an mbarrier parity wait can never run two phases ahead of its slot
 constexpr int X_STAGE_BYTES = BT * XK * 2;  // 32 KB
 constexpr int TMEM_COLS = 512;
 constexpr int D_COL = 0;
@@ -74,6 +76,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
            const __grid_constant__ CUtensorMap tm_m, const GemmP p) {
   using SM = Smem<BITS>;
   constexpr int S_W = GCfg<BITS>::S_W;
+  static_assert(S_W % DQ_GROUPS == 0 && S_A % DQ_GROUPS == 0, "slots must not be shared by dequant groups");
   constexpr int GB = GCfg<BITS>::GB;
   constexpr uint32_t W_BYTES = BN * GB;
   extern __shared__ uint8_t smem_raw[];

@@ -35,28 +35,37 @@ using namespace tc;
 constexpr int BN = 128;     // weight rows per unit (TMEM lanes, MMA M)
 constexpr int BT = 32;      // token columns (MMA N)
 constexpr int XK = 64;
-constexpr int X_STAGE = BT * XK * 2;  // 4 KB
-constexpr int S_X = 16;               // 8 units of activation lookahead
-constexpr int S_A = 3;
+constexpr int X_BLOCK = BT * XK * 2;  // 4 KB: [32 tokens][64 k] SW128 tile
 constexpr int DQ_GROUPS = 2;          // dequant warp-groups working on alternating units
-constexpr int TMEM_COLS = 256;        // 2 CTAs may share an SM without blocking each other's alloc
+// Ring depths are multiples of DQ_GROUPS: unit i uses W slot i % S_W and A slot i % S_A, so
+// every slot belongs to ONE group, which consumes its units in order -- an mbarrier parity
+// wait can then never be two phases ahead of the slot it waits on.
+constexpr int TMEM_COLS = 512;
 constexpr int D_COL = 0;              // 2 x 32 columns (double-buffered accumulator)
-constexpr int A_COL = 64;             // S_A x 64 columns
+constexpr int A_COL = 64;             // S_A x (64 * UG) columns
 constexpr int NUM_THREADS = 32 * (2 + 4 * DQ_GROUPS + 4);  // producer, MMA, dequant groups, epilogue
 constexpr uint32_t kIdescTc = make_idesc(BN, BT);
 
-template <int BITS>
-struct DCfg { static constexpr int S_W = BITS == 16 ? 3 : (BITS == 8 ? 6 : 10); };
+// UG = 128-k groups per unit (2 when k/128 is even: one TMA box each for codes, meta and
+// activations per 256 k, halving the per-byte issue overhead of the single producer thread)
+template <int BITS, int UG>
+struct DCfg {
+  static constexpr int S_W = BITS == 16 ? 4 : (BITS == 8 ? 4 : (UG == 2 ? 6 : 10));
+  static constexpr int S_A = UG == 2 ? 2 : 4;  // TMEM A slots of 64*UG columns
+  static constexpr int S_X = UG == 2 ? 4 : 8;  // activation ring, in units
+};
 
-template <int BITS>
+template <int BITS, int UG>
 struct DSmem {
-  static constexpr int S_W = DCfg<BITS>::S_W;
-  static constexpr int W_STAGE = ((BN * GCfg<BITS>::GB + 1023) / 1024) * 1024;
+  static constexpr int S_W = DCfg<BITS, UG>::S_W;
+  static constexpr int S_X = DCfg<BITS, UG>::S_X;
+  static constexpr int X_STAGE = 2 * UG * X_BLOCK;
+  static constexpr int W_STAGE = ((BN * GCfg<BITS>::GB * UG + 1023) / 1024) * 1024;
   static constexpr int OFF_X = 0;
   static constexpr int OFF_W = OFF_X + S_X * X_STAGE;
   static constexpr int OFF_META = OFF_W + S_W * W_STAGE;
-  static constexpr int OFF_BAR = OFF_META + S_W * BN * 4;
-  static constexpr int NUM_BARS = 2 * S_X + 2 * S_W + 2 * S_A + 4;
+  static constexpr int OFF_BAR = OFF_META + S_W * BN * 4 * UG;
+  static constexpr int NUM_BARS = 2 * S_X + 2 * S_W + 2 * DCfg<BITS, UG>::S_A + 4;
   static constexpr int OFF_MISC = OFF_BAR + NUM_BARS * 8;
   static constexpr int BYTES = OFF_MISC + 64 + 1024;
 };
@@ -70,7 +79,7 @@ struct TcP {
   int m;
   int n;
   int kg;
-  int U;      // units = (n / 128) * kg
+  int U;      // units = (n / 128) * (kg / UG)
   float* part;  // [CTAs][2][32 tokens][128 rows]
   int* cnt;     // [n / 128]
   unsigned long long* trace;  // debug: CTA 0 per-unit clock64 events (sq_debug_trace), or null
@@ -98,14 +107,18 @@ __device__ __forceinline__ void epi_store(const TcP& p, int64_t row, const float
   }
 }
 
-template <int BITS, int EPI>
+template <int BITS, int UG, int EPI>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
     k_gemv_tc(const __grid_constant__ CUtensorMap tm_x, const __grid_constant__ CUtensorMap tm_w,
               const __grid_constant__ CUtensorMap tm_m, const TcP p) {
-  using SM = DSmem<BITS>;
+  using SM = DSmem<BITS, UG>;
   constexpr int S_W = SM::S_W;
+  constexpr int S_A = DCfg<BITS, UG>::S_A;
+  static_assert(S_W % DQ_GROUPS == 0 && S_A % DQ_GROUPS == 0, "slots must not be shared by dequant groups");
+  constexpr int S_X = SM::S_X;
+  constexpr int X_STAGE = SM::X_STAGE;
   constexpr int GB = GCfg<BITS>::GB;
-  constexpr uint32_t W_BYTES = BN * GB;
+  constexpr uint32_t W_BYTES = BN * GB * UG;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + SM::OFF_BAR);
@@ -120,7 +133,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   uint32_t* misc = reinterpret_cast<uint32_t*>(smem + SM::OFF_MISC);  // [0] tmem base, [1..2] fixup flags
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int kg = p.kg;
+  const int kg = p.kg / UG;  // units per row tile
   const int C0 = rlo(blockIdx.x, p.U, gridDim.x), C1 = rlo(blockIdx.x + 1, p.U, gridDim.x);
   const int nunits = C1 - C0;
 
@@ -144,27 +157,29 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     // ---------------- producer: weights (+meta) and the activation slice of every unit
     {  // whole warp runs the loop (warp-uniform operands live in uniform registers); a leader issues
       for (int i = 0; i < nunits; ++i) {
-        const int u = C0 + i, rt = u / kg, g = u - rt * kg;
+        const int u = C0 + i, rt = u / kg, g = (u - rt * kg) * UG;  // first 128-k group of the unit
         const int sw = i % S_W, rw = i / S_W;
         mbar_wait(&empty_w[sw], (rw & 1) ^ 1);
         trace_ev(p, 0, i);
         uint8_t* wdst = smem + SM::OFF_W + sw * SM::W_STAGE;
-        if (elect_one()) mbar_arrive_expect_tx(&full_w[sw], W_BYTES + (BITS != 16 ? BN * 4 : 0));
+        if (elect_one()) mbar_arrive_expect_tx(&full_w[sw], W_BYTES + (BITS != 16 ? BN * 4 * UG : 0));
         if constexpr (BITS == 16) {
           if (elect_one()) tma_load_2d(wdst, &tm_w, &full_w[sw], g * 128, rt * BN);
           if (elect_one()) tma_load_2d(wdst + BN * 128, &tm_w, &full_w[sw], g * 128 + 64, rt * BN);
         } else {
+          // placement T16: box {GB bytes, 16 rows, UG groups, 8 row tiles} -> [tile][group][16][GB]
           if (elect_one()) tma_load_4d(wdst, &tm_w, &full_w[sw], 0, 0, g, rt * (BN / 16));
           trace_ev(p, 6, i);
-          if (elect_one()) tma_load_3d(smem + SM::OFF_META + sw * BN * 4, &tm_m, &full_w[sw], 0, g, rt * (BN / 16));
+          if (elect_one()) tma_load_3d(smem + SM::OFF_META + sw * BN * 4 * UG, &tm_m, &full_w[sw], 0, g, rt * (BN / 16));
           trace_ev(p, 7, i);
         }
-        for (int h = 0; h < 2; ++h) {
-          const int it = 2 * i + h, sx = it % S_X, rx = it / S_X;
+        {
+          const int sx = i % S_X, rx = i / S_X;
           mbar_wait(&empty_x[sx], (rx & 1) ^ 1);
           if (elect_one()) mbar_arrive_expect_tx(&full_x[sx], X_STAGE);
-          if (elect_one()) tma_load_2d(smem + SM::OFF_X + sx * X_STAGE, &tm_x, &full_x[sx], g * 128 + h * XK, 0);
-          trace_ev(p, 8 + h, i);
+          // activations: box {64 k, 32 tokens, 2*UG k-blocks} -> 2*UG SW128 tiles [32][64]
+          if (elect_one()) tma_load_3d(smem + SM::OFF_X + sx * X_STAGE, &tm_x, &full_x[sx], 0, 0, g * 2);
+          trace_ev(p, 8, i);
         }
       }
     }
@@ -185,19 +200,19 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         mbar_wait(&full_a[sa], ra & 1);
         trace_ev(p, 3, i);
         tc_fence_after();
-        for (int h = 0; h < 2; ++h) {
-          const int it = 2 * i + h, sx = it % S_X, rx = it / S_X;
+        {
+          const int sx = i % S_X, rx = i / S_X;
           mbar_wait(&full_x[sx], rx & 1);
-          trace_ev(p, 10 + 2 * h, i);
+          trace_ev(p, 10, i);
           tc_fence_after();
           const uint32_t xs = smem_u32(smem + SM::OFF_X + sx * X_STAGE);
 #pragma unroll
-          for (int kk = 0; kk < XK / 16; ++kk) {
-            const uint64_t bdesc = make_sw128_desc(xs + kk * 32);
-            const uint32_t a_tm = tmem + A_COL + sa * 64 + h * 32 + kk * 8;
-            if (elect_one()) tc_mma_ts(tmem + D_COL + dbuf * BT, a_tm, bdesc, kIdescTc, (seg_first && h == 0 && kk == 0) ? 0u : 1u);
+          for (int kk = 0; kk < 8 * UG; ++kk) {
+            const uint64_t bdesc = make_sw128_desc(xs + (kk >> 2) * X_BLOCK + (kk & 3) * 32);
+            const uint32_t a_tm = tmem + A_COL + sa * 64 * UG + kk * 8;
+            if (elect_one()) tc_mma_ts(tmem + D_COL + dbuf * BT, a_tm, bdesc, kIdescTc, (seg_first && kk == 0) ? 0u : 1u);
           }
-          trace_ev(p, 11 + 2 * h, i);
+          trace_ev(p, 11, i);
           if (elect_one()) tc_commit(&empty_x[sx]);
         }
         if (elect_one()) tc_commit(&empty_a[sa]);
@@ -222,8 +237,14 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       mbar_wait(&empty_a[sa], (ra & 1) ^ 1);
       if (threadIdx.x == 64) trace_ev(p, 5, i);
       tc_fence_after();
-      const uint32_t meta = reinterpret_cast<const uint32_t*>(smem + SM::OFF_META + sw * BN * 4)[r];
-      dequant_row_to_tmem<BITS>(smem + SM::OFF_W + sw * SM::W_STAGE, meta, r, tmem + lane_base + A_COL + sa * 64);
+#pragma unroll
+      for (int gg = 0; gg < UG; ++gg) {
+        // stage layout [tile][group][16 rows]: row r of group gg
+        const int ru = ((r >> 4) * UG + gg) * 16 + (r & 15);
+        const uint32_t meta = reinterpret_cast<const uint32_t*>(smem + SM::OFF_META + sw * BN * 4 * UG)[ru];
+        dequant_row_to_tmem<BITS>(smem + SM::OFF_W + sw * SM::W_STAGE, meta, r,
+                                  tmem + lane_base + A_COL + sa * 64 * UG + gg * 64, ru * GB);
+      }
       tc_wait_st();
       tc_fence_before();
       __syncwarp();
@@ -333,29 +354,38 @@ cudaError_t enc(CUtensorMap* m, CUtensorMapDataType dt, const void* ptr, int ran
   return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
 }
 
-template <int BITS, int EPI>
+template <int BITS, int UG, int EPI>
 cudaError_t launch_tc_be(const CUtensorMap& tx, const CUtensorMap& tw, const CUtensorMap& tm, const TcP& p, int nc,
                          cudaStream_t s) {
-  auto kern = k_gemv_tc<BITS, EPI>;
+  auto kern = k_gemv_tc<BITS, UG, EPI>;
   static bool attr = false;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, DSmem<BITS>::BYTES);
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, DSmem<BITS, UG>::BYTES);
     if (e != cudaSuccess) return e;
     attr = true;
   }
-  kern<<<nc, NUM_THREADS, DSmem<BITS>::BYTES, s>>>(tx, tw, tm, p);
+  kern<<<nc, NUM_THREADS, DSmem<BITS, UG>::BYTES, s>>>(tx, tw, tm, p);
   return cudaGetLastError();
+}
+
+template <int BITS, int UG>
+cudaError_t launch_tc_u(const CUtensorMap& tx, const CUtensorMap& tw, const CUtensorMap& tm, const TcP& p, int epi,
+                        int nc, cudaStream_t s) {
+  switch (epi) {
+    case SQ_EPI_F16: return launch_tc_be<BITS, UG, SQ_EPI_F16>(tx, tw, tm, p, nc, s);
+    case SQ_EPI_F16_RELU: return launch_tc_be<BITS, UG, SQ_EPI_F16_RELU>(tx, tw, tm, p, nc, s);
+    case SQ_EPI_F16_GELU: return launch_tc_be<BITS, UG, SQ_EPI_F16_GELU>(tx, tw, tm, p, nc, s);
+    default: return launch_tc_be<BITS, UG, SQ_EPI_F32_ACCUM>(tx, tw, tm, p, nc, s);
+  }
 }
 
 template <int BITS>
 cudaError_t launch_tc_b(const CUtensorMap& tx, const CUtensorMap& tw, const CUtensorMap& tm, const TcP& p, int epi,
-                        int nc, cudaStream_t s) {
-  switch (epi) {
-    case SQ_EPI_F16: return launch_tc_be<BITS, SQ_EPI_F16>(tx, tw, tm, p, nc, s);
-    case SQ_EPI_F16_RELU: return launch_tc_be<BITS, SQ_EPI_F16_RELU>(tx, tw, tm, p, nc, s);
-    case SQ_EPI_F16_GELU: return launch_tc_be<BITS, SQ_EPI_F16_GELU>(tx, tw, tm, p, nc, s);
-    default: return launch_tc_be<BITS, SQ_EPI_F32_ACCUM>(tx, tw, tm, p, nc, s);
+                        int nc, int ug, cudaStream_t s) {
+  if constexpr (BITS != 16) {
+    if (ug == 2) return launch_tc_u<BITS, 2>(tx, tw, tm, p, epi, nc, s);
   }
+  return launch_tc_u<BITS, 1>(tx, tw, tm, p, epi, nc, s);
 }
 
 unsigned long long* g_trace = nullptr;
@@ -380,10 +410,13 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
                            void* ws, cudaStream_t s) {
   CUtensorMap tx, tw, tm;
   memset(&tm, 0, sizeof(tm));
+  const int kg = (int)(w.k / 128);
+  const int ug = (w.bits != 16 && kg % 2 == 0) ? 2 : 1;
   {
-    const uint64_t dx[2] = {(uint64_t)w.k, (uint64_t)m}, sx[1] = {(uint64_t)ldx * 2};
-    const uint32_t bx[2] = {XK, BT};
-    cudaError_t e = enc(&tx, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, x, 2, dx, sx, bx, CU_TENSOR_MAP_SWIZZLE_128B);
+    // activations as [k/64][m][64]: one box {64, 32, 2*ug} per unit -> 2*ug SW128 tiles [32 tokens][64 k]
+    const uint64_t dx[3] = {64, (uint64_t)m, (uint64_t)w.k / 64}, sx[2] = {(uint64_t)ldx * 2, 128};
+    const uint32_t bx[3] = {XK, BT, (uint32_t)(2 * ug)};
+    cudaError_t e = enc(&tx, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, x, 3, dx, sx, bx, CU_TENSOR_MAP_SWIZZLE_128B);
     if (e != cudaSuccess) return e;
   }
   if (w.bits == 16) {
@@ -392,15 +425,15 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
     cudaError_t e = enc(&tw, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, w.packed, 2, dw, sw_, bw, CU_TENSOR_MAP_SWIZZLE_128B);
     if (e != cudaSuccess) return e;
   } else {
-    const uint64_t gb = 128 * w.bits / 8, kg = (uint64_t)w.k / 128, nt = (uint64_t)w.n / 16;
+    const uint64_t gb = 128 * w.bits / 8, nt = (uint64_t)w.n / 16;
     CUtensorMapSwizzle sw = w.bits == 8 ? CU_TENSOR_MAP_SWIZZLE_128B
                                         : (w.bits == 4 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_NONE);
     const uint64_t dw[4] = {gb, 16, kg, nt}, sw_[3] = {gb, 16 * gb, kg * 16 * gb};
-    const uint32_t bw[4] = {(uint32_t)gb, 16, 1, BN / 16};
+    const uint32_t bw[4] = {(uint32_t)gb, 16, (uint32_t)ug, BN / 16};
     cudaError_t e = enc(&tw, CU_TENSOR_MAP_DATA_TYPE_UINT8, w.packed, 4, dw, sw_, bw, sw);
     if (e != cudaSuccess) return e;
     const uint64_t dm[3] = {16, kg, nt}, sm_[2] = {64, kg * 64};
-    const uint32_t bm[3] = {16, 1, BN / 16};
+    const uint32_t bm[3] = {16, (uint32_t)ug, BN / 16};
     e = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, w.meta, 3, dm, sm_, bm, CU_TENSOR_MAP_SWIZZLE_NONE);
     if (e != cudaSuccess) return e;
   }
@@ -412,8 +445,8 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
   p.ldy = (int)ldy;
   p.m = m;
   p.n = (int)w.n;
-  p.kg = (int)(w.k / 128);
-  p.U = (int)((w.n / BN) * p.kg);
+  p.kg = kg;
+  p.U = (int)((w.n / BN) * (kg / ug));
   uint8_t* base = static_cast<uint8_t*>(ws);
   p.cnt = reinterpret_cast<int*>(base);
   p.part = reinterpret_cast<float*>(base + kCntBytes);
@@ -423,10 +456,10 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
   auto t = prof_begin(KC_GEMV, bytes, 2.0 * m * w.n * w.k, s);
   cudaError_t e;
   switch (w.bits) {
-    case 3: e = launch_tc_b<3>(tx, tw, tm, p, epi, nc, s); break;
-    case 4: e = launch_tc_b<4>(tx, tw, tm, p, epi, nc, s); break;
-    case 8: e = launch_tc_b<8>(tx, tw, tm, p, epi, nc, s); break;
-    default: e = launch_tc_b<16>(tx, tw, tm, p, epi, nc, s); break;
+    case 3: e = launch_tc_b<3>(tx, tw, tm, p, epi, nc, ug, s); break;
+    case 4: e = launch_tc_b<4>(tx, tw, tm, p, epi, nc, ug, s); break;
+    case 8: e = launch_tc_b<8>(tx, tw, tm, p, epi, nc, ug, s); break;
+    default: e = launch_tc_b<16>(tx, tw, tm, p, epi, nc, 1, s); break;
   }
   prof_end(t, s);
   count_launch();

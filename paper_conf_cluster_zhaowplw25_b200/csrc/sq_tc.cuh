@@ -20,7 +20,7 @@ struct GCfg<3> { static constexpr int GB = 48; static constexpr int S_W = 4; };
 template <>
 struct GCfg<4> { static constexpr int GB = 64; static constexpr int S_W = 4; };
 template <>
-struct GCfg<8> { static constexpr int GB = 128; static constexpr int S_W = 3; };
+struct GCfg<8> { static constexpr int GB = 128; static constexpr int S_W = 4; };
 template <>
 struct GCfg<16> { static constexpr int GB = 256; static constexpr int S_W = 2; };
 
@@ -48,12 +48,15 @@ __device__ __forceinline__ uint32_t hsub_fma(uint32_t h, uint32_t off2, uint32_t
 // Dequantize this thread's row (r) of one 128-k group into 64 half2 columns,
 // written to TMEM in 4 batches of 16 columns.
 template <int BITS>
-__device__ __forceinline__ void dequant_row_to_tmem(const uint8_t* wst, uint32_t meta, int r, uint32_t taddr) {
+// `row_off` = byte offset of this thread's row inside the stage (default r * GB); the swizzle
+// pattern only depends on r % 16 because every T16 unit starts on a 1-KB boundary.
+__device__ __forceinline__ void dequant_row_to_tmem(const uint8_t* wst, uint32_t meta, int r, uint32_t taddr,
+                                                    int row_off = -1) {
   const uint32_t s2 = (meta & 0xFFFFu) * 0x10001u;
   const uint32_t z2 = (meta >> 16) * 0x10001u;
   constexpr uint32_t K1024 = 0x64006400u, K64 = 0x54005400u;
   if constexpr (BITS == 4) {
-    const uint8_t* row = wst + r * 64;
+    const uint8_t* row = wst + (row_off >= 0 ? row_off : r * 64);
 #pragma unroll
     for (int b = 0; b < 4; ++b) {
       const int pc = b ^ ((r >> 1) & 3);  // SWIZZLE_64B
@@ -71,7 +74,7 @@ __device__ __forceinline__ void dequant_row_to_tmem(const uint8_t* wst, uint32_t
       tmem_st16(taddr + 16 * b, o);
     }
   } else if constexpr (BITS == 8) {
-    const uint8_t* row = wst + r * 128;
+    const uint8_t* row = wst + (row_off >= 0 ? row_off : r * 128);
 #pragma unroll
     for (int b = 0; b < 4; ++b) {
       uint32_t o[16];
@@ -89,7 +92,7 @@ __device__ __forceinline__ void dequant_row_to_tmem(const uint8_t* wst, uint32_t
       tmem_st16(taddr + 16 * b, o);
     }
   } else if constexpr (BITS == 3) {
-    const uint32_t* row = reinterpret_cast<const uint32_t*>(wst + r * 48);
+    const uint32_t* row = reinterpret_cast<const uint32_t*>(wst + (row_off >= 0 ? row_off : r * 48));
 #pragma unroll
     for (int bl = 0; bl < 4; ++bl) {
       const uint32_t L0 = row[3 * bl], L1 = row[3 * bl + 1], H = row[3 * bl + 2];
