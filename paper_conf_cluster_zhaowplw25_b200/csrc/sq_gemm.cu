@@ -80,7 +80,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   constexpr int GB = GCfg<BITS>::GB;
   constexpr uint32_t W_BYTES = BN * GB;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1-KB aligned (SW128 atoms); pointer arithmetic on smem_raw keeps the shared address space
+  // visible to the compiler (LDS, not generic LD)
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + SM::OFF_BAR);
   uint64_t* full_x = bars;
   uint64_t* empty_x = full_x + S_X;

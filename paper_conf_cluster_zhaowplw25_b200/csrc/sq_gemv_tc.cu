@@ -1,27 +1,33 @@
 // K2c — decode dequant-GEMV on tcgen05 for micro-batches of up to 32 tokens
 // (the pipeline's decode micro-batch xi = 32).  At 32 tokens a
 // decode linear does 64 flop per weight; legacy mma.sync tops out near
-// 535 TFLOP/s on B200 (measured), i.e. ~67 % of HBM speed at INT4, so the
-// contraction moves to the 5th-generation tensor cores:
+// 535 TFLOP/s on B200 (measured), below HBM speed at INT4, so the contraction
+// moves to the 5th-generation tensor cores:
 //
-//  * Work unit = 128 weight rows x one group (128 k).  Units are flattened
-//    row-tile-major / group-minor (placement T16 makes a unit 8 consecutive
-//    16-row units) and split evenly over one CTA per SM (stream-K): every SM
-//    streams the same number of bytes whatever the shape.
-//  * Producer warp: TMA 4-D box of packed codes + 3-D box of meta per unit,
-//    and the unit's activation slice [32 tokens x 128 k] (2 x SW128 boxes;
-//    tokens >= m are zero-filled by TMA).  6-deep weight ring.
-//  * 4 dequant warps (one thread per weight row): magic-number unpack,
-//    w~ = s*c + z in fp16 (HSUB2 + HFMA2), tcgen05.st into a TMEM A slot.
-//  * MMA thread: tcgen05.mma kind::f16, M = 128 rows, N = 32 tokens, K = 16,
-//    A from TMEM, B (activations) from SMEM; fp32 accumulator in TMEM,
-//    double-buffered per row-tile segment.
-//  * 4 epilogue warps: drain each finished segment; a tile fully inside the
-//    CTA is written directly (bias / activation / fp32 residual), a tile split
-//    across CTAs goes through a workspace and is finished by the last CTA in
-//    fixed CTA order (deterministic, counters self-reset).
-// Warp roles: 0 producer, 1 MMA (+TMEM alloc), 2..9 dequant (2 groups of 4, alternating
-// units so one group's tcgen05.st latency overlaps the other's unpack), 10..13 epilogue.
+//  * Unit = 128 weight rows x UG groups (UG*128 k): one MMA M-tile.  Units are
+//    grouped in PANELS of P <= 4 row tiles that share every activation slice
+//    [32 tokens x UG*128 k] (fetched once per P units): a TMA stream ingests
+//    ~45 GB/s per SM whether it hits L2 or HBM (measured, tools/mb_tma.cu), so
+//    activation bytes cost as much as weight bytes.
+//  * Work item = (panel, k-slice z < Z): the panel's k range is split in Z even
+//    slices.  (P, Z) are chosen per shape on the host to minimise the bytes the
+//    busiest SM ingests (weights + activations + partial sums) with about one
+//    item per SM (tc_plan).
+//  * Producer warp: per unit one 4-D TMA box of packed codes and one 3-D box of
+//    meta; per k-step one 3-D box of activations (tokens >= m zero-filled),
+//    issued one step behind the weights (it is only needed at MMA time).
+//  * 16 dequant warps (thread = weight row, warp = a quarter of the unit's k):
+//    magic-number unpack, w~ = s*c + z in fp16 (HSUB2 + HFMA2), tcgen05.st into
+//    TMEM A slot i % 3 while the MMA reads the others.
+//  * MMA warp: tcgen05.mma kind::f16, M = 128 rows, N = 32 tokens, K = 16, A
+//    from TMEM, B (activations) from SMEM; fp32 accumulators of the panel's P
+//    tiles in TMEM (P x 32 columns).
+//  * 4 epilogue warps drain an item: Z = 1 -> bias / activation / fp32 residual
+//    straight to y; Z > 1 -> fp32 partial to the workspace, and the last of the
+//    Z items to arrive (atomic counter) sums all Z partials of the panel in fixed
+//    z order at the end of its CTA (bulk copies into the then idle rings; all
+//    warps).  Deterministic; counters self-reset.
+// Warp roles: 0 producer, 1 MMA (+TMEM alloc), 2..17 dequant, 18..21 epilogue.
 #include <cuda.h>
 
 #include <cstring>
@@ -34,25 +40,28 @@ using namespace tc;
 
 constexpr int BN = 128;     // weight rows per unit (TMEM lanes, MMA M)
 constexpr int BT = 32;      // token columns (MMA N)
+constexpr int PMAX = 4;     // row tiles per panel (activation reuse), at most
 constexpr int XK = 64;
 constexpr int X_BLOCK = BT * XK * 2;  // 4 KB: [32 tokens][64 k] SW128 tile
-constexpr int DQ_GROUPS = 2;          // dequant warp-groups working on alternating units
-// Ring depths are multiples of DQ_GROUPS: unit i uses W slot i % S_W and A slot i % S_A, so
-// every slot belongs to ONE group, which consumes its units in order -- an mbarrier parity
-// wait can then never be two phases ahead of the slot it waits on.
+constexpr int DQ_WARPS = 8;           // dequant warps: 2 per TMEM lane quadrant, each half of the unit's k
 constexpr int TMEM_COLS = 512;
-constexpr int D_COL = 0;              // 2 x 32 columns (double-buffered accumulator)
-constexpr int A_COL = 64;             // S_A x (64 * UG) columns
-constexpr int NUM_THREADS = 32 * (2 + 4 * DQ_GROUPS + 4);  // producer, MMA, dequant groups, epilogue
+constexpr int D_COL = 0;              // P x 32 columns: the panel's accumulators
+constexpr int A_COL = PMAX * BT;      // S_A x (64 * UG) columns
+constexpr int NUM_THREADS = 32 * (2 + DQ_WARPS + 4);  // producer, MMA, dequant, epilogue
+constexpr int EPI_WARP0 = 2 + DQ_WARPS;
 constexpr uint32_t kIdescTc = make_idesc(BN, BT);
+constexpr int X_LAG = 1;              // activations of step q are fetched after the weights of step q + 1
 
-// UG = 128-k groups per unit (2 when k/128 is even: one TMA box each for codes, meta and
-// activations per 256 k, halving the per-byte issue overhead of the single producer thread)
+// UG = 128-k groups per unit, chosen so a weight stage is ~16 KB (INT3/INT4: 2, INT8: 1).
 template <int BITS, int UG>
 struct DCfg {
-  static constexpr int S_W = BITS == 16 ? 4 : (BITS == 8 ? 4 : (UG == 2 ? 6 : 10));
-  static constexpr int S_A = UG == 2 ? 2 : 4;  // TMEM A slots of 64*UG columns
-  static constexpr int S_X = UG == 2 ? 4 : 8;  // activation ring, in units
+  // weight ring: a slot lives TMA latency (~1.8k cycles) + wait for its group + dequant (~2k)
+  static constexpr int S_W = UG == 2 ? 9 : (BITS == 8 ? 9 : (BITS == 4 ? 18 : 24));
+  // TMEM A slots of 64*UG columns: the dequant warps fill slot i % S_A while the MMA reads the
+  // others (128 + 3 * 128 = 512 columns at UG = 2)
+  static constexpr int S_A = UG == 2 ? 3 : 6;
+  static constexpr int S_X = 3;  // activation ring, in steps
+  static_assert(A_COL + S_A * 64 * UG <= TMEM_COLS, "TMEM budget");
 };
 
 template <int BITS, int UG>
@@ -65,9 +74,11 @@ struct DSmem {
   static constexpr int OFF_W = OFF_X + S_X * X_STAGE;
   static constexpr int OFF_META = OFF_W + S_W * W_STAGE;
   static constexpr int OFF_BAR = OFF_META + S_W * BN * 4 * UG;
-  static constexpr int NUM_BARS = 2 * S_X + 2 * S_W + 2 * DCfg<BITS, UG>::S_A + 4;
+  static constexpr int NUM_BARS = 2 * S_X + 2 * S_W + 2 * DCfg<BITS, UG>::S_A + 2 + PMAX;
   static constexpr int OFF_MISC = OFF_BAR + NUM_BARS * 8;
-  static constexpr int BYTES = OFF_MISC + 64 + 1024;
+  static constexpr int BYTES = OFF_MISC + 256 + 1024;  // misc: tmem base, pending panels (<= 62)
+  static_assert(BYTES <= 227 * 1024, "shared memory budget");
+  static constexpr int ZMAX = OFF_BAR / (BT * BN * 4) < 8 ? OFF_BAR / (BT * BN * 4) : 8;  // partial tiles staged
 };
 
 struct TcP {
@@ -79,14 +90,26 @@ struct TcP {
   int m;
   int n;
   int kg;
-  int U;      // units = (n / 128) * (kg / UG)
-  float* part;  // [CTAs][2][32 tokens][128 rows]
-  int* cnt;     // [n / 128]
+  int nt;     // row tiles (n / 128)
+  int ks;     // k-steps per row (kg / UG)
+  int P;      // row tiles per panel (1..4)
+  int Z;      // k slices per panel
+  int I;      // work items = panels * Z
+  float* part;  // [items][PMAX tiles][32 tokens][128 rows] fp32 partial sums (Z > 1)
+  int* cnt;     // [panels]
   unsigned long long* trace;  // debug: CTA 0 per-unit clock64 events (sq_debug_trace), or null
 };
 
 __device__ __forceinline__ void trace_ev(const TcP& p, int ev, int i) {
   if (p.trace && blockIdx.x == 0 && i < 256) p.trace[ev * 256 + i] = clock64();
+}
+
+__device__ __forceinline__ void trace_cta(const TcP& p, int ev) {
+  if (p.trace && blockIdx.x < 256) {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    p.trace[ev * 256 + blockIdx.x] = t;
+  }
 }
 
 __device__ __forceinline__ int rlo(int i, int total, int parts) { return (int)(((long long)i * total) / parts); }
@@ -114,13 +137,14 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   using SM = DSmem<BITS, UG>;
   constexpr int S_W = SM::S_W;
   constexpr int S_A = DCfg<BITS, UG>::S_A;
-  static_assert(S_W % DQ_GROUPS == 0 && S_A % DQ_GROUPS == 0, "slots must not be shared by dequant groups");
   constexpr int S_X = SM::S_X;
   constexpr int X_STAGE = SM::X_STAGE;
   constexpr int GB = GCfg<BITS>::GB;
-  constexpr uint32_t W_BYTES = BN * GB * UG;
+  constexpr uint32_t W_BYTES = BN * GB * UG + BN * 4 * UG;  // codes + meta of one unit
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1-KB aligned (SW128 atoms); pointer arithmetic on smem_raw keeps the shared address space
+  // visible to the compiler (LDS, not generic LD)
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + SM::OFF_BAR);
   uint64_t* full_x = bars;
   uint64_t* empty_x = full_x + S_X;
@@ -128,123 +152,136 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   uint64_t* empty_w = full_w + S_W;
   uint64_t* full_a = empty_w + S_W;
   uint64_t* empty_a = full_a + S_A;
-  uint64_t* d_full = empty_a + S_A;   // [2]
-  uint64_t* d_empty = d_full + 2;     // [2]
-  uint32_t* misc = reinterpret_cast<uint32_t*>(smem + SM::OFF_MISC);  // [0] tmem base, [1..2] fixup flags
+  uint64_t* d_full = empty_a + S_A;
+  uint64_t* d_empty = d_full + 1;
+  uint64_t* red_bar = d_empty + 1;  // [PMAX]
+  uint32_t* misc = reinterpret_cast<uint32_t*>(smem + SM::OFF_MISC);  // [0] tmem base, [1] #pending, [2..] panels
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int kg = p.kg / UG;  // units per row tile
-  const int C0 = rlo(blockIdx.x, p.U, gridDim.x), C1 = rlo(blockIdx.x + 1, p.U, gridDim.x);
-  const int nunits = C1 - C0;
+  const int ks = p.ks, C = gridDim.x, P = p.P, Z = p.Z, I = p.I;
+  const int last_panel = (p.nt - 1) / P, p_last = p.nt - last_panel * P;  // tiles in the last panel
+  auto tiles_of = [&](int pn) { return pn == last_panel ? p_last : P; };
+  // item it = (panel it / Z, k-steps [j0, j1) of slice it % Z)
+  auto j0_of = [&](int it) { return (int)((long long)(it % Z) * ks / Z); };
+  auto j1_of = [&](int it) { return (int)((long long)(it % Z + 1) * ks / Z); };
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < S_X; ++i) { mbar_init(&full_x[i], 1); mbar_init(&empty_x[i], 1); }
-    for (int i = 0; i < S_W; ++i) { mbar_init(&full_w[i], 1); mbar_init(&empty_w[i], 4); }
-    for (int i = 0; i < S_A; ++i) { mbar_init(&full_a[i], 4); mbar_init(&empty_a[i], 1); }
-    for (int i = 0; i < 2; ++i) { mbar_init(&d_full[i], 1); mbar_init(&d_empty[i], 4); }
+    for (int i = 0; i < S_W; ++i) { mbar_init(&full_w[i], 1); mbar_init(&empty_w[i], DQ_WARPS); }
+    for (int i = 0; i < S_A; ++i) { mbar_init(&full_a[i], DQ_WARPS); mbar_init(&empty_a[i], 1); }
+    mbar_init(d_full, 1);
+    mbar_init(d_empty, 4);
+    for (int i = 0; i < PMAX; ++i) mbar_init(&red_bar[i], 1);
+    misc[1] = 0;
     fence_barrier_init();
     prefetch_tmap(&tm_x);
     prefetch_tmap(&tm_w);
-    if constexpr (BITS != 16) prefetch_tmap(&tm_m);
+    prefetch_tmap(&tm_m);
   }
   if (warp == 1) tmem_alloc(misc, TMEM_COLS);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
-  const uint32_t tmem = misc[0];
+  if (misc[0] != 0) __trap();  // a 512-column allocation owns all of TMEM: base is lane 0, column 0
+  constexpr uint32_t tmem = 0;
+  if (threadIdx.x == 0) trace_cta(p, 14);
 
   if (warp == 0) {
-    // ---------------- producer: weights (+meta) and the activation slice of every unit
-    {  // whole warp runs the loop (warp-uniform operands live in uniform registers); a leader issues
-      for (int i = 0; i < nunits; ++i) {
-        const int u = C0 + i, rt = u / kg, g = (u - rt * kg) * UG;  // first 128-k group of the unit
-        const int sw = i % S_W, rw = i / S_W;
-        mbar_wait(&empty_w[sw], (rw & 1) ^ 1);
-        trace_ev(p, 0, i);
-        uint8_t* wdst = smem + SM::OFF_W + sw * SM::W_STAGE;
-        if (elect_one()) mbar_arrive_expect_tx(&full_w[sw], W_BYTES + (BITS != 16 ? BN * 4 * UG : 0));
-        if constexpr (BITS == 16) {
-          if (elect_one()) tma_load_2d(wdst, &tm_w, &full_w[sw], g * 128, rt * BN);
-          if (elect_one()) tma_load_2d(wdst + BN * 128, &tm_w, &full_w[sw], g * 128 + 64, rt * BN);
-        } else {
-          // placement T16: box {GB bytes, 16 rows, UG groups, 8 row tiles} -> [tile][group][16][GB]
-          if (elect_one()) tma_load_4d(wdst, &tm_w, &full_w[sw], 0, 0, g, rt * (BN / 16));
-          trace_ev(p, 6, i);
-          if (elect_one()) tma_load_3d(smem + SM::OFF_META + sw * BN * 4 * UG, &tm_m, &full_w[sw], 0, g, rt * (BN / 16));
-          trace_ev(p, 7, i);
-        }
-        {
-          const int sx = i % S_X, rx = i / S_X;
-          mbar_wait(&empty_x[sx], (rx & 1) ^ 1);
-          if (elect_one()) mbar_arrive_expect_tx(&full_x[sx], X_STAGE);
-          // activations: box {64 k, 32 tokens, 2*UG k-blocks} -> 2*UG SW128 tiles [32][64]
-          if (elect_one()) tma_load_3d(smem + SM::OFF_X + sx * X_STAGE, &tm_x, &full_x[sx], 0, 0, g * 2);
+    // ---------------- producer.  The warp runs the loop and the waits; one elected lane issues.
+    int i = 0, q = 0, qx = 0;  // units, k-steps issued (weights), k-steps issued (activations)
+    int xj[X_LAG + 1];         // k-step of the pending activation fetches (ring of X_LAG + 1)
+    auto issue_x = [&](int j) {
+      const int sx = qx % S_X, rx = qx / S_X;
+      mbar_wait(&empty_x[sx], (rx & 1) ^ 1);
+      if (elect_one()) {
+        // box {64 k, 32 tokens, 2*UG k-blocks} -> 2*UG SW128 tiles [32][64]
+        mbar_arrive_expect_tx(&full_x[sx], X_STAGE);
+        tma_load_3d(smem + SM::OFF_X + sx * X_STAGE, &tm_x, &full_x[sx], 0, 0, j * UG * 2);
+      }
+      __syncwarp();
+      ++qx;
+    };
+    for (int it = blockIdx.x; it < I; it += C) {
+      const int pn = it / Z, j1 = j1_of(it), pp = tiles_of(pn);
+      for (int j = j0_of(it); j < j1; ++j, ++q) {
+        xj[q % (X_LAG + 1)] = j;
+        if (q >= X_LAG) issue_x(xj[(q - X_LAG) % (X_LAG + 1)]);
+        for (int t = 0; t < pp; ++t, ++i) {
+          const int sw = i % S_W, rw = i / S_W;
+          mbar_wait(&empty_w[sw], (rw & 1) ^ 1);
+          trace_ev(p, 0, i);
+          if (elect_one()) {
+            const int tile16 = (pn * P + t) * (BN / 16);
+            mbar_arrive_expect_tx(&full_w[sw], W_BYTES);
+            // placement T16: box {GB bytes, 16 rows, UG groups, 8 row tiles} -> [tile][group][16][GB]
+            tma_load_4d(smem + SM::OFF_W + sw * SM::W_STAGE, &tm_w, &full_w[sw], 0, 0, j * UG, tile16);
+            tma_load_3d(smem + SM::OFF_META + sw * BN * 4 * UG, &tm_m, &full_w[sw], 0, j * UG, tile16);
+          }
+          __syncwarp();
           trace_ev(p, 8, i);
         }
       }
     }
+    for (int r = q > X_LAG ? q - X_LAG : 0; r < q; ++r) issue_x(xj[r % (X_LAG + 1)]);
   } else if (warp == 1) {
-    // ---------------- MMA issuer
-    {  // whole warp runs the loop; the elected leader issues tcgen05.mma / commit
-      int seg = 0, dbuf = 0;
-      for (int i = 0; i < nunits; ++i) {
-        const int u = C0 + i, g = u % kg;
-        const bool seg_first = (i == 0) || g == 0;
-        const bool seg_last = (i == nunits - 1) || g == kg - 1;
-        if (seg_first) {
-          dbuf = seg & 1;
-          mbar_wait(&d_empty[dbuf], ((seg >> 1) & 1) ^ 1);
+    // ---------------- MMA issuer: the warp waits, one elected lane issues a unit's 8*UG MMAs and
+    // commits.  TMEM base is 0, so every operand is warp-uniform.
+    int i = 0, q = 0, n_item = 0;
+    for (int it = blockIdx.x; it < I; it += C, ++n_item) {
+      const int pn = it / Z, j0 = j0_of(it), j1 = j1_of(it), pp = tiles_of(pn);
+      mbar_wait(d_empty, (n_item & 1) ^ 1);  // the epilogue drained the previous item
+      for (int j = j0; j < j1; ++j, ++q) {
+        const int sx = q % S_X, rx = q / S_X;
+        mbar_wait(&full_x[sx], rx & 1);
+        const uint64_t bdesc0 = make_sw128_desc(smem_u32(smem + SM::OFF_X + sx * X_STAGE));
+        for (int t = 0; t < pp; ++t, ++i) {
+          const int sa = i % S_A, ra = i / S_A;
+          mbar_wait(&full_a[sa], ra & 1);
           tc_fence_after();
-        }
-        const int sa = i % S_A, ra = i / S_A;
-        mbar_wait(&full_a[sa], ra & 1);
-        trace_ev(p, 3, i);
-        tc_fence_after();
-        {
-          const int sx = i % S_X, rx = i / S_X;
-          mbar_wait(&full_x[sx], rx & 1);
-          trace_ev(p, 10, i);
-          tc_fence_after();
-          const uint32_t xs = smem_u32(smem + SM::OFF_X + sx * X_STAGE);
+          trace_ev(p, 3, i);
+          if (elect_one()) {
+            const uint32_t d_tm = tmem + D_COL + t * BT;
+            const uint32_t a_tm = tmem + A_COL + sa * 64 * UG;
 #pragma unroll
-          for (int kk = 0; kk < 8 * UG; ++kk) {
-            const uint64_t bdesc = make_sw128_desc(xs + (kk >> 2) * X_BLOCK + (kk & 3) * 32);
-            const uint32_t a_tm = tmem + A_COL + sa * 64 * UG + kk * 8;
-            if (elect_one()) tc_mma_ts(tmem + D_COL + dbuf * BT, a_tm, bdesc, kIdescTc, (seg_first && kk == 0) ? 0u : 1u);
+            for (int kk = 0; kk < 8 * UG; ++kk)
+              tc_mma_ts(d_tm, a_tm + kk * 8, bdesc0 + (uint64_t)(((kk >> 2) * X_BLOCK + (kk & 3) * 32) >> 4),
+                        kIdescTc, (j == j0 && kk == 0) ? 0u : 1u);
+            tc_commit(&empty_a[sa]);
+            if (t == pp - 1) {
+              tc_commit(&empty_x[sx]);
+              if (j == j1 - 1) tc_commit(d_full);
+            }
           }
-          trace_ev(p, 11, i);
-          if (elect_one()) tc_commit(&empty_x[sx]);
-        }
-        if (elect_one()) tc_commit(&empty_a[sa]);
-        trace_ev(p, 4, i);
-        if (seg_last) {
-          if (elect_one()) tc_commit(&d_full[dbuf]);
-          ++seg;
+          __syncwarp();
+          trace_ev(p, 4, i);
         }
       }
     }
-  } else if (warp < 2 + 4 * DQ_GROUPS) {
-    // ---------------- dequant warps: one thread per weight row; group gi takes units i = gi (mod 2)
+  } else if (warp < EPI_WARP0) {
+    // ---------------- dequant warps: thread = weight row (lane quadrant warp % 4); warp kh takes
+    // batches [kh*2*UG, kh*2*UG + 2*UG) of the unit's 4*UG 32-k batches.  All 8 warps work on
+    // every unit, so a unit's dequant latency is half of one warp's work.
+    int nunits = 0;
+    for (int it = blockIdx.x; it < I; it += C) nunits += (j1_of(it) - j0_of(it)) * tiles_of(it / Z);
+    constexpr int NBW = 2 * UG;                              // batches per warp
     const int sp = warp & 3;
-    const int gi = (warp - 2) >> 2;
+    const int kh = (warp - 2) >> 2;
+    const int gg = (kh * NBW) >> 2, b0 = (kh * NBW) & 3;  // group of the unit and first batch in it
     const int r = sp * 32 + lane;
+    const int ru = ((r >> 4) * UG + gg) * 16 + (r & 15);  // stage layout [tile][group][16 rows]
     const uint32_t lane_base = (uint32_t)(sp * 32) << 16;
-    for (int i = gi; i < nunits; i += DQ_GROUPS) {
-      const int sw = i % S_W, rw = i / S_W;
-      const int sa = i % S_A, ra = i / S_A;
-      mbar_wait(&full_w[sw], rw & 1);
-      if (threadIdx.x == 64) trace_ev(p, 1, i);
-      mbar_wait(&empty_a[sa], (ra & 1) ^ 1);
-      if (threadIdx.x == 64) trace_ev(p, 5, i);
+    const bool tr = (warp == 2 && lane == 0);
+    int sw = 0, pw = 0, sa = 0, pa = 0;  // ring slots and phases
+    for (int i = 0; i < nunits; ++i) {
+      mbar_wait(&full_w[sw], pw);
+      if (tr) trace_ev(p, 1, i);
+      mbar_wait(&empty_a[sa], pa ^ 1);
+      if (tr) trace_ev(p, 5, i);
       tc_fence_after();
-#pragma unroll
-      for (int gg = 0; gg < UG; ++gg) {
-        // stage layout [tile][group][16 rows]: row r of group gg
-        const int ru = ((r >> 4) * UG + gg) * 16 + (r & 15);
-        const uint32_t meta = reinterpret_cast<const uint32_t*>(smem + SM::OFF_META + sw * BN * 4 * UG)[ru];
-        dequant_row_to_tmem<BITS>(smem + SM::OFF_W + sw * SM::W_STAGE, meta, r,
-                                  tmem + lane_base + A_COL + sa * 64 * UG + gg * 64, ru * GB);
-      }
+      const uint32_t meta = reinterpret_cast<const uint32_t*>(smem + SM::OFF_META + sw * BN * 4 * UG)[ru];
+      dequant_row_batches<BITS, NBW < 4 ? NBW : 4>(smem + SM::OFF_W + sw * SM::W_STAGE, meta, r,
+                                                   tmem + lane_base + A_COL + sa * 64 * UG + gg * 64, ru * GB, b0);
+      if (tr) trace_ev(p, 12, i);
       tc_wait_st();
       tc_fence_before();
       __syncwarp();
@@ -252,78 +289,112 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         mbar_arrive(&empty_w[sw]);
         mbar_arrive(&full_a[sa]);
       }
-      if (threadIdx.x == 64 || threadIdx.x == 64 + 128) trace_ev(p, 2, i);
+      if (tr) trace_ev(p, 2, i);
+      if (++sw == S_W) { sw = 0; pw ^= 1; }
+      if (++sa == S_A) { sa = 0; pa ^= 1; }
     }
   } else {
-    // ---------------- epilogue warps: drain finished segments
+    // ---------------- epilogue warps: drain each item's accumulators
     const int sp = warp & 3;
     const int r = sp * 32 + lane;
     const uint32_t lane_base = (uint32_t)(sp * 32) << 16;
-    int seg = 0;
-    int i = 0;
-    while (i < nunits) {
-      const int u0 = C0 + i, rt = u0 / kg, g0 = u0 - rt * kg;
-      const int len = (kg - g0) < (nunits - i) ? (kg - g0) : (nunits - i);
-      const bool full = (g0 == 0) && (len == kg);
-      const int dbuf = seg & 1;
-      mbar_wait_sleepy(&d_full[dbuf], (seg >> 1) & 1);
+    const bool leader = threadIdx.x == EPI_WARP0 * 32;
+    int n_item = 0;
+    for (int it = blockIdx.x; it < I; it += C, ++n_item) {
+      const int pn = it / Z, pp = tiles_of(pn);
+      mbar_wait_sleepy(d_full, n_item & 1);
       tc_fence_after();
-      float v[BT];
-      {
-        uint32_t a[16], b[16];
-        tmem_ld16(tmem + lane_base + D_COL + dbuf * BT, a);
-        tmem_ld16(tmem + lane_base + D_COL + dbuf * BT + 16, b);
-        tc_wait_ld();
+      for (int t = 0; t < pp; ++t) {
+        float v[BT];
+        {
+          uint32_t a[16], b[16];
+          tmem_ld16(tmem + lane_base + D_COL + t * BT, a);
+          tmem_ld16(tmem + lane_base + D_COL + t * BT + 16, b);
+          tc_wait_ld();
 #pragma unroll
-        for (int t = 0; t < 16; ++t) { v[t] = __uint_as_float(a[t]); v[16 + t] = __uint_as_float(b[t]); }
+          for (int c = 0; c < 16; ++c) { v[c] = __uint_as_float(a[c]); v[16 + c] = __uint_as_float(b[c]); }
+        }
+        if (Z == 1) {
+          const int64_t row = (int64_t)(pn * P + t) * BN + r;
+          epi_store<EPI>(p, row, v, p.bias ? __half2float(p.bias[row]) : 0.f);
+        } else {
+          float* gp = p.part + (((int64_t)it * PMAX + t) * BT) * BN + r;  // [tok][row]: coalesced
+#pragma unroll
+          for (int c = 0; c < BT; ++c) __stcg(gp + c * BN, v[c]);
+        }
       }
       tc_fence_before();
       __syncwarp();
-      if (lane == 0) mbar_arrive(&d_empty[dbuf]);
-      const int64_t row = (int64_t)rt * BN + r;
-      const float bias = p.bias ? __half2float(p.bias[row]) : 0.f;
-      if (full) {
-        epi_store<EPI>(p, row, v, bias);
-      } else {
-        // partial tile: publish, the last contributing CTA reduces in fixed CTA order
-        const int slot = (C0 < rt * kg) ? 1 : 0;
-        float* gp = p.part + (((int64_t)blockIdx.x * 2 + slot) * BT) * BN;
-#pragma unroll
-        for (int t = 0; t < BT; ++t) __stcg(gp + t * BN + r, v[t]);
+      if (lane == 0) mbar_arrive(d_empty);  // accumulators drained: the MMA may start the next item
+      if (Z > 1) {
         __threadfence();
         asm volatile("bar.sync 1, 128;" ::: "memory");
-        if (threadIdx.x == (2 + 4 * DQ_GROUPS) * 32) {
-          const int NC = gridDim.x;
-          const int ca = (int)(((long long)(rt * kg + 1) * NC - 1) / p.U);
-          const int cb = (int)(((long long)((rt + 1) * kg) * NC - 1) / p.U);
-          const int old = atomicAdd(p.cnt + rt, 1);
-          misc[1] = (old == cb - ca) ? 1u : 0u;
-          misc[2] = (uint32_t)ca;
-          misc[3] = (uint32_t)cb;
+        if (leader && atomicAdd(p.cnt + pn, 1) == Z - 1) {  // last of the panel's Z items
+          p.cnt[pn] = 0;                                     // self-reset for the next launch
+          misc[2 + misc[1]] = (uint32_t)pn;
+          misc[1] = misc[1] + 1;
         }
-        asm volatile("bar.sync 1, 128;" ::: "memory");
-        if (misc[1]) {
-          __threadfence();
-          const int ca = (int)misc[2], cb = (int)misc[3];
-#pragma unroll
-          for (int t = 0; t < BT; ++t) v[t] = 0.f;
-          for (int c = ca; c <= cb; ++c) {
-            const int sl = (rlo(c, p.U, gridDim.x) < rt * kg) ? 1 : 0;
-            const float* qp = p.part + (((int64_t)c * 2 + sl) * BT) * BN;
-#pragma unroll
-            for (int t = 0; t < BT; ++t) v[t] += __ldcg(qp + t * BN + r);
-          }
-          epi_store<EPI>(p, row, v, bias);
-          if (threadIdx.x == (2 + 4 * DQ_GROUPS) * 32) p.cnt[rt] = 0;
-        }
-        asm volatile("bar.sync 1, 128;" ::: "memory");  // misc[] reuse
       }
-      ++seg;
-      i += len;
+    }
+  }
+  // ---------------- fix-up: this CTA sums the Z partials of the panels it finished last, in
+  // fixed z order, with every warp; the rings are idle now and stage Z partial tiles at a time.
+  __syncthreads();
+  const int npend = (int)misc[1];
+  if (threadIdx.x == 0) trace_cta(p, 11);
+  if (npend > 0) {
+    __threadfence();
+    constexpr uint32_t tile_bytes = BT * BN * 4;
+    float* sred = reinterpret_cast<float*>(smem);
+    const int batch = (int)(SM::OFF_BAR / (tile_bytes * Z)) < PMAX ? (int)(SM::OFF_BAR / (tile_bytes * Z)) : PMAX;
+    int use = 0;  // red_bar[b] completes once per batch
+    for (int e = 0; e < npend; ++e) {
+      const int pn = (int)misc[2 + e], pp = tiles_of(pn);
+      for (int t0 = 0; t0 < pp; t0 += batch, ++use) {
+        const int nb = pp - t0 < batch ? pp - t0 : batch;
+        if (threadIdx.x == 0) {  // all of the batch's partial tiles in flight at once, one barrier per tile
+          for (int b = 0; b < nb; ++b) {
+            mbar_arrive_expect_tx(&red_bar[b], tile_bytes * Z);
+            for (int z = 0; z < Z; ++z)
+              bulk_load(smem + (b * Z + z) * tile_bytes,
+                        p.part + ((int64_t)(pn * Z + z) * PMAX + t0 + b) * BT * BN, tile_bytes, &red_bar[b]);
+          }
+        }
+        for (int b = 0; b < nb; ++b) {
+          mbar_wait(&red_bar[b], use & 1);
+          if (threadIdx.x == 0 && b == 0 && e == 0 && t0 == 0) trace_cta(p, 10);
+          if (threadIdx.x == 0 && b == 1 && e == 0 && t0 == 0) trace_cta(p, 6);
+          if (threadIdx.x == 0 && b == 3 && e == 0 && t0 == 0) trace_cta(p, 7);
+          const int64_t row0 = (int64_t)(pn * P + t0 + b) * BN;
+          const float* sp_ = sred + b * Z * BT * BN;
+          if (threadIdx.x < 4 * BN) {  // thread = (row, token phase): one bias load, 8 independent tokens
+            const int rr = threadIdx.x % BN, tq = threadIdx.x / BN;
+            const float bias = p.bias ? __half2float(p.bias[row0 + rr]) : 0.f;
+#pragma unroll
+            for (int u = 0; u < BT / 4; ++u) {
+              const int tok = tq + 4 * u;
+              if (tok < p.m) {
+                float acc = 0.f;
+                for (int z = 0; z < Z; ++z) acc += sp_[z * BT * BN + tok * BN + rr];
+                acc += bias;
+                if constexpr (EPI == SQ_EPI_F32_ACCUM) {
+                  static_cast<float*>(p.y)[(int64_t)tok * p.ldy + row0 + rr] += acc;
+                } else {
+                  static_cast<__half*>(p.y)[(int64_t)tok * p.ldy + row0 + rr] = __float2half_rn(apply_act<EPI>(acc));
+                }
+              }
+            }
+          }
+        }
+        if (threadIdx.x == 0 && e == 0 && t0 == 0) trace_cta(p, 9);
+        __syncthreads();  // staging reuse
+        if (threadIdx.x == 0 && e == 0 && t0 == 0) trace_cta(p, 13);
+      }
     }
   }
   tc_fence_before();
   __syncthreads();
+  if (threadIdx.x == 0) trace_cta(p, 15);
   if (warp == 1) {
     tc_fence_after();
     tmem_dealloc(tmem, TMEM_COLS);
@@ -382,18 +453,51 @@ cudaError_t launch_tc_u(const CUtensorMap& tx, const CUtensorMap& tw, const CUte
 template <int BITS>
 cudaError_t launch_tc_b(const CUtensorMap& tx, const CUtensorMap& tw, const CUtensorMap& tm, const TcP& p, int epi,
                         int nc, int ug, cudaStream_t s) {
-  if constexpr (BITS != 16) {
+  if constexpr (BITS != 8) {
     if (ug == 2) return launch_tc_u<BITS, 2>(tx, tw, tm, p, epi, nc, s);
   }
   return launch_tc_u<BITS, 1>(tx, tw, tm, p, epi, nc, s);
 }
 
+// UG: groups per unit -- a ~16-KB weight stage (INT3/INT4 two groups when k/128 is even)
+int tc_ug(int bits, int kg) { return (bits != 8 && kg % 2 == 0) ? 2 : 1; }
+
+int tc_zmax(int bits, int ug) {
+  switch (bits * 4 + ug) {
+    case 3 * 4 + 1: return DSmem<3, 1>::ZMAX;
+    case 3 * 4 + 2: return DSmem<3, 2>::ZMAX;
+    case 4 * 4 + 1: return DSmem<4, 1>::ZMAX;
+    case 4 * 4 + 2: return DSmem<4, 2>::ZMAX;
+    default: return DSmem<8, 1>::ZMAX;
+  }
+}
+
+struct TcPlan { int P, Z, I, ctas; };
+
+// Panel width P and k split Z: minimise the bytes the busiest SM ingests -- weights + meta,
+// activation slices (once per k-step per panel, 32 token rows) and, for Z > 1, the Z partial
+// tiles the finishing CTA reads back -- over ceil(items / SMs) rounds.
+TcPlan tc_plan(int64_t n, int64_t k, int bits) {
+  const int64_t nt = n / BN, kg = k / 128;
+  const int ug = tc_ug(bits, (int)kg);
+  const int64_t ks = kg / ug, C = num_sms();
+  const double unit_w = BN * ug * 128.0 * bits / 8 + BN * 4.0 * ug, unit_x = ug * 128.0 * BT * 2;
+  TcPlan best{1, 1, 0, 0};
+  double best_cost = 1e300;
+  const int zmax = tc_zmax(bits, ug);
+  for (int P = 1; P <= PMAX; ++P) {
+    for (int Z = 1; Z <= zmax && Z <= ks; ++Z) {
+      const int64_t I = ((nt + P - 1) / P) * Z, rounds = (I + C - 1) / C;
+      if (Z > 1 && rounds > 62) continue;  // pending-panel list of the fix-up
+      const int64_t steps = (ks + Z - 1) / Z;
+      const double cost = rounds * (steps * (P * unit_w + unit_x) + (Z > 1 ? Z * P * (double)BT * BN * 4 : 0.0));
+      if (cost < best_cost * 0.999) { best_cost = cost; best = {P, Z, (int)I, (int)(I < C ? I : C)}; }
+    }
+  }
+  return best;
+}
 unsigned long long* g_trace = nullptr;
 
-int tc_ctas(int64_t U) {
-  const int64_t full = num_sms();
-  return (int)(U < full ? U : full);
-}
 
 }  // namespace
 
@@ -402,8 +506,13 @@ int tc_ctas(int64_t U) {
 constexpr size_t kCntBytes = (65536 / 16) * sizeof(int);
 
 size_t gemv_tc_workspace_bytes(int64_t n, int64_t k) {
-  const int64_t U = (n / BN) * (k / 128);
-  return kCntBytes + (size_t)tc_ctas(U) * 2 * BT * BN * sizeof(float) + 256;
+  // partials: [items][PMAX tiles][32 x 128] fp32, worst case over the bit widths
+  int64_t items = 0;
+  for (int bits : {3, 4, 8}) {
+    const TcPlan pl = tc_plan(n, k, bits);
+    if (pl.Z > 1 && pl.I > items) items = pl.I;
+  }
+  return kCntBytes + (size_t)items * PMAX * BT * BN * sizeof(float) + 256;
 }
 
 cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, int m, void* y, int64_t ldy, int epi,
@@ -411,7 +520,8 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
   CUtensorMap tx, tw, tm;
   memset(&tm, 0, sizeof(tm));
   const int kg = (int)(w.k / 128);
-  const int ug = (w.bits != 16 && kg % 2 == 0) ? 2 : 1;
+  if (w.bits == 16) return cudaErrorNotSupported;  // fp16 weights stay on the mma.sync path (gemv_path)
+  const int ug = tc_ug(w.bits, kg);
   {
     // activations as [k/64][m][64]: one box {64, 32, 2*ug} per unit -> 2*ug SW128 tiles [32 tokens][64 k]
     const uint64_t dx[3] = {64, (uint64_t)m, (uint64_t)w.k / 64}, sx[2] = {(uint64_t)ldx * 2, 128};
@@ -419,20 +529,15 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
     cudaError_t e = enc(&tx, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, x, 3, dx, sx, bx, CU_TENSOR_MAP_SWIZZLE_128B);
     if (e != cudaSuccess) return e;
   }
-  if (w.bits == 16) {
-    const uint64_t dw[2] = {(uint64_t)w.k, (uint64_t)w.n}, sw_[1] = {(uint64_t)w.k * 2};
-    const uint32_t bw[2] = {64, BN};
-    cudaError_t e = enc(&tw, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, w.packed, 2, dw, sw_, bw, CU_TENSOR_MAP_SWIZZLE_128B);
-    if (e != cudaSuccess) return e;
-  } else {
+  {
     const uint64_t gb = 128 * w.bits / 8, nt = (uint64_t)w.n / 16;
     CUtensorMapSwizzle sw = w.bits == 8 ? CU_TENSOR_MAP_SWIZZLE_128B
                                         : (w.bits == 4 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_NONE);
-    const uint64_t dw[4] = {gb, 16, kg, nt}, sw_[3] = {gb, 16 * gb, kg * 16 * gb};
+    const uint64_t dw[4] = {gb, 16, (uint64_t)kg, nt}, sw_[3] = {gb, 16 * gb, kg * 16 * gb};
     const uint32_t bw[4] = {(uint32_t)gb, 16, (uint32_t)ug, BN / 16};
     cudaError_t e = enc(&tw, CU_TENSOR_MAP_DATA_TYPE_UINT8, w.packed, 4, dw, sw_, bw, sw);
     if (e != cudaSuccess) return e;
-    const uint64_t dm[3] = {16, kg, nt}, sm_[2] = {64, kg * 64};
+    const uint64_t dm[3] = {16, (uint64_t)kg, nt}, sm_[2] = {64, (uint64_t)kg * 64};
     const uint32_t bm[3] = {16, (uint32_t)ug, BN / 16};
     e = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, w.meta, 3, dm, sm_, bm, CU_TENSOR_MAP_SWIZZLE_NONE);
     if (e != cudaSuccess) return e;
@@ -446,12 +551,17 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
   p.m = m;
   p.n = (int)w.n;
   p.kg = kg;
-  p.U = (int)((w.n / BN) * (kg / ug));
+  p.nt = (int)(w.n / BN);
+  p.ks = kg / ug;
+  const TcPlan pl = tc_plan(w.n, w.k, w.bits);
+  p.P = pl.P;
+  p.Z = pl.Z;
+  p.I = pl.I;
   uint8_t* base = static_cast<uint8_t*>(ws);
   p.cnt = reinterpret_cast<int*>(base);
   p.part = reinterpret_cast<float*>(base + kCntBytes);
   p.trace = g_trace;
-  const int nc = tc_ctas(p.U);
+  const int nc = pl.ctas;
   const double bytes = (double)w.n * w.k * w.bits / 8.0 + (w.bits != 16 ? (double)w.n * (w.k / 128) * 4.0 : 0.0);
   auto t = prof_begin(KC_GEMV, bytes, 2.0 * m * w.n * w.k, s);
   cudaError_t e;
@@ -459,7 +569,7 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
     case 3: e = launch_tc_b<3>(tx, tw, tm, p, epi, nc, ug, s); break;
     case 4: e = launch_tc_b<4>(tx, tw, tm, p, epi, nc, ug, s); break;
     case 8: e = launch_tc_b<8>(tx, tw, tm, p, epi, nc, ug, s); break;
-    default: e = launch_tc_b<16>(tx, tw, tm, p, epi, nc, 1, s); break;
+    default: e = cudaErrorNotSupported; break;
   }
   prof_end(t, s);
   count_launch();
@@ -469,5 +579,5 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
 }  // namespace sq
 
 // debug only (not part of include/sq.h): record CTA 0's per-unit clock64 events of the
-// tcgen05 decode kernel into a device buffer of 14 x 256 uint64 (tools/trace_tc.py)
+// tcgen05 decode kernel into a device buffer of 16 x 256 uint64 (rows 14/15: per-CTA globaltimer start/end) (tools/trace_tc.py)
 extern "C" void sq_debug_trace(void* dev_buf) { sq::g_trace = static_cast<unsigned long long*>(dev_buf); }

@@ -45,20 +45,21 @@ __device__ __forceinline__ uint32_t hsub_fma(uint32_t h, uint32_t off2, uint32_t
   return *reinterpret_cast<uint32_t*>(&r);
 }
 
-// Dequantize this thread's row (r) of one 128-k group into 64 half2 columns,
-// written to TMEM in 4 batches of 16 columns.
-template <int BITS>
-// `row_off` = byte offset of this thread's row inside the stage (default r * GB); the swizzle
-// pattern only depends on r % 16 because every T16 unit starts on a 1-KB boundary.
-__device__ __forceinline__ void dequant_row_to_tmem(const uint8_t* wst, uint32_t meta, int r, uint32_t taddr,
-                                                    int row_off = -1) {
+// Dequantize batches [B0, B0 + NB) (32 k each) of this thread's row (r) of one 128-k group into
+// half2 columns taddr + 16 b .. + 15 (w~ = s*c + z), one tcgen05.st per batch.  `row_off` = byte
+// offset of the row inside the stage (default r * GB); the swizzle pattern only depends on
+// r % 16 because every T16 unit starts on a 1-KB boundary.  B0 must be warp-uniform.
+template <int BITS, int NB>
+__device__ __forceinline__ void dequant_row_batches(const uint8_t* wst, uint32_t meta, int r, uint32_t taddr,
+                                                    int row_off, int B0) {
   const uint32_t s2 = (meta & 0xFFFFu) * 0x10001u;
   const uint32_t z2 = (meta >> 16) * 0x10001u;
   constexpr uint32_t K1024 = 0x64006400u, K64 = 0x54005400u;
   if constexpr (BITS == 4) {
     const uint8_t* row = wst + (row_off >= 0 ? row_off : r * 64);
 #pragma unroll
-    for (int b = 0; b < 4; ++b) {
+    for (int bi = 0; bi < NB; ++bi) {
+      const int b = B0 + bi;
       const int pc = b ^ ((r >> 1) & 3);  // SWIZZLE_64B
       uint4 v = *reinterpret_cast<const uint4*>(row + pc * 16);
       const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
@@ -76,7 +77,8 @@ __device__ __forceinline__ void dequant_row_to_tmem(const uint8_t* wst, uint32_t
   } else if constexpr (BITS == 8) {
     const uint8_t* row = wst + (row_off >= 0 ? row_off : r * 128);
 #pragma unroll
-    for (int b = 0; b < 4; ++b) {
+    for (int bi = 0; bi < NB; ++bi) {
+      const int b = B0 + bi;
       uint32_t o[16];
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
@@ -94,7 +96,8 @@ __device__ __forceinline__ void dequant_row_to_tmem(const uint8_t* wst, uint32_t
   } else if constexpr (BITS == 3) {
     const uint32_t* row = reinterpret_cast<const uint32_t*>(wst + (row_off >= 0 ? row_off : r * 48));
 #pragma unroll
-    for (int bl = 0; bl < 4; ++bl) {
+    for (int bi = 0; bi < NB; ++bi) {
+      const int bl = B0 + bi;
       const uint32_t L0 = row[3 * bl], L1 = row[3 * bl + 1], H = row[3 * bl + 2];
       uint32_t o[16];
 #pragma unroll
@@ -115,7 +118,8 @@ __device__ __forceinline__ void dequant_row_to_tmem(const uint8_t* wst, uint32_t
   } else {
     // fp16: two SW128 regions (k 0..63, 64..127) of [128 rows x 128 B]
 #pragma unroll
-    for (int b = 0; b < 4; ++b) {
+    for (int bi = 0; bi < NB; ++bi) {
+      const int b = B0 + bi;
       const uint8_t* region = wst + (b >> 1) * (128 * 128) + r * 128;
       uint32_t o[16];
 #pragma unroll
@@ -129,6 +133,12 @@ __device__ __forceinline__ void dequant_row_to_tmem(const uint8_t* wst, uint32_t
   }
 }
 
+// the whole 128-k group of this thread's row: 64 half2 columns at taddr .. taddr + 63
+template <int BITS>
+__device__ __forceinline__ void dequant_row_to_tmem(const uint8_t* wst, uint32_t meta, int r, uint32_t taddr,
+                                                    int row_off = -1) {
+  dequant_row_batches<BITS, 4>(wst, meta, r, taddr, row_off, 0);
+}
 
 // Fetch the 128-row x 1-group weight tile (8 T16 units, each 16*GB contiguous bytes at unit
 // index t*kg + g) and its meta (8 x 64 B) with 16 bulk copies onto one mbarrier.

@@ -131,8 +131,9 @@ def test_decode_parity(bits, m):
 
 @pytest.mark.parametrize("bits", [3, 4, 8, 16])
 @pytest.mark.parametrize("epi", [1, 2, 3])
-def test_decode_epilogues(bits, epi):
-    n, k, m = 272, 640, 3
+@pytest.mark.parametrize("n,m", [(272, 3), (640, 32)])
+def test_decode_epilogues(bits, epi, n, m):
+    k = 640
     qo, qg = _make(bits, n, k, seed=300)
     x = synth.act_f16(301, m, k)
     lin = O.linear(x, qo)
@@ -146,13 +147,28 @@ def test_decode_epilogues(bits, epi):
 
 
 @pytest.mark.parametrize("bits", [3, 4, 8, 16])
-def test_decode_deterministic(bits):
-    n, k, m = 2048, 1536, 7
+@pytest.mark.parametrize("m", [7, 32])
+def test_decode_deterministic(bits, m):
+    n, k = 2048, 1536
     qo, qg = _make(bits, n, k, seed=400)
     x = synth.act_f16(401, m, k)
     a = _run_linear("decode", qg, x, 0)
     b = _run_linear("decode", qg, x, 0)
     assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("bits", [3, 4, 8])
+@pytest.mark.parametrize("m", [12, 32])
+@pytest.mark.parametrize("n,k", [(640, 9216), (128, 4992), (1920, 384)])
+def test_decode_tc_split_panels(bits, m, n, k):
+    """tcgen05 path (m > 8): panels split over many CTAs (fix-up order), a ragged last panel,
+    one-tile panels and odd k/128 (one group per unit)."""
+    qo, qg = _make(bits, n, k, seed=500 + n)
+    x = synth.act_f16(501 + m, m, k)
+    ref = O.linear(x, qo)
+    y = _run_linear("decode", qg, x, 0)
+    assert normwise(y, ref) <= TOL, (n, k, normwise(y, ref))
+    assert np.array_equal(y, _run_linear("decode", qg, x, 0))
 
 
 @pytest.mark.parametrize("bits", [3, 4, 8])

@@ -12,17 +12,35 @@ q = sq.QLinear.from_fp16(wd, bits)
 x = torch.randn(m, k, device="cuda").half()
 y = torch.empty(m, n, device="cuda", dtype=torch.float16)
 ws = torch.zeros(sq.sq_linear_workspace_bytes(q, m), dtype=torch.uint8, device="cuda")
-tr = torch.zeros(14 * 256, dtype=torch.int64, device="cuda")
+tr = torch.zeros(16 * 256, dtype=torch.int64, device="cuda")
 sq.lib().sq_debug_trace.argtypes = [ctypes.c_void_p]
 for _ in range(3):
     sq.sq_linear_decode(q, x, y, 0, ws=ws)
 sq.lib().sq_debug_trace(tr.data_ptr())
 sq.sq_linear_decode(q, x, y, 0, ws=ws)
 torch.cuda.synchronize()
-t = tr.view(14, 256).cpu().numpy().astype("int64")
+t = tr.view(16, 256).cpu().numpy().astype("int64")
 t0 = t[0, 0]
 U = (n // 128) * (k // 128); per = U // 148
 print("units on CTA0:", per)
-print(" i  Wwait    Wtma  metatma   X0tma   X1tma dq_done mma_Ardy  x0rdy  mma0done  x1rdy mma1done mma_end")
-for i in range(min(per, 48)):
-    print(f"{i:2d} " + " ".join(f"{(t[e, i] - t0) if t[e, i] else -1:8d}" for e in (0, 6, 7, 8, 9, 2, 3, 10, 11, 12, 13, 4)))
+cols = [("prodW", 0), ("prodIss", 8), ("dqW", 1), ("dqSlot", 5), ("dqCalc", 12), ("dqDone", 2), ("mmaRdy", 3), ("mmaIss", 4)]
+print(" i " + " ".join(f"{c:>8s}" for c, _ in cols))
+for i in range(min(per, 64)):
+    print(f"{i:2d} " + " ".join(f"{(t[e, i] - t0) if t[e, i] else -1:8d}" for _, e in cols))
+ns = min(148, int((t[14] > 0).sum()))
+g0 = t[14, :ns].min()
+st, en = (t[14, :ns] - g0) / 1e3, (t[15, :ns] - g0) / 1e3
+print(f"CTA start us: min {st.min():.2f} max {st.max():.2f}; end us: min {en.min():.2f} med {sorted(en)[ns // 2]:.2f} max {en.max():.2f}")
+print("slowest CTAs:", [(int(c), round(float(en[c]), 2)) for c in en.argsort()[-8:]])
+print("ends:", " ".join(f"{e:.1f}" for e in en[:40]))
+fx = (t[11, :ns] - g0) / 1e3
+land = (t[10, :ns] - g0) / 1e3
+red = [c for c in range(ns) if t[10, c] > t[14, c]]
+print("reducers:", len(red), "fixup start->first tile landed->end us:", [(round(float(fx[c]), 1), round(float(land[c]), 1), round(float(en[c]), 1)) for c in red[:6]])
+print("non-reducers fixup start:", [round(float(fx[c]), 1) for c in range(ns) if c not in red][:8])
+done = (t[9, :ns] - g0) / 1e3
+sync = (t[13, :ns] - g0) / 1e3
+print("reducers compute-done / after-sync:", [(round(float(done[c]), 1), round(float(sync[c]), 1)) for c in red[:6]])
+l1 = (t[6, :ns] - g0) / 1e3
+l3 = (t[7, :ns] - g0) / 1e3
+print("reducers tile1/tile3 landed:", [(round(float(l1[c]), 1), round(float(l3[c]), 1)) for c in red[:6]])
