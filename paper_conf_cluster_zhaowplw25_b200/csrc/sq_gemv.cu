@@ -499,7 +499,8 @@ size_t gemv_workspace_bytes(int64_t n, int64_t k, int64_t m) {
   return a > b ? a : b;
 }
 
-// K2 (mma.sync, register unpack) for m <= 8; K2c (tcgen05, TMEM dequant) for 8 < m <= 32.
+// K2 (mma.sync, register unpack) for m <= 8; K2c (tcgen05: TMEM dequant, or fp16 weights straight
+// from SMEM) for 8 < m <= 32.
 // SQ_GEMV_PATH=mma|tc overrides (benchmarking).
 int gemv_path(int64_t n, int m, int bits) {
   static int forced = -2;
@@ -507,7 +508,7 @@ int gemv_path(int64_t n, int m, int bits) {
     const char* e = getenv("SQ_GEMV_PATH");
     forced = !e ? -1 : (e[0] == 't' ? 1 : (e[0] == 'm' ? 0 : -1));
   }
-  if (n % 128 || bits == 16) return 0;  // fp16 weights: 2 B/weight keeps even m = 32 HBM-bound on mma.sync
+  if (n % 128) return 0;
   if (forced >= 0) return forced;
   return m > 8 ? 1 : 0;
 }

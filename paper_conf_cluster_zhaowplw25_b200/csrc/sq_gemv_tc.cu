@@ -56,7 +56,7 @@ constexpr int X_LAG = 1;              // activations of step q are fetched after
 template <int BITS, int UG>
 struct DCfg {
   // weight ring: a slot lives TMA latency (~1.8k cycles) + wait for its group + dequant (~2k)
-  static constexpr int S_W = UG == 2 ? 9 : (BITS == 8 ? 9 : (BITS == 4 ? 18 : 24));
+  static constexpr int S_W = BITS == 16 ? 5 : (UG == 2 ? 9 : (BITS == 8 ? 9 : (BITS == 4 ? 18 : 24)));
   // TMEM A slots of 64*UG columns: the dequant warps fill slot i % S_A while the MMA reads the
   // others (128 + 3 * 128 = 512 columns at UG = 2)
   static constexpr int S_A = UG == 2 ? 3 : 6;
@@ -73,7 +73,7 @@ struct DSmem {
   static constexpr int OFF_X = 0;
   static constexpr int OFF_W = OFF_X + S_X * X_STAGE;
   static constexpr int OFF_META = OFF_W + S_W * W_STAGE;
-  static constexpr int OFF_BAR = OFF_META + S_W * BN * 4 * UG;
+  static constexpr int OFF_BAR = OFF_META + (BITS == 16 ? 0 : S_W * BN * 4 * UG);
   static constexpr int NUM_BARS = 2 * S_X + 2 * S_W + 2 * DCfg<BITS, UG>::S_A + 2 + PMAX;
   static constexpr int OFF_MISC = OFF_BAR + NUM_BARS * 8;
   static constexpr int BYTES = OFF_MISC + 256 + 1024;  // misc: tmem base, pending panels (<= 62)
@@ -140,7 +140,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   constexpr int S_X = SM::S_X;
   constexpr int X_STAGE = SM::X_STAGE;
   constexpr int GB = GCfg<BITS>::GB;
-  constexpr uint32_t W_BYTES = BN * GB * UG + BN * 4 * UG;  // codes + meta of one unit
+  constexpr uint32_t W_BYTES = BN * GB * UG + (BITS == 16 ? 0 : BN * 4 * UG);  // codes + meta of one unit
   extern __shared__ uint8_t smem_raw[];
   // 1-KB aligned (SW128 atoms); pointer arithmetic on smem_raw keeps the shared address space
   // visible to the compiler (LDS, not generic LD)
@@ -167,7 +167,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < S_X; ++i) { mbar_init(&full_x[i], 1); mbar_init(&empty_x[i], 1); }
-    for (int i = 0; i < S_W; ++i) { mbar_init(&full_w[i], 1); mbar_init(&empty_w[i], DQ_WARPS); }
+    // fp16 weights are the MMA's A operand straight from SMEM: the MMA commit frees the slot
+    for (int i = 0; i < S_W; ++i) { mbar_init(&full_w[i], 1); mbar_init(&empty_w[i], BITS == 16 ? 1 : DQ_WARPS); }
     for (int i = 0; i < S_A; ++i) { mbar_init(&full_a[i], DQ_WARPS); mbar_init(&empty_a[i], 1); }
     mbar_init(d_full, 1);
     mbar_init(d_empty, 4);
@@ -176,7 +177,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     fence_barrier_init();
     prefetch_tmap(&tm_x);
     prefetch_tmap(&tm_w);
-    prefetch_tmap(&tm_m);
+    if constexpr (BITS != 16) prefetch_tmap(&tm_m);
   }
   if (warp == 1) tmem_alloc(misc, TMEM_COLS);
   tc_fence_before();
@@ -212,10 +213,17 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           trace_ev(p, 0, i);
           if (elect_one()) {
             const int tile16 = (pn * P + t) * (BN / 16);
+            uint8_t* wdst = smem + SM::OFF_W + sw * SM::W_STAGE;
             mbar_arrive_expect_tx(&full_w[sw], W_BYTES);
-            // placement T16: box {GB bytes, 16 rows, UG groups, 8 row tiles} -> [tile][group][16][GB]
-            tma_load_4d(smem + SM::OFF_W + sw * SM::W_STAGE, &tm_w, &full_w[sw], 0, 0, j * UG, tile16);
-            tma_load_3d(smem + SM::OFF_META + sw * BN * 4 * UG, &tm_m, &full_w[sw], 0, j * UG, tile16);
+            if constexpr (BITS == 16) {
+              // row-major fp16 [n][k]: two SW128 boxes [128 rows][64 k] = the MMA's K-major A tiles
+              tma_load_2d(wdst, &tm_w, &full_w[sw], j * 128, (pn * P + t) * BN);
+              tma_load_2d(wdst + BN * 128, &tm_w, &full_w[sw], j * 128 + 64, (pn * P + t) * BN);
+            } else {
+              // placement T16: box {GB bytes, 16 rows, UG groups, 8 row tiles} -> [tile][group][16][GB]
+              tma_load_4d(wdst, &tm_w, &full_w[sw], 0, 0, j * UG, tile16);
+              tma_load_3d(smem + SM::OFF_META + sw * BN * 4 * UG, &tm_m, &full_w[sw], 0, j * UG, tile16);
+            }
           }
           __syncwarp();
           trace_ev(p, 8, i);
@@ -235,6 +243,31 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         mbar_wait(&full_x[sx], rx & 1);
         const uint64_t bdesc0 = make_sw128_desc(smem_u32(smem + SM::OFF_X + sx * X_STAGE));
         for (int t = 0; t < pp; ++t, ++i) {
+          if constexpr (BITS == 16) {
+            // A (fp16 weights) straight from the W stage: two SW128 [128 x 64] tiles
+            const int sw = i % S_W, rw = i / S_W;
+            mbar_wait(&full_w[sw], rw & 1);
+            tc_fence_after();
+            trace_ev(p, 3, i);
+            if (elect_one()) {
+              const uint32_t d_tm = tmem + D_COL + t * BT;
+              const uint64_t adesc0 = make_sw128_desc(smem_u32(smem + SM::OFF_W + sw * SM::W_STAGE));
+#pragma unroll
+              for (int kk = 0; kk < 8; ++kk) {
+                const uint64_t off = (uint64_t)(((kk >> 2) * BN * 128 + (kk & 3) * 32) >> 4);
+                const uint64_t boff = (uint64_t)(((kk >> 2) * X_BLOCK + (kk & 3) * 32) >> 4);
+                tc_mma_ss(d_tm, adesc0 + off, bdesc0 + boff, kIdescTc, (j == j0 && kk == 0) ? 0u : 1u);
+              }
+              tc_commit(&empty_w[sw]);
+              if (t == pp - 1) {
+                tc_commit(&empty_x[sx]);
+                if (j == j1 - 1) tc_commit(d_full);
+              }
+            }
+            __syncwarp();
+            trace_ev(p, 4, i);
+            continue;
+          }
           const int sa = i % S_A, ra = i / S_A;
           mbar_wait(&full_a[sa], ra & 1);
           tc_fence_after();
@@ -262,7 +295,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     // batches [kh*2*UG, kh*2*UG + 2*UG) of the unit's 4*UG 32-k batches.  All 8 warps work on
     // every unit, so a unit's dequant latency is half of one warp's work.
     int nunits = 0;
-    for (int it = blockIdx.x; it < I; it += C) nunits += (j1_of(it) - j0_of(it)) * tiles_of(it / Z);
+    if constexpr (BITS != 16)
+      for (int it = blockIdx.x; it < I; it += C) nunits += (j1_of(it) - j0_of(it)) * tiles_of(it / Z);
     constexpr int NBW = 2 * UG;                              // batches per warp
     const int sp = warp & 3;
     const int kh = (warp - 2) >> 2;
@@ -367,8 +401,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           if (threadIdx.x == 0 && b == 3 && e == 0 && t0 == 0) trace_cta(p, 7);
           const int64_t row0 = (int64_t)(pn * P + t0 + b) * BN;
           const float* sp_ = sred + b * Z * BT * BN;
-          if (threadIdx.x < 4 * BN) {  // thread = (row, token phase): one bias load, 8 independent tokens
-            const int rr = threadIdx.x % BN, tq = threadIdx.x / BN;
+          for (int th = threadIdx.x; th < 4 * BN; th += NUM_THREADS) {  // (row, token phase): 8 tokens each
+            const int rr = th % BN, tq = th / BN;
             const float bias = p.bias ? __half2float(p.bias[row0 + rr]) : 0.f;
 #pragma unroll
             for (int u = 0; u < BT / 4; ++u) {
@@ -453,14 +487,14 @@ cudaError_t launch_tc_u(const CUtensorMap& tx, const CUtensorMap& tw, const CUte
 template <int BITS>
 cudaError_t launch_tc_b(const CUtensorMap& tx, const CUtensorMap& tw, const CUtensorMap& tm, const TcP& p, int epi,
                         int nc, int ug, cudaStream_t s) {
-  if constexpr (BITS != 8) {
+  if constexpr (BITS == 3 || BITS == 4) {
     if (ug == 2) return launch_tc_u<BITS, 2>(tx, tw, tm, p, epi, nc, s);
   }
   return launch_tc_u<BITS, 1>(tx, tw, tm, p, epi, nc, s);
 }
 
 // UG: groups per unit -- a ~16-KB weight stage (INT3/INT4 two groups when k/128 is even)
-int tc_ug(int bits, int kg) { return (bits != 8 && kg % 2 == 0) ? 2 : 1; }
+int tc_ug(int bits, int kg) { return (bits <= 4 && kg % 2 == 0) ? 2 : 1; }
 
 int tc_zmax(int bits, int ug) {
   switch (bits * 4 + ug) {
@@ -468,6 +502,7 @@ int tc_zmax(int bits, int ug) {
     case 3 * 4 + 2: return DSmem<3, 2>::ZMAX;
     case 4 * 4 + 1: return DSmem<4, 1>::ZMAX;
     case 4 * 4 + 2: return DSmem<4, 2>::ZMAX;
+    case 16 * 4 + 1: return DSmem<16, 1>::ZMAX;
     default: return DSmem<8, 1>::ZMAX;
   }
 }
@@ -481,7 +516,7 @@ TcPlan tc_plan(int64_t n, int64_t k, int bits) {
   const int64_t nt = n / BN, kg = k / 128;
   const int ug = tc_ug(bits, (int)kg);
   const int64_t ks = kg / ug, C = num_sms();
-  const double unit_w = BN * ug * 128.0 * bits / 8 + BN * 4.0 * ug, unit_x = ug * 128.0 * BT * 2;
+  const double unit_w = BN * ug * 128.0 * bits / 8 + (bits == 16 ? 0.0 : BN * 4.0 * ug), unit_x = ug * 128.0 * BT * 2;
   TcPlan best{1, 1, 0, 0};
   double best_cost = 1e300;
   const int zmax = tc_zmax(bits, ug);
@@ -508,7 +543,7 @@ constexpr size_t kCntBytes = (65536 / 16) * sizeof(int);
 size_t gemv_tc_workspace_bytes(int64_t n, int64_t k) {
   // partials: [items][PMAX tiles][32 x 128] fp32, worst case over the bit widths
   int64_t items = 0;
-  for (int bits : {3, 4, 8}) {
+  for (int bits : {3, 4, 8, 16}) {
     const TcPlan pl = tc_plan(n, k, bits);
     if (pl.Z > 1 && pl.I > items) items = pl.I;
   }
@@ -520,7 +555,6 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
   CUtensorMap tx, tw, tm;
   memset(&tm, 0, sizeof(tm));
   const int kg = (int)(w.k / 128);
-  if (w.bits == 16) return cudaErrorNotSupported;  // fp16 weights stay on the mma.sync path (gemv_path)
   const int ug = tc_ug(w.bits, kg);
   {
     // activations as [k/64][m][64]: one box {64, 32, 2*ug} per unit -> 2*ug SW128 tiles [32 tokens][64 k]
@@ -529,7 +563,12 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
     cudaError_t e = enc(&tx, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, x, 3, dx, sx, bx, CU_TENSOR_MAP_SWIZZLE_128B);
     if (e != cudaSuccess) return e;
   }
-  {
+  if (w.bits == 16) {
+    const uint64_t dw[2] = {(uint64_t)w.k, (uint64_t)w.n}, sw_[1] = {(uint64_t)w.k * 2};
+    const uint32_t bw[2] = {64, BN};
+    cudaError_t e = enc(&tw, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, w.packed, 2, dw, sw_, bw, CU_TENSOR_MAP_SWIZZLE_128B);
+    if (e != cudaSuccess) return e;
+  } else {
     const uint64_t gb = 128 * w.bits / 8, nt = (uint64_t)w.n / 16;
     CUtensorMapSwizzle sw = w.bits == 8 ? CU_TENSOR_MAP_SWIZZLE_128B
                                         : (w.bits == 4 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_NONE);
@@ -569,7 +608,7 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
     case 3: e = launch_tc_b<3>(tx, tw, tm, p, epi, nc, ug, s); break;
     case 4: e = launch_tc_b<4>(tx, tw, tm, p, epi, nc, ug, s); break;
     case 8: e = launch_tc_b<8>(tx, tw, tm, p, epi, nc, ug, s); break;
-    default: e = cudaErrorNotSupported; break;
+    default: e = launch_tc_b<16>(tx, tw, tm, p, epi, nc, 1, s); break;
   }
   prof_end(t, s);
   count_launch();
