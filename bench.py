@@ -322,7 +322,8 @@ def run_ours(args, wl):
     if dom:
         r = kern[dom]
         roof = {"bound": r["bound"], "achieved": round(r["achieved"], 2), "peak": r["peak"], "unit": r["unit"],
-                "frac": round(r["frac"], 4), "traffic": traffic_for(dom), "kernel": dom,
+                "frac": round(r["frac"], 4), "traffic": traffic_for(dom, r.get("bytes_per_launch")), "kernel": dom,
+                "traffic_src": "profiles/traffic.json (ncu --set full dram bytes / algorithmic bytes of one launch)",
                 "peak_src": pk["src"] + (" sustained" if r["bound"] == "tensor" else " copy")}
 
     # ---------------- e2e: host buffers through the C-ABI, copies inside the timed region
@@ -390,13 +391,20 @@ def run_ours(args, wl):
         dist.destroy_process_group()
 
 
-def traffic_for(kernel: str):
-    """dram bytes per launch of the dominant kernel from the committed ncu capture (profiles/)."""
+def traffic_for(kernel: str, per_launch: float | None = None):
+    """DRAM bytes per launch of the dominant kernel from the committed ncu --set full capture
+    (profiles/traffic.json): the captured launch's dram/algorithmic ratio applied to this run's
+    algorithmic bytes per launch (so `traffic` and `achieved` count the same launches)."""
     try:
         with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
-            return json.load(f).get(kernel)
+            t = json.load(f).get(kernel)
     except Exception:
         return None
+    if not t:
+        return None
+    if per_launch is not None and t.get("ratio"):
+        return round(t["ratio"] * per_launch)
+    return t.get("dram_bytes")
 
 
 def main():
