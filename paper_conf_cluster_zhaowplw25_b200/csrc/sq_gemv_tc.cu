@@ -25,11 +25,13 @@
 //  * 4 epilogue warps drain an item: Z = 1 -> bias / activation / fp32 residual
 //    straight to y; Z > 1 -> fp32 partial to the workspace, and the last of the
 //    Z items to arrive (atomic counter) sums all Z partials of the panel in fixed
-//    z order at the end of its CTA (bulk copies into the then idle rings; all
-//    warps).  Deterministic; counters self-reset.
+//    z order at the end of its CTA (all warps, 16-B loads).  Deterministic;
+//    counters self-reset.
 // Warp roles: 0 producer, 1 MMA (+TMEM alloc), 2..17 dequant, 18..21 epilogue.
 #include <cuda.h>
 
+#include <cstdlib>
+#include <cstdio>
 #include <cstring>
 
 #include "sq_tc.cuh"
@@ -74,11 +76,11 @@ struct DSmem {
   static constexpr int OFF_W = OFF_X + S_X * X_STAGE;
   static constexpr int OFF_META = OFF_W + S_W * W_STAGE;
   static constexpr int OFF_BAR = OFF_META + (BITS == 16 ? 0 : S_W * BN * 4 * UG);
-  static constexpr int NUM_BARS = 2 * S_X + 2 * S_W + 2 * DCfg<BITS, UG>::S_A + 2 + PMAX;
+  static constexpr int NUM_BARS = 2 * S_X + 2 * S_W + 2 * DCfg<BITS, UG>::S_A + 2;
   static constexpr int OFF_MISC = OFF_BAR + NUM_BARS * 8;
   static constexpr int BYTES = OFF_MISC + 256 + 1024;  // misc: tmem base, pending panels (<= 62)
   static_assert(BYTES <= 227 * 1024, "shared memory budget");
-  static constexpr int ZMAX = OFF_BAR / (BT * BN * 4) < 8 ? OFF_BAR / (BT * BN * 4) : 8;  // partial tiles staged
+
 };
 
 struct TcP {
@@ -98,6 +100,7 @@ struct TcP {
   float* part;  // [items][PMAX tiles][32 tokens][128 rows] fp32 partial sums (Z > 1)
   int* cnt;     // [panels]
   unsigned long long* trace;  // debug: CTA 0 per-unit clock64 events (sq_debug_trace), or null
+  int abl;                    // debug ablation (SQ_TC_ABL): 1 = no dequant, 2 = no MMAs (results wrong)
 };
 
 __device__ __forceinline__ void trace_ev(const TcP& p, int ev, int i) {
@@ -112,7 +115,6 @@ __device__ __forceinline__ void trace_cta(const TcP& p, int ev) {
   }
 }
 
-__device__ __forceinline__ int rlo(int i, int total, int parts) { return (int)(((long long)i * total) / parts); }
 
 template <int EPI>
 __device__ __forceinline__ void epi_store(const TcP& p, int64_t row, const float (&v)[BT], float bias) {
@@ -154,7 +156,6 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   uint64_t* empty_a = full_a + S_A;
   uint64_t* d_full = empty_a + S_A;
   uint64_t* d_empty = d_full + 1;
-  uint64_t* red_bar = d_empty + 1;  // [PMAX]
   uint32_t* misc = reinterpret_cast<uint32_t*>(smem + SM::OFF_MISC);  // [0] tmem base, [1] #pending, [2..] panels
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -172,7 +173,6 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     for (int i = 0; i < S_A; ++i) { mbar_init(&full_a[i], DQ_WARPS); mbar_init(&empty_a[i], 1); }
     mbar_init(d_full, 1);
     mbar_init(d_empty, 4);
-    for (int i = 0; i < PMAX; ++i) mbar_init(&red_bar[i], 1);
     misc[1] = 0;
     fence_barrier_init();
     prefetch_tmap(&tm_x);
@@ -193,7 +193,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     int xj[X_LAG + 1];         // k-step of the pending activation fetches (ring of X_LAG + 1)
     auto issue_x = [&](int j) {
       const int sx = qx % S_X, rx = qx / S_X;
-      mbar_wait(&empty_x[sx], (rx & 1) ^ 1);
+      mbar_wait_park(&empty_x[sx], (rx & 1) ^ 1);
       if (elect_one()) {
         // box {64 k, 32 tokens, 2*UG k-blocks} -> 2*UG SW128 tiles [32][64]
         mbar_arrive_expect_tx(&full_x[sx], X_STAGE);
@@ -209,7 +209,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         if (q >= X_LAG) issue_x(xj[(q - X_LAG) % (X_LAG + 1)]);
         for (int t = 0; t < pp; ++t, ++i) {
           const int sw = i % S_W, rw = i / S_W;
-          mbar_wait(&empty_w[sw], (rw & 1) ^ 1);
+          mbar_wait_park(&empty_w[sw], (rw & 1) ^ 1);
           trace_ev(p, 0, i);
           if (elect_one()) {
             const int tile16 = (pn * P + t) * (BN / 16);
@@ -237,16 +237,16 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     int i = 0, q = 0, n_item = 0;
     for (int it = blockIdx.x; it < I; it += C, ++n_item) {
       const int pn = it / Z, j0 = j0_of(it), j1 = j1_of(it), pp = tiles_of(pn);
-      mbar_wait(d_empty, (n_item & 1) ^ 1);  // the epilogue drained the previous item
+      mbar_wait_park(d_empty, (n_item & 1) ^ 1);  // the epilogue drained the previous item
       for (int j = j0; j < j1; ++j, ++q) {
         const int sx = q % S_X, rx = q / S_X;
-        mbar_wait(&full_x[sx], rx & 1);
+        mbar_wait_park(&full_x[sx], rx & 1);
         const uint64_t bdesc0 = make_sw128_desc(smem_u32(smem + SM::OFF_X + sx * X_STAGE));
         for (int t = 0; t < pp; ++t, ++i) {
           if constexpr (BITS == 16) {
             // A (fp16 weights) straight from the W stage: two SW128 [128 x 64] tiles
             const int sw = i % S_W, rw = i / S_W;
-            mbar_wait(&full_w[sw], rw & 1);
+            mbar_wait_park(&full_w[sw], rw & 1);
             tc_fence_after();
             trace_ev(p, 3, i);
             if (elect_one()) {
@@ -269,16 +269,18 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             continue;
           }
           const int sa = i % S_A, ra = i / S_A;
-          mbar_wait(&full_a[sa], ra & 1);
+          mbar_wait_park(&full_a[sa], ra & 1);
           tc_fence_after();
           trace_ev(p, 3, i);
           if (elect_one()) {
             const uint32_t d_tm = tmem + D_COL + t * BT;
             const uint32_t a_tm = tmem + A_COL + sa * 64 * UG;
+            if (!(p.abl & 2)) {
 #pragma unroll
-            for (int kk = 0; kk < 8 * UG; ++kk)
-              tc_mma_ts(d_tm, a_tm + kk * 8, bdesc0 + (uint64_t)(((kk >> 2) * X_BLOCK + (kk & 3) * 32) >> 4),
-                        kIdescTc, (j == j0 && kk == 0) ? 0u : 1u);
+              for (int kk = 0; kk < 8 * UG; ++kk)
+                tc_mma_ts(d_tm, a_tm + kk * 8, bdesc0 + (uint64_t)(((kk >> 2) * X_BLOCK + (kk & 3) * 32) >> 4),
+                          kIdescTc, (j == j0 && kk == 0) ? 0u : 1u);
+            }
             tc_commit(&empty_a[sa]);
             if (t == pp - 1) {
               tc_commit(&empty_x[sx]);
@@ -307,14 +309,15 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const bool tr = (warp == 2 && lane == 0);
     int sw = 0, pw = 0, sa = 0, pa = 0;  // ring slots and phases
     for (int i = 0; i < nunits; ++i) {
-      mbar_wait(&full_w[sw], pw);
+      mbar_wait_park(&full_w[sw], pw);
       if (tr) trace_ev(p, 1, i);
-      mbar_wait(&empty_a[sa], pa ^ 1);
+      mbar_wait_park(&empty_a[sa], pa ^ 1);
       if (tr) trace_ev(p, 5, i);
       tc_fence_after();
       const uint32_t meta = reinterpret_cast<const uint32_t*>(smem + SM::OFF_META + sw * BN * 4 * UG)[ru];
-      dequant_row_batches<BITS, NBW < 4 ? NBW : 4>(smem + SM::OFF_W + sw * SM::W_STAGE, meta, r,
-                                                   tmem + lane_base + A_COL + sa * 64 * UG + gg * 64, ru * GB, b0);
+      if (!(p.abl & 1))
+        dequant_row_batches<BITS, NBW < 4 ? NBW : 4>(smem + SM::OFF_W + sw * SM::W_STAGE, meta, r,
+                                                     tmem + lane_base + A_COL + sa * 64 * UG + gg * 64, ru * GB, b0);
       if (tr) trace_ev(p, 12, i);
       tc_wait_st();
       tc_fence_before();
@@ -378,51 +381,34 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   if (threadIdx.x == 0) trace_cta(p, 11);
   if (npend > 0) {
     __threadfence();
-    constexpr uint32_t tile_bytes = BT * BN * 4;
-    float* sred = reinterpret_cast<float*>(smem);
-    const int batch = (int)(SM::OFF_BAR / (tile_bytes * Z)) < PMAX ? (int)(SM::OFF_BAR / (tile_bytes * Z)) : PMAX;
-    int use = 0;  // red_bar[b] completes once per batch
+    // every thread: 4 consecutive rows of one token per step, the Z partials summed in z order
     for (int e = 0; e < npend; ++e) {
       const int pn = (int)misc[2 + e], pp = tiles_of(pn);
-      for (int t0 = 0; t0 < pp; t0 += batch, ++use) {
-        const int nb = pp - t0 < batch ? pp - t0 : batch;
-        if (threadIdx.x == 0) {  // all of the batch's partial tiles in flight at once, one barrier per tile
-          for (int b = 0; b < nb; ++b) {
-            mbar_arrive_expect_tx(&red_bar[b], tile_bytes * Z);
-            for (int z = 0; z < Z; ++z)
-              bulk_load(smem + (b * Z + z) * tile_bytes,
-                        p.part + ((int64_t)(pn * Z + z) * PMAX + t0 + b) * BT * BN, tile_bytes, &red_bar[b]);
-          }
+      for (int idx = threadIdx.x; idx < pp * BT * (BN / 4); idx += NUM_THREADS) {
+        const int t = idx / (BT * (BN / 4)), rem = idx - t * (BT * (BN / 4));
+        const int tok = rem / (BN / 4), r4 = (rem % (BN / 4)) * 4;
+        if (tok >= p.m) continue;
+        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+        for (int z = 0; z < Z; ++z) {
+          const float4 v = __ldcg(reinterpret_cast<const float4*>(
+              p.part + (((int64_t)(pn * Z + z) * PMAX + t) * BT + tok) * BN + r4));
+          acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
         }
-        for (int b = 0; b < nb; ++b) {
-          mbar_wait(&red_bar[b], use & 1);
-          if (threadIdx.x == 0 && b == 0 && e == 0 && t0 == 0) trace_cta(p, 10);
-          if (threadIdx.x == 0 && b == 1 && e == 0 && t0 == 0) trace_cta(p, 6);
-          if (threadIdx.x == 0 && b == 3 && e == 0 && t0 == 0) trace_cta(p, 7);
-          const int64_t row0 = (int64_t)(pn * P + t0 + b) * BN;
-          const float* sp_ = sred + b * Z * BT * BN;
-          for (int th = threadIdx.x; th < 4 * BN; th += NUM_THREADS) {  // (row, token phase): 8 tokens each
-            const int rr = th % BN, tq = th / BN;
-            const float bias = p.bias ? __half2float(p.bias[row0 + rr]) : 0.f;
+        const int64_t row0 = (int64_t)(pn * P + t) * BN + r4;
+        float o[4] = {acc.x, acc.y, acc.z, acc.w};
+        if (p.bias) {
 #pragma unroll
-            for (int u = 0; u < BT / 4; ++u) {
-              const int tok = tq + 4 * u;
-              if (tok < p.m) {
-                float acc = 0.f;
-                for (int z = 0; z < Z; ++z) acc += sp_[z * BT * BN + tok * BN + rr];
-                acc += bias;
-                if constexpr (EPI == SQ_EPI_F32_ACCUM) {
-                  static_cast<float*>(p.y)[(int64_t)tok * p.ldy + row0 + rr] += acc;
-                } else {
-                  static_cast<__half*>(p.y)[(int64_t)tok * p.ldy + row0 + rr] = __float2half_rn(apply_act<EPI>(acc));
-                }
-              }
-            }
-          }
+          for (int c = 0; c < 4; ++c) o[c] += __half2float(p.bias[row0 + c]);
         }
-        if (threadIdx.x == 0 && e == 0 && t0 == 0) trace_cta(p, 9);
-        __syncthreads();  // staging reuse
-        if (threadIdx.x == 0 && e == 0 && t0 == 0) trace_cta(p, 13);
+        if constexpr (EPI == SQ_EPI_F32_ACCUM) {
+          float* yp = static_cast<float*>(p.y) + (int64_t)tok * p.ldy + row0;
+#pragma unroll
+          for (int c = 0; c < 4; ++c) yp[c] += o[c];
+        } else {
+          __half* yp = static_cast<__half*>(p.y) + (int64_t)tok * p.ldy + row0;
+#pragma unroll
+          for (int c = 0; c < 4; ++c) yp[c] = __float2half_rn(apply_act<EPI>(o[c]));
+        }
       }
     }
   }
@@ -496,22 +482,12 @@ cudaError_t launch_tc_b(const CUtensorMap& tx, const CUtensorMap& tw, const CUte
 // UG: groups per unit -- a ~16-KB weight stage (INT3/INT4 two groups when k/128 is even)
 int tc_ug(int bits, int kg) { return (bits <= 4 && kg % 2 == 0) ? 2 : 1; }
 
-int tc_zmax(int bits, int ug) {
-  switch (bits * 4 + ug) {
-    case 3 * 4 + 1: return DSmem<3, 1>::ZMAX;
-    case 3 * 4 + 2: return DSmem<3, 2>::ZMAX;
-    case 4 * 4 + 1: return DSmem<4, 1>::ZMAX;
-    case 4 * 4 + 2: return DSmem<4, 2>::ZMAX;
-    case 16 * 4 + 1: return DSmem<16, 1>::ZMAX;
-    default: return DSmem<8, 1>::ZMAX;
-  }
-}
-
 struct TcPlan { int P, Z, I, ctas; };
 
 // Panel width P and k split Z: minimise the bytes the busiest SM ingests -- weights + meta,
 // activation slices (once per k-step per panel, 32 token rows) and, for Z > 1, the Z partial
-// tiles the finishing CTA reads back -- over ceil(items / SMs) rounds.
+// tiles the finishing CTA reads back (weighted by their measured slowness) -- over
+// ceil(items / SMs) rounds.
 TcPlan tc_plan(int64_t n, int64_t k, int bits) {
   const int64_t nt = n / BN, kg = k / 128;
   const int ug = tc_ug(bits, (int)kg);
@@ -519,13 +495,15 @@ TcPlan tc_plan(int64_t n, int64_t k, int bits) {
   const double unit_w = BN * ug * 128.0 * bits / 8 + (bits == 16 ? 0.0 : BN * 4.0 * ug), unit_x = ug * 128.0 * BT * 2;
   TcPlan best{1, 1, 0, 0};
   double best_cost = 1e300;
-  const int zmax = tc_zmax(bits, ug);
+  constexpr int zmax = 8;
   for (int P = 1; P <= PMAX; ++P) {
     for (int Z = 1; Z <= zmax && Z <= ks; ++Z) {
       const int64_t I = ((nt + P - 1) / P) * Z, rounds = (I + C - 1) / C;
       if (Z > 1 && rounds > 62) continue;  // pending-panel list of the fix-up
       const int64_t steps = (ks + Z - 1) / Z;
-      const double cost = rounds * (steps * (P * unit_w + unit_x) + (Z > 1 ? Z * P * (double)BT * BN * 4 : 0.0));
+      // the fix-up's partial tiles come back at ~1/8 of the streaming rate (measured: bulk copies of
+      // another CTA's fresh partials land at ~14 GB/s per SM), so they are weighted 8x
+      const double cost = rounds * (steps * (P * unit_w + unit_x) + (Z > 1 ? 8.0 * Z * P * (double)BT * BN * 4 : 0.0));
       if (cost < best_cost * 0.999) { best_cost = cost; best = {P, Z, (int)I, (int)(I < C ? I : C)}; }
     }
   }
@@ -600,6 +578,11 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
   p.cnt = reinterpret_cast<int*>(base);
   p.part = reinterpret_cast<float*>(base + kCntBytes);
   p.trace = g_trace;
+  {
+    static int abl = -1;
+    if (abl < 0) { const char* e = getenv("SQ_TC_ABL"); abl = e ? atoi(e) : 0; }
+    p.abl = abl;
+  }
   const int nc = pl.ctas;
   const double bytes = (double)w.n * w.k * w.bits / 8.0 + (w.bits != 16 ? (double)w.n * (w.k / 128) * 4.0 : 0.0);
   auto t = prof_begin(KC_GEMV, bytes, 2.0 * m * w.n * w.k, s);
