@@ -168,6 +168,12 @@ def run_reference(args, wl):
 
 
 # ------------------------------------------------------------------ decode GEMV sweep (configs[1])
+def flush_l2(buf):
+    # evict L2 by READING a 2 x L2 buffer: a write flush leaves ~126 MB of dirty lines whose
+    # write-back then runs inside the timed kernel (measured: ~13 us on every launch)
+    buf.sum()
+
+
 def gemv_sweep(reps=10):
     import torch
     import synth
@@ -175,14 +181,14 @@ def gemv_sweep(reps=10):
     pk = peaks()
     dev = torch.device("cuda")
     l2 = torch.cuda.get_device_properties(0).L2_cache_size
-    flush = torch.empty(2 * l2 // 4 + 1024, dtype=torch.float32, device=dev)
+    flush = torch.zeros(2 * l2 // 4 + 1024, dtype=torch.float32, device=dev)
     out = []
     for (n, k) in ((5120, 5120), (20480, 5120), (5120, 20480)):
         wd = torch.empty((n, k), dtype=torch.float16, device=dev)
         synth.device_weight_f16(wd.data_ptr(), 4242, n, k)
         for bits in (3, 4, 8):
             q = sq.QLinear.from_fp16(wd, bits)
-            for m in (1, 8):
+            for m in (1, 8, 32):
                 x = torch.randn(m, k, device=dev).half()
                 y = torch.empty(m, n, device=dev, dtype=torch.float16)
                 ws = torch.zeros(sq.sq_linear_workspace_bytes(q, m), dtype=torch.uint8, device=dev)
@@ -191,7 +197,10 @@ def gemv_sweep(reps=10):
                     sq.sq_linear_decode(q, x, y, 0, xsum=xs, ws=ws)
                 ts = []
                 for _ in range(reps):
-                    flush.zero_()
+                    flush_l2(flush)
+                    # keep the GPU busy while the host marshals the launch, so the events
+                    # time the kernel and not the host call
+                    torch.cuda._sleep(200_000)
                     e0 = torch.cuda.Event(enable_timing=True)
                     e1 = torch.cuda.Event(enable_timing=True)
                     e0.record()

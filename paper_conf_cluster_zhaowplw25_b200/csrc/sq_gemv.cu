@@ -167,6 +167,87 @@ __device__ __forceinline__ int range_lo(int i, int total, int parts) {
   return (int)(((long long)i * total) / parts);
 }
 
+// CTA-level reduction of split tiles (fixed warp order), then cross-CTA fix-up: a tile that
+// straddles two CTAs is finished by the last CTA to arrive (atomic counter), summing the CTA
+// partials in fixed CTA order.  Deterministic; counters self-reset.
+template <int TOK, int EPI>
+__device__ __forceinline__ void reduce_tail(const GemvP& p, const float* part_s, int C0, int C1, int R, int warp,
+                                            int lane, int g, int q) {
+  constexpr int NJ = NT<TOK>::v;
+  const int kg = p.kg;
+  if (R <= 0) return;
+  const int t_first = C0 / kg, t_last = (C1 - 1) / kg;
+  for (int t = t_first + warp; t <= t_last; t += kWarps) {
+    const int lo = t * kg > C0 ? t * kg : C0;
+    const int hi = (t + 1) * kg < C1 ? (t + 1) * kg : C1;  // exclusive
+    const int wa = (int)(((long long)(lo - C0 + 1) * kWarps - 1) / R);
+    const int wb = (int)(((long long)(hi - C0) * kWarps - 1) / R);
+    if (wa == wb && lo == t * kg && hi == (t + 1) * kg) continue;  // one warp stored it directly
+    float v[NJ][4];
+#pragma unroll
+    for (int j = 0; j < NJ; ++j)
+#pragma unroll
+      for (int i = 0; i < 4; ++i) v[j][i] = 0.f;
+    for (int wi = wa; wi <= wb; ++wi) {
+      const int wlo = C0 + range_lo(wi, R, kWarps), whi = C0 + range_lo(wi + 1, R, kWarps);
+      if (whi <= wlo) continue;  // empty warp range
+      const int sl = (wlo < t * kg) ? 1 : 0;
+      const float* qp = part_s + ((wi * 2 + sl) * TOK) * kRows;
+#pragma unroll
+      for (int j = 0; j < NJ; ++j)
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+          const int tok = 8 * j + 2 * q + e;
+          v[j][e] += qp[tok * kRows + g];
+          v[j][2 + e] += qp[tok * kRows + g + 8];
+        }
+    }
+    if (lo == t * kg && hi == (t + 1) * kg) {  // tile entirely inside this CTA
+      store_out<TOK, EPI>(p, t, g, q, v);
+      continue;
+    }
+    // straddles a CTA boundary: publish this CTA's partial, the last CTA reduces
+    const int cslot = (C0 < t * kg) ? 1 : 0;
+    float* gp = p.part + (((int64_t)blockIdx.x * 2 + cslot) * TOK) * kRows;
+#pragma unroll
+    for (int j = 0; j < NJ; ++j)
+#pragma unroll
+      for (int e = 0; e < 2; ++e) {
+        const int tok = 8 * j + 2 * q + e;
+        __stcg(gp + tok * kRows + g, v[j][e]);
+        __stcg(gp + tok * kRows + g + 8, v[j][2 + e]);
+      }
+    __threadfence();
+    __syncwarp();
+    const int NC = gridDim.x;
+    const int ca = (int)(((long long)(t * kg + 1) * NC - 1) / p.U);
+    const int cb2 = (int)(((long long)((t + 1) * kg) * NC - 1) / p.U);
+    int old = 0;
+    if (lane == 0) old = atomicAdd(p.cnt + t, 1);
+    old = __shfl_sync(0xffffffff, old, 0);
+    if (old != cb2 - ca) continue;
+    __threadfence();
+#pragma unroll
+    for (int j = 0; j < NJ; ++j)
+#pragma unroll
+      for (int i = 0; i < 4; ++i) v[j][i] = 0.f;
+    for (int c = ca; c <= cb2; ++c) {
+      const int sl = (range_lo(c, p.U, NC) < t * kg) ? 1 : 0;
+      const float* qp = p.part + (((int64_t)c * 2 + sl) * TOK) * kRows;
+#pragma unroll
+      for (int j = 0; j < NJ; ++j)
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+          const int tok = 8 * j + 2 * q + e;
+          v[j][e] += __ldcg(qp + tok * kRows + g);
+          v[j][2 + e] += __ldcg(qp + tok * kRows + g + 8);
+        }
+    }
+    store_out<TOK, EPI>(p, t, g, q, v);
+    if (lane == 0) p.cnt[t] = 0;
+  }
+}
+
 template <int BITS, int TOK, int EPI>
 __global__ void __launch_bounds__(kThreads, 1) k_gemv(const GemvP p) {
   constexpr int LU = Cfg<BITS>::LU;
@@ -344,78 +425,202 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemv(const GemvP p) {
   }
   __syncthreads();
 
-  // ---- CTA-level reduction of split tiles (fixed warp order), then cross-CTA fix-up
-  if (R <= 0) return;
-  const int t_first = C0 / kg, t_last = (C1 - 1) / kg;
-  for (int t = t_first + warp; t <= t_last; t += kWarps) {
-    const int lo = t * kg > C0 ? t * kg : C0;
-    const int hi = (t + 1) * kg < C1 ? (t + 1) * kg : C1;  // exclusive
-    const int wa = (int)(((long long)(lo - C0 + 1) * kWarps - 1) / R);
-    const int wb = (int)(((long long)(hi - C0) * kWarps - 1) / R);
-    if (wa == wb && lo == t * kg && hi == (t + 1) * kg) continue;  // one warp stored it directly
-    float v[NJ][4];
-#pragma unroll
-    for (int j = 0; j < NJ; ++j)
-#pragma unroll
-      for (int i = 0; i < 4; ++i) v[j][i] = 0.f;
-    for (int wi = wa; wi <= wb; ++wi) {
-      const int wlo = C0 + range_lo(wi, R, kWarps), whi = C0 + range_lo(wi + 1, R, kWarps);
-      if (whi <= wlo) continue;  // empty warp range
-      const int sl = (wlo < t * kg) ? 1 : 0;
-      const float* qp = part_s + ((wi * 2 + sl) * TOK) * kRows;
-#pragma unroll
-      for (int j = 0; j < NJ; ++j)
-#pragma unroll
-        for (int e = 0; e < 2; ++e) {
-          const int tok = 8 * j + 2 * q + e;
-          v[j][e] += qp[tok * kRows + g];
-          v[j][2 + e] += qp[tok * kRows + g + 8];
-        }
-    }
-    if (lo == t * kg && hi == (t + 1) * kg) {  // tile entirely inside this CTA
-      store_out<TOK, EPI>(p, t, g, q, v);
-      continue;
-    }
-    // straddles a CTA boundary: publish this CTA's partial, the last CTA reduces
-    const int cslot = (C0 < t * kg) ? 1 : 0;
-    float* gp = p.part + (((int64_t)blockIdx.x * 2 + cslot) * TOK) * kRows;
-#pragma unroll
-    for (int j = 0; j < NJ; ++j)
-#pragma unroll
-      for (int e = 0; e < 2; ++e) {
-        const int tok = 8 * j + 2 * q + e;
-        __stcg(gp + tok * kRows + g, v[j][e]);
-        __stcg(gp + tok * kRows + g + 8, v[j][2 + e]);
-      }
-    __threadfence();
-    __syncwarp();
-    const int NC = gridDim.x;
-    const int ca = (int)(((long long)(t * kg + 1) * NC - 1) / p.U);
-    const int cb2 = (int)(((long long)((t + 1) * kg) * NC - 1) / p.U);
-    int old = 0;
-    if (lane == 0) old = atomicAdd(p.cnt + t, 1);
-    old = __shfl_sync(0xffffffff, old, 0);
-    if (old != cb2 - ca) continue;
-    __threadfence();
-#pragma unroll
-    for (int j = 0; j < NJ; ++j)
-#pragma unroll
-      for (int i = 0; i < 4; ++i) v[j][i] = 0.f;
-    for (int c = ca; c <= cb2; ++c) {
-      const int sl = (range_lo(c, p.U, NC) < t * kg) ? 1 : 0;
-      const float* qp = p.part + (((int64_t)c * 2 + sl) * TOK) * kRows;
-#pragma unroll
-      for (int j = 0; j < NJ; ++j)
-#pragma unroll
-        for (int e = 0; e < 2; ++e) {
-          const int tok = 8 * j + 2 * q + e;
-          v[j][e] += __ldcg(qp + tok * kRows + g);
-          v[j][2 + e] += __ldcg(qp + tok * kRows + g + 8);
-        }
-    }
-    store_out<TOK, EPI>(p, t, g, q, v);
-    if (lane == 0) p.cnt[t] = 0;
+  reduce_tail<TOK, EPI>(p, part_s, C0, C1, R, warp, lane, g, q);
+}
+
+// ---------------------------------------------------------------- K2 with a bulk-copy SMEM ring
+// Quantized weights (placement T16): a warp's unit range is ONE contiguous byte range (and so is
+// its meta), so each warp streams it with cp.async.bulk into its own S-slot shared-memory ring
+// (CH units per slot, one mbarrier per slot, lane 0 issues): ~150 KB in flight per SM instead of
+// the 4-unit register ring, decoupling HBM latency from the warps.  Unpack, mma.sync, the
+// factorised scale/zero and the reductions are those of k_gemv.
+template <int BITS, int TOK>
+struct QRing {
+  static constexpr int UB = 16 * Cfg<BITS>::GB;                   // codes bytes per unit
+  static constexpr int UM = 64;                                   // meta bytes per unit
+  static constexpr int PART = kWarps * 2 * TOK * kRows * 4;      // split-tile partials
+  static constexpr int BARS = kWarps * 8 * 8;                     // <= 8 mbarriers per warp
+  static constexpr int CH = BITS == 8 ? 2 : (BITS == 4 ? 3 : 4);  // units per slot (3.3-4.2 KB)
+  static constexpr int SLOT = CH * (UB + UM);
+  static constexpr int S0 = (227 * 1024 - PART - BARS - 128) / kWarps / SLOT;
+  static constexpr int S = S0 > 8 ? 8 : S0;
+  static constexpr int BYTES = PART + BARS + kWarps * S * SLOT;
+  static_assert(S >= 2, "ring depth");
+  static_assert(BYTES <= 227 * 1024, "shared memory budget");
+};
+
+// this lane's codes of one row of the unit in shared memory (p = row start + lane offset)
+template <int BITS>
+__device__ __forceinline__ void lds_codes(const uint8_t* p, uint32_t* c) {
+  if constexpr (BITS == 4) {
+    const uint4 v = *reinterpret_cast<const uint4*>(p);
+    c[0] = v.x; c[1] = v.y; c[2] = v.z; c[3] = v.w;
+  } else if constexpr (BITS == 8) {
+    // k in [16q, 16q+16) and [64+16q, 64+16q+16): conflict-free 16-B phases
+    const uint4 v0 = *reinterpret_cast<const uint4*>(p), v1 = *reinterpret_cast<const uint4*>(p + 64);
+    c[0] = v0.x; c[1] = v0.y; c[2] = v0.z; c[3] = v0.w;
+    c[4] = v1.x; c[5] = v1.y; c[6] = v1.z; c[7] = v1.w;
+  } else {
+    const uint32_t* w = reinterpret_cast<const uint32_t*>(p);
+    c[0] = w[0]; c[1] = w[1]; c[2] = w[2];
   }
+}
+
+template <int BITS, int TOK, int EPI>
+__global__ void __launch_bounds__(kThreads, 1) k_gemv_q(const GemvP p) {
+  using RC = QRing<BITS, TOK>;
+  constexpr int LU = Cfg<BITS>::LU;
+  constexpr int GB = Cfg<BITS>::GB;
+  constexpr int NJ = NT<TOK>::v;
+  constexpr int CH = RC::CH, S = RC::S, UB = RC::UB, SLOT = RC::SLOT;
+  extern __shared__ float4 smem4[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>(smem4);
+  float* part_s = reinterpret_cast<float*>(smem);  // [16 warps][2][TOK][16]
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + RC::PART) + (threadIdx.x >> 5) * 8;
+
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31, g = lane >> 2, q = lane & 3;
+  const int kg = p.kg, m = p.m;
+  const int C0 = range_lo(blockIdx.x, p.U, gridDim.x), C1 = range_lo(blockIdx.x + 1, p.U, gridDim.x);
+  const int R = C1 - C0;
+  const int u0 = C0 + range_lo(warp, R, kWarps), u1 = C0 + range_lo(warp + 1, R, kWarps);
+  const int nunits = u1 - u0;
+  const int head_tile = u0 / kg;
+  const int grp0 = u0 - head_tile * kg;
+  uint8_t* ring = smem + RC::PART + RC::BARS + warp * S * SLOT;
+
+  // ---- the warp's own ring: lane 0 initialises its barriers and keeps S slots in flight
+  const int nch = (nunits + CH - 1) / CH;
+  auto issue = [&](int c) {
+    const int slot = c % S;
+    const int nu = nunits - c * CH < CH ? nunits - c * CH : CH;
+    const int64_t u = (int64_t)u0 + (int64_t)c * CH;
+    mbar_arrive_expect_tx(&bar[slot], (uint32_t)(nu * (UB + 64)));
+    bulk_load(ring + slot * SLOT, p.packed + u * UB, (uint32_t)(nu * UB), &bar[slot]);
+    bulk_load(ring + slot * SLOT + CH * UB, p.meta + u * 16, (uint32_t)(nu * 64), &bar[slot]);
+  };
+  if (lane == 0) {
+    for (int i = 0; i < S; ++i) mbar_init(&bar[i], 1);
+    fence_barrier_init();
+    for (int c = 0; c < S && c < nch; ++c) issue(c);
+  }
+  __syncwarp();
+
+  // activation fragment pointers for token n8-tile j: row 8j + g (predicated off beyond m); the
+  // lane's k set matches its codes: [32q, 32q+32) (INT3/INT4) or [16q,16q+16) u [64+16q, 80+16q) (INT8)
+  const int xq = BITS == 8 ? q * 16 : q * 32;
+  const __half* xrow[NJ];
+  bool xon[NJ];
+#pragma unroll
+  for (int j = 0; j < NJ; ++j) {
+    xon[j] = (8 * j + g) < m;
+    xrow[j] = p.x + (int64_t)(xon[j] ? 8 * j + g : 0) * p.ldx + xq;
+  }
+  uint32_t xt1[16];
+#pragma unroll
+  for (int i = 0; i < 16; ++i) xt1[i] = 0u;
+
+  int tile = head_tile, grp = grp0;
+  bool seg_from_start = (grp0 == 0);
+  float acc[NJ][4];
+#pragma unroll
+  for (int j = 0; j < NJ; ++j)
+#pragma unroll
+    for (int i = 0; i < 4; ++i) acc[j][i] = 0.f;
+  const int lane_off = BITS == 8 ? q * 16 : q * lane_bytes<BITS>();
+
+  for (int c = 0; c < nch; ++c) {
+    const int slot = c % S;
+    mbar_wait(&bar[slot], (uint32_t)((c / S) & 1));
+    const uint8_t* cs = ring + slot * SLOT;
+    const uint32_t* ms = reinterpret_cast<const uint32_t*>(cs + CH * UB);
+#pragma unroll
+    for (int s = 0; s < CH; ++s) {
+      const int ui = c * CH + s;
+      if (ui >= nunits) break;
+      uint32_t cw0[LU], cw1[LU];
+      lds_codes<BITS>(cs + s * UB + g * GB + lane_off, cw0);
+      lds_codes<BITS>(cs + s * UB + (g + 8) * GB + lane_off, cw1);
+      const uint32_t mr0 = ms[s * 16 + g], mr1 = ms[s * 16 + g + 8];
+#pragma unroll
+      for (int j = 0; j < NJ; ++j) {
+        const __half* xp = xrow[j] + grp * 128;
+        uint32_t xloc[16];
+        uint32_t* xtj = NJ == 1 ? xt1 : xloc;
+        if (NJ > 1) {
+#pragma unroll
+          for (int i = 0; i < 16; ++i) xloc[i] = 0u;
+        }
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const int xo = BITS == 8 ? (i < 2 ? 8 * i : 64 + 8 * (i - 2)) : 8 * i;
+          ldg_v4_pred(xtj + 4 * i, xp + xo, xon[j]);
+        }
+        const float4 xsv = __ldg(reinterpret_cast<const float4*>(p.xsum + grp * kXsTok + 8 * j + 2 * q));
+        float d0[4], d1[4];  // two independent HMMA chains (even / odd chunks)
+        {
+          uint32_t a[4], b[4];
+          frag<BITS>(cw0, 0, a[0], a[2]);
+          frag<BITS>(cw1, 0, a[1], a[3]);
+          frag<BITS>(cw0, 1, b[0], b[2]);
+          frag<BITS>(cw1, 1, b[1], b[3]);
+          mma_16816_zc(d0, a, xtj[0], xtj[1]);
+          mma_16816_zc(d1, b, xtj[2], xtj[3]);
+        }
+#pragma unroll
+        for (int t = 2; t < 8; t += 2) {
+          uint32_t a[4], b[4];
+          frag<BITS>(cw0, t, a[0], a[2]);
+          frag<BITS>(cw1, t, a[1], a[3]);
+          frag<BITS>(cw0, t + 1, b[0], b[2]);
+          frag<BITS>(cw1, t + 1, b[1], b[3]);
+          mma_16816(d0, a, xtj[2 * t], xtj[2 * t + 1], d0);
+          mma_16816(d1, b, xtj[2 * t + 2], xtj[2 * t + 3], d1);
+        }
+        const float d[4] = {d0[0] + d1[0], d0[1] + d1[1], d0[2] + d1[2], d0[3] + d1[3]};
+        const float2 f0 = __half22float2(*reinterpret_cast<const __half2*>(&mr0));  // (s, z) row g
+        const float2 f1 = __half22float2(*reinterpret_cast<const __half2*>(&mr1));  // row g+8
+        // (xs, xoff) of tokens 2q, 2q+1: xs = sum x, xoff = sum off_k x
+        const float xs0 = xsv.x + xsv.y, xs1 = xsv.z + xsv.w;
+        const float xo0 = BITS == 4 ? fmaf(1024.f, xsv.x, 64.f * xsv.y) : (BITS == 3 ? 8.f * xs0 : 1024.f * xs0);
+        const float xo1 = BITS == 4 ? fmaf(1024.f, xsv.z, 64.f * xsv.w) : (BITS == 3 ? 8.f * xs1 : 1024.f * xs1);
+        // y += s * (D - xoff) + z * xs
+        acc[j][0] = fmaf(-f0.x, xo0, fmaf(f0.y, xs0, fmaf(f0.x, d[0], acc[j][0])));
+        acc[j][1] = fmaf(-f0.x, xo1, fmaf(f0.y, xs1, fmaf(f0.x, d[1], acc[j][1])));
+        acc[j][2] = fmaf(-f1.x, xo0, fmaf(f1.y, xs0, fmaf(f1.x, d[2], acc[j][2])));
+        acc[j][3] = fmaf(-f1.x, xo1, fmaf(f1.y, xs1, fmaf(f1.x, d[3], acc[j][3])));
+      }
+
+      // ---- segment end: row tile finished or this warp's run finished
+      const bool tile_end = (grp == kg - 1);
+      if (tile_end || ui == nunits - 1) {
+        if (seg_from_start && tile_end) {
+          store_out<TOK, EPI>(p, tile, g, q, acc);
+        } else {
+          const int sl = (tile == head_tile) ? 0 : 1;  // head / tail tile of this warp
+          float* pp = part_s + ((warp * 2 + sl) * TOK) * kRows;
+#pragma unroll
+          for (int j = 0; j < NJ; ++j)
+#pragma unroll
+            for (int e = 0; e < 2; ++e) {
+              const int tok = 8 * j + 2 * q + e;
+              pp[tok * kRows + g] = acc[j][e];
+              pp[tok * kRows + g + 8] = acc[j][2 + e];
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < NJ; ++j)
+#pragma unroll
+          for (int i = 0; i < 4; ++i) acc[j][i] = 0.f;
+        seg_from_start = true;
+      }
+      if (++grp == kg) { grp = 0; ++tile; }
+    }
+    __syncwarp();  // every lane's reads of this slot are done (their values fed the MMAs)
+    if (lane == 0 && c + S < nch) issue(c + S);
+  }
+  __syncthreads();
+  reduce_tail<TOK, EPI>(p, part_s, C0, C1, R, warp, lane, g, q);
 }
 
 // xsum[g][t] = (sum_{k%4<2} x[t,k], sum_{k%4>=2} x[t,k]) over group g, t < 32 (0 for t >= m);
@@ -444,8 +649,15 @@ size_t gemv_smem(int tok, int kg) { return (size_t)kWarps * 2 * tok * kRows * 4 
 
 template <int BITS, int TOK, int EPI>
 cudaError_t launch_e(const GemvP& p, cudaStream_t s) {
-  auto kern = k_gemv<BITS, TOK, EPI>;
-  const size_t smem = gemv_smem(TOK, p.kg);
+  void (*kern)(const GemvP);
+  size_t smem;
+  if constexpr (BITS == 16) {
+    kern = k_gemv<BITS, TOK, EPI>;
+    smem = gemv_smem(TOK, p.kg);
+  } else {
+    kern = k_gemv_q<BITS, TOK, EPI>;
+    smem = (size_t)QRing<BITS, TOK>::BYTES;
+  }
   static size_t attr = 0;
   if (smem > attr) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -500,7 +712,7 @@ size_t gemv_workspace_bytes(int64_t n, int64_t k, int64_t m) {
 }
 
 // K2 (mma.sync, register unpack) for m <= 8; K2c (tcgen05: TMEM dequant, or fp16 weights straight
-// from SMEM) for 8 < m <= 32.
+// from SMEM) for 8 < m <= 32.  K2 takes the activation group sums (xsum; computed here if null).
 // SQ_GEMV_PATH=mma|tc overrides (benchmarking).
 int gemv_path(int64_t n, int m, int bits) {
   static int forced = -2;

@@ -45,7 +45,11 @@ constexpr int BT = 32;      // token columns (MMA N)
 constexpr int PMAX = 4;     // row tiles per panel (activation reuse), at most
 constexpr int XK = 64;
 constexpr int X_BLOCK = BT * XK * 2;  // 4 KB: [32 tokens][64 k] SW128 tile
-constexpr int DQ_WARPS = 8;           // dequant warps: 2 per TMEM lane quadrant, each half of the unit's k
+#ifndef SQ_TC_DQ_WARPS
+#define SQ_TC_DQ_WARPS 16
+#endif
+constexpr int DQ_WARPS = SQ_TC_DQ_WARPS;  // dequant warps, in DQ_GROUPS groups of 8
+constexpr int DQ_GROUPS = DQ_WARPS / 8;    // group q dequantizes units i = q (mod DQ_GROUPS)
 constexpr int TMEM_COLS = 512;
 constexpr int D_COL = 0;              // P x 32 columns: the panel's accumulators
 constexpr int A_COL = PMAX * BT;      // S_A x (64 * UG) columns
@@ -58,12 +62,14 @@ constexpr int X_LAG = 1;              // activations of step q are fetched after
 template <int BITS, int UG>
 struct DCfg {
   // weight ring: a slot lives TMA latency (~1.8k cycles) + wait for its group + dequant (~2k)
-  static constexpr int S_W = BITS == 16 ? 5 : (UG == 2 ? 9 : (BITS == 8 ? 9 : (BITS == 4 ? 18 : 24)));
+  // (quantized rings are multiples of DQ_GROUPS so each slot is owned by one dequant group)
+  static constexpr int S_W = BITS == 16 ? 5 : (UG == 2 ? 10 : (BITS == 8 ? 10 : (BITS == 4 ? 18 : 24)));
   // TMEM A slots of 64*UG columns: the dequant warps fill slot i % S_A while the MMA reads the
-  // others (128 + 3 * 128 = 512 columns at UG = 2)
-  static constexpr int S_A = UG == 2 ? 3 : 6;
+  // others (slots are owned by one dequant group: multiples of DQ_GROUPS)
+  static constexpr int A_SLOT = 64 * UG;
+  static constexpr int S_A = UG == 2 ? 2 : 6;
   static constexpr int S_X = 3;  // activation ring, in steps
-  static_assert(A_COL + S_A * 64 * UG <= TMEM_COLS, "TMEM budget");
+  static_assert(BITS == 16 || A_COL + S_A * A_SLOT <= TMEM_COLS, "TMEM budget");
 };
 
 template <int BITS, int UG>
@@ -103,12 +109,15 @@ struct TcP {
   int abl;                    // debug ablation (SQ_TC_ABL): 1 = no dequant, 2 = no MMAs (results wrong)
 };
 
+#ifndef SQ_TC_DEBUG
+#define SQ_TC_DEBUG 0  // 1: clock64 trace (sq_debug_trace) and SQ_TC_ABL ablations compiled in
+#endif
 __device__ __forceinline__ void trace_ev(const TcP& p, int ev, int i) {
-  if (p.trace && blockIdx.x == 0 && i < 256) p.trace[ev * 256 + i] = clock64();
+  if (SQ_TC_DEBUG && p.trace && blockIdx.x == 0 && i < 256) p.trace[ev * 256 + i] = clock64();
 }
 
 __device__ __forceinline__ void trace_cta(const TcP& p, int ev) {
-  if (p.trace && blockIdx.x < 256) {
+  if (SQ_TC_DEBUG && p.trace && blockIdx.x < 256) {
     uint64_t t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     p.trace[ev * 256 + blockIdx.x] = t;
@@ -169,8 +178,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   if (threadIdx.x == 0) {
     for (int i = 0; i < S_X; ++i) { mbar_init(&full_x[i], 1); mbar_init(&empty_x[i], 1); }
     // fp16 weights are the MMA's A operand straight from SMEM: the MMA commit frees the slot
-    for (int i = 0; i < S_W; ++i) { mbar_init(&full_w[i], 1); mbar_init(&empty_w[i], BITS == 16 ? 1 : DQ_WARPS); }
-    for (int i = 0; i < S_A; ++i) { mbar_init(&full_a[i], DQ_WARPS); mbar_init(&empty_a[i], 1); }
+    for (int i = 0; i < S_W; ++i) { mbar_init(&full_w[i], 1); mbar_init(&empty_w[i], BITS == 16 ? 1 : 8); }
+    for (int i = 0; i < S_A; ++i) { mbar_init(&full_a[i], 8); mbar_init(&empty_a[i], 1); }
     mbar_init(d_full, 1);
     mbar_init(d_empty, 4);
     misc[1] = 0;
@@ -274,8 +283,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           trace_ev(p, 3, i);
           if (elect_one()) {
             const uint32_t d_tm = tmem + D_COL + t * BT;
-            const uint32_t a_tm = tmem + A_COL + sa * 64 * UG;
-            if (!(p.abl & 2)) {
+            const uint32_t a_tm = tmem + A_COL + sa * DCfg<BITS, UG>::A_SLOT;
+            if (!(SQ_TC_DEBUG && (p.abl & 2))) {
 #pragma unroll
               for (int kk = 0; kk < 8 * UG; ++kk)
                 tc_mma_ts(d_tm, a_tm + kk * 8, bdesc0 + (uint64_t)(((kk >> 2) * X_BLOCK + (kk & 3) * 32) >> 4),
@@ -293,31 +302,37 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       }
     }
   } else if (warp < EPI_WARP0) {
-    // ---------------- dequant warps: thread = weight row (lane quadrant warp % 4); warp kh takes
-    // batches [kh*2*UG, kh*2*UG + 2*UG) of the unit's 4*UG 32-k batches.  All 8 warps work on
-    // every unit, so a unit's dequant latency is half of one warp's work.
+    // ---------------- dequant warps: DQ_GROUPS groups of 8; group dg takes units i = dg (mod
+    // DQ_GROUPS).  Thread = weight row (lane quadrant warp % 4); warp kh of the group takes batches
+    // [kh*2*UG, kh*2*UG + 2*UG) of the unit's 4*UG 32-k batches.  Slots of both rings are owned by
+    // one group (ring depths are multiples of DQ_GROUPS), so phases follow from i alone.
+    static_assert(BITS == 16 || (S_W % DQ_GROUPS == 0 && S_A % DQ_GROUPS == 0), "ring slots owned by one dequant group");
     int nunits = 0;
     if constexpr (BITS != 16)
       for (int it = blockIdx.x; it < I; it += C) nunits += (j1_of(it) - j0_of(it)) * tiles_of(it / Z);
     constexpr int NBW = 2 * UG;                              // batches per warp
     const int sp = warp & 3;
-    const int kh = (warp - 2) >> 2;
+    const int dg = (warp - 2) >> 3;
+    const int kh = ((warp - 2) >> 2) & 1;
     const int gg = (kh * NBW) >> 2, b0 = (kh * NBW) & 3;  // group of the unit and first batch in it
     const int r = sp * 32 + lane;
     const int ru = ((r >> 4) * UG + gg) * 16 + (r & 15);  // stage layout [tile][group][16 rows]
     const uint32_t lane_base = (uint32_t)(sp * 32) << 16;
     const bool tr = (warp == 2 && lane == 0);
-    int sw = 0, pw = 0, sa = 0, pa = 0;  // ring slots and phases
-    for (int i = 0; i < nunits; ++i) {
-      mbar_wait_park(&full_w[sw], pw);
+    for (int i = dg; i < nunits; i += DQ_GROUPS) {
+      const int sw = i % S_W, sa = i % S_A;
+      mbar_wait_park(&full_w[sw], (uint32_t)((i / S_W) & 1));
       if (tr) trace_ev(p, 1, i);
-      mbar_wait_park(&empty_a[sa], pa ^ 1);
+      mbar_wait_park(&empty_a[sa], (uint32_t)(((i / S_A) & 1) ^ 1));
       if (tr) trace_ev(p, 5, i);
       tc_fence_after();
       const uint32_t meta = reinterpret_cast<const uint32_t*>(smem + SM::OFF_META + sw * BN * 4 * UG)[ru];
-      if (!(p.abl & 1))
-        dequant_row_batches<BITS, NBW < 4 ? NBW : 4>(smem + SM::OFF_W + sw * SM::W_STAGE, meta, r,
-                                                     tmem + lane_base + A_COL + sa * 64 * UG + gg * 64, ru * GB, b0);
+      const uint32_t a_tm = tmem + lane_base + A_COL + sa * DCfg<BITS, UG>::A_SLOT;
+      if constexpr (BITS != 16) {
+        if (!(SQ_TC_DEBUG && (p.abl & 1)))
+          dequant_row_batches<BITS, NBW < 4 ? NBW : 4>(smem + SM::OFF_W + sw * SM::W_STAGE, meta, r,
+                                                       a_tm + gg * 64, ru * GB, b0);
+      }
       if (tr) trace_ev(p, 12, i);
       tc_wait_st();
       tc_fence_before();
@@ -327,8 +342,6 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         mbar_arrive(&full_a[sa]);
       }
       if (tr) trace_ev(p, 2, i);
-      if (++sw == S_W) { sw = 0; pw ^= 1; }
-      if (++sa == S_A) { sa = 0; pa ^= 1; }
     }
   } else {
     // ---------------- epilogue warps: drain each item's accumulators
@@ -339,7 +352,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     int n_item = 0;
     for (int it = blockIdx.x; it < I; it += C, ++n_item) {
       const int pn = it / Z, pp = tiles_of(pn);
-      mbar_wait_sleepy(d_full, n_item & 1);
+      mbar_wait_park(d_full, n_item & 1);
       tc_fence_after();
       for (int t = 0; t < pp; ++t) {
         float v[BT];
@@ -518,14 +531,21 @@ unsigned long long* g_trace = nullptr;
 // launch self-reset to 0, so consecutive linears of any n can share one workspace).
 constexpr size_t kCntBytes = (65536 / 16) * sizeof(int);
 
+size_t gemv_tc_xsum_offset(int64_t n, int64_t k);
+
+// [counters][partials: [items][PMAX tiles][32 x 128] fp32, worst case over the bit widths][xsum]
 size_t gemv_tc_workspace_bytes(int64_t n, int64_t k) {
-  // partials: [items][PMAX tiles][32 x 128] fp32, worst case over the bit widths
+  return gemv_tc_xsum_offset(n, k) + xsum_bytes(k) + 256;
+}
+
+// the activation group sums (when the caller passes none) follow the partials
+size_t gemv_tc_xsum_offset(int64_t n, int64_t k) {
   int64_t items = 0;
   for (int bits : {3, 4, 8, 16}) {
     const TcPlan pl = tc_plan(n, k, bits);
     if (pl.Z > 1 && pl.I > items) items = pl.I;
   }
-  return kCntBytes + (size_t)items * PMAX * BT * BN * sizeof(float) + 256;
+  return (kCntBytes + (size_t)items * PMAX * BT * BN * sizeof(float) + 255) / 256 * 256;
 }
 
 cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, int m, void* y, int64_t ldy, int epi,

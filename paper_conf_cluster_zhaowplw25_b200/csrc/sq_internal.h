@@ -35,6 +35,7 @@ cudaError_t launch_gemv(const sq_qweight& w, const __half* x, int64_t ldx, int m
                         const float2* xsum, void* ws, cudaStream_t s);
 
 size_t gemv_tc_workspace_bytes(int64_t n, int64_t k);
+size_t gemv_tc_xsum_offset(int64_t n, int64_t k);
 cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, int m, void* y, int64_t ldy, int epi,
                            void* ws, cudaStream_t s);
 int gemv_path(int64_t n, int m, int bits);  // 0 = mma.sync (K2), 1 = tcgen05 (K2c)

@@ -96,31 +96,34 @@ sq_status stage_forward(const sq_layer* layers, int n_layers, int phase, const f
   cudaError_t e = cudaSuccess;
   for (int l = 0; l < n_layers && e == cudaSuccess; ++l) {
     const sq_layer& L = layers[l];
+    // per-group activation sums only for linears on the mma.sync decode path (K2); the tcgen05
+    // decode (K2c) dequantizes the weights and needs none
     const bool q = L.bits != 16;
+    auto k2 = [&](const sq_qweight& w) { return dec && q && gemv_path(w.n, (int)T, w.bits) == 0; };
     const float* xr = (l == 0) ? x_in : x_out;
     const bool copy = (l == 0 && x_in != x_out);
     // a = LN(x) (layer 0 also initialises the residual buffer x_out = x_in)
-    e = launch_layernorm_f16(xr, T, h1, a16, (dec && q) ? xs : nullptr, copy ? x_in : nullptr, copy ? x_out : nullptr, s);
+    e = launch_layernorm_f16(xr, T, h1, a16, k2(L.qkv) ? xs : nullptr, copy ? x_in : nullptr, copy ? x_out : nullptr, s);
     if (e) break;
-    e = lin(L.qkv, a16, h1, qkv16, 3 * h1, SQ_EPI_F16, (dec && q) ? xs : nullptr);
+    e = lin(L.qkv, a16, h1, qkv16, 3 * h1, SQ_EPI_F16, k2(L.qkv) ? xs : nullptr);
     if (e) break;
     // attention stub: attn = v = qkv[:, 2h1:3h1] (R12)
     const __half* v = qkv16 + 2 * h1;
-    if (dec && q) {
+    if (k2(L.o)) {
       e = launch_xsum(v, 3 * h1, T, h1, xs, s);
       if (e) break;
     }
-    e = lin(L.o, v, 3 * h1, x_out, h1, SQ_EPI_F32_ACCUM, (dec && q) ? xs : nullptr);
+    e = lin(L.o, v, 3 * h1, x_out, h1, SQ_EPI_F32_ACCUM, k2(L.o) ? xs : nullptr);
     if (e) break;
-    e = launch_layernorm_f16(x_out, T, h1, a16, (dec && q) ? xs : nullptr, nullptr, nullptr, s);
+    e = launch_layernorm_f16(x_out, T, h1, a16, k2(L.fc1) ? xs : nullptr, nullptr, nullptr, s);
     if (e) break;
-    e = lin(L.fc1, a16, h1, u16, h2, L.act == 0 ? SQ_EPI_F16_RELU : SQ_EPI_F16_GELU, (dec && q) ? xs : nullptr);
+    e = lin(L.fc1, a16, h1, u16, h2, L.act == 0 ? SQ_EPI_F16_RELU : SQ_EPI_F16_GELU, k2(L.fc1) ? xs : nullptr);
     if (e) break;
-    if (dec && q) {
+    if (k2(L.fc2)) {
       e = launch_xsum(u16, h2, T, h2, xs, s);
       if (e) break;
     }
-    e = lin(L.fc2, u16, h2, x_out, h1, SQ_EPI_F32_ACCUM, (dec && q) ? xs : nullptr);
+    e = lin(L.fc2, u16, h2, x_out, h1, SQ_EPI_F32_ACCUM, k2(L.fc2) ? xs : nullptr);
     if (e) break;
     if (qkv_dbg && l == n_layers - 1)
       e = cudaMemcpyAsync(qkv_dbg, qkv16, (size_t)T * 3 * h1 * 2, cudaMemcpyDeviceToDevice, s);

@@ -1,6 +1,6 @@
 """Decode GEMV sweep (configs[1]: OPT-13B linear shapes, bits 3/4/8/16, M 1..32).
 
-L2 flushed between timed reps (write a 2 x L2 buffer); CUDA events on the launch
+L2 flushed between timed reps (read a 2 x L2 buffer); CUDA events on the launch
 stream; median of reps.  GB/s = algorithmic bytes (codes + meta) / time.
 """
 import argparse
@@ -15,16 +15,31 @@ import synth
 import paper_conf_cluster_zhaowplw25_b200 as sq
 
 
+def flush_l2(buf):
+    # evict L2 by READING a 2 x L2 buffer: a write flush leaves ~126 MB of dirty lines whose
+    # write-back then runs inside the timed kernel (measured: ~13 us on every launch)
+    if FLUSH == "write":
+        buf.zero_()
+    else:
+        buf.sum()
+
+
+FLUSH = "read"
+
+
 def main():
+    global FLUSH
     ap = argparse.ArgumentParser()
     ap.add_argument("--reps", type=int, default=20)
     ap.add_argument("--bits", default="3,4,8,16")
     ap.add_argument("--ms", default="1,8,32")
     ap.add_argument("--shapes", default="5120x5120,20480x5120,5120x20480")
+    ap.add_argument("--flush", default="read", choices=["read", "write"])
     a = ap.parse_args()
+    FLUSH = a.flush
     dev = torch.device("cuda")
     l2 = torch.cuda.get_device_properties(0).L2_cache_size
-    flush = torch.empty(2 * l2 // 4 + 1024, dtype=torch.float32, device=dev)
+    flush = torch.zeros(2 * l2 // 4 + 1024, dtype=torch.float32, device=dev)
     out = []
     for shp in a.shapes.split(","):
         n, k = map(int, shp.split("x"))
@@ -42,7 +57,10 @@ def main():
                     sq.sq_linear_decode(q, x, y, 0, xsum=xs, ws=ws)
                 ts = []
                 for _ in range(a.reps):
-                    flush.zero_()
+                    flush_l2(flush)
+                    # keep the GPU busy while the host marshals the launch, so the events
+                    # time the kernel and not the host call
+                    torch.cuda._sleep(200_000)
                     e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
                     e0.record()
                     sq.sq_linear_decode(q, x, y, 0, xsum=xs, ws=ws)

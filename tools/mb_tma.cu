@@ -17,10 +17,12 @@
 
 using namespace sq;
 
-constexpr int MAXST = 13, STAGE = 16384;
+constexpr int MAXST = 13;
+int STAGE = 16384;
+__constant__ int d_stage = 16384;
 
 __global__ void __launch_bounds__(64, 1) k_tma(const __grid_constant__ CUtensorMap tm, const uint8_t* src,
-                                                int pattern, int iters, uint64_t span_units, int STAGES) {
+                                                int pattern, int iters, uint64_t span_units, int STAGES, uint32_t stage_bytes) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   __shared__ uint64_t full[MAXST], empty[MAXST];
@@ -35,15 +37,17 @@ __global__ void __launch_bounds__(64, 1) k_tma(const __grid_constant__ CUtensorM
       const int s = i % STAGES, ph = (i / STAGES) & 1;
       mbar_wait(&empty[s], ph ^ 1);
       if (elect_one()) {
-        const uint64_t unit = ((uint64_t)blockIdx.x * iters + i) % span_units;  // 16 KB unit index
-        uint8_t* dst = smem + s * STAGE;
-        mbar_arrive_expect_tx(&full[s], STAGE);
-        if (pattern == 0) tma_load_2d(dst, &tm, &full[s], 0, (int)(unit * 128));
-        else if (pattern == 1) tma_load_4d(dst, &tm, &full[s], 0, 0, 0, (int)(unit * 8));
+        const uint64_t unit = ((uint64_t)blockIdx.x * iters + i) % span_units;  // stage-sized unit index
+        uint8_t* dst = smem + s * stage_bytes;
+        mbar_arrive_expect_tx(&full[s], stage_bytes);
+        if ((pattern & 15) == 0) tma_load_2d(dst, &tm, &full[s], 0, (int)(unit * (pattern >> 4)));
+        else if (pattern == 1 || pattern >= 5 && pattern <= 7) tma_load_4d(dst, &tm, &full[s], 0, 0, 0, (int)(unit * 8));
+        else if (pattern == 8)
+          for (int j = 0; j < 16; ++j) bulk_load(dst + j * 1024, src + unit * stage_bytes + j * 1024, 1024, &full[s]);
         else if (pattern == 2) tma_load_2d(dst, &tm, &full[s], 0, (int)(unit * 8));
-        else if (pattern == 3) bulk_load(dst, src + unit * STAGE, STAGE, &full[s]);
+        else if ((pattern & 15) == 3) bulk_load(dst, src + unit * stage_bytes, stage_bytes, &full[s]);
         else
-          for (int j = 0; j < 8; ++j) bulk_load(dst + j * 2048, src + unit * STAGE + j * 2048, 2048, &full[s]);
+          for (int j = 0; j < 8; ++j) bulk_load(dst + j * 2048, src + unit * stage_bytes + j * 2048, 2048, &full[s]);
       }
       __syncwarp();
     }
@@ -74,49 +78,36 @@ int main() {
   cudaMalloc(&buf, big);
   cudaMemset(buf, 1, big);
   const int iters = 2048;
-  const char* names[5] = {"2D fp16 {64,128} SW128", "4D u8 {64,16,2,8} SW64", "2D u64 {256,8}", "bulk 16KB x1",
-                          "bulk 2KB x8"};
+  const char* names[9] = {"2D fp16 {64,128} SW128", "4D u8 {64,16,2,8} SW64", "2D u64 {256,8}", "bulk 16KB x1",
+                          "bulk 2KB x8", "4D u8 {128,8,2,8} SW128", "4D u8 {48,16,2,8} none (12KB)",
+                          "4D u8 {128,6,2,8} none (12KB)", "bulk 1KB x16"};
   for (int cfg = 0; cfg < 6; ++cfg) {
-  const int STAGES = cfg < 3 ? 8 : (cfg == 3 ? 4 : 12);
-  const int smem = cfg == 0 ? 8 * STAGE + 2048 : (cfg == 1 ? 12 * STAGE + 2048 : (cfg == 2 ? 8 * STAGE + 2048 : STAGES * STAGE + 2048));
-  cudaFuncSetAttribute(k_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  for (int l2 = 0; l2 < 1; ++l2) {
-    const uint64_t span = l2 ? (4ull << 20) / STAGE : big / STAGE;
-    for (int p = 0; p < 4; p += 3) {
-      CUtensorMap tm{};
-      cuuint32_t es[4] = {1, 1, 1, 1};
-      CUresult r = CUDA_SUCCESS;
-      if (p == 0) {
-        cuuint64_t d[2] = {64, big / 128}, st[1] = {128};
-        cuuint32_t b[2] = {64, 128};
-        r = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, buf, d, st, b, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-      } else if (p == 1) {
-        cuuint64_t d[4] = {64, 16, 2, big / 2048}, st[3] = {64, 1024, 2048};
-        cuuint32_t b[4] = {64, 16, 2, 8};
-        r = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT8, 4, buf, d, st, b, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-      } else if (p == 2) {
-        cuuint64_t d[2] = {256, big / 2048}, st[1] = {2048};
-        cuuint32_t b[2] = {256, 8};
-        r = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT64, 2, buf, d, st, b, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-      }
-      if (r != CUDA_SUCCESS) { printf("encode failed p=%d r=%d\n", p, (int)r); continue; }
-      k_tma<<<sms, 64, smem>>>(tm, buf, p, 64, span, STAGES);
-      cudaEvent_t e0, e1;
-      cudaEventCreate(&e0); cudaEventCreate(&e1);
-      cudaEventRecord(e0);
-      k_tma<<<sms, 64, smem>>>(tm, buf, p, iters, span, STAGES);
-      cudaEventRecord(e1);
-      cudaError_t err = cudaDeviceSynchronize();
-      if (err != cudaSuccess) { printf("error %s\n", cudaGetErrorString(err)); return 1; }
-      float ms; cudaEventElapsedTime(&ms, e0, e1);
-      const double bytes = (double)sms * iters * STAGE;
-      printf("smem=%3dKB st=%2d %s %-26s %8.1f GB/s  %6.1f ns per 16 KB stage per SM\n", smem / 1024, STAGES, l2 ? "L2 " : "HBM", names[p],
-             bytes / (ms * 1e-3) / 1e9, ms * 1e6 / iters);
+    const int sb = cfg < 3 ? 8192 << cfg : 8192 << (cfg - 3);
+    const int p = cfg < 3 ? 0 : 3;
+    const int STAGES = sb <= 16384 ? 8 : 6;
+    const int smem = STAGES * sb + 2048;
+    cudaFuncSetAttribute(k_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    const uint64_t span = big / sb;
+    CUtensorMap tm{};
+    cuuint32_t es[4] = {1, 1, 1, 1};
+    if (p == 0) {
+      cuuint64_t d[2] = {64, big / 128}, st[1] = {128};
+      cuuint32_t b[2] = {64, (cuuint32_t)(sb / 128)};
+      enc(&tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, buf, d, st, b, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+          CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     }
-  }
+    k_tma<<<sms, 64, smem>>>(tm, buf, p + 16 * (sb / 128), 64, span, STAGES, sb);
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0); cudaEventCreate(&e1);
+    cudaEventRecord(e0);
+    k_tma<<<sms, 64, smem>>>(tm, buf, p + 16 * (sb / 128), iters, span, STAGES, sb);
+    cudaEventRecord(e1);
+    cudaError_t err = cudaDeviceSynchronize();
+    if (err != cudaSuccess) { printf("error %s\n", cudaGetErrorString(err)); return 1; }
+    float ms; cudaEventElapsedTime(&ms, e0, e1);
+    const double bytes = (double)sms * iters * sb;
+    printf("stage %6d B x%d %s: %8.1f GB/s  %6.1f GB/s per SM  %.3f us per stage\n", sb, STAGES, p == 0 ? "2D box" : "bulk  ",
+           bytes / (ms * 1e-3) / 1e9, bytes / (ms * 1e-3) / 1e9 / sms, ms * 1e3 / iters);
   }
   return 0;
 }
