@@ -26,6 +26,10 @@ FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "--expt-relaxe
          "-Xptxas", "-v,-warn-spills"]
 
 
+# debug builds only (e.g. SQ_NVCC_EXTRA="-DSQ_TC_DEBUG=1" for the tcgen05 decode trace)
+EXTRA = os.environ.get("SQ_NVCC_EXTRA", "").split()
+
+
 def nccl_dir() -> str:
     import importlib.util
     spec = importlib.util.find_spec("nvidia")
@@ -60,7 +64,7 @@ def build(verbose: bool = False, force: bool = False) -> str:
         o = os.path.join(OBJ, os.path.basename(s) + ".o")
         objs.append(o)
         if force or not _newer(o, [s, *headers, __file__]):
-            jobs.append([NVCC, *ARCH, *FLAGS, *inc, "-c", s, "-o", o])
+            jobs.append([NVCC, *ARCH, *FLAGS, *EXTRA, *inc, "-c", s, "-o", o])
     logs = []
     with cf.ThreadPoolExecutor(max_workers=os.cpu_count() or 4) as ex:
         for log in ex.map(_run, jobs):

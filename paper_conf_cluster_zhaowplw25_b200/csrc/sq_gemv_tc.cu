@@ -42,7 +42,8 @@ using namespace tc;
 
 constexpr int BN = 128;     // weight rows per unit (TMEM lanes, MMA M)
 constexpr int BT = 32;      // token columns (MMA N)
-constexpr int PMAX = 4;     // row tiles per panel (activation reuse), at most
+constexpr int PMAX = 8;     // row tiles per panel (activation reuse), at most
+constexpr int kCnt2 = 2048;  // second per-panel counter (fix-up done) at cnt + kCnt2
 constexpr int XK = 64;
 constexpr int X_BLOCK = BT * XK * 2;  // 4 KB: [32 tokens][64 k] SW128 tile
 #ifndef SQ_TC_DQ_WARPS
@@ -56,7 +57,7 @@ constexpr int A_COL = PMAX * BT;      // S_A x (64 * UG) columns
 constexpr int NUM_THREADS = 32 * (2 + DQ_WARPS + 4);  // producer, MMA, dequant, epilogue
 constexpr int EPI_WARP0 = 2 + DQ_WARPS;
 constexpr uint32_t kIdescTc = make_idesc(BN, BT);
-constexpr int X_LAG = 1;              // activations of step q are fetched after the weights of step q + 1
+constexpr int X_LAG = 0;              // activations of step q are fetched just before its weights (X_LAG > 0 deadlocks once P * (X_LAG + 1) > S_W)
 
 // UG = 128-k groups per unit, chosen so a weight stage is ~16 KB (INT3/INT4: 2, INT8: 1).
 template <int BITS, int UG>
@@ -67,7 +68,7 @@ struct DCfg {
   // TMEM A slots of 64*UG columns: the dequant warps fill slot i % S_A while the MMA reads the
   // others (slots are owned by one dequant group: multiples of DQ_GROUPS)
   static constexpr int A_SLOT = 64 * UG;
-  static constexpr int S_A = UG == 2 ? 2 : 6;
+  static constexpr int S_A = UG == 2 ? 2 : 4;
   static constexpr int S_X = 3;  // activation ring, in steps
   static_assert(BITS == 16 || A_COL + S_A * A_SLOT <= TMEM_COLS, "TMEM budget");
 };
@@ -376,53 +377,59 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(d_empty);  // accumulators drained: the MMA may start the next item
-      if (Z > 1) {
+      if (Z > 1) {  // publish this slice's partial (one item per CTA when Z > 1)
         __threadfence();
         asm volatile("bar.sync 1, 128;" ::: "memory");
-        if (leader && atomicAdd(p.cnt + pn, 1) == Z - 1) {  // last of the panel's Z items
-          p.cnt[pn] = 0;                                     // self-reset for the next launch
-          misc[2 + misc[1]] = (uint32_t)pn;
-          misc[1] = misc[1] + 1;
-        }
+        if (leader) atomicAdd(p.cnt + pn, 1);
       }
     }
   }
-  // ---------------- fix-up: this CTA sums the Z partials of the panels it finished last, in
-  // fixed z order, with every warp; the rings are idle now and stage Z partial tiles at a time.
+  // ---------------- split-k fix-up (Z > 1: one item per CTA, all Z items of a panel resident):
+  // wait until the panel's Z partials are published, then this CTA reduces its 1/Z share of the
+  // panel's outputs, summing the partials in fixed z order (deterministic).  The last CTA to finish
+  // resets the panel's two counters for the next launch.
   __syncthreads();
-  const int npend = (int)misc[1];
   if (threadIdx.x == 0) trace_cta(p, 11);
-  if (npend > 0) {
-    __threadfence();
-    // every thread: 4 consecutive rows of one token per step, the Z partials summed in z order
-    for (int e = 0; e < npend; ++e) {
-      const int pn = (int)misc[2 + e], pp = tiles_of(pn);
-      for (int idx = threadIdx.x; idx < pp * BT * (BN / 4); idx += NUM_THREADS) {
-        const int t = idx / (BT * (BN / 4)), rem = idx - t * (BT * (BN / 4));
-        const int tok = rem / (BN / 4), r4 = (rem % (BN / 4)) * 4;
-        if (tok >= p.m) continue;
-        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
-        for (int z = 0; z < Z; ++z) {
-          const float4 v = __ldcg(reinterpret_cast<const float4*>(
-              p.part + (((int64_t)(pn * Z + z) * PMAX + t) * BT + tok) * BN + r4));
-          acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
-        }
-        const int64_t row0 = (int64_t)(pn * P + t) * BN + r4;
-        float o[4] = {acc.x, acc.y, acc.z, acc.w};
-        if (p.bias) {
-#pragma unroll
-          for (int c = 0; c < 4; ++c) o[c] += __half2float(p.bias[row0 + c]);
-        }
-        if constexpr (EPI == SQ_EPI_F32_ACCUM) {
-          float* yp = static_cast<float*>(p.y) + (int64_t)tok * p.ldy + row0;
-#pragma unroll
-          for (int c = 0; c < 4; ++c) yp[c] += o[c];
-        } else {
-          __half* yp = static_cast<__half*>(p.y) + (int64_t)tok * p.ldy + row0;
-#pragma unroll
-          for (int c = 0; c < 4; ++c) yp[c] = __float2half_rn(apply_act<EPI>(o[c]));
-        }
+  if (Z > 1 && (int)blockIdx.x < I) {
+    const int it = blockIdx.x, pn = it / Z, z = it % Z, pp = tiles_of(pn);
+    if (threadIdx.x == 0) {
+      volatile int* c = p.cnt + pn;
+      while (*c < Z) __nanosleep(64);
+      __threadfence();
+    }
+    __syncthreads();
+    const int nel = pp * BT * (BN / 4);  // (tile, token, 4 rows)
+    const int e0 = (int)((long long)z * nel / Z), e1 = (int)((long long)(z + 1) * nel / Z);
+    for (int idx = e0 + threadIdx.x; idx < e1; idx += NUM_THREADS) {
+      const int t = idx / (BT * (BN / 4)), rem = idx - t * (BT * (BN / 4));
+      const int tok = rem / (BN / 4), r4 = (rem % (BN / 4)) * 4;
+      if (tok >= p.m) continue;
+      float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int zz = 0; zz < Z; ++zz) {
+        const float4 v = __ldcg(reinterpret_cast<const float4*>(
+            p.part + (((int64_t)(pn * Z + zz) * PMAX + t) * BT + tok) * BN + r4));
+        acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
       }
+      const int64_t row0 = (int64_t)(pn * P + t) * BN + r4;
+      float o[4] = {acc.x, acc.y, acc.z, acc.w};
+      if (p.bias) {
+#pragma unroll
+        for (int c = 0; c < 4; ++c) o[c] += __half2float(p.bias[row0 + c]);
+      }
+      if constexpr (EPI == SQ_EPI_F32_ACCUM) {
+        float* yp = static_cast<float*>(p.y) + (int64_t)tok * p.ldy + row0;
+#pragma unroll
+        for (int c = 0; c < 4; ++c) yp[c] += o[c];
+      } else {
+        __half* yp = static_cast<__half*>(p.y) + (int64_t)tok * p.ldy + row0;
+#pragma unroll
+        for (int c = 0; c < 4; ++c) yp[c] = __float2half_rn(apply_act<EPI>(o[c]));
+      }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0 && atomicAdd(p.cnt + kCnt2 + pn, 1) == Z - 1) {
+      p.cnt[pn] = 0;
+      p.cnt[kCnt2 + pn] = 0;
     }
   }
   tc_fence_before();
@@ -497,10 +504,11 @@ int tc_ug(int bits, int kg) { return (bits <= 4 && kg % 2 == 0) ? 2 : 1; }
 
 struct TcPlan { int P, Z, I, ctas; };
 
-// Panel width P and k split Z: minimise the bytes the busiest SM ingests -- weights + meta,
-// activation slices (once per k-step per panel, 32 token rows) and, for Z > 1, the Z partial
-// tiles the finishing CTA reads back (weighted by their measured slowness) -- over
-// ceil(items / SMs) rounds.
+// Panel width P and k split Z: minimise the bytes the busiest SM ingests -- weights + meta and the
+// activation slice of every panel k-step (activation bytes cost as much as weight bytes in the
+// per-SM TMA pipeline, ~45-50 GB/s per SM, tools/mb_tma.cu) -- plus, for Z > 1, the split-k fix-up
+// (partials written and re-read, the panel-wide wait).  Z > 1 requires a single round (every item
+// resident: the fix-up waits for the panel's other items).
 TcPlan tc_plan(int64_t n, int64_t k, int bits) {
   const int64_t nt = n / BN, kg = k / 128;
   const int ug = tc_ug(bits, (int)kg);
@@ -508,15 +516,14 @@ TcPlan tc_plan(int64_t n, int64_t k, int bits) {
   const double unit_w = BN * ug * 128.0 * bits / 8 + (bits == 16 ? 0.0 : BN * 4.0 * ug), unit_x = ug * 128.0 * BT * 2;
   TcPlan best{1, 1, 0, 0};
   double best_cost = 1e300;
-  constexpr int zmax = 8;
+  constexpr int zmax = 32;
   for (int P = 1; P <= PMAX; ++P) {
     for (int Z = 1; Z <= zmax && Z <= ks; ++Z) {
       const int64_t I = ((nt + P - 1) / P) * Z, rounds = (I + C - 1) / C;
-      if (Z > 1 && rounds > 62) continue;  // pending-panel list of the fix-up
+      if (Z > 1 && rounds > 1) continue;
       const int64_t steps = (ks + Z - 1) / Z;
-      // the fix-up's partial tiles come back at ~1/8 of the streaming rate (measured: bulk copies of
-      // another CTA's fresh partials land at ~14 GB/s per SM), so they are weighted 8x
-      const double cost = rounds * (steps * (P * unit_w + unit_x) + (Z > 1 ? 8.0 * Z * P * (double)BT * BN * 4 : 0.0));
+      const double fix = Z > 1 ? 2.0 * P * BT * BN * 4 + 131072.0 : 0.0;
+      const double cost = rounds * steps * (P * unit_w + unit_x) + fix;
       if (cost < best_cost * 0.999) { best_cost = cost; best = {P, Z, (int)I, (int)(I < C ? I : C)}; }
     }
   }
@@ -540,7 +547,7 @@ size_t gemv_tc_workspace_bytes(int64_t n, int64_t k) {
 
 // the activation group sums (when the caller passes none) follow the partials
 size_t gemv_tc_xsum_offset(int64_t n, int64_t k) {
-  int64_t items = 0;
+  int64_t items = getenv("SQ_TC_PZ") ? 2 * num_sms() : 0;  // room for forced splits (experiments)
   for (int bits : {3, 4, 8, 16}) {
     const TcPlan pl = tc_plan(n, k, bits);
     if (pl.Z > 1 && pl.I > items) items = pl.I;
@@ -590,7 +597,20 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
   p.kg = kg;
   p.nt = (int)(w.n / BN);
   p.ks = kg / ug;
-  const TcPlan pl = tc_plan(w.n, w.k, w.bits);
+  TcPlan pl = tc_plan(w.n, w.k, w.bits);
+  {
+    // experiments only: SQ_TC_PZ="P,Z" forces the panel width and k split
+    static int fp = -1, fz = -1;
+    if (fp < 0) {
+      const char* e = getenv("SQ_TC_PZ");
+      fp = 0;
+      if (e && sscanf(e, "%d,%d", &fp, &fz) != 2) fp = 0;
+    }
+    if (fp > 0 && fp <= PMAX && fz >= 1 && fz <= p.ks) {
+      const int64_t I = ((p.nt + fp - 1) / fp) * (int64_t)fz;
+      if (fz == 1 || I <= num_sms()) pl = {fp, fz, (int)I, (int)(I < num_sms() ? I : num_sms())};
+    }
+  }
   p.P = pl.P;
   p.Z = pl.Z;
   p.I = pl.I;
