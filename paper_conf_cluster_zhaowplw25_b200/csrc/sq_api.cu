@@ -1,6 +1,7 @@
 // C-ABI entry points of libsq (include/sq.h): argument validation (before any
 // launch), error state, launch accounting and the event-based profiler.
 #include <atomic>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <mutex>
@@ -23,6 +24,15 @@ sq_status fail(sq_status st, const char* fmt, ...) {
 sq_status cuda_check(cudaError_t e, const char* what) {
   if (e == cudaSuccess) return SQ_OK;
   return fail(SQ_ECUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+bool pdl_enabled() {
+  static int on = -1;
+  if (on < 0) {
+    const char* e = getenv("SQ_PDL");
+    on = (e && e[0] == '0') ? 0 : 1;
+  }
+  return on == 1;
 }
 
 int num_sms() {

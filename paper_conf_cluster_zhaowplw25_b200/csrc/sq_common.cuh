@@ -239,6 +239,11 @@ __device__ __forceinline__ void tmem_st8(uint32_t taddr, const uint32_t (&r)[8])
                : "memory");
 }
 
+// PDL (see launch_pdl): wait for the previous kernel of the stream (complete, memory visible);
+// allow the next one to be scheduled
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31; }
 __device__ __forceinline__ uint32_t warp_id_sync() { return __shfl_sync(0xffffffff, threadIdx.x >> 5, 0); }
 __device__ __forceinline__ bool elect_one() {

@@ -128,7 +128,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           if (elect_one()) tma_load_2d(wdst + BN * 128, &tm_w, &full_w[sw], g * 128 + 64, (int32_t)n0);
         } else {
           // placement T16: 4-D box {GB bytes, 16 rows, 1 group, 8 row tiles} -> [128 rows][GB]
-          if (elect_one()) tma_load_4d(wdst, &tm_w, &full_w[sw], 0, 0, g, (int32_t)(n0 / 16));
+          if (elect_one()) tma_load_3d(wdst, &tm_w, &full_w[sw], 0, g * (BITS == 3 ? 3 : (BITS == 4 ? 8 : 16)), (int32_t)(n0 / 16));
           if (elect_one()) tma_load_3d(smem + SM::OFF_META + sw * BN * 4, &tm_m, &full_w[sw], 0, g, (int32_t)(n0 / 16));
         }
         for (int h = 0; h < 2; ++h, ++it_x) {
@@ -299,11 +299,11 @@ cudaError_t launch_gemm(const sq_qweight& w, const __half* x, int64_t ldx, int64
   } else {
     // placement T16: [n/16 tiles][kg groups][16 rows][GB bytes]
     const uint64_t gb = 128 * w.bits / 8, kg = (uint64_t)w.k / 128, nt = (uint64_t)w.n / 16;
-    CUtensorMapSwizzle sw = w.bits == 8 ? CU_TENSOR_MAP_SWIZZLE_128B
-                                        : (w.bits == 4 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_NONE);
-    const uint64_t dw[4] = {gb, 16, kg, nt}, sw_[3] = {gb, 16 * gb, kg * 16 * gb};
-    const uint32_t bw[4] = {(uint32_t)gb, 16, 1, BN / 16};
-    e = encode_nd(&tw, CU_TENSOR_MAP_DATA_TYPE_UINT8, w.packed, 4, dw, sw_, bw, sw);
+    const WLines wl = wlines(w.bits);  // T16 units as long TMA lines (sq_tc.cuh)
+    const uint64_t dw[3] = {(uint64_t)wl.line, kg * wl.lpu, nt}, sw_[2] = {(uint64_t)wl.line, kg * 16 * gb};
+    const uint32_t bw[3] = {(uint32_t)wl.line, (uint32_t)wl.lpu, BN / 16};
+    e = encode_nd(&tw, CU_TENSOR_MAP_DATA_TYPE_UINT8, w.packed, 3, dw, sw_, bw,
+                  wl.sw128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE);
     if (e == cudaSuccess) {
       const uint64_t dm[3] = {16, kg, nt}, sm_[2] = {64, kg * 64};
       const uint32_t bm[3] = {16, 1, BN / 16};

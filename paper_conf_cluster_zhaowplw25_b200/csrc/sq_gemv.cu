@@ -304,6 +304,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemv(const GemvP p) {
 #pragma unroll
   for (int j = 0; j < D; ++j)
     if (j < nunits) issue(j);
+  // PDL: the weight fetches above are independent of the previous kernel; everything below is not
+  pdl_trigger();
+  pdl_wait();
 
   // ---- stage (xs, xoff) per (group, token) in shared memory (overlaps the weight loads):
   //      xs = sum x, xoff = sum off_k x  (off = 1024 INT8, 1024 / 64 for the two nibble slots of L4, 8 INT3)
@@ -505,6 +508,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemv_q(const GemvP p) {
     for (int c = 0; c < S && c < nch; ++c) issue(c);
   }
   __syncwarp();
+  // PDL: the weight fetches above are independent of the previous kernel; everything below is not
+  pdl_trigger();
+  pdl_wait();
 
   // activation fragment pointers for token n8-tile j: row 8j + g (predicated off beyond m); the
   // lane's k set matches its codes: [32q, 32q+32) (INT3/INT4) or [16q,16q+16) u [64+16q, 80+16q) (INT8)
@@ -627,6 +633,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemv_q(const GemvP p) {
 // one warp per (g, t), fixed summation order.
 __global__ void k_xsum(const __half* __restrict__ x, int64_t ldx, int64_t m, int kg, float2* __restrict__ out) {
   const int64_t id = (int64_t)blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5);
+  pdl_trigger();
+  pdl_wait();
   if (id >= (int64_t)kg * kXsTok) return;
   const int lane = threadIdx.x & 31;
   const int64_t g = id / kXsTok, t = id % kXsTok;
@@ -664,8 +672,7 @@ cudaError_t launch_e(const GemvP& p, cudaStream_t s) {
     if (e != cudaSuccess) return e;
     attr = smem;
   }
-  kern<<<(unsigned)p.W, kThreads, smem, s>>>(p);
-  return cudaGetLastError();
+  return launch_pdl(kern, dim3((unsigned)p.W), dim3(kThreads), smem, s, p);
 }
 
 template <int BITS, int TOK>
@@ -728,10 +735,10 @@ int gemv_path(int64_t n, int m, int bits) {
 cudaError_t launch_xsum(const __half* x, int64_t ldx, int64_t m, int64_t k, float2* xsum, cudaStream_t s) {
   const int64_t items = (k / 128) * kXsTok;
   auto t = prof_begin(KC_GLUE, (double)m * k * 2 + items * 8.0, 0, s);
-  k_xsum<<<(unsigned)((items + 7) / 8), 256, 0, s>>>(x, ldx, m, (int)(k / 128), xsum);
+  cudaError_t e = launch_pdl(k_xsum, dim3((unsigned)((items + 7) / 8)), dim3(256), 0, s, x, ldx, m, (int)(k / 128), xsum);
   prof_end(t, s);
   count_launch();
-  return cudaGetLastError();
+  return e;
 }
 
 cudaError_t launch_gemv(const sq_qweight& w, const __half* x, int64_t ldx, int m, void* y, int64_t ldy, int epi,

@@ -42,15 +42,23 @@ using namespace tc;
 
 constexpr int BN = 128;     // weight rows per unit (TMEM lanes, MMA M)
 constexpr int BT = 32;      // token columns (MMA N)
-constexpr int PMAX = 8;     // row tiles per panel (activation reuse), at most
+#ifndef SQ_TC_DEEP_A
+#define SQ_TC_DEEP_A 1  // 1: panels of <= 4 tiles, 1.5x deeper TMEM A ring (3 slots of 2 groups / 6 of 1)
+#endif
+constexpr int PMAX = SQ_TC_DEEP_A ? 4 : 8;  // row tiles per panel (activation reuse), at most
 constexpr int kCnt2 = 2048;  // second per-panel counter (fix-up done) at cnt + kCnt2
 constexpr int XK = 64;
 constexpr int X_BLOCK = BT * XK * 2;  // 4 KB: [32 tokens][64 k] SW128 tile
 #ifndef SQ_TC_DQ_WARPS
 #define SQ_TC_DQ_WARPS 16
 #endif
-constexpr int DQ_WARPS = SQ_TC_DQ_WARPS;  // dequant warps, in DQ_GROUPS groups of 8
-constexpr int DQ_GROUPS = DQ_WARPS / 8;    // group q dequantizes units i = q (mod DQ_GROUPS)
+#ifndef SQ_TC_DQ_PER_GROUP
+#define SQ_TC_DQ_PER_GROUP 8
+#endif
+constexpr int DQ_WARPS = SQ_TC_DQ_WARPS;        // dequant warps, in DQ_GROUPS groups of DQ_PER_GROUP
+constexpr int DQ_PER_GROUP = SQ_TC_DQ_PER_GROUP;  // 4 lane quadrants x KH k-parts of one unit
+constexpr int DQ_KH = DQ_PER_GROUP / 4;
+constexpr int DQ_GROUPS = DQ_WARPS / DQ_PER_GROUP;  // group q dequantizes units i = q (mod DQ_GROUPS)
 constexpr int TMEM_COLS = 512;
 constexpr int D_COL = 0;              // P x 32 columns: the panel's accumulators
 constexpr int A_COL = PMAX * BT;      // S_A x (64 * UG) columns
@@ -68,7 +76,7 @@ struct DCfg {
   // TMEM A slots of 64*UG columns: the dequant warps fill slot i % S_A while the MMA reads the
   // others (slots are owned by one dequant group: multiples of DQ_GROUPS)
   static constexpr int A_SLOT = 64 * UG;
-  static constexpr int S_A = UG == 2 ? 2 : 4;
+  static constexpr int S_A = SQ_TC_DEEP_A ? (UG == 2 ? 3 : 6) : (UG == 2 ? 2 : 4);
   static constexpr int S_X = 3;  // activation ring, in steps
   static_assert(BITS == 16 || A_COL + S_A * A_SLOT <= TMEM_COLS, "TMEM budget");
 };
@@ -153,6 +161,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   constexpr int X_STAGE = SM::X_STAGE;
   constexpr int GB = GCfg<BITS>::GB;
   constexpr uint32_t W_BYTES = BN * GB * UG + (BITS == 16 ? 0 : BN * 4 * UG);  // codes + meta of one unit
+  constexpr int LPU = BITS == 3 ? 3 : (BITS == 4 ? 8 : 16);  // TMA lines per T16 unit (wlines)
   extern __shared__ uint8_t smem_raw[];
   // 1-KB aligned (SW128 atoms); pointer arithmetic on smem_raw keeps the shared address space
   // visible to the compiler (LDS, not generic LD)
@@ -179,8 +188,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   if (threadIdx.x == 0) {
     for (int i = 0; i < S_X; ++i) { mbar_init(&full_x[i], 1); mbar_init(&empty_x[i], 1); }
     // fp16 weights are the MMA's A operand straight from SMEM: the MMA commit frees the slot
-    for (int i = 0; i < S_W; ++i) { mbar_init(&full_w[i], 1); mbar_init(&empty_w[i], BITS == 16 ? 1 : 8); }
-    for (int i = 0; i < S_A; ++i) { mbar_init(&full_a[i], 8); mbar_init(&empty_a[i], 1); }
+    for (int i = 0; i < S_W; ++i) { mbar_init(&full_w[i], 1); mbar_init(&empty_w[i], BITS == 16 ? 1 : DQ_PER_GROUP); }
+    for (int i = 0; i < S_A; ++i) { mbar_init(&full_a[i], DQ_PER_GROUP); mbar_init(&empty_a[i], 1); }
     mbar_init(d_full, 1);
     mbar_init(d_empty, 4);
     misc[1] = 0;
@@ -189,6 +198,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     prefetch_tmap(&tm_w);
     if constexpr (BITS != 16) prefetch_tmap(&tm_m);
   }
+  pdl_trigger();  // the next kernel may be scheduled as soon as SMs free up
   if (warp == 1) tmem_alloc(misc, TMEM_COLS);
   tc_fence_before();
   __syncthreads();
@@ -212,16 +222,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       __syncwarp();
       ++qx;
     };
-    for (int it = blockIdx.x; it < I; it += C) {
-      const int pn = it / Z, j1 = j1_of(it), pp = tiles_of(pn);
-      for (int j = j0_of(it); j < j1; ++j, ++q) {
-        xj[q % (X_LAG + 1)] = j;
-        if (q >= X_LAG) issue_x(xj[(q - X_LAG) % (X_LAG + 1)]);
-        for (int t = 0; t < pp; ++t, ++i) {
-          const int sw = i % S_W, rw = i / S_W;
-          mbar_wait_park(&empty_w[sw], (rw & 1) ^ 1);
-          trace_ev(p, 0, i);
-          if (elect_one()) {
+    auto issue_w = [&](int i, int pn, int t, int j) {
+      const int sw = i % S_W;
+      if (elect_one()) {
             const int tile16 = (pn * P + t) * (BN / 16);
             uint8_t* wdst = smem + SM::OFF_W + sw * SM::W_STAGE;
             mbar_arrive_expect_tx(&full_w[sw], W_BYTES);
@@ -230,12 +233,33 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
               tma_load_2d(wdst, &tm_w, &full_w[sw], j * 128, (pn * P + t) * BN);
               tma_load_2d(wdst + BN * 128, &tm_w, &full_w[sw], j * 128 + 64, (pn * P + t) * BN);
             } else {
-              // placement T16: box {GB bytes, 16 rows, UG groups, 8 row tiles} -> [tile][group][16][GB]
-              tma_load_4d(wdst, &tm_w, &full_w[sw], 0, 0, j * UG, tile16);
+              // placement T16 as lines: box {line, lpu * UG lines, 8 row tiles} -> [tile][group][16][GB]
+              tma_load_3d(wdst, &tm_w, &full_w[sw], 0, j * UG * LPU, tile16);
               tma_load_3d(smem + SM::OFF_META + sw * BN * 4 * UG, &tm_m, &full_w[sw], 0, j * UG, tile16);
             }
-          }
-          __syncwarp();
+      }
+      __syncwarp();
+    };
+    // PDL: weights never depend on the previous kernel -- fill the whole ring before waiting for
+    // it (these first S_W slots are free, no empty wait); activations only after the wait
+    int pre = 0;
+    for (int it = blockIdx.x; it < I && pre < S_W; it += C) {
+      const int pn = it / Z, j1 = j1_of(it), pp = tiles_of(pn);
+      for (int j = j0_of(it); j < j1 && pre < S_W; ++j)
+        for (int t = 0; t < pp && pre < S_W; ++t, ++pre) issue_w(pre, pn, t, j);
+    }
+    pdl_wait();
+    for (int it = blockIdx.x; it < I; it += C) {
+      const int pn = it / Z, j1 = j1_of(it), pp = tiles_of(pn);
+      for (int j = j0_of(it); j < j1; ++j, ++q) {
+        xj[q % (X_LAG + 1)] = j;
+        if (q >= X_LAG) issue_x(xj[(q - X_LAG) % (X_LAG + 1)]);
+        for (int t = 0; t < pp; ++t, ++i) {
+          if (i < pre) continue;
+          const int sw = i % S_W, rw = i / S_W;
+          mbar_wait_park(&empty_w[sw], (rw & 1) ^ 1);
+          trace_ev(p, 0, i);
+          issue_w(i, pn, t, j);
           trace_ev(p, 8, i);
         }
       }
@@ -307,14 +331,16 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     // DQ_GROUPS).  Thread = weight row (lane quadrant warp % 4); warp kh of the group takes batches
     // [kh*2*UG, kh*2*UG + 2*UG) of the unit's 4*UG 32-k batches.  Slots of both rings are owned by
     // one group (ring depths are multiples of DQ_GROUPS), so phases follow from i alone.
-    static_assert(BITS == 16 || (S_W % DQ_GROUPS == 0 && S_A % DQ_GROUPS == 0), "ring slots owned by one dequant group");
+    // (SQ_TC_DEEP_A: A slots alternate between the groups; in-order MMA completion keeps every
+    // waiter within one phase of the slot's barrier)
+    static_assert(BITS == 16 || (S_W % DQ_GROUPS == 0 && (SQ_TC_DEEP_A || S_A % DQ_GROUPS == 0)), "ring slots owned by one dequant group");
     int nunits = 0;
     if constexpr (BITS != 16)
       for (int it = blockIdx.x; it < I; it += C) nunits += (j1_of(it) - j0_of(it)) * tiles_of(it / Z);
-    constexpr int NBW = 2 * UG;                              // batches per warp
+    constexpr int NBW = 4 * UG / DQ_KH;                      // batches per warp
     const int sp = warp & 3;
-    const int dg = (warp - 2) >> 3;
-    const int kh = ((warp - 2) >> 2) & 1;
+    const int dg = (warp - 2) / DQ_PER_GROUP;
+    const int kh = ((warp - 2) >> 2) % DQ_KH;
     const int gg = (kh * NBW) >> 2, b0 = (kh * NBW) & 3;  // group of the unit and first batch in it
     const int r = sp * 32 + lane;
     const int ru = ((r >> 4) * UG + gg) * 16 + (r & 15);  // stage layout [tile][group][16 rows]
@@ -350,6 +376,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const int r = sp * 32 + lane;
     const uint32_t lane_base = (uint32_t)(sp * 32) << 16;
     const bool leader = threadIdx.x == EPI_WARP0 * 32;
+    pdl_wait();  // y / partial writes below
     int n_item = 0;
     for (int it = blockIdx.x; it < I; it += C, ++n_item) {
       const int pn = it / Z, pp = tiles_of(pn);
@@ -390,6 +417,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   // resets the panel's two counters for the next launch.
   __syncthreads();
   if (threadIdx.x == 0) trace_cta(p, 11);
+  pdl_wait();  // (returns at once: the producer already waited)
   if (Z > 1 && (int)blockIdx.x < I) {
     const int it = blockIdx.x, pn = it / Z, z = it % Z, pp = tiles_of(pn);
     if (threadIdx.x == 0) {
@@ -475,8 +503,7 @@ cudaError_t launch_tc_be(const CUtensorMap& tx, const CUtensorMap& tw, const CUt
     if (e != cudaSuccess) return e;
     attr = true;
   }
-  kern<<<nc, NUM_THREADS, DSmem<BITS, UG>::BYTES, s>>>(tx, tw, tm, p);
-  return cudaGetLastError();
+  return launch_pdl(kern, dim3(nc), dim3(NUM_THREADS), DSmem<BITS, UG>::BYTES, s, tx, tw, tm, p);
 }
 
 template <int BITS, int UG>
@@ -574,12 +601,13 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
     cudaError_t e = enc(&tw, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, w.packed, 2, dw, sw_, bw, CU_TENSOR_MAP_SWIZZLE_128B);
     if (e != cudaSuccess) return e;
   } else {
+    // T16 units as lines: [n/16 tiles][kg * lpu lines][line bytes]; box = UG units of 8 tiles
     const uint64_t gb = 128 * w.bits / 8, nt = (uint64_t)w.n / 16;
-    CUtensorMapSwizzle sw = w.bits == 8 ? CU_TENSOR_MAP_SWIZZLE_128B
-                                        : (w.bits == 4 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_NONE);
-    const uint64_t dw[4] = {gb, 16, (uint64_t)kg, nt}, sw_[3] = {gb, 16 * gb, kg * 16 * gb};
-    const uint32_t bw[4] = {(uint32_t)gb, 16, (uint32_t)ug, BN / 16};
-    cudaError_t e = enc(&tw, CU_TENSOR_MAP_DATA_TYPE_UINT8, w.packed, 4, dw, sw_, bw, sw);
+    const WLines wl = wlines(w.bits);
+    const uint64_t dw[3] = {(uint64_t)wl.line, (uint64_t)kg * wl.lpu, nt}, sw_[2] = {(uint64_t)wl.line, kg * 16 * gb};
+    const uint32_t bw[3] = {(uint32_t)wl.line, (uint32_t)(wl.lpu * ug), BN / 16};
+    cudaError_t e = enc(&tw, CU_TENSOR_MAP_DATA_TYPE_UINT8, w.packed, 3, dw, sw_, bw,
+                        wl.sw128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE);
     if (e != cudaSuccess) return e;
     const uint64_t dm[3] = {16, (uint64_t)kg, nt}, sm_[2] = {64, (uint64_t)kg * 64};
     const uint32_t bm[3] = {16, (uint32_t)ug, BN / 16};

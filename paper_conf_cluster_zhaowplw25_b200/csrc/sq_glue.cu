@@ -31,6 +31,8 @@ __global__ void __launch_bounds__(kLnThreads) k_layernorm(const float* __restric
                                                           const float* __restrict__ copy_src, float* __restrict__ copy_dst) {
   constexpr int MAXV = 14;  // up to d = 14 * 1024 = 14336 (BLOOM-176B h1)
   __shared__ float red[kLnThreads / 32];
+  pdl_trigger();
+  pdl_wait();
   const int64_t row = blockIdx.x;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const float* xr = x + row * d;
@@ -93,6 +95,8 @@ __global__ void __launch_bounds__(kLnThreads) k_layernorm(const float* __restric
 // dst[r, 0:d] = src[r * sstride, 0:d] for r < rows (fp32, d % 4 == 0)
 __global__ void k_copy_rows(const float* __restrict__ src, int64_t sstride, int64_t rows, int64_t d,
                             float* __restrict__ dst, int64_t dstride) {
+  pdl_trigger();
+  pdl_wait();
   const int64_t r = blockIdx.y;
   for (int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 4; c < d; c += (int64_t)gridDim.x * blockDim.x * 4)
     *reinterpret_cast<float4*>(dst + r * dstride + c) = *reinterpret_cast<const float4*>(src + r * sstride + c);
@@ -104,19 +108,21 @@ cudaError_t launch_layernorm_f16(const float* x, int64_t rows, int64_t d, __half
                                  const float* copy_src, float* copy_dst, cudaStream_t s) {
   if (d % 128 || d > 14 * 1024) return cudaErrorInvalidValue;
   auto t = prof_begin(KC_GLUE, (double)rows * d * (4 + 2 + (copy_dst ? 8 : 0)), 0, s);
-  k_layernorm<true><<<(unsigned)rows, kLnThreads, 0, s>>>(x, d, y, xsum, 32, copy_src, copy_dst);
+  cudaError_t e = launch_pdl(k_layernorm<true>, dim3((unsigned)rows), dim3(kLnThreads), 0, s, x, d, (void*)y, xsum, 32,
+                             copy_src, copy_dst);
   prof_end(t, s);
   count_launch();
-  return cudaGetLastError();
+  return e;
 }
 
 cudaError_t launch_layernorm_f32(const float* x, int64_t rows, int64_t d, float* y, cudaStream_t s) {
   if (d % 128 || d > 14 * 1024) return cudaErrorInvalidValue;
   auto t = prof_begin(KC_GLUE, (double)rows * d * 8, 0, s);
-  k_layernorm<false><<<(unsigned)rows, kLnThreads, 0, s>>>(x, d, y, nullptr, 0, nullptr, nullptr);
+  cudaError_t e = launch_pdl(k_layernorm<false>, dim3((unsigned)rows), dim3(kLnThreads), 0, s, x, d, (void*)y,
+                             (float2*)nullptr, 0, (const float*)nullptr, (float*)nullptr);
   prof_end(t, s);
   count_launch();
-  return cudaGetLastError();
+  return e;
 }
 
 cudaError_t launch_copy_rows(const float* src, int64_t sstride, int64_t rows, int64_t d, float* dst, int64_t dstride,
@@ -124,10 +130,10 @@ cudaError_t launch_copy_rows(const float* src, int64_t sstride, int64_t rows, in
   if (rows <= 0) return cudaSuccess;
   dim3 grid((unsigned)((d / 4 + 255) / 256), (unsigned)rows);
   auto t = prof_begin(KC_GLUE, (double)rows * d * 8, 0, s);
-  k_copy_rows<<<grid, 256, 0, s>>>(src, sstride, rows, d, dst, dstride);
+  cudaError_t e = launch_pdl(k_copy_rows, grid, dim3(256), 0, s, src, sstride, rows, d, dst, dstride);
   prof_end(t, s);
   count_launch();
-  return cudaGetLastError();
+  return e;
 }
 
 }  // namespace sq

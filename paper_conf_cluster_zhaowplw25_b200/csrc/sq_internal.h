@@ -57,4 +57,27 @@ sq_status check_layers(const sq_layer* layers, int n_layers, const char* who);
 
 int num_sms();
 
+// ---- programmatic dependent launch (PDL) ----
+// Decode kernels are launched with programmatic stream serialization: the next kernel of the
+// stream may be scheduled while this one drains, runs its prologue (barriers, TMEM, and the
+// first weight fetches -- weights never depend on the previous kernel), and blocks in
+// griddepcontrol.wait (pdl_wait) before it touches anything the previous kernel produces or
+// consumes.  Every kernel launched this way calls pdl_wait before its first dependent access.
+// SQ_PDL=0 disables the attribute (plain stream order).
+bool pdl_enabled();
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, static_cast<Args&&>(args)...);
+}
+
 }  // namespace sq

@@ -2,9 +2,11 @@
 // decode GEMV (K2c): SW128 smem descriptors, the instruction descriptor, and the
 // per-row dequantization of one 128-k group straight into tensor memory.
 //
-// Packed weight stages are [128 rows][GB bytes] fetched by one 4-D TMA box (8 T16 units of
-// 16 rows) with SWIZZLE_64B (INT4) / SWIZZLE_128B (INT8) / none (INT3, 48-B rows are
-// conflict-free); fp16 weight stages are two SW128 [128][128 B] tiles.  tcgen05.st is
+// Packed weight stages are [128 rows][GB bytes] fetched by one 3-D TMA box whose rows are
+// 128-B lines (INT4: two weight rows per line; INT8: one) under SWIZZLE_128B, or 256-B lines
+// without swizzle (INT3: 48-B weight rows are conflict-free) -- the TMA engine moves short box
+// rows slowly (64-B rows measured at ~60 % of the 128-B rate), so the box rows are made long;
+// fp16 weight stages are two SW128 [128][128 B] tiles.  tcgen05.st is
 // .sync.aligned: its TMEM column address must be warp-uniform, so the chunk order is static
 // and bank conflicts are avoided by the TMA swizzle, not by per-thread reordering.
 #pragma once
@@ -23,6 +25,15 @@ template <>
 struct GCfg<8> { static constexpr int GB = 128; static constexpr int S_W = 4; };
 template <>
 struct GCfg<16> { static constexpr int GB = 256; static constexpr int S_W = 2; };
+
+// Geometry of the packed-weight tensor map (placement T16 viewed as lines): line bytes, lines per
+// (16-row, 1-group) unit, swizzle (0 none, 1 SWIZZLE_128B).  Box = {line, lines_per_unit * UG, 8}.
+struct WLines { int line, lpu, sw128; };
+inline WLines wlines(int bits) {
+  if (bits == 3) return {256, 3, 0};   // 768 B per unit
+  if (bits == 4) return {128, 8, 1};   // 1 KB per unit
+  return {128, 16, 1};                 // INT8: 2 KB per unit
+}
 
 __device__ __forceinline__ uint64_t make_sw128_desc(uint32_t saddr) {
   uint64_t d = 0;
@@ -67,12 +78,16 @@ __device__ __forceinline__ void dequant_row_batches(const uint8_t* wst, uint32_t
   const uint32_t z2 = (meta >> 16) * 0x10001u;
   constexpr uint32_t K1024 = 0x64006400u, K64 = 0x54005400u;
   if constexpr (BITS == 4) {
-    const uint8_t* row = wst + (row_off >= 0 ? row_off : r * 64);
+    // the stage is a sequence of 128-B lines (two 64-B rows each) under SWIZZLE_128B: logical chunk
+    // (row & 1) * 4 + b of line row / 2 sits at physical chunk ^ (line & 7)
+    const int lo = row_off >= 0 ? row_off : r * 64;
+    const uint8_t* line = wst + (lo & ~127);
+    const int h4 = (lo >> 4) & 4, swz = (lo >> 7) & 7;
 #pragma unroll
     for (int bi = 0; bi < NB; ++bi) {
       const int b = B0 + bi;
-      const int pc = b ^ ((r >> 1) & 3);  // SWIZZLE_64B
-      uint4 v = *reinterpret_cast<const uint4*>(row + pc * 16);
+      const int pc = (h4 | b) ^ swz;
+      uint4 v = *reinterpret_cast<const uint4*>(line + pc * 16);
       const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
       uint32_t o[16];
 #pragma unroll
@@ -178,12 +193,13 @@ __device__ __forceinline__ void unpack_sc_row_batches(const uint8_t* wst, uint32
   if constexpr (BITS == 4) {
     const uint32_t nbA = neg_off_s(sb, 1024.f, ok_a), nbB = neg_off_s(sb, 64.f, ok_b);
     const bool fast = ok_a;  // ok_a implies ok_b
-    const uint8_t* row = wst + row_off;
+    const uint8_t* line = wst + (row_off & ~127);
+    const int h4 = (row_off >> 4) & 4, swz = (row_off >> 7) & 7;
 #pragma unroll
     for (int bi = 0; bi < NB; ++bi) {
       const int b = B0 + bi;
-      const int pc = b ^ ((r >> 1) & 3);  // SWIZZLE_64B
-      uint4 v = *reinterpret_cast<const uint4*>(row + pc * 16);
+      const int pc = (h4 | b) ^ swz;  // 128-B lines under SWIZZLE_128B (see dequant_row_batches)
+      uint4 v = *reinterpret_cast<const uint4*>(line + pc * 16);
       const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
       uint32_t o[16];
       if (fast) {

@@ -23,6 +23,7 @@ def main():
     ap.add_argument("--shapes", default="5120x5120,20480x5120,36864x9216")
     ap.add_argument("--n-launch", type=int, default=60)
     ap.add_argument("--min-bytes", type=float, default=400e6)
+    ap.add_argument("--graph", action="store_true", help="replay the launches from one CUDA graph (no host time)")
     a = ap.parse_args()
     dev = torch.device("cuda")
     for shp in a.shapes.split(","):
@@ -42,15 +43,32 @@ def main():
                 for i in range(2 * R):
                     sq.sq_linear_decode(qs[i % R], x, y, 0, xsum=xs, ws=ws)
                 torch.cuda.synchronize()
-                torch.cuda._sleep(1_000_000)  # GPU busy while the host enqueues the launches
                 e0 = torch.cuda.Event(enable_timing=True)
                 e1 = torch.cuda.Event(enable_timing=True)
-                e0.record()
-                for i in range(a.n_launch):
-                    sq.sq_linear_decode(qs[i % R], x, y, 0, xsum=xs, ws=ws)
-                e1.record()
-                torch.cuda.synchronize()
-                us = e0.elapsed_time(e1) * 1e3 / a.n_launch
+                if a.graph:
+                    g = torch.cuda.CUDAGraph()
+                    with torch.cuda.graph(g):
+                        for i in range(a.n_launch):
+                            sq.sq_linear_decode(qs[i % R], x, y, 0, xsum=xs, ws=ws)
+                    g.replay()
+                    torch.cuda.synchronize()
+                    best = 1e30
+                    for _ in range(5):
+                        e0.record()
+                        g.replay()
+                        e1.record()
+                        torch.cuda.synchronize()
+                        best = min(best, e0.elapsed_time(e1))
+                    us = best * 1e3 / a.n_launch
+                    del g
+                else:
+                    torch.cuda._sleep(1_000_000)  # GPU busy while the host enqueues the launches
+                    e0.record()
+                    for i in range(a.n_launch):
+                        sq.sq_linear_decode(qs[i % R], x, y, 0, xsum=xs, ws=ws)
+                    e1.record()
+                    torch.cuda.synchronize()
+                    us = e0.elapsed_time(e1) * 1e3 / a.n_launch
                 print(json.dumps({"n": n, "k": k, "bits": bits, "m": m, "copies": R, "us": round(us, 2),
                                   "GBps": round(q0.nbytes() / us / 1e3, 1)}), flush=True)
             del qs, q0
