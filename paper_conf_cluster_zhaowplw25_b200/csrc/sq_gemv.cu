@@ -535,92 +535,98 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemv_q(const GemvP p) {
     for (int i = 0; i < 4; ++i) acc[j][i] = 0.f;
   const int lane_off = BITS == 8 ? q * 16 : q * lane_bytes<BITS>();
 
+  // one unit: codes of rows g / g+8 from the slot, activation fragment from L1, 8 HMMAs, the
+  // per-group factorised scale / zero, segment end (row tile finished or end of the warp's run)
+  auto unit = [&](const uint8_t* cs, const uint32_t* ms, int s, int ui) {
+    uint32_t cw0[LU], cw1[LU];
+    lds_codes<BITS>(cs + s * UB + g * GB + lane_off, cw0);
+    lds_codes<BITS>(cs + s * UB + (g + 8) * GB + lane_off, cw1);
+    const uint32_t mr0 = ms[s * 16 + g], mr1 = ms[s * 16 + g + 8];
+#pragma unroll
+    for (int j = 0; j < NJ; ++j) {
+      const uint4* xp = reinterpret_cast<const uint4*>(xrow[j] + grp * 128);
+      uint32_t xloc[16];
+      uint32_t* xtj = NJ == 1 ? xt1 : xloc;
+      if (xon[j]) {
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const int xo = BITS == 8 ? (i < 2 ? i : 8 + (i - 2)) : i;  // 16-B units
+          const uint4 v = __ldg(xp + xo);
+          xtj[4 * i] = v.x; xtj[4 * i + 1] = v.y; xtj[4 * i + 2] = v.z; xtj[4 * i + 3] = v.w;
+        }
+      } else if (NJ > 1) {
+#pragma unroll
+        for (int i = 0; i < 16; ++i) xloc[i] = 0u;
+      }
+      const float4 xsv = __ldg(reinterpret_cast<const float4*>(p.xsum + grp * kXsTok + 8 * j + 2 * q));
+      float d0[4], d1[4];  // two independent HMMA chains (even / odd chunks)
+      {
+        uint32_t a[4], b[4];
+        frag<BITS>(cw0, 0, a[0], a[2]);
+        frag<BITS>(cw1, 0, a[1], a[3]);
+        frag<BITS>(cw0, 1, b[0], b[2]);
+        frag<BITS>(cw1, 1, b[1], b[3]);
+        mma_16816_zc(d0, a, xtj[0], xtj[1]);
+        mma_16816_zc(d1, b, xtj[2], xtj[3]);
+      }
+#pragma unroll
+      for (int t = 2; t < 8; t += 2) {
+        uint32_t a[4], b[4];
+        frag<BITS>(cw0, t, a[0], a[2]);
+        frag<BITS>(cw1, t, a[1], a[3]);
+        frag<BITS>(cw0, t + 1, b[0], b[2]);
+        frag<BITS>(cw1, t + 1, b[1], b[3]);
+        mma_16816(d0, a, xtj[2 * t], xtj[2 * t + 1], d0);
+        mma_16816(d1, b, xtj[2 * t + 2], xtj[2 * t + 3], d1);
+      }
+      const float d[4] = {d0[0] + d1[0], d0[1] + d1[1], d0[2] + d1[2], d0[3] + d1[3]};
+      const float2 f0 = __half22float2(*reinterpret_cast<const __half2*>(&mr0));  // (s, z) row g
+      const float2 f1 = __half22float2(*reinterpret_cast<const __half2*>(&mr1));  // row g+8
+      // (xs, xoff) of tokens 2q, 2q+1: xs = sum x, xoff = sum off_k x
+      const float xs0 = xsv.x + xsv.y, xs1 = xsv.z + xsv.w;
+      const float xo0 = BITS == 4 ? fmaf(1024.f, xsv.x, 64.f * xsv.y) : (BITS == 3 ? 8.f * xs0 : 1024.f * xs0);
+      const float xo1 = BITS == 4 ? fmaf(1024.f, xsv.z, 64.f * xsv.w) : (BITS == 3 ? 8.f * xs1 : 1024.f * xs1);
+      // y += s * (D - xoff) + z * xs
+      acc[j][0] = fmaf(-f0.x, xo0, fmaf(f0.y, xs0, fmaf(f0.x, d[0], acc[j][0])));
+      acc[j][1] = fmaf(-f0.x, xo1, fmaf(f0.y, xs1, fmaf(f0.x, d[1], acc[j][1])));
+      acc[j][2] = fmaf(-f1.x, xo0, fmaf(f1.y, xs0, fmaf(f1.x, d[2], acc[j][2])));
+      acc[j][3] = fmaf(-f1.x, xo1, fmaf(f1.y, xs1, fmaf(f1.x, d[3], acc[j][3])));
+    }
+    const bool tile_end = (grp == kg - 1);
+    if (tile_end || ui == nunits - 1) {
+      if (seg_from_start && tile_end) {
+        store_out<TOK, EPI>(p, tile, g, q, acc);
+      } else {
+        const int sl = (tile == head_tile) ? 0 : 1;  // head / tail tile of this warp
+        float* pp = part_s + ((warp * 2 + sl) * TOK) * kRows;
+#pragma unroll
+        for (int j = 0; j < NJ; ++j)
+#pragma unroll
+          for (int e = 0; e < 2; ++e) {
+            const int tok = 8 * j + 2 * q + e;
+            pp[tok * kRows + g] = acc[j][e];
+            pp[tok * kRows + g + 8] = acc[j][2 + e];
+          }
+      }
+#pragma unroll
+      for (int j = 0; j < NJ; ++j)
+#pragma unroll
+        for (int i = 0; i < 4; ++i) acc[j][i] = 0.f;
+      seg_from_start = true;
+    }
+    if (++grp == kg) { grp = 0; ++tile; }
+  };
+
   for (int c = 0; c < nch; ++c) {
     const int slot = c % S;
     mbar_wait(&bar[slot], (uint32_t)((c / S) & 1));
     const uint8_t* cs = ring + slot * SLOT;
     const uint32_t* ms = reinterpret_cast<const uint32_t*>(cs + CH * UB);
+    if (c * CH + CH <= nunits) {  // full slot (warp-uniform): straight-line body
 #pragma unroll
-    for (int s = 0; s < CH; ++s) {
-      const int ui = c * CH + s;
-      if (ui >= nunits) break;
-      uint32_t cw0[LU], cw1[LU];
-      lds_codes<BITS>(cs + s * UB + g * GB + lane_off, cw0);
-      lds_codes<BITS>(cs + s * UB + (g + 8) * GB + lane_off, cw1);
-      const uint32_t mr0 = ms[s * 16 + g], mr1 = ms[s * 16 + g + 8];
-#pragma unroll
-      for (int j = 0; j < NJ; ++j) {
-        const __half* xp = xrow[j] + grp * 128;
-        uint32_t xloc[16];
-        uint32_t* xtj = NJ == 1 ? xt1 : xloc;
-        if (NJ > 1) {
-#pragma unroll
-          for (int i = 0; i < 16; ++i) xloc[i] = 0u;
-        }
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const int xo = BITS == 8 ? (i < 2 ? 8 * i : 64 + 8 * (i - 2)) : 8 * i;
-          ldg_v4_pred(xtj + 4 * i, xp + xo, xon[j]);
-        }
-        const float4 xsv = __ldg(reinterpret_cast<const float4*>(p.xsum + grp * kXsTok + 8 * j + 2 * q));
-        float d0[4], d1[4];  // two independent HMMA chains (even / odd chunks)
-        {
-          uint32_t a[4], b[4];
-          frag<BITS>(cw0, 0, a[0], a[2]);
-          frag<BITS>(cw1, 0, a[1], a[3]);
-          frag<BITS>(cw0, 1, b[0], b[2]);
-          frag<BITS>(cw1, 1, b[1], b[3]);
-          mma_16816_zc(d0, a, xtj[0], xtj[1]);
-          mma_16816_zc(d1, b, xtj[2], xtj[3]);
-        }
-#pragma unroll
-        for (int t = 2; t < 8; t += 2) {
-          uint32_t a[4], b[4];
-          frag<BITS>(cw0, t, a[0], a[2]);
-          frag<BITS>(cw1, t, a[1], a[3]);
-          frag<BITS>(cw0, t + 1, b[0], b[2]);
-          frag<BITS>(cw1, t + 1, b[1], b[3]);
-          mma_16816(d0, a, xtj[2 * t], xtj[2 * t + 1], d0);
-          mma_16816(d1, b, xtj[2 * t + 2], xtj[2 * t + 3], d1);
-        }
-        const float d[4] = {d0[0] + d1[0], d0[1] + d1[1], d0[2] + d1[2], d0[3] + d1[3]};
-        const float2 f0 = __half22float2(*reinterpret_cast<const __half2*>(&mr0));  // (s, z) row g
-        const float2 f1 = __half22float2(*reinterpret_cast<const __half2*>(&mr1));  // row g+8
-        // (xs, xoff) of tokens 2q, 2q+1: xs = sum x, xoff = sum off_k x
-        const float xs0 = xsv.x + xsv.y, xs1 = xsv.z + xsv.w;
-        const float xo0 = BITS == 4 ? fmaf(1024.f, xsv.x, 64.f * xsv.y) : (BITS == 3 ? 8.f * xs0 : 1024.f * xs0);
-        const float xo1 = BITS == 4 ? fmaf(1024.f, xsv.z, 64.f * xsv.w) : (BITS == 3 ? 8.f * xs1 : 1024.f * xs1);
-        // y += s * (D - xoff) + z * xs
-        acc[j][0] = fmaf(-f0.x, xo0, fmaf(f0.y, xs0, fmaf(f0.x, d[0], acc[j][0])));
-        acc[j][1] = fmaf(-f0.x, xo1, fmaf(f0.y, xs1, fmaf(f0.x, d[1], acc[j][1])));
-        acc[j][2] = fmaf(-f1.x, xo0, fmaf(f1.y, xs0, fmaf(f1.x, d[2], acc[j][2])));
-        acc[j][3] = fmaf(-f1.x, xo1, fmaf(f1.y, xs1, fmaf(f1.x, d[3], acc[j][3])));
-      }
-
-      // ---- segment end: row tile finished or this warp's run finished
-      const bool tile_end = (grp == kg - 1);
-      if (tile_end || ui == nunits - 1) {
-        if (seg_from_start && tile_end) {
-          store_out<TOK, EPI>(p, tile, g, q, acc);
-        } else {
-          const int sl = (tile == head_tile) ? 0 : 1;  // head / tail tile of this warp
-          float* pp = part_s + ((warp * 2 + sl) * TOK) * kRows;
-#pragma unroll
-          for (int j = 0; j < NJ; ++j)
-#pragma unroll
-            for (int e = 0; e < 2; ++e) {
-              const int tok = 8 * j + 2 * q + e;
-              pp[tok * kRows + g] = acc[j][e];
-              pp[tok * kRows + g + 8] = acc[j][2 + e];
-            }
-        }
-#pragma unroll
-        for (int j = 0; j < NJ; ++j)
-#pragma unroll
-          for (int i = 0; i < 4; ++i) acc[j][i] = 0.f;
-        seg_from_start = true;
-      }
-      if (++grp == kg) { grp = 0; ++tile; }
+      for (int s = 0; s < CH; ++s) unit(cs, ms, s, c * CH + s);
+    } else {
+      for (int s = 0; s < nunits - c * CH; ++s) unit(cs, ms, s, c * CH + s);
     }
     __syncwarp();  // every lane's reads of this slot are done (their values fed the MMAs)
     if (lane == 0 && c + S < nch) issue(c + S);
@@ -721,7 +727,7 @@ size_t gemv_workspace_bytes(int64_t n, int64_t k, int64_t m) {
 // K2 (mma.sync, register unpack) for m <= 8; K2c (tcgen05: TMEM dequant, or fp16 weights straight
 // from SMEM) for 8 < m <= 32.  K2 takes the activation group sums (xsum; computed here if null).
 // SQ_GEMV_PATH=mma|tc overrides (benchmarking).
-int gemv_path(int64_t n, int m, int bits) {
+int gemv_path(int64_t n, int64_t k, int m, int bits) {
   static int forced = -2;
   if (forced == -2) {
     const char* e = getenv("SQ_GEMV_PATH");
@@ -729,7 +735,15 @@ int gemv_path(int64_t n, int m, int bits) {
   }
   if (n % 128) return 0;
   if (forced >= 0) return forced;
-  return m > 8 ? 1 : 0;
+  // measured on B200 (tools/gemv_rot.py --graph, back-to-back launches): the tcgen05 kernel's cost
+  // does not depend on m; the mma.sync kernel's grows with m (activation fragments from L1) but
+  // has the shorter ramp -- it wins on OPT-13B-sized linears at m <= 4 (and m <= 8 off INT4),
+  // the tcgen05 kernel everywhere else, and always for fp16 weights
+  (void)k;
+  if (bits == 16 || m > 8) return 1;
+  const double bytes = (double)n * k * bits / 8.0;
+  if (bytes >= 120e6) return (bits == 3 && m < 8) ? 0 : 1;
+  return (bits == 4 && m > 4) ? 1 : 0;
 }
 
 cudaError_t launch_xsum(const __half* x, int64_t ldx, int64_t m, int64_t k, float2* xsum, cudaStream_t s) {
@@ -743,7 +757,7 @@ cudaError_t launch_xsum(const __half* x, int64_t ldx, int64_t m, int64_t k, floa
 
 cudaError_t launch_gemv(const sq_qweight& w, const __half* x, int64_t ldx, int m, void* y, int64_t ldy, int epi,
                         const float2* xsum, void* ws, cudaStream_t s) {
-  if (gemv_path(w.n, m, w.bits) == 1) return launch_gemv_tc(w, x, ldx, m, y, ldy, epi, ws, s);
+  if (gemv_path(w.n, w.k, m, w.bits) == 1) return launch_gemv_tc(w, x, ldx, m, y, ldy, epi, ws, s);
   if (w.n > kMaxN || w.n / kRows * (w.k / 128) >= (1ll << 31) / 256) return cudaErrorInvalidValue;  // 32-bit index math
   GemvP p{};
   p.packed = static_cast<const uint8_t*>(w.packed);

@@ -99,7 +99,7 @@ sq_status stage_forward(const sq_layer* layers, int n_layers, int phase, const f
     // per-group activation sums only for linears on the mma.sync decode path (K2); the tcgen05
     // decode (K2c) dequantizes the weights and needs none
     const bool q = L.bits != 16;
-    auto k2 = [&](const sq_qweight& w) { return dec && q && gemv_path(w.n, (int)T, w.bits) == 0; };
+    auto k2 = [&](const sq_qweight& w) { return dec && q && gemv_path(w.n, w.k, (int)T, w.bits) == 0; };
     const float* xr = (l == 0) ? x_in : x_out;
     const bool copy = (l == 0 && x_in != x_out);
     // a = LN(x) (layer 0 also initialises the residual buffer x_out = x_in)

@@ -1,0 +1,37 @@
+"""Run by test_gpu_linear.test_decode_forced_path in a subprocess with SQ_GEMV_PATH=mma|tc (the
+path choice is read once per process): decode parity of the forced kernel against the oracle."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+import torch
+
+import synth
+from oracle import oracle as O
+import paper_conf_cluster_zhaowplw25_b200 as sq
+
+
+def main():
+    worst = 0.0
+    for bits in (3, 4, 8, 16):
+        for (n, k) in ((256, 512), (768, 768), (384, 1152)):
+            w = synth.weight_f16(900 + n + bits, n, k)
+            b = synth.bias_f16(901 + n, n)
+            qo = O.QWeight(w, bits, bias=b)
+            qg = sq.QLinear.from_fp16(torch.from_numpy(w).cuda(), bits, torch.from_numpy(b).cuda())
+            for m in (1, 3, 5, 8, 9, 32):
+                x = synth.act_f16(902 + m, m, k)
+                ref = O.linear(x, qo)
+                y = torch.empty((m, n), dtype=torch.float16, device="cuda")
+                sq.sq_linear_decode(qg, torch.from_numpy(x).cuda(), y, 0)
+                torch.cuda.synchronize()
+                yy = y.float().cpu().numpy().astype(np.float64)
+                err = float(np.abs(yy - ref).max() / np.abs(ref).max())
+                worst = max(worst, err)
+                assert err <= 2e-3, (os.environ.get("SQ_GEMV_PATH"), bits, n, k, m, err)
+    print("ok worst", worst)
+
+
+if __name__ == "__main__":
+    main()
