@@ -36,9 +36,25 @@
 
 #include "sq_tc.cuh"
 
+#ifndef SQ_TC_WAIT
+#define SQ_TC_WAIT 0  // experiments: 0 = try_wait with a suspend-time hint, 1 = try_wait spin, 2 = test_wait spin
+#endif
+
 namespace sq {
 namespace {
 using namespace tc;
+
+__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile("{\n\t.reg .pred p;\n\tmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+               : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void wait_bar(uint64_t* bar, uint32_t parity) {
+  if (SQ_TC_WAIT == 0) mbar_wait_park(bar, parity);
+  else if (SQ_TC_WAIT == 1) mbar_wait(bar, parity);
+  else while (!mbar_test(bar, parity)) {}
+}
 
 constexpr int BN = 128;     // weight rows per unit (TMEM lanes, MMA M)
 constexpr int BT = 32;      // token columns (MMA N)
@@ -213,7 +229,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     int xj[X_LAG + 1];         // k-step of the pending activation fetches (ring of X_LAG + 1)
     auto issue_x = [&](int j) {
       const int sx = qx % S_X, rx = qx / S_X;
-      mbar_wait_park(&empty_x[sx], (rx & 1) ^ 1);
+      wait_bar(&empty_x[sx], (rx & 1) ^ 1);
       if (elect_one()) {
         // box {64 k, 32 tokens, 2*UG k-blocks} -> 2*UG SW128 tiles [32][64]
         mbar_arrive_expect_tx(&full_x[sx], X_STAGE);
@@ -257,7 +273,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         for (int t = 0; t < pp; ++t, ++i) {
           if (i < pre) continue;
           const int sw = i % S_W, rw = i / S_W;
-          mbar_wait_park(&empty_w[sw], (rw & 1) ^ 1);
+          wait_bar(&empty_w[sw], (rw & 1) ^ 1);
           trace_ev(p, 0, i);
           issue_w(i, pn, t, j);
           trace_ev(p, 8, i);
@@ -271,16 +287,16 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     int i = 0, q = 0, n_item = 0;
     for (int it = blockIdx.x; it < I; it += C, ++n_item) {
       const int pn = it / Z, j0 = j0_of(it), j1 = j1_of(it), pp = tiles_of(pn);
-      mbar_wait_park(d_empty, (n_item & 1) ^ 1);  // the epilogue drained the previous item
+      wait_bar(d_empty, (n_item & 1) ^ 1);  // the epilogue drained the previous item
       for (int j = j0; j < j1; ++j, ++q) {
         const int sx = q % S_X, rx = q / S_X;
-        mbar_wait_park(&full_x[sx], rx & 1);
+        wait_bar(&full_x[sx], rx & 1);
         const uint64_t bdesc0 = make_sw128_desc(smem_u32(smem + SM::OFF_X + sx * X_STAGE));
         for (int t = 0; t < pp; ++t, ++i) {
           if constexpr (BITS == 16) {
             // A (fp16 weights) straight from the W stage: two SW128 [128 x 64] tiles
             const int sw = i % S_W, rw = i / S_W;
-            mbar_wait_park(&full_w[sw], rw & 1);
+            wait_bar(&full_w[sw], rw & 1);
             tc_fence_after();
             trace_ev(p, 3, i);
             if (elect_one()) {
@@ -303,7 +319,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             continue;
           }
           const int sa = i % S_A, ra = i / S_A;
-          mbar_wait_park(&full_a[sa], ra & 1);
+          wait_bar(&full_a[sa], ra & 1);
           tc_fence_after();
           trace_ev(p, 3, i);
           if (elect_one()) {
@@ -348,9 +364,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const bool tr = (warp == 2 && lane == 0);
     for (int i = dg; i < nunits; i += DQ_GROUPS) {
       const int sw = i % S_W, sa = i % S_A;
-      mbar_wait_park(&full_w[sw], (uint32_t)((i / S_W) & 1));
+      wait_bar(&full_w[sw], (uint32_t)((i / S_W) & 1));
       if (tr) trace_ev(p, 1, i);
-      mbar_wait_park(&empty_a[sa], (uint32_t)(((i / S_A) & 1) ^ 1));
+      wait_bar(&empty_a[sa], (uint32_t)(((i / S_A) & 1) ^ 1));
       if (tr) trace_ev(p, 5, i);
       tc_fence_after();
       const uint32_t meta = reinterpret_cast<const uint32_t*>(smem + SM::OFF_META + sw * BN * 4 * UG)[ru];
@@ -380,7 +396,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     int n_item = 0;
     for (int it = blockIdx.x; it < I; it += C, ++n_item) {
       const int pn = it / Z, pp = tiles_of(pn);
-      mbar_wait_park(d_full, n_item & 1);
+      wait_bar(d_full, n_item & 1);
       tc_fence_after();
       for (int t = 0; t < pp; ++t) {
         float v[BT];
