@@ -84,6 +84,26 @@ sq_status sq_pack(const uint8_t* codes_dev, const void* scales_dev, const void* 
                   int64_t n, int64_t k, int bits, int group, void* packed_dev, void* meta_dev,
                   sq_stream_t stream);
 
+/* ------------------------------------------------------------------------
+ * f2 — inputs of the variance indicator (Proposition 1, eq. 3, P:186-192;
+ *   Theorem 1):  omega_{i,b} = sum_{o in layer i} D_{W_o} S_{W_o}(b)^2 G(X_o),
+ *   G(X) = Var[X] / 4 for round-to-nearest (deterministic) quantization.
+ *   sq_scale_sq_sums: W fp16 [n,k] (8-B aligned), groups of `group` (32/64/128) along k;
+ *     for each b = bits_host[i] (2..8, n_bits <= 8) out_dev[i] = sum_g group * s_g(b)^2 (fp64)
+ *     with s_g(b) = fp16(fp32(mx - mn) / (2^b - 1)) -- exactly the scale sq_quantize_groups
+ *     stores (R5), i.e. D_W * S_W(b)^2 with per-group scales (R17).  k % 128 == 0.
+ *     ws_dev: sq_scale_sq_sums_workspace_bytes(n, k) bytes, 8-B aligned.  Deterministic.
+ *   sq_act_moments: x fp16 [count] (calibration activations X_o, any shape flattened) ->
+ *     out_dev[0] = E[X], out_dev[1] = Var[X] (population), fp64.  Deterministic.
+ *   omega is assembled on the host from these (paper_conf_cluster_zhaowplw25_b200.indicator).
+ * ------------------------------------------------------------------------ */
+size_t sq_scale_sq_sums_workspace_bytes(int64_t n, int64_t k);
+sq_status sq_scale_sq_sums(const void* w_dev, int64_t n, int64_t k, int group, const int32_t* bits_host,
+                           int n_bits, double* out_dev, void* ws_dev, size_t ws_bytes, sq_stream_t stream);
+size_t sq_act_moments_workspace_bytes(int64_t count);
+sq_status sq_act_moments(const void* x_dev, int64_t count, double* out_dev, void* ws_dev, size_t ws_bytes,
+                         sq_stream_t stream);
+
 /* One quantized linear: non-owning view of device memory. */
 typedef struct {
   int32_t bits;          /* 3, 4, 8, or 16 (16 = fp16 weight, not quantized, R7) */

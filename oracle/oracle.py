@@ -7,6 +7,10 @@ It never imports the CUDA package, and the CUDA package never imports it.
 
 Functions whose pin is missing are marked "parity unpinned" (none at present;
 throughput has no paper number to pin).
+
+f2 (variance indicator, eq. 3): scale_sq_sum / act_moments / variance_indicator, pinned by
+closed-form scales (grid-spanning groups), constant groups (omega = 0) and Theorem 1's
+bound on the realised rounding error (tests/test_indicator.py).
 """
 from __future__ import annotations
 
@@ -69,6 +73,36 @@ def quantize_groups(w: np.ndarray, bits: int, group: int = 128):
     z = np.empty((n, k // group), np.float16)
     _check(_lib().oq_quantize_groups(_p(w), n, k, bits, group, _p(codes), _p(s), _p(z)), "quantize")
     return codes, s, z
+
+
+def scale_sq_sum(w: np.ndarray, bits: int, group: int = 128) -> float:
+    """f2, eq. (3) weight term: D_W * S_W(b)^2 with the per-group scale of reading R4
+    (R17) = sum over groups of group * s_g(b)^2, s_g(b) the scale O1 stores.  fp64."""
+    _, s, _ = quantize_groups(w, bits, group)
+    sd = s.astype(np.float64)
+    return float(np.sum(group * sd * sd))
+
+
+def act_moments(x: np.ndarray) -> tuple[float, float]:
+    """E[X], Var[X] (population) over all elements, fp64 (G(X) of eq. 3 is Var[X]/4)."""
+    xd = np.asarray(x, np.float64).ravel()
+    mu = float(np.sum(xd) / xd.size)
+    return mu, float(np.sum((xd - mu) ** 2) / xd.size)
+
+
+def variance_indicator(weights: list[np.ndarray], acts: list[np.ndarray], bits: int, group: int = 128,
+                       stochastic: bool = False) -> float:
+    """Proposition 1, eq. (3): omega_{i,b} = sum_o D_{W_o} S_{W_o}(b)^2 G(X_o) over the
+    linear operators o of a layer; G(X) = Var[X]/4 (deterministic rounding) or (E[X]^2 + Var[X])/6
+    (stochastic).  bits == 16 (not quantized, R7) -> 0."""
+    if bits == 16:
+        return 0.0
+    om = 0.0
+    for w, x in zip(weights, acts):
+        mu, var = act_moments(x)
+        g = (mu * mu + var) / 6.0 if stochastic else var / 4.0
+        om += scale_sq_sum(w, bits, group) * g
+    return om
 
 
 def pack(codes: np.ndarray, scales: np.ndarray, zeros: np.ndarray, bits: int, group: int = 128):

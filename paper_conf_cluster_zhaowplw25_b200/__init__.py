@@ -98,7 +98,8 @@ EXPORTED = [
     "sq_stage_workspace_bytes", "sq_stage_forward", "sq_layernorm_f32", "sq_comm_unique_id_bytes",
     "sq_comm_get_unique_id", "sq_comm_init", "sq_comm_init_local", "sq_comm_destroy",
     "sq_pipeline_workspace_bytes", "sq_pipeline_run", "sq_plan_check", "sq_profile_enable", "sq_profile_read",
-    "sq_launch_count", "sq_pipeline_schedule",
+    "sq_launch_count", "sq_pipeline_schedule", "sq_scale_sq_sums_workspace_bytes", "sq_scale_sq_sums",
+    "sq_act_moments_workspace_bytes", "sq_act_moments",
 ]
 
 
@@ -121,6 +122,11 @@ _opt("sq_pipeline_run", ctypes.c_int, ctypes.POINTER(sq_plan), ctypes.c_int, cty
      P, P, P, P, ctypes.c_size_t, ctypes.POINTER(sq_run_stats), P)
 _opt("sq_plan_check", ctypes.c_int, ctypes.POINTER(sq_plan))
 _opt("sq_pipeline_schedule", I64, ctypes.POINTER(sq_plan), ctypes.c_int, ctypes.POINTER(sq_sched_op), I64)
+_opt("sq_scale_sq_sums_workspace_bytes", ctypes.c_size_t, I64, I64)
+_opt("sq_scale_sq_sums", ctypes.c_int, P, I64, I64, ctypes.c_int, ctypes.POINTER(I32), ctypes.c_int, P, P,
+     ctypes.c_size_t, P)
+_opt("sq_act_moments_workspace_bytes", ctypes.c_size_t, I64)
+_opt("sq_act_moments", ctypes.c_int, P, I64, P, P, ctypes.c_size_t, P)
 
 
 def _check(st: int) -> None:
@@ -215,6 +221,30 @@ def sq_linear_prefill(w: QLinear, x: torch.Tensor, y: torch.Tensor, epi: int = S
     _check(_L.sq_linear_prefill(ctypes.byref(w.c), _ptr(x), x.stride(0), m, _ptr(y), y.stride(0), epi,
                                 _stream(stream)))
     return y
+
+
+# ---------------------------------------------------------------- f2: variance indicator inputs
+def sq_scale_sq_sums(w: torch.Tensor, bits=(3, 4, 8), group: int = 128, stream=None) -> list[float]:
+    """sum_g group * s_g(b)^2 for each b (fp64, on the GPU), W fp16 [n, k] contiguous."""
+    assert w.is_cuda and w.dtype == torch.float16 and w.dim() == 2 and w.is_contiguous()
+    n, k = w.shape
+    bl = (I32 * len(bits))(*bits)
+    out = torch.empty(len(bits), dtype=torch.float64, device=w.device)
+    nb = _L.sq_scale_sq_sums_workspace_bytes(n, k)
+    ws = torch.empty(max(nb, 8), dtype=torch.uint8, device=w.device)
+    _check(_L.sq_scale_sq_sums(_ptr(w), n, k, group, bl, len(bits), _ptr(out), _ptr(ws), ws.numel(), _stream(stream)))
+    return [float(v) for v in out.cpu()]
+
+
+def sq_act_moments(x: torch.Tensor, stream=None) -> tuple[float, float]:
+    """(E[X], Var[X]) of fp16 activations (all elements), fp64 on the GPU."""
+    assert x.is_cuda and x.dtype == torch.float16 and x.is_contiguous()
+    out = torch.empty(2, dtype=torch.float64, device=x.device)
+    nb = _L.sq_act_moments_workspace_bytes(x.numel())
+    ws = torch.empty(max(nb, 8), dtype=torch.uint8, device=x.device)
+    _check(_L.sq_act_moments(_ptr(x), x.numel(), _ptr(out), _ptr(ws), ws.numel(), _stream(stream)))
+    o = out.cpu()
+    return float(o[0]), float(o[1])
 
 
 def sq_profile_enable(on: bool = True) -> None:

@@ -51,3 +51,15 @@ def test_invalid_arguments_rejected_before_launch():
     w = sq.sq_qweight(4, 128, 16, 100, 16, 16, None)
     st = L.sq_linear_decode(ctypes.byref(w), None, 128, 1, None, 8, 0, None, None, 0, None)
     assert st == sq.SQ_EINVAL
+
+
+def test_indicator_arguments_rejected_before_launch():
+    import paper_conf_cluster_zhaowplw25_b200 as sq
+    L = sq.lib()
+    bits = (ctypes.c_int32 * 2)(4, 9)
+    st = L.sq_scale_sq_sums(None, 8, 128, 128, bits, 2, None, None, 0, None)
+    assert st == sq.SQ_EINVAL and b"bits" in L.sq_last_error()
+    st = L.sq_scale_sq_sums(None, 8, 100, 128, bits, 1, None, None, 0, None)
+    assert st == sq.SQ_EINVAL
+    assert L.sq_scale_sq_sums_workspace_bytes(8, 100) == 0
+    assert L.sq_act_moments(None, 0, None, None, 0, None) == sq.SQ_EINVAL
