@@ -7,7 +7,7 @@ regression over profiled sample points:
   decode  (memory-bound, "MOPs"):                    t_dec(v, t + s)  ~ [1, v, v (t+s), (t+s)]
 
 with v the micro-batch size, s the prompt length and t + s the past sequence length.  Here the
-samples are our own kernels (``sq_stage_forward`` on a 3-layer synthetic stage, CUDA events), fitted per
+samples are our own kernels (``sq_stage_forward`` on an 8-layer synthetic stage, CUDA events), fitted per
 bit width by least squares; the model error on unseen workloads is reported like the paper's
 < 6 %.  The attention stub (reading R12) has no KV cache, so the (t+s) terms fit to ~0 on
 this path; they are kept so the model has the paper's form.
@@ -87,17 +87,18 @@ class LatencyModel:
 
 # ---------------------------------------------------------------- profiling (GPU)
 def profile(h1: int, h2: int, bits_set=(3, 4, 8, 16), pre_points=((1, 128), (1, 512), (2, 256), (4, 512), (8, 512)),
-            dec_points=((1, 256), (8, 512), (16, 384), (32, 640), (32, 1024)), reps: int = 5, act: int = 0) -> list[dict]:
-    """Time sq_stage_forward per bit width on a stage of 3 synthetic layers (so the per-layer time
-    includes the steady-state launch overlap of consecutive layers, as in a real stage) and divide
-    by 3: prefill v sequences x s tokens, decode v tokens (past length ctx).  3 distinct layers
-    stream their weights from HBM."""
+            dec_points=((1, 256), (8, 512), (16, 384), (32, 640), (32, 1024)), reps: int = 5, act: int = 0,
+            n_layers: int = 8) -> list[dict]:
+    """Time sq_stage_forward per bit width on a stage of ``n_layers`` synthetic layers (so the
+    per-layer time includes the steady-state launch overlap of consecutive layers, as in a real
+    stage) and divide by n_layers: prefill v sequences x s tokens, decode v tokens (past length
+    ctx).  Distinct layers: every weight byte streams from HBM."""
     import torch
     from . import SQ_DECODE, SQ_PREFILL
     from .runtime import StageWorkspace, build_layers, layer_array, sq_stage_forward
     out = []
     for b in bits_set:
-        copies = build_layers(3, h1, h2, [b] * 3, act=act)
+        copies = build_layers(n_layers, h1, h2, [b] * n_layers, act=act)
         arr = layer_array(copies)
         max_tok = max(v * s for v, s in pre_points)
         ws = StageWorkspace(copies, max_tok)
