@@ -73,6 +73,47 @@ def test_stage_parity_opt125m(opt125m, phase, T):
     assert normwise(qkv.float().cpu().numpy(), ref_qkv) <= TOL
 
 
+@pytest.mark.parametrize("T", [1, 8, 32])
+def test_decode_stage_cuda_graph(opt125m, T):
+    """configs[0] decode step captured in ONE CUDA graph (SURVEY D-1): the stage forward is
+    asynchronous on the caller's stream and allocation-free, so it captures as-is (PDL edges
+    included); replays equal the eager run bitwise and the oracle within 2e-3."""
+    sq, R = rt()
+    bits, g, o = opt125m
+    x = synth.hidden_f32(700 + T, T, H1)
+    ws = R.StageWorkspace(g, T)
+    xi = torch.from_numpy(x).cuda()
+    xo_eager = torch.empty_like(xi)
+    R.sq_stage_forward(g, 1, xi, xo_eager, ws)
+    torch.cuda.synchronize()
+    xo = torch.empty_like(xi)
+    arr = R.layer_array(g)
+    side = torch.cuda.Stream()
+    side.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(side):  # warm-up on the capture stream
+        R.sq_stage_forward(g, 1, xi, xo, ws, arr=arr)
+    torch.cuda.current_stream().wait_stream(side)
+    torch.cuda.synchronize()
+    graph = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(graph):
+        R.sq_stage_forward(g, 1, xi, xo, ws, arr=arr)
+    for _ in range(3):
+        xo.zero_()
+        graph.replay()
+    torch.cuda.synchronize()
+    assert torch.equal(xo, xo_eager)
+    ref, _ = O.stage(o, x.astype(np.float64))
+    assert normwise(xo.cpu().numpy(), ref) <= TOL
+    # graph replay vs eager launches: per-step latency of the 12-layer decode step
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(20):
+        graph.replay()
+    e1.record()
+    torch.cuda.synchronize()
+    print(f"configs[0] decode step T={T}: {e0.elapsed_time(e1) / 20 * 1e3:.1f} us per step (CUDA graph)")
+
+
 def test_stage_in_place_and_gelu():
     sq, R = rt()
     bits = [4, 16]
