@@ -88,7 +88,8 @@ template <int BITS, int UG>
 struct DCfg {
   // weight ring: a slot lives TMA latency (~1.8k cycles) + wait for its group + dequant (~2k)
   // (quantized rings are multiples of DQ_GROUPS so each slot is owned by one dequant group)
-  static constexpr int S_W = BITS == 16 ? 5 : (UG == 2 ? 10 : (BITS == 8 ? 10 : (BITS == 4 ? 18 : 24)));
+  static constexpr int S_W0 = UG == 2 ? 10 : (BITS == 8 ? 10 : (BITS == 4 ? 18 : 24));
+  static constexpr int S_W = BITS == 16 ? 5 : (S_W0 / DQ_GROUPS) * DQ_GROUPS;
   // TMEM A slots of 64*UG columns: the dequant warps fill slot i % S_A while the MMA reads the
   // others (slots are owned by one dequant group: multiples of DQ_GROUPS)
   static constexpr int A_SLOT = 64 * UG;
