@@ -153,17 +153,22 @@ __device__ __forceinline__ void trace_cta(const TcP& p, int ev) {
 
 template <int EPI>
 __device__ __forceinline__ void epi_store(const TcP& p, int64_t row, const float (&v)[BT], float bias) {
+  if constexpr (EPI == SQ_EPI_F32_ACCUM) {
+    // residual read-modify-write: every load before any store (no per-token L2 round trip chain)
+    float* yb = static_cast<float*>(p.y) + row;
 #pragma unroll
-  for (int t = 0; t < BT; ++t) {
-    if (t < p.m) {
-      const float o = v[t] + bias;
-      if constexpr (EPI == SQ_EPI_F32_ACCUM) {
-        float* yp = static_cast<float*>(p.y) + (int64_t)t * p.ldy + row;
-        *yp += o;
-      } else {
-        static_cast<__half*>(p.y)[(int64_t)t * p.ldy + row] = __float2half_rn(apply_act<EPI>(o));
-      }
+    for (int h = 0; h < BT; h += 16) {
+      float r[16];
+#pragma unroll
+      for (int t = 0; t < 16; ++t) r[t] = h + t < p.m ? __ldcg(yb + (int64_t)(h + t) * p.ldy) : 0.f;
+#pragma unroll
+      for (int t = 0; t < 16; ++t)
+        if (h + t < p.m) yb[(int64_t)(h + t) * p.ldy] = r[t] + (v[h + t] + bias);
     }
+  } else {
+#pragma unroll
+    for (int t = 0; t < BT; ++t)
+      if (t < p.m) static_cast<__half*>(p.y)[(int64_t)t * p.ldy + row] = __float2half_rn(apply_act<EPI>(v[t] + bias));
   }
 }
 
