@@ -257,7 +257,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             } else {
               // placement T16 as lines: box {line, lpu * UG lines, 8 row tiles} -> [tile][group][16][GB]
               tma_load_3d(wdst, &tm_w, &full_w[sw], 0, j * UG * LPU, tile16);
-              tma_load_3d(smem + SM::OFF_META + sw * BN * 4 * UG, &tm_m, &full_w[sw], 0, j * UG, tile16);
+              tma_load_2d(smem + SM::OFF_META + sw * BN * 4 * UG, &tm_m, &full_w[sw], j * UG * 16, tile16);
             }
       }
       __syncwarp();
@@ -631,9 +631,11 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
     cudaError_t e = enc(&tw, CU_TENSOR_MAP_DATA_TYPE_UINT8, w.packed, 3, dw, sw_, bw,
                         wl.sw128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE);
     if (e != cudaSuccess) return e;
-    const uint64_t dm[3] = {16, (uint64_t)kg, nt}, sm_[2] = {64, (uint64_t)kg * 64};
-    const uint32_t bm[3] = {16, (uint32_t)ug, BN / 16};
-    e = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, w.meta, 3, dm, sm_, bm, CU_TENSOR_MAP_SWIZZLE_NONE);
+    // meta as [n/16 tiles][kg * 16] u32: one box row = the UG groups of a tile (64 * UG contiguous
+    // bytes), 8 rows per unit (a 3-D {16, UG, 8} box would move 16 rows of 64 B)
+    const uint64_t dm[2] = {(uint64_t)kg * 16, nt}, sm_[1] = {(uint64_t)kg * 64};
+    const uint32_t bm[2] = {(uint32_t)(16 * ug), BN / 16};
+    e = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, w.meta, 2, dm, sm_, bm, CU_TENSOR_MAP_SWIZZLE_NONE);
     if (e != cudaSuccess) return e;
   }
   TcP p{};

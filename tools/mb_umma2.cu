@@ -66,6 +66,35 @@ __global__ void __launch_bounds__(32 * 18, 1) k_umma2(long long* out, int iters,
   if (warp == 0) { tc_fence_after(); tmem_dealloc(0, 512); }
 }
 
+// pure tcgen05.st throughput: W warps each issue `iters` st.32x32b.x16 (2 KB per warp-instruction),
+// with a wait::st every `batch` stores; bytes per cycle per SM from clock64 on warp 0
+__global__ void __launch_bounds__(32 * 17, 1) k_st(long long* out, int iters, int batch, int nwarps) {
+  __shared__ uint32_t tbase;
+  const int warp = threadIdx.x >> 5;
+  if (warp == 0) tmem_alloc(&tbase, 512);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  long long t0 = clock64();
+  if (warp < nwarps) {
+    const uint32_t lane_base = (uint32_t)((warp & 3) * 32) << 16;
+    uint32_t v[16];
+#pragma unroll
+    for (int i = 0; i < 16; ++i) v[i] = (uint32_t)i;
+    for (int i = 0; i < iters; ++i) {
+      tmem_st16(lane_base + ((i * 16 + (warp >> 2) * 128) & 511), v);
+      if ((i + 1) % batch == 0) tc_wait_st();
+    }
+    tc_wait_st();
+  }
+  __syncthreads();
+  long long t1 = clock64();
+  if (threadIdx.x == 0) { out[2 * blockIdx.x] = t0; out[2 * blockIdx.x + 1] = t1; }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 0) { tc_fence_after(); tmem_dealloc(0, 512); }
+}
+
 int main() {
   int sms = 0;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
@@ -83,6 +112,18 @@ int main() {
     printf("mode %d (%s) st_warps %2d: %.1f cycles per M128 N32 K16 MMA\n", cs.mode,
            cs.mode == 0 ? "same D" : (cs.mode == 1 ? "D over 4 tiles" : "D over 4 tiles + tcgen05.st"), cs.w,
            (double)(h[1] - h[0]) / iters);
+  }
+  for (int w : {4, 8, 16}) {
+    for (int batch : {1, 4, 16}) {
+      const int iters = 4096;
+      k_st<<<sms, 32 * 17>>>(d, iters, batch, w);
+      cudaError_t err = cudaDeviceSynchronize();
+      if (err != cudaSuccess) { printf("error %s\n", cudaGetErrorString(err)); return 1; }
+      long long h[2];
+      cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost);
+      const double bytes = (double)w * iters * 2048;
+      printf("tcgen05.st.32x32b.x16: %2d warps, wait every %2d: %.1f B/cycle per SM\n", w, batch, bytes / (double)(h[1] - h[0]));
+    }
   }
   return 0;
 }
