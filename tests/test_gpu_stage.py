@@ -198,3 +198,24 @@ def test_stage_opt13b_layer_teacher_forced(bits):
         rows = [0, T // 2, T - 1]
         ref, _ = O.stage(o, x[rows].astype(np.float64))
         assert normwise(xo.cpu().numpy()[rows], ref) <= TOL
+
+
+@pytest.mark.parametrize("bits", [3, 4])  # (8 and 16 at full OPT-13B size above; ~70 s of oracle each)
+def test_stage_opt66b_layer_bench_config(bits):
+    """One OPT-66B-shaped layer (d = 9216, configs[3]) in the launch configuration bench.py times:
+    decode micro-batch xi = 32 tokens and prefill micro-batch eta x s = 8 x 512 = 4096 tokens;
+    oracle teacher-forced on sampled rows (first, middle, last)."""
+    sq, R = rt()
+    h1, h2 = 9216, 36864
+    g = R.build_layers(1, h1, h2, [bits], layer_offset=21)
+    o = oracle_layers(1, h1, h2, [bits], layer_offset=21)
+    for phase, T in ((1, 32), (0, 4096)):
+        x = synth.hidden_f32(31 + T, T, h1)
+        ws = R.StageWorkspace(g, T)
+        xi = torch.from_numpy(x).cuda()
+        xo = torch.empty_like(xi)
+        R.sq_stage_forward(g, phase, xi, xo, ws)
+        torch.cuda.synchronize()
+        rows = [0, T // 2 + 1, T - 1]
+        ref, _ = O.stage(o, x[rows].astype(np.float64))
+        assert normwise(xo.cpu().numpy()[rows], ref) <= TOL, (phase, T)
