@@ -37,6 +37,10 @@ WORKLOADS = {
     # BASELINE.json configs[3]
     "opt66b": dict(name="configs[3] OPT-66B-shaped 64 layers, uneven mixed-bit pipeline, prompt 512 + 128 decode tokens",
                    h1=9216, h2=36864, L=64, act=0, eta=8, xi=32, s=512, n_dec=128, b_per_gpu=32, balanced=True),
+    # BASELINE.json configs[4]: BLOOM-176B-shaped (d = 14336, fused QKV, GeLU), 70 layers, INT3/INT4 50/50
+    "bloom176b": dict(name="configs[4] BLOOM-176B-shaped 70 layers, INT3/INT4-mixed, uneven pipeline with micro-batching",
+                      h1=14336, h2=57344, L=70, act=1, eta=8, xi=32, s=512, n_dec=128, b_per_gpu=32, balanced=True,
+                      choices=(3, 4)),
     # BASELINE.json configs[0] (small; for quick runs)
     "opt125m": dict(name="configs[0] OPT-125m-shaped 12 layers, bits {3,4,8,16}, prefill 1x32 + 8 decode steps",
                     h1=768, h2=3072, L=12, act=0, eta=1, xi=1, s=32, n_dec=8, b_per_gpu=1, balanced=False),
@@ -241,7 +245,7 @@ def run_ours(args, wl):
 
     B = wl["b_per_gpu"] * P
     L, h1, h2 = wl["L"], wl["h1"], wl["h2"]
-    bits = [int(b) for b in synth.bits_plan(2, L, balanced=wl["balanced"])]
+    bits = [int(b) for b in synth.bits_plan(2, L, choices=wl.get("choices", (3, 4, 8, 16)), balanced=wl["balanced"])]
     costs = PL.phase_costs(bits, h1, h2, B, wl["eta"], wl["xi"], wl["s"], wl["n_dec"], pk["hbm_gbs"],
                            pk["tflops_sustained"])
     sol = PL.partition_layers(costs, P)

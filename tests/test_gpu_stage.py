@@ -219,3 +219,23 @@ def test_stage_opt66b_layer_bench_config(bits):
         rows = [0, T // 2 + 1, T - 1]
         ref, _ = O.stage(o, x[rows].astype(np.float64))
         assert normwise(xo.cpu().numpy()[rows], ref) <= TOL, (phase, T)
+
+
+def test_stage_bloom_width_layer():
+    """configs[4] width: d = 14336 (BLOOM-176B LayerNorm, fused QKV 43008 x 14336, GeLU), with a
+    reduced FFN (h2 = 4096) to bound the oracle's cost; decode 32 tokens and prefill 512 tokens,
+    oracle teacher-forced on sampled rows."""
+    sq, R = rt()
+    h1, h2 = 14336, 4096
+    g = R.build_layers(1, h1, h2, [4], act=1, layer_offset=69)
+    o = oracle_layers(1, h1, h2, [4], act=1, layer_offset=69)
+    for phase, T in ((1, 32), (0, 512)):
+        x = synth.hidden_f32(41 + T, T, h1)
+        ws = R.StageWorkspace(g, T)
+        xi = torch.from_numpy(x).cuda()
+        xo = torch.empty_like(xi)
+        R.sq_stage_forward(g, phase, xi, xo, ws)
+        torch.cuda.synchronize()
+        rows = [0, T - 1]
+        ref, _ = O.stage(o, x[rows].astype(np.float64))
+        assert normwise(xo.cpu().numpy()[rows], ref) <= TOL, (phase, T)
