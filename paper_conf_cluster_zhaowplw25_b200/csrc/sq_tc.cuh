@@ -159,121 +159,6 @@ __device__ __forceinline__ void dequant_row_batches(const uint8_t* wst, uint32_t
   }
 }
 
-// Decode variant (K2c): the A operand holds s*c only -- the zero-point term z * sum(x) of the group
-// is added by one extra MMA per unit (z columns x activation group sums, decode kernel).  With the
-// magic-number code v = off + c (exact), s*c = v*s + (-off*s) is ONE HFMA2 per pair: -off*s is exact
-// in fp16 (power-of-two scaling) and the FMA rounds once, to fp16(s*c).  Rows whose -off*s would
-// overflow fp16 (|s| >= 65504/off, pathological outlier groups) take (v - off)*s (HSUB2 + HMUL2).
-// Offsets: INT4 1024 / 64 (low / high nibble slot of L4), INT8 1024 (PRMT), INT3 8 (code placed
-// under exponent 2^3, as in K2).  Same batch/swizzle conventions as dequant_row_batches.
-__device__ __forceinline__ uint32_t hfma2_u(uint32_t a, uint32_t b, uint32_t c) {
-  __half2 r = __hfma2(*reinterpret_cast<__half2*>(&a), *reinterpret_cast<__half2*>(&b), *reinterpret_cast<__half2*>(&c));
-  return *reinterpret_cast<uint32_t*>(&r);
-}
-__device__ __forceinline__ uint32_t hsub_mul_u(uint32_t v, uint32_t off2, uint32_t s2) {
-  __half2 c = __hsub2(*reinterpret_cast<__half2*>(&v), *reinterpret_cast<__half2*>(&off2));
-  __half2 r = __hmul2(c, *reinterpret_cast<__half2*>(&s2));
-  return *reinterpret_cast<uint32_t*>(&r);
-}
-// -off * s as half2 (exact unless it overflows; `ok` false then)
-__device__ __forceinline__ uint32_t neg_off_s(uint32_t s_bits, float off, bool& ok) {
-  const float nb = -off * __half2float(__ushort_as_half((unsigned short)s_bits));
-  ok = fabsf(nb) <= 65504.f;
-  const uint32_t h = __half_as_ushort(__float2half_rn(nb));
-  return h * 0x10001u;
-}
-
-template <int BITS, int NB>
-__device__ __forceinline__ void unpack_sc_row_batches(const uint8_t* wst, uint32_t meta, int r, uint32_t taddr,
-                                                      int row_off, int B0) {
-  const uint32_t sb = meta & 0xFFFFu;
-  const uint32_t s2 = sb * 0x10001u;
-  constexpr uint32_t K1024 = 0x64006400u, K64 = 0x54005400u, K8 = 0x48004800u;
-  bool ok_a, ok_b;
-  if constexpr (BITS == 4) {
-    const uint32_t nbA = neg_off_s(sb, 1024.f, ok_a), nbB = neg_off_s(sb, 64.f, ok_b);
-    const bool fast = ok_a;  // ok_a implies ok_b
-    const uint8_t* line = wst + (row_off & ~127);
-    const int h4 = (row_off >> 4) & 4, swz = (row_off >> 7) & 7;
-#pragma unroll
-    for (int bi = 0; bi < NB; ++bi) {
-      const int b = B0 + bi;
-      const int pc = (h4 | b) ^ swz;  // 128-B lines under SWIZZLE_128B (see dequant_row_batches)
-      uint4 v = *reinterpret_cast<const uint4*>(line + pc * 16);
-      const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
-      uint32_t o[16];
-      if (fast) {
-#pragma unroll
-        for (int w = 0; w < 4; ++w) {
-          const uint32_t x = wv[w], x8 = x >> 8;
-          o[4 * w + 0] = hfma2_u(lop3_and_or(x, 0x000F000Fu, K1024), s2, nbA);
-          o[4 * w + 1] = hfma2_u(lop3_and_or(x, 0x00F000F0u, K64), s2, nbB);
-          o[4 * w + 2] = hfma2_u(lop3_and_or(x8, 0x000F000Fu, K1024), s2, nbA);
-          o[4 * w + 3] = hfma2_u(lop3_and_or(x8, 0x00F000F0u, K64), s2, nbB);
-        }
-      } else {
-#pragma unroll
-        for (int w = 0; w < 4; ++w) {
-          const uint32_t x = wv[w], x8 = x >> 8;
-          o[4 * w + 0] = hsub_mul_u(lop3_and_or(x, 0x000F000Fu, K1024), K1024, s2);
-          o[4 * w + 1] = hsub_mul_u(lop3_and_or(x, 0x00F000F0u, K64), K64, s2);
-          o[4 * w + 2] = hsub_mul_u(lop3_and_or(x8, 0x000F000Fu, K1024), K1024, s2);
-          o[4 * w + 3] = hsub_mul_u(lop3_and_or(x8, 0x00F000F0u, K64), K64, s2);
-        }
-      }
-      tmem_st16(taddr + 16 * b, o);
-    }
-  } else if constexpr (BITS == 8) {
-    const uint32_t nbA = neg_off_s(sb, 1024.f, ok_a);
-    const uint8_t* row = wst + row_off;
-#pragma unroll
-    for (int bi = 0; bi < NB; ++bi) {
-      const int b = B0 + bi;
-      uint32_t o[16];
-#pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        const int c = 2 * b + h, pc = c ^ (r & 7);  // SWIZZLE_128B
-        uint4 v = *reinterpret_cast<const uint4*>(row + pc * 16);
-        const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
-#pragma unroll
-        for (int t = 0; t < 4; ++t) {
-          const uint32_t lo = prmt(wv[t], 0x64646464u, 0x4140u), hi = prmt(wv[t], 0x64646464u, 0x4342u);
-          o[8 * h + 2 * t] = ok_a ? hfma2_u(lo, s2, nbA) : hsub_mul_u(lo, K1024, s2);
-          o[8 * h + 2 * t + 1] = ok_a ? hfma2_u(hi, s2, nbA) : hsub_mul_u(hi, K1024, s2);
-        }
-      }
-      tmem_st16(taddr + 16 * b, o);
-    }
-  } else {
-    static_assert(BITS == 3, "unpack_sc_row_batches: 3/4/8 bits");
-    const uint32_t nbA = neg_off_s(sb, 8.f, ok_a);
-    const uint32_t* row = reinterpret_cast<const uint32_t*>(wst + row_off);
-#pragma unroll
-    for (int bi = 0; bi < NB; ++bi) {
-      const int bl = B0 + bi;
-      const uint32_t L0 = row[3 * bl], L1 = row[3 * bl + 1], H = row[3 * bl + 2];
-      uint32_t o[16];
-#pragma unroll
-      for (int a = 0; a < 2; ++a) {
-        const uint32_t La = a ? L1 : L0;
-#pragma unroll
-        for (int i = 0; i < 8; ++i) {
-          // low two bits -> mantissa bits 7..8, high bit -> bit 9, under exponent 2^3: half2(8 + c)
-          const int sl = 7 - 2 * i;
-          const uint32_t l = sl >= 0 ? (La << sl) : (La >> (-sl));
-          const int sh = i + 8 * a - 9;
-          const uint32_t hs = sh >= 0 ? (H >> sh) : (H << (-sh));
-          uint32_t t;
-          asm("lop3.b32 %0, %1, %2, %3, 0xD8;" : "=r"(t) : "r"(hs), "r"(l), "r"(0x01800180u));  // mask ? l : hs
-          const uint32_t v = lop3_and_or(t, 0x03800380u, K8);
-          o[8 * a + i] = ok_a ? hfma2_u(v, s2, nbA) : hsub_mul_u(v, K8, s2);
-        }
-      }
-      tmem_st16(taddr + 16 * bl, o);
-    }
-  }
-}
-
 // the whole 128-k group of this thread's row: 64 half2 columns at taddr .. taddr + 63
 template <int BITS>
 __device__ __forceinline__ void dequant_row_to_tmem(const uint8_t* wst, uint32_t meta, int r, uint32_t taddr,
