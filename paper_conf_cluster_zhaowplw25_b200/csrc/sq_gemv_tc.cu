@@ -81,6 +81,9 @@ constexpr int A_COL = PMAX * BT;      // S_A x (64 * UG) columns
 constexpr int NUM_THREADS = 32 * (2 + DQ_WARPS + 4);  // producer, MMA, dequant, epilogue
 constexpr int EPI_WARP0 = 2 + DQ_WARPS;
 constexpr uint32_t kIdescTc = make_idesc(BN, BT);
+#ifndef SQ_TC_XLDG
+#define SQ_TC_XLDG 0  // 1: the epilogue warps load the activation slices (LDG -> STS), 0: TMA (measured: 0 is faster)
+#endif
 constexpr int X_LAG = 0;              // activations of step q are fetched just before its weights (X_LAG > 0 deadlocks once P * (X_LAG + 1) > S_W)
 
 // UG = 128-k groups per unit, chosen so a weight stage is ~16 KB (INT3/INT4: 2, INT8: 1).
@@ -133,6 +136,8 @@ struct TcP {
   int* cnt;     // [panels]
   unsigned long long* trace;  // debug: CTA 0 per-unit clock64 events (sq_debug_trace), or null
   int abl;                    // debug ablation (SQ_TC_ABL): 1 = no dequant, 2 = no MMAs (results wrong)
+  const __half* x;            // activations [m][ldx] (SQ_TC_XLDG: loaded by the epilogue warps)
+  int ldx;
 };
 
 #ifndef SQ_TC_DEBUG
@@ -208,7 +213,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   auto j1_of = [&](int it) { return (int)((long long)(it % Z + 1) * ks / Z); };
 
   if (threadIdx.x == 0) {
-    for (int i = 0; i < S_X; ++i) { mbar_init(&full_x[i], 1); mbar_init(&empty_x[i], 1); }
+    for (int i = 0; i < S_X; ++i) { mbar_init(&full_x[i], SQ_TC_XLDG ? 4 : 1); mbar_init(&empty_x[i], 1); }
     // fp16 weights are the MMA's A operand straight from SMEM: the MMA commit frees the slot
     for (int i = 0; i < S_W; ++i) { mbar_init(&full_w[i], 1); mbar_init(&empty_w[i], BITS == 16 ? 1 : DQ_PER_GROUP); }
     for (int i = 0; i < S_A; ++i) { mbar_init(&full_a[i], DQ_PER_GROUP); mbar_init(&empty_a[i], 1); }
@@ -227,7 +232,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   tc_fence_after();
   if (misc[0] != 0) __trap();  // a 512-column allocation owns all of TMEM: base is lane 0, column 0
   constexpr uint32_t tmem = 0;
-  if (threadIdx.x == 0) trace_cta(p, 14);
+  if (threadIdx.x == 0) { trace_cta(p, 14); trace_ev(p, 13, 0); }
 
   if (warp == 0) {
     // ---------------- producer.  The warp runs the loop and the waits; one elected lane issues.
@@ -268,14 +273,18 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     for (int it = blockIdx.x; it < I && pre < S_W; it += C) {
       const int pn = it / Z, j1 = j1_of(it), pp = tiles_of(pn);
       for (int j = j0_of(it); j < j1 && pre < S_W; ++j)
-        for (int t = 0; t < pp && pre < S_W; ++t, ++pre) issue_w(pre, pn, t, j);
+        for (int t = 0; t < pp && pre < S_W; ++t, ++pre) {
+          issue_w(pre, pn, t, j);
+          trace_ev(p, 0, pre);
+        }
     }
     pdl_wait();
+    trace_ev(p, 7, 0);
     for (int it = blockIdx.x; it < I; it += C) {
       const int pn = it / Z, j1 = j1_of(it), pp = tiles_of(pn);
       for (int j = j0_of(it); j < j1; ++j, ++q) {
         xj[q % (X_LAG + 1)] = j;
-        if (q >= X_LAG) issue_x(xj[(q - X_LAG) % (X_LAG + 1)]);
+        if (!SQ_TC_XLDG && q >= X_LAG) issue_x(xj[(q - X_LAG) % (X_LAG + 1)]);
         for (int t = 0; t < pp; ++t, ++i) {
           if (i < pre) continue;
           const int sw = i % S_W, rw = i / S_W;
@@ -286,7 +295,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         }
       }
     }
-    for (int r = q > X_LAG ? q - X_LAG : 0; r < q; ++r) issue_x(xj[r % (X_LAG + 1)]);
+    if (!SQ_TC_XLDG)
+      for (int r = q > X_LAG ? q - X_LAG : 0; r < q; ++r) issue_x(xj[r % (X_LAG + 1)]);
   } else if (warp == 1) {
     // ---------------- MMA issuer: the warp waits, one elected lane issues a unit's 8*UG MMAs and
     // commits.  TMEM base is 0, so every operand is warp-uniform.
@@ -297,6 +307,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       for (int j = j0; j < j1; ++j, ++q) {
         const int sx = q % S_X, rx = q / S_X;
         wait_bar(&full_x[sx], rx & 1);
+        trace_ev(p, 6, q);
         const uint64_t bdesc0 = make_sw128_desc(smem_u32(smem + SM::OFF_X + sx * X_STAGE));
         for (int t = 0; t < pp; ++t, ++i) {
           if constexpr (BITS == 16) {
@@ -398,10 +409,39 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const int r = sp * 32 + lane;
     const uint32_t lane_base = (uint32_t)(sp * 32) << 16;
     const bool leader = threadIdx.x == EPI_WARP0 * 32;
-    pdl_wait();  // y / partial writes below
-    int n_item = 0;
+    pdl_wait();  // activation loads, y / partial writes below
+    int n_item = 0, qx = 0;
+    const int ew = warp - EPI_WARP0;  // 0..3
     for (int it = blockIdx.x; it < I; it += C, ++n_item) {
       const int pn = it / Z, pp = tiles_of(pn);
+      if (SQ_TC_XLDG) {
+        // activation slices of this item's k-steps: [32 tokens][UG*128 k] fp16 as 2*UG SW128 tiles
+        // [32][64] (tokens >= m zero), written with generic stores then handed to the tensor core
+        // (fence.proxy.async) -- off the TMA engine, whose per-SM ingest the weight stream needs
+        constexpr int CHUNKS = 2 * UG * BT * 8;  // 16-B chunks per step
+        for (int j = j0_of(it); j < j1_of(it); ++j, ++qx) {
+          const int sx = qx % S_X, rx = qx / S_X;
+          wait_bar(&empty_x[sx], (rx & 1) ^ 1);
+          uint8_t* xs = smem + SM::OFF_X + sx * X_STAGE;
+          uint4 v[CHUNKS / 128];
+#pragma unroll
+          for (int u = 0; u < CHUNKS / 128; ++u) {
+            const int c = (u * 128) + ew * 32 + lane;  // chunk: tile c / 256, row (c / 8) % 32, col c % 8
+            const int tt = c >> 8, r = (c >> 3) & 31, lc = c & 7;
+            v[u] = r < p.m ? __ldg(reinterpret_cast<const uint4*>(p.x + (int64_t)r * p.ldx + (int64_t)j * UG * 128 + tt * 64 + lc * 8))
+                           : make_uint4(0u, 0u, 0u, 0u);
+          }
+#pragma unroll
+          for (int u = 0; u < CHUNKS / 128; ++u) {
+            const int c = (u * 128) + ew * 32 + lane;
+            const int tt = c >> 8, r = (c >> 3) & 31, lc = c & 7;
+            *reinterpret_cast<uint4*>(xs + tt * X_BLOCK + r * 128 + ((lc ^ (r & 7)) << 4)) = v[u];
+          }
+          fence_proxy_async_smem();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&full_x[sx]);
+        }
+      }
       wait_bar(d_full, n_item & 1);
       tc_fence_after();
       for (int t = 0; t < pp; ++t) {
@@ -675,6 +715,8 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
     if (abl < 0) { const char* e = getenv("SQ_TC_ABL"); abl = e ? atoi(e) : 0; }
     p.abl = abl;
   }
+  p.x = x;
+  p.ldx = (int)ldx;
   const int nc = pl.ctas;
   const double bytes = (double)w.n * w.k * w.bits / 8.0 + (w.bits != 16 ? (double)w.n * (w.k / 128) * 4.0 : 0.0);
   auto t = prof_begin(KC_GEMV, bytes, 2.0 * m * w.n * w.k, s);
