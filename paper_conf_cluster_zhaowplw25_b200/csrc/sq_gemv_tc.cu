@@ -226,6 +226,38 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     if constexpr (BITS != 16) prefetch_tmap(&tm_m);
   }
   pdl_trigger();  // the next kernel may be scheduled as soon as SMs free up
+  constexpr int LPU_ = BITS == 3 ? 3 : (BITS == 4 ? 8 : 16);
+  // TMA of weight unit i (panel pn, tile t, k-step j) into ring slot i % S_W; one thread
+  auto issue_w1 = [&](int i, int pn, int t, int j) {
+    const int sw = i % S_W;
+    const int tile16 = (pn * P + t) * (BN / 16);
+    uint8_t* wdst = smem + SM::OFF_W + sw * SM::W_STAGE;
+    const bool no_meta = SQ_TC_DEBUG && (p.abl & 16), no_w = SQ_TC_DEBUG && (p.abl & 32);
+    mbar_arrive_expect_tx(&full_w[sw], (BITS == 16 ? BN * 256u : (uint32_t)(BN * GCfg<BITS>::GB * UG + BN * 4 * UG)) -
+                                           (no_meta && BITS != 16 ? BN * 4 * UG : 0) -
+                                           (no_w ? BN * GCfg<BITS>::GB * UG : 0));
+    if constexpr (BITS == 16) {
+      // row-major fp16 [n][k]: two SW128 boxes [128 rows][64 k] = the MMA's K-major A tiles
+      tma_load_2d(wdst, &tm_w, &full_w[sw], j * 128, (pn * P + t) * BN);
+      tma_load_2d(wdst + BN * 128, &tm_w, &full_w[sw], j * 128 + 64, (pn * P + t) * BN);
+    } else {
+      // placement T16 as lines: box {line, lpu * UG lines, 8 row tiles} -> [tile][group][16][GB]
+      if (!no_w) tma_load_3d(wdst, &tm_w, &full_w[sw], 0, j * UG * LPU_, tile16);
+      if (!no_meta) tma_load_2d(smem + SM::OFF_META + sw * BN * 4 * UG, &tm_m, &full_w[sw], j * UG * 16, tile16);
+    }
+  };
+  // PDL: weights never depend on the previous kernel -- thread 0 fills the whole weight ring right
+  // after the barrier init, before the other warps are released (a producer warp sharing its SMSP
+  // with waiting warps issued only ~1 unit per 0.4 us here, measured)
+  int pre = 0;
+  if (warp == 0) {
+    for (int it = blockIdx.x; it < I && pre < S_W; it += C) {
+      const int pn = it / Z, j1 = j1_of(it), pp = tiles_of(pn);
+      for (int j = j0_of(it); j < j1 && pre < S_W; ++j)
+        for (int t = 0; t < pp && pre < S_W; ++t, ++pre)
+          if (lane == 0) issue_w1(pre, pn, t, j);
+    }
+  }
   if (warp == 1) tmem_alloc(misc, TMEM_COLS);
   tc_fence_before();
   __syncthreads();
@@ -250,34 +282,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       ++qx;
     };
     auto issue_w = [&](int i, int pn, int t, int j) {
-      const int sw = i % S_W;
-      if (elect_one()) {
-            const int tile16 = (pn * P + t) * (BN / 16);
-            uint8_t* wdst = smem + SM::OFF_W + sw * SM::W_STAGE;
-            mbar_arrive_expect_tx(&full_w[sw], W_BYTES);
-            if constexpr (BITS == 16) {
-              // row-major fp16 [n][k]: two SW128 boxes [128 rows][64 k] = the MMA's K-major A tiles
-              tma_load_2d(wdst, &tm_w, &full_w[sw], j * 128, (pn * P + t) * BN);
-              tma_load_2d(wdst + BN * 128, &tm_w, &full_w[sw], j * 128 + 64, (pn * P + t) * BN);
-            } else {
-              // placement T16 as lines: box {line, lpu * UG lines, 8 row tiles} -> [tile][group][16][GB]
-              tma_load_3d(wdst, &tm_w, &full_w[sw], 0, j * UG * LPU, tile16);
-              tma_load_2d(smem + SM::OFF_META + sw * BN * 4 * UG, &tm_m, &full_w[sw], j * UG * 16, tile16);
-            }
-      }
+      if (elect_one()) issue_w1(i, pn, t, j);
       __syncwarp();
     };
-    // PDL: weights never depend on the previous kernel -- fill the whole ring before waiting for
-    // it (these first S_W slots are free, no empty wait); activations only after the wait
-    int pre = 0;
-    for (int it = blockIdx.x; it < I && pre < S_W; it += C) {
-      const int pn = it / Z, j1 = j1_of(it), pp = tiles_of(pn);
-      for (int j = j0_of(it); j < j1 && pre < S_W; ++j)
-        for (int t = 0; t < pp && pre < S_W; ++t, ++pre) {
-          issue_w(pre, pn, t, j);
-          trace_ev(p, 0, pre);
-        }
-    }
     pdl_wait();
     trace_ev(p, 7, 0);
     for (int it = blockIdx.x; it < I; it += C) {
