@@ -138,7 +138,23 @@ struct TcP {
   int abl;                    // debug ablation (SQ_TC_ABL): 1 = no dequant, 2 = no MMAs (results wrong)
   const __half* x;            // activations [m][ldx] (SQ_TC_XLDG: loaded by the epilogue warps)
   int ldx;
+  int cl;                     // Z > 1 items of a panel form a thread-block cluster: DSMEM reduction
 };
+
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+// address of the same shared-memory byte in cluster CTA `rank`
+__device__ __forceinline__ uint32_t dsmem_addr(uint32_t local, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(local), "r"(rank));
+  return r;
+}
+__device__ __forceinline__ float4 ld_dsmem_f4(uint32_t addr) {
+  float4 v;
+  asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(addr) : "memory");
+  return v;
+}
 
 #ifndef SQ_TC_DEBUG
 #define SQ_TC_DEBUG 0  // 1: clock64 trace (sq_debug_trace) and SQ_TC_ABL ablations compiled in
@@ -464,6 +480,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         if (Z == 1) {
           const int64_t row = (int64_t)(pn * P + t) * BN + r;
           epi_store<EPI>(p, row, v, p.bias ? __half2float(p.bias[row]) : 0.f);
+        } else if (p.cl) {
+          // the weight ring is idle once the item's MMAs completed (one item per CTA when Z > 1)
+          float* sp_ = reinterpret_cast<float*>(smem + SM::OFF_W) + (t * BT) * BN + r;  // [tile][tok][row]
+#pragma unroll
+          for (int c = 0; c < BT; ++c) sp_[c * BN] = v[c];
         } else {
           float* gp = p.part + (((int64_t)it * PMAX + t) * BT) * BN + r;  // [tok][row]: coalesced
 #pragma unroll
@@ -473,7 +494,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(d_empty);  // accumulators drained: the MMA may start the next item
-      if (Z > 1) {  // publish this slice's partial (one item per CTA when Z > 1)
+      if (Z > 1 && !p.cl) {  // publish this slice's partial (one item per CTA when Z > 1)
         __threadfence();
         asm volatile("bar.sync 1, 128;" ::: "memory");
         if (leader) atomicAdd(p.cnt + pn, 1);
@@ -488,7 +509,48 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   if (threadIdx.x == 0) trace_cta(p, 11);
   // (no griddepcontrol.wait here: everything below is ordered after the producer's wait by the
   // CTA barrier, and a redundant wait by all 704 threads measured ~2 us)
-  if (Z > 1 && (int)blockIdx.x < I) {
+  if (Z > 1 && p.cl) {
+    // cluster of the panel's Z items: partials stay in each CTA's shared memory; CTA z sums its
+    // 1/Z share over the Z CTAs in fixed order through DSMEM (deterministic), then a second cluster
+    // barrier keeps every partial alive until all peers have read it
+    static_assert(PMAX * BT * BN * 4 <= SM::S_W * SM::W_STAGE, "partials fit the weight ring");
+    const int it = blockIdx.x, pn = it / Z, z = it % Z, pp = tiles_of(pn);
+    cluster_sync_all();
+    const uint32_t base = smem_u32(smem + SM::OFF_W);
+    const int nel = pp * BT * (BN / 4);
+    const int e0 = (int)((long long)z * nel / Z), e1 = (int)((long long)(z + 1) * nel / Z);
+    for (int idx = e0 + threadIdx.x; idx < e1; idx += NUM_THREADS) {
+      const int t = idx / (BT * (BN / 4)), rem = idx - t * (BT * (BN / 4));
+      const int tok = rem / (BN / 4), r4 = (rem % (BN / 4)) * 4;
+      if (tok >= p.m) continue;
+      const uint32_t off = (uint32_t)(((t * BT + tok) * BN + r4) * 4);
+      float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int zz = 0; zz < Z; ++zz) {
+        const float4 v = ld_dsmem_f4(dsmem_addr(base + off, (uint32_t)zz));
+        acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
+      }
+      const int64_t row0 = (int64_t)(pn * P + t) * BN + r4;
+      float o[4] = {acc.x, acc.y, acc.z, acc.w};
+      if (p.bias) {
+#pragma unroll
+        for (int c = 0; c < 4; ++c) o[c] += __half2float(p.bias[row0 + c]);
+      }
+      if constexpr (EPI == SQ_EPI_F32_ACCUM) {
+        float* yp = static_cast<float*>(p.y) + (int64_t)tok * p.ldy + row0;
+        const float4 y0 = __ldcg(reinterpret_cast<const float4*>(yp));
+        *reinterpret_cast<float4*>(yp) = make_float4(y0.x + o[0], y0.y + o[1], y0.z + o[2], y0.w + o[3]);
+      } else {
+        __half* yp = static_cast<__half*>(p.y) + (int64_t)tok * p.ldy + row0;
+        const __half2 h01 = __floats2half2_rn(apply_act<EPI>(o[0]), apply_act<EPI>(o[1]));
+        const __half2 h23 = __floats2half2_rn(apply_act<EPI>(o[2]), apply_act<EPI>(o[3]));
+        uint2 pk;
+        pk.x = *reinterpret_cast<const uint32_t*>(&h01);
+        pk.y = *reinterpret_cast<const uint32_t*>(&h23);
+        *reinterpret_cast<uint2*>(yp) = pk;
+      }
+    }
+    cluster_sync_all();
+  } else if (Z > 1 && (int)blockIdx.x < I) {
     const int it = blockIdx.x, pn = it / Z, z = it % Z, pp = tiles_of(pn);
     if (threadIdx.x == 0) {
       volatile int* c = p.cnt + pn;
@@ -564,16 +626,43 @@ cudaError_t enc(CUtensorMap* m, CUtensorMapDataType dt, const void* ptr, int ran
 }
 
 template <int BITS, int UG, int EPI>
-cudaError_t launch_tc_be(const CUtensorMap& tx, const CUtensorMap& tw, const CUtensorMap& tm, const TcP& p, int nc,
+cudaError_t launch_tc_be(const CUtensorMap& tx, const CUtensorMap& tw, const CUtensorMap& tm, const TcP& p0, int nc,
                          cudaStream_t s) {
   auto kern = k_gemv_tc<BITS, UG, EPI>;
   static bool attr = false;
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, DSmem<BITS, UG>::BYTES);
     if (e != cudaSuccess) return e;
+    cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
     attr = true;
   }
-  return launch_pdl(kern, dim3(nc), dim3(NUM_THREADS), DSmem<BITS, UG>::BYTES, s, tx, tw, tm, p);
+  TcP p = p0;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(nc);
+  cfg.blockDim = dim3(NUM_THREADS);
+  cfg.dynamicSmemBytes = DSmem<BITS, UG>::BYTES;
+  cfg.stream = s;
+  cudaLaunchAttribute at[2];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+  at[1].id = cudaLaunchAttributeClusterDimension;
+  at[1].val.clusterDim.x = p.Z;
+  at[1].val.clusterDim.y = 1;
+  at[1].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  if (p.cl) {
+    // the panel's Z items as one cluster, only if every cluster of the grid can be resident at once
+    // (the DSMEM reduction waits for all Z CTAs); else the global-memory fix-up
+    cfg.numAttrs = 2;
+    int ncl = 0;
+    if (cudaOccupancyMaxActiveClusters(&ncl, kern, &cfg) != cudaSuccess || ncl * p.Z < nc) {
+      cudaGetLastError();
+      p.cl = 0;
+      cfg.numAttrs = 1;
+    }
+  }
+  return cudaLaunchKernelEx(&cfg, kern, tx, tw, tm, p);
 }
 
 template <int BITS, int UG>
@@ -725,6 +814,11 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
   }
   p.x = x;
   p.ldx = (int)ldx;
+  {
+    static int cl = -1;  // SQ_TC_CLUSTER=0 disables the cluster/DSMEM split-k reduction
+    if (cl < 0) { const char* e = getenv("SQ_TC_CLUSTER"); cl = (e && e[0] == '0') ? 0 : 1; }
+    p.cl = (cl && pl.Z > 1 && pl.Z <= 8 && pl.I == pl.ctas && pl.I % pl.Z == 0) ? 1 : 0;
+  }
   const int nc = pl.ctas;
   const double bytes = (double)w.n * w.k * w.bits / 8.0 + (w.bits != 16 ? (double)w.n * (w.k / 128) * 4.0 : 0.0);
   auto t = prof_begin(KC_GEMV, bytes, 2.0 * m * w.n * w.k, s);
