@@ -229,14 +229,18 @@ def test_one_token_prefill_equals_decode_function():
     assert normwise(a, ref) <= TOL and normwise(b, ref) <= TOL
 
 
-@pytest.mark.parametrize("path", ["mma", "tc"])
+@pytest.mark.parametrize("path", ["mma", "tc", "tc-nocluster"])
 def test_decode_forced_path(path):
     """Both decode kernels (mma.sync K2 and tcgen05 K2c) for every bit width and m in 1..32, whatever
-    the automatic choice (gemv_path) would pick: SQ_GEMV_PATH forces one (read once per process)."""
+    the automatic choice (gemv_path) would pick: SQ_GEMV_PATH forces one (read once per process).
+    "tc-nocluster" forces K2c's global-memory split-k fix-up instead of the cluster/DSMEM reduction
+    (SQ_TC_CLUSTER=0), the fallback taken when the clusters cannot all be resident."""
     import os
     import subprocess
     import sys
-    env = dict(os.environ, SQ_GEMV_PATH=path)
+    env = dict(os.environ, SQ_GEMV_PATH=path.split("-")[0])
+    if path == "tc-nocluster":
+        env["SQ_TC_CLUSTER"] = "0"
     script = os.path.join(os.path.dirname(os.path.abspath(__file__)), "_decode_path_check.py")
     r = subprocess.run([sys.executable, script], env=env, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
