@@ -91,12 +91,12 @@ template <int BITS, int UG>
 struct DCfg {
   // weight ring: a slot lives TMA latency (~1.8k cycles) + wait for its group + dequant (~2k)
   // (quantized rings are multiples of DQ_GROUPS so each slot is owned by one dequant group)
-  static constexpr int S_W0 = UG == 2 ? 10 : (BITS == 8 ? 10 : (BITS == 4 ? 18 : 24));
+  static constexpr int S_W0 = UG == 3 ? 6 : (UG == 2 ? 10 : (BITS == 8 ? 10 : (BITS == 4 ? 18 : 24)));
   static constexpr int S_W = BITS == 16 ? 5 : (S_W0 / DQ_GROUPS) * DQ_GROUPS;
   // TMEM A slots of 64*UG columns: the dequant warps fill slot i % S_A while the MMA reads the
   // others (slots are owned by one dequant group: multiples of DQ_GROUPS)
   static constexpr int A_SLOT = 64 * UG;
-  static constexpr int S_A = SQ_TC_DEEP_A ? (UG == 2 ? 3 : 6) : (UG == 2 ? 2 : 4);
+  static constexpr int S_A = UG == 3 ? 2 : (SQ_TC_DEEP_A ? (UG == 2 ? 3 : 6) : (UG == 2 ? 2 : 4));
   static constexpr int S_X = 3;  // activation ring, in steps
   static_assert(BITS == 16 || A_COL + S_A * A_SLOT <= TMEM_COLS, "TMEM budget");
 };
@@ -409,12 +409,25 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       wait_bar(&empty_a[sa], (uint32_t)(((i / S_A) & 1) ^ 1));
       if (tr) trace_ev(p, 5, i);
       tc_fence_after();
-      const uint32_t meta = reinterpret_cast<const uint32_t*>(smem + SM::OFF_META + sw * BN * 4 * UG)[ru];
+      const uint32_t* mt = reinterpret_cast<const uint32_t*>(smem + SM::OFF_META + sw * BN * 4 * UG);
       const uint32_t a_tm = tmem + lane_base + A_COL + sa * DCfg<BITS, UG>::A_SLOT;
-      if constexpr (BITS != 16) {
+      const uint8_t* wst = smem + SM::OFF_W + sw * SM::W_STAGE;
+      if constexpr (BITS != 16 && UG == 3) {
+        // 12 batches over 3 groups, 6 per warp: kh 0 -> group 0 batches 0..3 + group 1 batches 0..1,
+        // kh 1 -> group 1 batches 2..3 + group 2 batches 0..3 (one meta word per group)
+        static_assert(DQ_KH == 2, "UG = 3 splits the unit's k in two warp halves");
+        const int ru1 = ru + 16;  // (gg = 0 here) the row's entry of group 1 / group 2 in the stage
+        if (kh == 0) {
+          dequant_row_batches<BITS, 4>(wst, mt[ru], r, a_tm, ru * GB, 0);
+          dequant_row_batches<BITS, 2>(wst, mt[ru1], r, a_tm + 64, ru1 * GB, 0);
+        } else {
+          const int ru0 = ru - 16 * gg;
+          dequant_row_batches<BITS, 2>(wst, mt[ru0 + 16], r, a_tm + 64, (ru0 + 16) * GB, 2);
+          dequant_row_batches<BITS, 4>(wst, mt[ru0 + 32], r, a_tm + 128, (ru0 + 32) * GB, 0);
+        }
+      } else if constexpr (BITS != 16) {
         if (!(SQ_TC_DEBUG && (p.abl & 1)))
-          dequant_row_batches<BITS, NBW < 4 ? NBW : 4>(smem + SM::OFF_W + sw * SM::W_STAGE, meta, r,
-                                                       a_tm + gg * 64, ru * GB, b0);
+          dequant_row_batches<BITS, NBW < 4 ? NBW : 4>(wst, mt[ru], r, a_tm + gg * 64, ru * GB, b0);
       }
       if (tr) trace_ev(p, 12, i);
       tc_wait_st();
@@ -681,12 +694,21 @@ cudaError_t launch_tc_b(const CUtensorMap& tx, const CUtensorMap& tw, const CUte
                         int nc, int ug, cudaStream_t s) {
   if constexpr (BITS == 3 || BITS == 4) {
     if (ug == 2) return launch_tc_u<BITS, 2>(tx, tw, tm, p, epi, nc, s);
+    if (ug == 3) return launch_tc_u<BITS, 3>(tx, tw, tm, p, epi, nc, s);
   }
   return launch_tc_u<BITS, 1>(tx, tw, tm, p, epi, nc, s);
 }
 
 // UG: groups per unit -- a ~16-KB weight stage (INT3/INT4 two groups when k/128 is even)
-int tc_ug(int bits, int kg) { return (bits <= 4 && kg % 2 == 0) ? 2 : 1; }
+// INT3/INT4 take three groups per unit when 3 | k/128 (a ~24 KB INT4 stage, 2 TMEM A slots): one
+// hand-off chain per 1.5x the bytes; measured +5-8 % INT4 GB/s on OPT-66B shapes (tools/exp_ug3.sh).
+// SQ_TC_UG3=0 restores two.
+int tc_ug(int bits, int kg) {
+  static int ug3 = -1;
+  if (ug3 < 0) { const char* e = getenv("SQ_TC_UG3"); ug3 = (e && e[0] == '0') ? 0 : 1; }
+  if (ug3 && bits <= 4 && kg % 3 == 0) return 3;
+  return (bits <= 4 && kg % 2 == 0) ? 2 : 1;
+}
 
 struct TcPlan { int P, Z, I, ctas; };
 

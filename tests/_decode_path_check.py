@@ -33,7 +33,7 @@ def main():
                 # fp32-residual epilogue (o / fc2): y_f32 += x W~^T + bias
                 y0 = synth.act_f16(903 + m, m, n).astype(np.float32)
                 ya = torch.from_numpy(y0.copy()).cuda()
-                sq.sq_linear_decode(qg, torch.from_numpy(x).cuda(), ya, 1)
+                sq.sq_linear_decode(qg, torch.from_numpy(x).cuda(), ya, sq.SQ_EPI_F32_ACCUM)
                 torch.cuda.synchronize()
                 dy = ya.cpu().numpy().astype(np.float64) - y0.astype(np.float64)
                 err = float(np.abs(dy - ref).max() / np.abs(ref).max())
