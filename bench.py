@@ -111,10 +111,21 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------ CPU oracle sample
-def oracle_sample(wl: dict, tokens: int = 16, row_frac: int = 8):
-    """Bounded oracle sample: oq_linear (fp64, plain loops) on the first n/row_frac rows of each
-    of the 4 linears of one 4-bit layer of the workload, `tokens` tokens.  Returns
-    (seconds, token-layer passes represented = tokens * row_frac... scaled by caller)."""
+def cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    import platform
+    return platform.processor() or "unknown"
+
+
+def oracle_layer_seconds(wl: dict, bits: int, tokens: int, row_frac: int) -> float:
+    """Bounded oracle sample: oq_linear (fp64, plain loops) on the first n/row_frac rows of each of the
+    4 linears of one layer of the workload at `bits`, `tokens` tokens.  Seconds of host time."""
     import numpy as np
     import synth
     from oracle import oracle as O
@@ -123,57 +134,97 @@ def oracle_sample(wl: dict, tokens: int = 16, row_frac: int = 8):
     qws = {}
     for name, (n, k) in dims.items():
         rows = np.arange(n // row_frac)
-        w = synth.weight_f16(synth.weight_seed(0, name), n, k, rows=rows)
-        qws[name] = O.QWeight(w, 4)
+        qws[name] = O.QWeight(synth.weight_f16(synth.weight_seed(0, name), n, k, rows=rows), bits)
     x1 = synth.act_f16(5, tokens, h1)
     x2 = synth.act_f16(6, tokens, h2)
     t0 = time.perf_counter()
     for name, (n, k) in dims.items():
         O.linear(x1 if k == h1 else x2, qws[name])
-    dt = time.perf_counter() - t0
-    return dt
+    return time.perf_counter() - t0
 
 
-def cpu_tokens_per_s(wl: dict, dt: float, tokens: int, row_frac: int, B: int) -> float:
-    # one full layer for `tokens` tokens ~ dt * row_frac; the workload runs L layers over
-    # (B*s prefill + B*n_dec decode) token rows and yields B*(1+n_dec) output tokens
-    per_token_layer = dt * row_frac / tokens
-    total = per_token_layer * wl["L"] * (B * wl["s"] + B * wl["n_dec"])
+def workload_bits(wl: dict) -> list[int]:
+    import synth
+    return [int(b) for b in synth.bits_plan(2, wl["L"], choices=wl.get("choices", (3, 4, 8, 16)),
+                                            balanced=wl["balanced"])]
+
+
+def oracle_tokens_per_s(wl: dict, B: int, per_bit_s: dict, tokens: int, row_frac: int) -> float:
+    """Extrapolate per-bit layer samples to the workload: sum over its layers (their own bits) of the
+    per-token layer time x the token rows the run processes (B*s prefill + B*n_dec decode)."""
+    bits = workload_bits(wl)
+    per_token = sum(per_bit_s[b] * row_frac / tokens for b in bits)
+    total = per_token * (B * wl["s"] + B * wl["n_dec"])
     return B * (1 + wl["n_dec"]) / total
+
+
+def cpu_baseline(wl: dict, B: int, tokens: int, row_frac: int, one_thread: bool = True) -> dict:
+    """The oracle as it stands, on this host: per bit width present in the workload, at all cores and
+    (optionally) at one thread; value = the workload's tokens/s at all cores."""
+    from oracle import oracle as O
+    ncores = len(os.sched_getaffinity(0))
+    present = sorted(set(workload_bits(wl)))
+    allc, one = {}, {}
+    O.set_threads(ncores)
+    for b in present:
+        allc[b] = oracle_layer_seconds(wl, b, tokens, row_frac)
+    if one_thread:
+        O.set_threads(1)
+        for b in present:
+            one[b] = oracle_layer_seconds(wl, b, tokens, row_frac)
+        O.set_threads(ncores)
+    out = {"value": oracle_tokens_per_s(wl, B, allc, tokens, row_frac), "unit": "tokens/s", "cores": ncores,
+           "kind": "oracle", "cpu": cpu_model(),
+           "sample": (f"oq_linear fp64 on the first 1/{row_frac} of the rows of the 4 linears of one layer per bit width "
+                      f"{present}, {tokens} tokens; extrapolated over the workload's {wl['L']} layers (their own bits) "
+                      f"x (B*s + B*n_dec) token rows"),
+           "layer_s_all_cores": {str(b): round(allc[b], 4) for b in present}}
+    if one_thread:
+        out["value_1_thread"] = oracle_tokens_per_s(wl, B, one, tokens, row_frac)
+        out["layer_s_1_thread"] = {str(b): round(one[b], 4) for b in present}
+    return out
 
 
 def run_reference(args, wl):
     rank, world, _ = dist_env()
     if rank != 0:
         return
+    from oracle import oracle as O
     ncores = len(os.sched_getaffinity(0))
-    os.environ.setdefault("OMP_NUM_THREADS", str(ncores))
+    O.set_threads(ncores)
     B = wl["b_per_gpu"] * max(1, args.gpus)
     tokens, frac = args.cpu_tokens, args.cpu_row_frac
+    present = sorted(set(workload_bits(wl)))
+
+    def one_step():
+        t0 = time.perf_counter()
+        per = {b: oracle_layer_seconds(wl, b, tokens, frac) for b in present}
+        return time.perf_counter() - t0, oracle_tokens_per_s(wl, B, per, tokens, frac)
+
     for _ in range(args.warmup):
-        oracle_sample(wl, tokens, frac)
+        one_step()
     vals, ts = [], []
     for _ in range(args.steps):
-        dt = oracle_sample(wl, tokens, frac)
+        dt, v = one_step()
         ts.append(dt)
-        vals.append(cpu_tokens_per_s(wl, dt, tokens, frac, B))
+        vals.append(v)
     v = statistics.median(vals)
-    sample = (f"oq_linear fp64 on the first 1/{frac} of the rows of the 4 linears of one 4-bit "
-              f"{wl['name'].split(' ')[1]} layer, {tokens} tokens, extrapolated to L={wl['L']} layers x "
+    sample = (f"per step: oq_linear fp64 on the first 1/{frac} of the rows of the 4 linears of one layer per bit "
+              f"width {present}, {tokens} tokens, extrapolated over the workload's {wl['L']} layers x "
               f"(B*s + B*n_dec) token rows")
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "tokens/s", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * statistics.median(ts),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": wl["name"], "B": B},
-            "cpu_baseline": {"value": v, "unit": "tokens/s", "cores": int(os.environ["OMP_NUM_THREADS"]),
-                             "kind": "oracle", "sample": sample},
+            "cpu_baseline": {"value": v, "unit": "tokens/s", "cores": ncores, "kind": "oracle", "sample": sample,
+                             "cpu": cpu_model()},
             "e2e": {"value": v, "unit": "tokens/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
 # ------------------------------------------------------------------ decode GEMV sweep (configs[1])
-def gemv_sweep(n_launch=40):
-    """configs[1]: OPT-13B linear shapes, bits 3/4/8, micro-batch 1/8/32.  Each point is a decode
+def gemv_sweep(n_launch=40, ms=(1, 2, 4, 8, 16, 32), bit_list=(3, 4, 8, 16)):
+    """configs[1]: OPT-13B linear shapes, bits 3/4/8 (+ fp16 as the reference row), micro-batch 1..32.  Each point is a decode
     step's worth of back-to-back linears: n_launch launches cycling over R distinct copies of the
     quantized weight (R copies > 2 x L2, so every launch streams its weights from HBM), captured in
     one CUDA graph (launch gaps hidden by PDL, as in the stage forward); best of 3 replays.
@@ -188,11 +239,12 @@ def gemv_sweep(n_launch=40):
     for (n, k) in ((5120, 5120), (20480, 5120), (5120, 20480)):
         wd = torch.empty((n, k), dtype=torch.float16, device=dev)
         synth.device_weight_f16(wd.data_ptr(), 4242, n, k)
-        for bits in (3, 4, 8):
+        for bits in bit_list:
             q0 = sq.QLinear.from_fp16(wd, bits)
             R = max(2, int(2 * l2 // q0.nbytes()) + 2)
-            qs = [q0] + [sq.QLinear(bits, n, k, q0.packed.clone(), q0.meta.clone()) for _ in range(R - 1)]
-            for m in (1, 8, 32):
+            qs = [q0] + [sq.QLinear(bits, n, k, q0.packed.clone(), None if q0.meta is None else q0.meta.clone())
+                         for _ in range(R - 1)]
+            for m in ms:
                 x = torch.randn(m, k, device=dev).half()
                 y = torch.empty(m, n, device=dev, dtype=torch.float16)
                 ws = torch.zeros(sq.sq_linear_workspace_bytes(q0, m), dtype=torch.uint8, device=dev)
@@ -234,18 +286,28 @@ def run_ours(args, wl):
     from paper_conf_cluster_zhaowplw25_b200 import plan as PL
 
     rank, world, local = dist_env()
-    assert world == args.gpus or world == 1, "launch N>1 with torchrun --nproc-per-node N"
+    if world != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}; run `python bench.py --gpus N` "
+                         f"(it launches the N ranks itself) or torchrun --nproc-per-node N")
     P = world
     torch.cuda.set_device(local)
     dist = None
+    selfcheck = None
     if P > 1:
         import torch.distributed as dist
         dist.init_process_group("gloo")
+        # the NCCL pipeline must equal the single-process virtual pipeline bitwise before anything is timed
+        from paper_conf_cluster_zhaowplw25_b200.selfcheck import pipeline_bitwise_check
+        selfcheck = pipeline_bitwise_check(rank, P, dist)
+        if not selfcheck["pipeline_bitwise_ok"]:
+            if rank == 0:
+                print(json.dumps({"error": "NCCL pipeline differs from the virtual pipeline", **selfcheck}), flush=True)
+            raise SystemExit(1)
     pk = peaks()
 
     B = wl["b_per_gpu"] * P
     L, h1, h2 = wl["L"], wl["h1"], wl["h2"]
-    bits = [int(b) for b in synth.bits_plan(2, L, choices=wl.get("choices", (3, 4, 8, 16)), balanced=wl["balanced"])]
+    bits = workload_bits(wl)
     costs = PL.phase_costs(bits, h1, h2, B, wl["eta"], wl["xi"], wl["s"], wl["n_dec"], pk["hbm_gbs"],
                            pk["tflops_sustained"])
     sol = PL.partition_layers(costs, P)
@@ -378,23 +440,24 @@ def run_ours(args, wl):
         ems = max_over_ranks(f0.elapsed_time(f1))
         e2e = {"value": tokens / (ems / 1e3), "unit": "tokens/s",
                "h2d_bytes_per_step": int(sum_over_ranks(x0.numel() * 4 if first else 0)),
-               "d2h_bytes_per_step": int(sum_over_ranks(out.numel() * 4 if last else 0))}
+               "d2h_bytes_per_step": int(sum_over_ranks(out.numel() * 4 if last else 0)),
+               "copies": "pinned host -> device embeddings before, device -> pinned host outputs after every "
+                         "sq_pipeline_run call (torch copy_ on the run's stream, inside the timed region)"}
 
     # ---------------- side measurements on rank 0 at N = 1
     extra = {}
     cpu = None
     if rank == 0 and P == 1:
         if not args.no_gemv_sweep:
-            extra["decode_gemv"] = {"workload": "configs[1] OPT-13B linear shapes; 40 back-to-back launches over > 2 x L2 of distinct weight copies in one CUDA graph, best of 3",
+            extra["decode_gemv"] = {"workload": "configs[1] OPT-13B linear shapes, m = 1..32, bits 3/4/8 (+16); 40 back-to-back launches over > 2 x L2 of distinct weight copies in one CUDA graph, best of 3",
                                     "results": gemv_sweep()}
+        if not args.no_gemm_sweep:
+            extra["prefill_gemm"] = {"workload": "configs[2] OPT-30B linear shapes (fused qkv 21504x7168, o 7168^2, fc1 28672x7168, fc2 7168x28672) at M = 8 x 512 = 4096 tokens, bits 3/4/8/16; median of 5 event-timed launches after 2 warm-up",
+                                     "results": gemm_sweep(pk)}
+        if not args.no_configs0:
+            extra["configs0"] = configs0_latency()
         if not args.no_cpu:
-            ncores = len(os.sched_getaffinity(0))
-            os.environ["OMP_NUM_THREADS"] = str(ncores)
-            dt = oracle_sample(wl, args.cpu_tokens, args.cpu_row_frac)
-            cpu = {"value": cpu_tokens_per_s(wl, dt, args.cpu_tokens, args.cpu_row_frac, B), "unit": "tokens/s",
-                   "cores": ncores, "kind": "oracle",
-                   "sample": (f"oq_linear fp64 on the first 1/{args.cpu_row_frac} of the rows of the 4 linears of "
-                              f"one 4-bit layer, {args.cpu_tokens} tokens, {dt:.2f} s, extrapolated to the workload")}
+            cpu = cpu_baseline(wl, B, args.cpu_tokens, args.cpu_row_frac)
     if rank == 0:
         st = stats[-1]
         line = {
@@ -411,7 +474,11 @@ def run_ours(args, wl):
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk,
             "kernels": kern,
             "phase_ms_rank0": {"prefill": st["t_prefill_ms"], "decode": st["t_decode_ms"]},
+            "gpus_active": P,
         }
+        if selfcheck is not None:
+            line["pipeline_bitwise_ok"] = selfcheck["pipeline_bitwise_ok"]
+            line["selfcheck"] = selfcheck
         line.update(extra)
         print(json.dumps(line), flush=True)
     if comm:
@@ -419,6 +486,118 @@ def run_ours(args, wl):
     if dist:
         dist.barrier()
         dist.destroy_process_group()
+
+
+def spawn_ranks(n: int) -> None:
+    """`python bench.py --gpus N` without torchrun: re-exec under torch.distributed.run with one rank per
+    GPU (never silently measure fewer GPUs than asked for)."""
+    import socket
+    import torch
+    have = torch.cuda.device_count()
+    if have < n:
+        print(json.dumps({"metric": METRIC, "error": f"--gpus {n} requested but only {have} CUDA device(s) visible",
+                          "n_gpus": n, "gpus_active": have}), flush=True)
+        raise SystemExit(1)
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+    os.execv(sys.executable, cmd)
+
+
+# ------------------------------------------------------------------ prefill GEMM sweep (configs[2])
+def gemm_sweep(pk: dict, reps: int = 5):
+    """configs[2]: OPT-30B linear shapes at M = eta * s = 8 * 512 = 4096 tokens, bits 3/4/8/16.  TFLOP/s =
+    2 M N K / event-timed launch duration (median of `reps` after 2 warm-up launches); fractions of the
+    measured bf16 dense peaks (burst and sustained)."""
+    import torch
+    import synth
+    import paper_conf_cluster_zhaowplw25_b200 as sq
+    h1, h2, M = 7168, 28672, 4096
+    out = []
+    x = torch.empty((M, h2), dtype=torch.float16, device="cuda")
+    synth.device_fill_f16(x.data_ptr(), 9, 0, x.numel(), 1.0, False)
+    for name, (n, k) in (("qkv", (3 * h1, h1)), ("o", (h1, h1)), ("fc1", (h2, h1)), ("fc2", (h1, h2))):
+        wd = torch.empty((n, k), dtype=torch.float16, device="cuda")
+        synth.device_weight_f16(wd.data_ptr(), synth.weight_seed(0, name), n, k)
+        xk = x[:, :k].contiguous()
+        y = torch.empty((M, n), dtype=torch.float16, device="cuda")
+        for bits in (3, 4, 8, 16):
+            q = sq.QLinear.from_fp16(wd, bits)
+            for _ in range(2):
+                sq.sq_linear_prefill(q, xk, y, 0)
+            ts = []
+            for _ in range(reps):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                sq.sq_linear_prefill(q, xk, y, 0)
+                e1.record()
+                torch.cuda.synchronize()
+                ts.append(e0.elapsed_time(e1))
+            ms = statistics.median(ts)
+            tf = 2.0 * M * n * k / (ms / 1e3) / 1e12
+            out.append({"linear": name, "n": n, "k": k, "bits": bits, "m": M, "us": round(ms * 1e3, 1),
+                        "TFLOPs": round(tf, 1), "frac_burst": round(tf / pk["tflops"], 3),
+                        "frac_sustained": round(tf / pk["tflops_sustained"], 3)})
+            del q
+        del wd, xk, y
+    return out
+
+
+# ------------------------------------------------------------------ configs[0] latency
+def configs0_latency(runs: int = 20):
+    """BASELINE.json configs[0] (OPT-125m shapes, 12 layers, bits {3,4,8,16}, G = 128, one sequence: prefill
+    1 x 32 tokens + 8 decode steps, 1 GPU): per-run latency through sq_pipeline_run, and the decode step
+    (all 12 layers at 1 token) captured in one CUDA graph."""
+    import torch
+    import synth
+    from paper_conf_cluster_zhaowplw25_b200 import runtime as R
+    wl = WORKLOADS["opt125m"]
+    h1, h2, L = wl["h1"], wl["h2"], wl["L"]
+    bits = workload_bits(wl)
+    g = R.build_layers(L, h1, h2, bits)
+    plan = R.Plan(bits, [0] * L, h1, h2, 1, 1, 1, wl["s"], wl["n_dec"])
+    ws = R.PipelineWorkspace(plan, g, 0)
+    x0 = torch.empty((1, wl["s"], h1), dtype=torch.float32, device="cuda")
+    synth.device_fill_f32(x0.data_ptr(), 1, 0, x0.numel(), 1.0, False)
+    out = torch.zeros((1, 1 + wl["n_dec"], h1), dtype=torch.float32, device="cuda")
+    arr = R.layer_array(g)
+    for _ in range(3):
+        R.sq_pipeline_run(plan, 0, g, None, x0, out, ws, arr=arr)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(runs):
+        R.sq_pipeline_run(plan, 0, g, None, x0, out, ws, arr=arr)
+    e1.record()
+    torch.cuda.synchronize()
+    run_ms = e0.elapsed_time(e1) / runs
+    # decode step (12 layers, 1 token) as one CUDA graph
+    sw = R.StageWorkspace(g, 1)
+    xi = torch.zeros((1, h1), dtype=torch.float32, device="cuda")
+    xo = torch.empty_like(xi)
+    side = torch.cuda.Stream()
+    side.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(side):
+        R.sq_stage_forward(g, 1, xi, xo, sw, arr=arr)
+    torch.cuda.current_stream().wait_stream(side)
+    torch.cuda.synchronize()
+    graph = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(graph):
+        R.sq_stage_forward(g, 1, xi, xo, sw, arr=arr)
+    graph.replay()
+    torch.cuda.synchronize()
+    e0.record()
+    for _ in range(100):
+        graph.replay()
+    e1.record()
+    torch.cuda.synchronize()
+    step_us = e0.elapsed_time(e1) / 100 * 1e3
+    return {"workload": wl["name"], "bits": bits, "ms_per_run": round(run_ms, 3),
+            "tokens_per_s": round((1 + wl["n_dec"]) / (run_ms / 1e3), 1),
+            "decode_step_us_cuda_graph": round(step_us, 1),
+            "note": "one sequence; per-run = prefill 32 tokens + 8 decode steps through sq_pipeline_run (P = 1)"}
 
 
 def traffic_for(kernel: str, per_launch: float | None = None):
@@ -447,10 +626,14 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-gemv-sweep", action="store_true")
+    ap.add_argument("--no-gemm-sweep", action="store_true")
+    ap.add_argument("--no-configs0", action="store_true")
     ap.add_argument("--cpu-tokens", type=int, default=8)
     ap.add_argument("--cpu-row-frac", type=int, default=8)
     args = ap.parse_args()
     wl = WORKLOADS[args.workload]
+    if args.impl == "ours" and args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        spawn_ranks(args.gpus)  # does not return
     if args.impl == "reference":
         run_reference(args, wl)
     else:

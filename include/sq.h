@@ -9,8 +9,9 @@
  * Conventions for every entry point
  *  - Pointers named *_dev are DEVICE pointers (any CUDA allocation on the
  *    current device); *_host are host pointers.  The caller owns all memory;
- *    the library never allocates in a hot call (only sq_comm_* and the first
- *    TMA-descriptor cache fill allocate host memory).
+ *    the library never allocates in a hot call (only sq_comm_* and the
+ *    per-thread TMA-descriptor cache -- one entry per distinct (pointer, shape,
+ *    box) the first time it is seen -- allocate host memory).
  *  - `stream` is a cudaStream_t (NULL = legacy default stream).  Kernels are
  *    enqueued asynchronously; device faults surface at the next sync.
  *  - Every call returns sq_status and never throws.  All validation happens
@@ -197,7 +198,8 @@ typedef struct sq_comm sq_comm;   /* owns NCCL link communicators + comm streams
 size_t sq_comm_unique_id_bytes(void);                         /* 128 */
 sq_status sq_comm_get_unique_id(uint8_t* id_host);            /* rank 0; broadcast by caller */
 /* One process per GPU; id_host from sq_comm_get_unique_id on rank 0 (world comm),
- * nranks = number of pipeline stages.  Collective over all ranks. */
+ * nranks = number of pipeline stages (any P >= 1: one 2-rank NCCL communicator per link
+ * r -> r+1 mod P, built with up to three ncclCommSplit calls).  Collective over all ranks. */
 sq_status sq_comm_init(sq_comm** out, const uint8_t* id_host, int nranks, int rank);
 /* Single-process "virtual pipeline": every stage on the current device, transfers
  * are device copies.  Bitwise reference for the multi-GPU run. */

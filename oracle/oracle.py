@@ -51,8 +51,17 @@ def _lib() -> ctypes.CDLL:
         L.oq_stage.argtypes = [P, ctypes.c_int, P, I64, I64, P]
         L.oq_packed_bytes.argtypes = [I64, I64, ctypes.c_int]
         L.oq_packed_bytes.restype = ctypes.c_size_t
+        L.oq_set_threads.argtypes = [ctypes.c_int]
+        L.oq_set_threads.restype = None
+        L.oq_max_threads.restype = ctypes.c_int
         _L = L
     return _L
+
+
+def set_threads(n: int) -> int:
+    """OpenMP threads of the oracle's parallel loops (timing only); returns the new maximum."""
+    _lib().oq_set_threads(int(n))
+    return int(_lib().oq_max_threads())
 
 
 def _p(a: np.ndarray | None):

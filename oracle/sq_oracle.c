@@ -20,7 +20,8 @@
  *   oq_pack/oq_unpack   Layouts L3/L4/L8 + tiling T16 of DESIGN.md (paper silent).  Pinned by
  *                       hand-derived golden words (tests/golden/pack_words.txt),
  *                       round trip, and the P:160 byte count.
- *   oq_dequant_row      x~ = s_x x^ + q_x, exact in fp64.
+ *   oq_dequant_row      x~ = s_x x^ + q_x, exact in fp64, saturated at 65504 (R20).
+ *                       Pinned by the hand-computed +-65504 group (tests/test_oracle_pins.py).
  *   oq_linear           y = x W~^T (+ bias) in fp64 (weight-only W.A16).  Pinned by
  *                       numpy fp64 matmul at bits = 16 and on grid-aligned weights,
  *                       Theorem 1 variance bound.
@@ -29,6 +30,7 @@
  *                       attention stub (R12); pinned by composition checks.
  */
 #include <math.h>
+#include <omp.h>
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
@@ -47,6 +49,10 @@ static uint16_t f2h(float f) {
 }
 
 float oq_h2f(uint16_t h) { return h2f(h); }
+
+/* host threads of the parallel loops (timing the oracle at 1 thread and at all cores; no arithmetic) */
+void oq_set_threads(int n) { omp_set_num_threads(n > 0 ? n : 1); }
+int oq_max_threads(void) { return omp_get_max_threads(); }
 uint16_t oq_f2h(float f) { return f2h(f); }
 
 /* ---------------- O1: round-to-nearest per-group min/max quantization ----------------
@@ -177,9 +183,13 @@ int oq_unpack(const uint8_t* packed, int64_t n, int64_t k, int bits, uint8_t* co
 }
 
 /* ---------------- O4: dequantize one row of a packed weight into fp64 ----------------
- * x~ = s x^ + q, exact in fp64 (s, q fp16; x^ < 256).  bits == 16: the fp16
+ * x~ = s x^ + q, exact in fp64 (s, q fp16; x^ < 256), then saturated to the fp16
+ * finite range (reading R20: the dequantized weight is an fp16 operand of the W.A16 product,
+ * P:93; only the top can overflow, since q = group min >= -65504 and s x^ >= 0, and the
+ * saturation never moves x~ away from x, because every x <= 65504).  bits == 16: the fp16
  * weight itself (reading R7: FP16 layers are not quantized).
  */
+#define OQ_F16_MAX 65504.0
 static void dequant_row(const uint8_t* packed, const uint32_t* meta, int64_t n, int64_t k,
                         int bits, int group, int64_t r, double* out, uint8_t* tmp_codes) {
   (void)group; (void)n; (void)tmp_codes;
@@ -193,7 +203,8 @@ static void dequant_row(const uint8_t* packed, const uint32_t* meta, int64_t n, 
     uint32_t m = meta[unit_off(r, kk / 128, kg)];
     double s = (double)h2f((uint16_t)(m & 0xFFFF));
     double z = (double)h2f((uint16_t)(m >> 16));
-    out[kk] = s * (double)code_at(packed, r, kk, kg, bits) + z;
+    const double wt = s * (double)code_at(packed, r, kk, kg, bits) + z;
+    out[kk] = wt > OQ_F16_MAX ? OQ_F16_MAX : wt;
   }
 }
 

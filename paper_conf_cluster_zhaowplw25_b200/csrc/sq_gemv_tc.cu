@@ -23,10 +23,13 @@
 //    from TMEM, B (activations) from SMEM; fp32 accumulators of the panel's P
 //    tiles in TMEM (P x 32 columns).
 //  * 4 epilogue warps drain an item: Z = 1 -> bias / activation / fp32 residual
-//    straight to y; Z > 1 -> fp32 partial to the workspace, and the last of the
-//    Z items to arrive (atomic counter) sums all Z partials of the panel in fixed
-//    z order at the end of its CTA (all warps, 16-B loads).  Deterministic;
-//    counters self-reset.
+//    straight to y; Z > 1 (one item per CTA) -> the panel's Z CTAs form a
+//    thread-block cluster, each leaves its fp32 partial in its own shared memory
+//    and CTA z reduces 1/Z of the panel over the cluster through DSMEM in fixed z
+//    order.  When the clusters cannot all be resident, the partials go to the
+//    workspace instead and the grid is launched cooperatively (co-resident by
+//    construction): every CTA waits for its panel's Z partials, then reduces its
+//    1/Z share in fixed z order.  Deterministic; counters self-reset.
 // Warp roles: 0 producer, 1 MMA (+TMEM alloc), 2..17 dequant, 18..21 epilogue.
 #include <cuda.h>
 
@@ -36,43 +39,21 @@
 
 #include "sq_tc.cuh"
 
-#ifndef SQ_TC_WAIT
-#define SQ_TC_WAIT 0  // experiments: 0 = try_wait with a suspend-time hint, 1 = try_wait spin, 2 = test_wait spin
-#endif
-
 namespace sq {
 namespace {
 using namespace tc;
 
-__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
-  uint32_t ok;
-  asm volatile("{\n\t.reg .pred p;\n\tmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
-               : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
-  return ok != 0;
-}
-__device__ __forceinline__ void wait_bar(uint64_t* bar, uint32_t parity) {
-  if (SQ_TC_WAIT == 0) mbar_wait_park(bar, parity);
-  else if (SQ_TC_WAIT == 1) mbar_wait(bar, parity);
-  else while (!mbar_test(bar, parity)) {}
-}
+// barrier waits: try_wait with a suspend-time hint (measured equal to spinning try_wait / test_wait)
+__device__ __forceinline__ void wait_bar(uint64_t* bar, uint32_t parity) { mbar_wait_park(bar, parity); }
 
 constexpr int BN = 128;     // weight rows per unit (TMEM lanes, MMA M)
 constexpr int BT = 32;      // token columns (MMA N)
-#ifndef SQ_TC_DEEP_A
-#define SQ_TC_DEEP_A 1  // 1: panels of <= 4 tiles, 1.5x deeper TMEM A ring (3 slots of 2 groups / 6 of 1)
-#endif
-constexpr int PMAX = SQ_TC_DEEP_A ? 4 : 8;  // row tiles per panel (activation reuse), at most
+constexpr int PMAX = 4;     // row tiles per panel (activation reuse), at most
 constexpr int kCnt2 = 2048;  // second per-panel counter (fix-up done) at cnt + kCnt2
 constexpr int XK = 64;
 constexpr int X_BLOCK = BT * XK * 2;  // 4 KB: [32 tokens][64 k] SW128 tile
-#ifndef SQ_TC_DQ_WARPS
-#define SQ_TC_DQ_WARPS 16
-#endif
-#ifndef SQ_TC_DQ_PER_GROUP
-#define SQ_TC_DQ_PER_GROUP 8
-#endif
-constexpr int DQ_WARPS = SQ_TC_DQ_WARPS;        // dequant warps, in DQ_GROUPS groups of DQ_PER_GROUP
-constexpr int DQ_PER_GROUP = SQ_TC_DQ_PER_GROUP;  // 4 lane quadrants x KH k-parts of one unit
+constexpr int DQ_WARPS = 16;      // dequant warps, in DQ_GROUPS groups of DQ_PER_GROUP (8 / 24 measured: no gain)
+constexpr int DQ_PER_GROUP = 8;   // 4 lane quadrants x KH k-parts of one unit
 constexpr int DQ_KH = DQ_PER_GROUP / 4;
 constexpr int DQ_GROUPS = DQ_WARPS / DQ_PER_GROUP;  // group q dequantizes units i = q (mod DQ_GROUPS)
 constexpr int TMEM_COLS = 512;
@@ -81,10 +62,6 @@ constexpr int A_COL = PMAX * BT;      // S_A x (64 * UG) columns
 constexpr int NUM_THREADS = 32 * (2 + DQ_WARPS + 4);  // producer, MMA, dequant, epilogue
 constexpr int EPI_WARP0 = 2 + DQ_WARPS;
 constexpr uint32_t kIdescTc = make_idesc(BN, BT);
-#ifndef SQ_TC_XLDG
-#define SQ_TC_XLDG 0  // 1: the epilogue warps load the activation slices (LDG -> STS), 0: TMA (measured: 0 is faster)
-#endif
-constexpr int X_LAG = 0;              // activations of step q are fetched just before its weights (X_LAG > 0 deadlocks once P * (X_LAG + 1) > S_W)
 
 // UG = 128-k groups per unit, chosen so a weight stage is ~16 KB (INT3/INT4: 2, INT8: 1).
 template <int BITS, int UG>
@@ -96,7 +73,7 @@ struct DCfg {
   // TMEM A slots of 64*UG columns: the dequant warps fill slot i % S_A while the MMA reads the
   // others (slots are owned by one dequant group: multiples of DQ_GROUPS)
   static constexpr int A_SLOT = 64 * UG;
-  static constexpr int S_A = UG == 3 ? 2 : (SQ_TC_DEEP_A ? (UG == 2 ? 3 : 6) : (UG == 2 ? 2 : 4));
+  static constexpr int S_A = UG == 3 ? 2 : (UG == 2 ? 3 : 6);
   static constexpr int S_X = 3;  // activation ring, in steps
   static_assert(BITS == 16 || A_COL + S_A * A_SLOT <= TMEM_COLS, "TMEM budget");
 };
@@ -134,10 +111,7 @@ struct TcP {
   int I;      // work items = panels * Z
   float* part;  // [items][PMAX tiles][32 tokens][128 rows] fp32 partial sums (Z > 1)
   int* cnt;     // [panels]
-  unsigned long long* trace;  // debug: CTA 0 per-unit clock64 events (sq_debug_trace), or null
-  int abl;                    // debug ablation (SQ_TC_ABL): 1 = no dequant, 2 = no MMAs (results wrong)
-  const __half* x;            // activations [m][ldx] (SQ_TC_XLDG: loaded by the epilogue warps)
-  int ldx;
+  unsigned long long* trace;  // debug build (SQ_TC_DEBUG): CTA 0 per-unit clock64 events (sq_debug_trace), or null
   int cl;                     // Z > 1 items of a panel form a thread-block cluster: DSMEM reduction
 };
 
@@ -157,7 +131,7 @@ __device__ __forceinline__ float4 ld_dsmem_f4(uint32_t addr) {
 }
 
 #ifndef SQ_TC_DEBUG
-#define SQ_TC_DEBUG 0  // 1: clock64 trace (sq_debug_trace) and SQ_TC_ABL ablations compiled in
+#define SQ_TC_DEBUG 0  // 1: clock64 trace (sq_debug_trace) and the SQ_TC_PZ plan override compiled in
 #endif
 __device__ __forceinline__ void trace_ev(const TcP& p, int ev, int i) {
   if (SQ_TC_DEBUG && p.trace && blockIdx.x == 0 && i < 256) p.trace[ev * 256 + i] = clock64();
@@ -229,7 +203,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   auto j1_of = [&](int it) { return (int)((long long)(it % Z + 1) * ks / Z); };
 
   if (threadIdx.x == 0) {
-    for (int i = 0; i < S_X; ++i) { mbar_init(&full_x[i], SQ_TC_XLDG ? 4 : 1); mbar_init(&empty_x[i], 1); }
+    for (int i = 0; i < S_X; ++i) { mbar_init(&full_x[i], 1); mbar_init(&empty_x[i], 1); }
     // fp16 weights are the MMA's A operand straight from SMEM: the MMA commit frees the slot
     for (int i = 0; i < S_W; ++i) { mbar_init(&full_w[i], 1); mbar_init(&empty_w[i], BITS == 16 ? 1 : DQ_PER_GROUP); }
     for (int i = 0; i < S_A; ++i) { mbar_init(&full_a[i], DQ_PER_GROUP); mbar_init(&empty_a[i], 1); }
@@ -248,18 +222,15 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const int sw = i % S_W;
     const int tile16 = (pn * P + t) * (BN / 16);
     uint8_t* wdst = smem + SM::OFF_W + sw * SM::W_STAGE;
-    const bool no_meta = SQ_TC_DEBUG && (p.abl & 16), no_w = SQ_TC_DEBUG && (p.abl & 32);
-    mbar_arrive_expect_tx(&full_w[sw], (BITS == 16 ? BN * 256u : (uint32_t)(BN * GCfg<BITS>::GB * UG + BN * 4 * UG)) -
-                                           (no_meta && BITS != 16 ? BN * 4 * UG : 0) -
-                                           (no_w ? BN * GCfg<BITS>::GB * UG : 0));
+    mbar_arrive_expect_tx(&full_w[sw], BITS == 16 ? BN * 256u : (uint32_t)(BN * GCfg<BITS>::GB * UG + BN * 4 * UG));
     if constexpr (BITS == 16) {
       // row-major fp16 [n][k]: two SW128 boxes [128 rows][64 k] = the MMA's K-major A tiles
       tma_load_2d(wdst, &tm_w, &full_w[sw], j * 128, (pn * P + t) * BN);
       tma_load_2d(wdst + BN * 128, &tm_w, &full_w[sw], j * 128 + 64, (pn * P + t) * BN);
     } else {
       // placement T16 as lines: box {line, lpu * UG lines, 8 row tiles} -> [tile][group][16][GB]
-      if (!no_w) tma_load_3d(wdst, &tm_w, &full_w[sw], 0, j * UG * LPU_, tile16);
-      if (!no_meta) tma_load_2d(smem + SM::OFF_META + sw * BN * 4 * UG, &tm_m, &full_w[sw], j * UG * 16, tile16);
+      tma_load_3d(wdst, &tm_w, &full_w[sw], 0, j * UG * LPU_, tile16);
+      tma_load_2d(smem + SM::OFF_META + sw * BN * 4 * UG, &tm_m, &full_w[sw], j * UG * 16, tile16);
     }
   };
   // PDL: weights never depend on the previous kernel -- thread 0 fills the whole weight ring right
@@ -284,8 +255,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 
   if (warp == 0) {
     // ---------------- producer.  The warp runs the loop and the waits; one elected lane issues.
-    int i = 0, q = 0, qx = 0;  // units, k-steps issued (weights), k-steps issued (activations)
-    int xj[X_LAG + 1];         // k-step of the pending activation fetches (ring of X_LAG + 1)
+    int i = 0, qx = 0;  // units issued, k-steps issued (activations)
     auto issue_x = [&](int j) {
       const int sx = qx % S_X, rx = qx / S_X;
       wait_bar(&empty_x[sx], (rx & 1) ^ 1);
@@ -305,9 +275,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     trace_ev(p, 7, 0);
     for (int it = blockIdx.x; it < I; it += C) {
       const int pn = it / Z, j1 = j1_of(it), pp = tiles_of(pn);
-      for (int j = j0_of(it); j < j1; ++j, ++q) {
-        xj[q % (X_LAG + 1)] = j;
-        if (!SQ_TC_XLDG && q >= X_LAG) issue_x(xj[(q - X_LAG) % (X_LAG + 1)]);
+      for (int j = j0_of(it); j < j1; ++j) {
+        issue_x(j);  // the step's activation slice, just before its weights
         for (int t = 0; t < pp; ++t, ++i) {
           if (i < pre) continue;
           const int sw = i % S_W, rw = i / S_W;
@@ -318,8 +287,6 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         }
       }
     }
-    if (!SQ_TC_XLDG)
-      for (int r = q > X_LAG ? q - X_LAG : 0; r < q; ++r) issue_x(xj[r % (X_LAG + 1)]);
   } else if (warp == 1) {
     // ---------------- MMA issuer: the warp waits, one elected lane issues a unit's 8*UG MMAs and
     // commits.  TMEM base is 0, so every operand is warp-uniform.
@@ -365,12 +332,10 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           if (elect_one()) {
             const uint32_t d_tm = tmem + D_COL + t * BT;
             const uint32_t a_tm = tmem + A_COL + sa * DCfg<BITS, UG>::A_SLOT;
-            if (!(SQ_TC_DEBUG && (p.abl & 2))) {
 #pragma unroll
-              for (int kk = 0; kk < 8 * UG; ++kk)
-                tc_mma_ts(d_tm, a_tm + kk * 8, bdesc0 + (uint64_t)(((kk >> 2) * X_BLOCK + (kk & 3) * 32) >> 4),
-                          kIdescTc, (j == j0 && kk == 0) ? 0u : 1u);
-            }
+            for (int kk = 0; kk < 8 * UG; ++kk)
+              tc_mma_ts(d_tm, a_tm + kk * 8, bdesc0 + (uint64_t)(((kk >> 2) * X_BLOCK + (kk & 3) * 32) >> 4),
+                        kIdescTc, (j == j0 && kk == 0) ? 0u : 1u);
             tc_commit(&empty_a[sa]);
             if (t == pp - 1) {
               tc_commit(&empty_x[sx]);
@@ -387,9 +352,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     // DQ_GROUPS).  Thread = weight row (lane quadrant warp % 4); warp kh of the group takes batches
     // [kh*2*UG, kh*2*UG + 2*UG) of the unit's 4*UG 32-k batches.  Slots of both rings are owned by
     // one group (ring depths are multiples of DQ_GROUPS), so phases follow from i alone.
-    // (SQ_TC_DEEP_A: A slots alternate between the groups; in-order MMA completion keeps every
-    // waiter within one phase of the slot's barrier)
-    static_assert(BITS == 16 || (S_W % DQ_GROUPS == 0 && (SQ_TC_DEEP_A || S_A % DQ_GROUPS == 0)), "ring slots owned by one dequant group");
+    // (A slots alternate between the groups; in-order MMA completion keeps every waiter within one
+    // phase of the slot's barrier)
+    static_assert(BITS == 16 || S_W % DQ_GROUPS == 0, "weight ring slots owned by one dequant group");
     int nunits = 0;
     if constexpr (BITS != 16)
       for (int it = blockIdx.x; it < I; it += C) nunits += (j1_of(it) - j0_of(it)) * tiles_of(it / Z);
@@ -426,8 +391,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           dequant_row_batches<BITS, 4>(wst, mt[ru0 + 32], r, a_tm + 128, (ru0 + 32) * GB, 0);
         }
       } else if constexpr (BITS != 16) {
-        if (!(SQ_TC_DEBUG && (p.abl & 1)))
-          dequant_row_batches<BITS, NBW < 4 ? NBW : 4>(wst, mt[ru], r, a_tm + gg * 64, ru * GB, b0);
+        dequant_row_batches<BITS, NBW < 4 ? NBW : 4>(wst, mt[ru], r, a_tm + gg * 64, ru * GB, b0);
       }
       if (tr) trace_ev(p, 12, i);
       tc_wait_st();
@@ -445,39 +409,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const int r = sp * 32 + lane;
     const uint32_t lane_base = (uint32_t)(sp * 32) << 16;
     const bool leader = threadIdx.x == EPI_WARP0 * 32;
-    if (SQ_TC_XLDG) pdl_wait();  // activation loads below; y / partial writes follow the producer's wait
-    int n_item = 0, qx = 0;
-    const int ew = warp - EPI_WARP0;  // 0..3
+    int n_item = 0;
     for (int it = blockIdx.x; it < I; it += C, ++n_item) {
       const int pn = it / Z, pp = tiles_of(pn);
-      if (SQ_TC_XLDG) {
-        // activation slices of this item's k-steps: [32 tokens][UG*128 k] fp16 as 2*UG SW128 tiles
-        // [32][64] (tokens >= m zero), written with generic stores then handed to the tensor core
-        // (fence.proxy.async) -- off the TMA engine, whose per-SM ingest the weight stream needs
-        constexpr int CHUNKS = 2 * UG * BT * 8;  // 16-B chunks per step
-        for (int j = j0_of(it); j < j1_of(it); ++j, ++qx) {
-          const int sx = qx % S_X, rx = qx / S_X;
-          wait_bar(&empty_x[sx], (rx & 1) ^ 1);
-          uint8_t* xs = smem + SM::OFF_X + sx * X_STAGE;
-          uint4 v[CHUNKS / 128];
-#pragma unroll
-          for (int u = 0; u < CHUNKS / 128; ++u) {
-            const int c = (u * 128) + ew * 32 + lane;  // chunk: tile c / 256, row (c / 8) % 32, col c % 8
-            const int tt = c >> 8, r = (c >> 3) & 31, lc = c & 7;
-            v[u] = r < p.m ? __ldg(reinterpret_cast<const uint4*>(p.x + (int64_t)r * p.ldx + (int64_t)j * UG * 128 + tt * 64 + lc * 8))
-                           : make_uint4(0u, 0u, 0u, 0u);
-          }
-#pragma unroll
-          for (int u = 0; u < CHUNKS / 128; ++u) {
-            const int c = (u * 128) + ew * 32 + lane;
-            const int tt = c >> 8, r = (c >> 3) & 31, lc = c & 7;
-            *reinterpret_cast<uint4*>(xs + tt * X_BLOCK + r * 128 + ((lc ^ (r & 7)) << 4)) = v[u];
-          }
-          fence_proxy_async_smem();
-          __syncwarp();
-          if (lane == 0) mbar_arrive(&full_x[sx]);
-        }
-      }
       wait_bar(d_full, n_item & 1);
       tc_fence_after();
       for (int t = 0; t < pp; ++t) {
@@ -614,30 +548,6 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   }
 }
 
-typedef CUresult (*EncodeFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
-                             const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
-                             CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
-
-cudaError_t enc(CUtensorMap* m, CUtensorMapDataType dt, const void* ptr, int rank, const uint64_t* dims,
-                const uint64_t* strides, const uint32_t* box, CUtensorMapSwizzle sw) {
-  static EncodeFn fn = nullptr;
-  if (!fn) {
-    void* f = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) != cudaSuccess ||
-        q != cudaDriverEntryPointSuccess)
-      return cudaErrorNotSupported;
-    fn = reinterpret_cast<EncodeFn>(f);
-  }
-  cuuint64_t d[5], st[4];
-  cuuint32_t b[5], es[5];
-  for (int i = 0; i < rank; ++i) { d[i] = dims[i]; b[i] = box[i]; es[i] = 1; }
-  for (int i = 0; i + 1 < rank; ++i) st[i] = strides[i];
-  CUresult r = fn(m, dt, (cuuint32_t)rank, const_cast<void*>(ptr), d, st, b, es, CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
-                  CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
-}
-
 template <int BITS, int UG, int EPI>
 cudaError_t launch_tc_be(const CUtensorMap& tx, const CUtensorMap& tw, const CUtensorMap& tm, const TcP& p0, int nc,
                          cudaStream_t s) {
@@ -655,27 +565,47 @@ cudaError_t launch_tc_be(const CUtensorMap& tx, const CUtensorMap& tw, const CUt
   cfg.blockDim = dim3(NUM_THREADS);
   cfg.dynamicSmemBytes = DSmem<BITS, UG>::BYTES;
   cfg.stream = s;
-  cudaLaunchAttribute at[2];
-  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  at[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
-  at[1].id = cudaLaunchAttributeClusterDimension;
-  at[1].val.clusterDim.x = p.Z;
-  at[1].val.clusterDim.y = 1;
-  at[1].val.clusterDim.z = 1;
+  cudaLaunchAttribute at[3];
+  int na = 0;
+  at[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[na++].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
   cfg.attrs = at;
-  cfg.numAttrs = 1;
   if (p.cl) {
     // the panel's Z items as one cluster, only if every cluster of the grid can be resident at once
-    // (the DSMEM reduction waits for all Z CTAs); else the global-memory fix-up
-    cfg.numAttrs = 2;
-    int ncl = 0;
-    if (cudaOccupancyMaxActiveClusters(&ncl, kern, &cfg) != cudaSuccess || ncl * p.Z < nc) {
-      cudaGetLastError();
-      p.cl = 0;
-      cfg.numAttrs = 1;
+    // (the DSMEM reduction waits for all Z CTAs); the occupancy answer is cached per Z
+    static int ncl_of_z[33];
+    static bool init = false;
+    if (!init) { for (int& v : ncl_of_z) v = -1; init = true; }
+    at[na].id = cudaLaunchAttributeClusterDimension;
+    at[na].val.clusterDim.x = p.Z;
+    at[na].val.clusterDim.y = 1;
+    at[na].val.clusterDim.z = 1;
+    cfg.numAttrs = na + 1;
+    int& ncl = ncl_of_z[p.Z];
+    if (ncl < 0) {
+      int v = 0;
+      if (cudaOccupancyMaxActiveClusters(&v, kern, &cfg) != cudaSuccess) { cudaGetLastError(); v = 0; }
+      ncl = v;
     }
+    if (ncl * p.Z >= nc) ++na;
+    else p.cl = 0;
   }
-  return cudaLaunchKernelEx(&cfg, kern, tx, tw, tm, p);
+  if (!p.cl && p.Z > 1) {
+    // global-memory split-k fix-up: a panel's CTAs wait for each other's partials, so the grid (one
+    // item per SM) is launched cooperatively -- co-residency is guaranteed even when other kernels
+    // (NCCL on the pipeline's comm streams) hold SMs
+    at[na].id = cudaLaunchAttributeCooperative;
+    at[na++].val.cooperative = 1;
+  }
+  cfg.numAttrs = na;
+  cudaError_t e = cudaLaunchKernelEx(&cfg, kern, tx, tw, tm, p);
+  if (e != cudaSuccess && na > 1 && pdl_enabled()) {
+    // a driver that rejects PDL together with a cluster / cooperative launch: plain stream order
+    cudaGetLastError();
+    at[0].val.programmaticStreamSerializationAllowed = 0;
+    e = cudaLaunchKernelEx(&cfg, kern, tx, tw, tm, p);
+  }
+  return e;
 }
 
 template <int BITS, int UG>
@@ -701,12 +631,9 @@ cudaError_t launch_tc_b(const CUtensorMap& tx, const CUtensorMap& tw, const CUte
 
 // UG: groups per unit -- a ~16-KB weight stage (INT3/INT4 two groups when k/128 is even)
 // INT3/INT4 take three groups per unit when 3 | k/128 (a ~24 KB INT4 stage, 2 TMEM A slots): one
-// hand-off chain per 1.5x the bytes; measured +5-8 % INT4 GB/s on OPT-66B shapes (tools/exp_ug3.sh).
-// SQ_TC_UG3=0 restores two.
+// hand-off chain per 1.5x the bytes; measured +5-8 % INT4 GB/s on OPT-66B shapes.
 int tc_ug(int bits, int kg) {
-  static int ug3 = -1;
-  if (ug3 < 0) { const char* e = getenv("SQ_TC_UG3"); ug3 = (e && e[0] == '0') ? 0 : 1; }
-  if (ug3 && bits <= 4 && kg % 3 == 0) return 3;
+  if (bits <= 4 && kg % 3 == 0) return 3;
   return (bits <= 4 && kg % 2 == 0) ? 2 : 1;
 }
 
@@ -755,7 +682,7 @@ size_t gemv_tc_workspace_bytes(int64_t n, int64_t k) {
 
 // the activation group sums (when the caller passes none) follow the partials
 size_t gemv_tc_xsum_offset(int64_t n, int64_t k) {
-  int64_t items = getenv("SQ_TC_PZ") ? 2 * num_sms() : 0;  // room for forced splits (experiments)
+  int64_t items = SQ_TC_DEBUG && getenv("SQ_TC_PZ") ? 2 * num_sms() : 0;  // room for forced splits (debug build)
   for (int bits : {3, 4, 8, 16}) {
     const TcPlan pl = tc_plan(n, k, bits);
     if (pl.Z > 1 && pl.I > items) items = pl.I;
@@ -773,13 +700,13 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
     // activations as [k/64][m][64]: one box {64, 32, 2*ug} per unit -> 2*ug SW128 tiles [32 tokens][64 k]
     const uint64_t dx[3] = {64, (uint64_t)m, (uint64_t)w.k / 64}, sx[2] = {(uint64_t)ldx * 2, 128};
     const uint32_t bx[3] = {XK, BT, (uint32_t)(2 * ug)};
-    cudaError_t e = enc(&tx, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, x, 3, dx, sx, bx, CU_TENSOR_MAP_SWIZZLE_128B);
+    cudaError_t e = encode_nd(&tx, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, x, 3, dx, sx, bx, CU_TENSOR_MAP_SWIZZLE_128B);
     if (e != cudaSuccess) return e;
   }
   if (w.bits == 16) {
     const uint64_t dw[2] = {(uint64_t)w.k, (uint64_t)w.n}, sw_[1] = {(uint64_t)w.k * 2};
     const uint32_t bw[2] = {64, BN};
-    cudaError_t e = enc(&tw, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, w.packed, 2, dw, sw_, bw, CU_TENSOR_MAP_SWIZZLE_128B);
+    cudaError_t e = encode_nd(&tw, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, w.packed, 2, dw, sw_, bw, CU_TENSOR_MAP_SWIZZLE_128B);
     if (e != cudaSuccess) return e;
   } else {
     // T16 units as lines: [n/16 tiles][kg * lpu lines][line bytes]; box = UG units of 8 tiles
@@ -787,14 +714,14 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
     const WLines wl = wlines(w.bits);
     const uint64_t dw[3] = {(uint64_t)wl.line, (uint64_t)kg * wl.lpu, nt}, sw_[2] = {(uint64_t)wl.line, kg * 16 * gb};
     const uint32_t bw[3] = {(uint32_t)wl.line, (uint32_t)(wl.lpu * ug), BN / 16};
-    cudaError_t e = enc(&tw, CU_TENSOR_MAP_DATA_TYPE_UINT8, w.packed, 3, dw, sw_, bw,
+    cudaError_t e = encode_nd(&tw, CU_TENSOR_MAP_DATA_TYPE_UINT8, w.packed, 3, dw, sw_, bw,
                         wl.sw128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE);
     if (e != cudaSuccess) return e;
     // meta as [n/16 tiles][kg * 16] u32: one box row = the UG groups of a tile (64 * UG contiguous
     // bytes), 8 rows per unit (a 3-D {16, UG, 8} box would move 16 rows of 64 B)
     const uint64_t dm[2] = {(uint64_t)kg * 16, nt}, sm_[1] = {(uint64_t)kg * 64};
     const uint32_t bm[2] = {(uint32_t)(16 * ug), BN / 16};
-    e = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, w.meta, 2, dm, sm_, bm, CU_TENSOR_MAP_SWIZZLE_NONE);
+    e = encode_nd(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, w.meta, 2, dm, sm_, bm, CU_TENSOR_MAP_SWIZZLE_NONE);
     if (e != cudaSuccess) return e;
   }
   TcP p{};
@@ -810,9 +737,9 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
   p.ks = kg / ug;
   TcPlan pl = tc_plan(w.n, w.k, w.bits);
   {
-    // experiments only: SQ_TC_PZ="P,Z" forces the panel width and k split
+    // debug build only: SQ_TC_PZ="P,Z" forces the panel width and k split
     static int fp = -1, fz = -1;
-    if (fp < 0) {
+    if (SQ_TC_DEBUG && fp < 0) {
       const char* e = getenv("SQ_TC_PZ");
       fp = 0;
       if (e && sscanf(e, "%d,%d", &fp, &fz) != 2) fp = 0;
@@ -829,13 +756,6 @@ cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, in
   p.cnt = reinterpret_cast<int*>(base);
   p.part = reinterpret_cast<float*>(base + kCntBytes);
   p.trace = g_trace;
-  {
-    static int abl = -1;
-    if (abl < 0) { const char* e = getenv("SQ_TC_ABL"); abl = e ? atoi(e) : 0; }
-    p.abl = abl;
-  }
-  p.x = x;
-  p.ldx = (int)ldx;
   {
     static int cl = -1;  // SQ_TC_CLUSTER=0 disables the cluster/DSMEM split-k reduction
     if (cl < 0) { const char* e = getenv("SQ_TC_CLUSTER"); cl = (e && e[0] == '0') ? 0 : 1; }

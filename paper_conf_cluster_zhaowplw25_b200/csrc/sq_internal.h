@@ -2,6 +2,7 @@
 #pragma once
 #include <cstdarg>
 #include <cstdint>
+#include <cuda.h>
 #include <cuda_fp16.h>
 #include <cuda_runtime.h>
 
@@ -56,6 +57,10 @@ sq_status stage_forward(const sq_layer* layers, int n_layers, int phase, const f
 sq_status check_layers(const sq_layer* layers, int n_layers, const char* who);
 
 int num_sms();
+
+// ---- TMA descriptors (sq_tmap.cu): cuTensorMapEncodeTiled behind a per-thread cache
+cudaError_t encode_nd(CUtensorMap* m, CUtensorMapDataType dt, const void* ptr, int rank, const uint64_t* dims,
+                      const uint64_t* strides_bytes, const uint32_t* box, CUtensorMapSwizzle sw);
 
 // ---- programmatic dependent launch (PDL) ----
 // Decode kernels are launched with programmatic stream serialization: the next kernel of the

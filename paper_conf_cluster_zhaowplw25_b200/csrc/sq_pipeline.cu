@@ -183,7 +183,6 @@ sq_status sq_comm_get_unique_id(uint8_t* id_host) {
 sq_status sq_comm_init(sq_comm** out, const uint8_t* id_host, int nranks, int rank) {
   if (!out || !id_host || nranks < 1 || rank < 0 || rank >= nranks)
     return fail(SQ_EINVAL, "sq_comm_init: bad arguments");
-  if (nranks > 1 && nranks % 2) return fail(SQ_ENOTSUP, "sq_comm_init: odd stage counts > 1 not implemented");
   sq_comm* c = new sq_comm();
   c->nranks = nranks;
   c->rank = rank;
@@ -192,17 +191,29 @@ sq_status sq_comm_init(sq_comm** out, const uint8_t* id_host, int nranks, int ra
     memcpy(&id, id_host, sizeof(id));
     sq_status st = nccl_check(ncclCommInitRank(&c->world, nranks, id, rank), "ncclCommInitRank");
     if (st) { delete c; return st; }
-    // links L_j = (j -> j+1 mod P).  Split A holds the even links, split B the odd ones;
-    // inside a link the sender is comm-rank 0 (key 0), the receiver comm-rank 1.
+    // One 2-rank communicator per link L_j = (j -> j+1 mod P), sender comm-rank 0 (key 0), receiver
+    // comm-rank 1.  ncclCommSplit gives each rank one colour per call, and every rank sits on two links
+    // (it sends on L_r and receives on L_{r-1}), so the links are spread over three split calls with no
+    // rank twice in one call: A = even j < P-1, B = odd j, C = the wrap link L_{P-1} when P is odd
+    // (for even P it is odd and lands in B).  Ranks outside a call's links pass NCCL_SPLIT_NOCOLOR.
     const int P = nranks, r = rank;
-    ncclComm_t a = nullptr, b = nullptr;
-    const int colorA = r / 2, keyA = r % 2;                       // even r: sender of L_r; odd r: receiver of L_{r-1}
-    const int colorB = (r % 2) ? r / 2 : ((r - 1 + P) % P) / 2;   // odd r: sender of L_r; even r: receiver of L_{r-1}
-    const int keyB = (r % 2) ? 0 : 1;
-    if ((st = nccl_check(ncclCommSplit(c->world, colorA, keyA, &a, nullptr), "ncclCommSplit(A)"))) { delete c; return st; }
-    if ((st = nccl_check(ncclCommSplit(c->world, colorB, keyB, &b, nullptr), "ncclCommSplit(B)"))) { delete c; return st; }
-    c->send_comm = (r % 2 == 0) ? a : b;
-    c->recv_comm = (r % 2 == 0) ? b : a;
+    auto call_of = [P](int j) { return (j == P - 1 && P % 2) ? 2 : (j % 2); };
+    const int send_link = r, recv_link = (r - 1 + P) % P;
+    ncclComm_t got[3] = {nullptr, nullptr, nullptr};
+    for (int call = 0; call < 3; ++call) {
+      int color = NCCL_SPLIT_NOCOLOR, key = 0;
+      if (call_of(send_link) == call) { color = send_link; key = 0; }
+      else if (call_of(recv_link) == call) { color = recv_link; key = 1; }
+      if (call == 2 && P % 2 == 0) continue;  // no third call for even P (identical on every rank)
+      st = nccl_check(ncclCommSplit(c->world, color, key, &got[call], nullptr), "ncclCommSplit");
+      if (st) {
+        for (ncclComm_t g : got) if (g) ncclCommDestroy(g);
+        sq_comm_destroy(c);
+        return st;
+      }
+    }
+    c->send_comm = got[call_of(send_link)];
+    c->recv_comm = got[call_of(recv_link)];
   }
   cudaStreamCreateWithFlags(&c->s_send, cudaStreamNonBlocking);
   cudaStreamCreateWithFlags(&c->s_recv, cudaStreamNonBlocking);

@@ -61,19 +61,33 @@ constexpr uint32_t make_idesc(int M, int N) {
   return (1u << 4) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
 }
 
+// w~ = s*c + z in one fp16 FMA (c exact after the magic-number subtraction).  SAT: saturate at the fp16
+// maximum (reading R20) -- only a group with s*(2^b - 1) + z >= 65520 can overflow to +inf, and such
+// groups take this variant (one extra HMNMX2 per pair); q = group min keeps the bottom finite.
+template <bool SAT = false>
 __device__ __forceinline__ uint32_t hsub_fma(uint32_t h, uint32_t off2, uint32_t s2, uint32_t z2) {
   __half2 c = __hsub2(*reinterpret_cast<__half2*>(&h), *reinterpret_cast<__half2*>(&off2));
   __half2 r = __hfma2(c, *reinterpret_cast<__half2*>(&s2), *reinterpret_cast<__half2*>(&z2));
+  if constexpr (SAT) r = __hmin2(r, __half2half2(__ushort_as_half((unsigned short)0x7BFFu)));
   return *reinterpret_cast<uint32_t*>(&r);
+}
+
+// true if some code of the group may dequantize beyond the fp16 maximum (conservative: fp32 rounding
+// of s*qmax + z is monotone, and overflow needs the exact value >= 65520)
+template <int BITS>
+__device__ __forceinline__ bool group_may_overflow(uint32_t meta) {
+  const float s = __half2float(__ushort_as_half((unsigned short)(meta & 0xFFFFu)));
+  const float z = __half2float(__ushort_as_half((unsigned short)(meta >> 16)));
+  return fmaf(s, (float)((1 << BITS) - 1), z) >= 65504.f;
 }
 
 // Dequantize batches [B0, B0 + NB) (32 k each) of this thread's row (r) of one 128-k group into
 // half2 columns taddr + 16 b .. + 15 (w~ = s*c + z), one tcgen05.st per batch.  `row_off` = byte
 // offset of the row inside the stage (default r * GB); the swizzle pattern only depends on
 // r % 16 because every T16 unit starts on a 1-KB boundary.  B0 must be warp-uniform.
-template <int BITS, int NB>
-__device__ __forceinline__ void dequant_row_batches(const uint8_t* wst, uint32_t meta, int r, uint32_t taddr,
-                                                    int row_off, int B0) {
+template <int BITS, int NB, bool SAT>
+__device__ __forceinline__ void dequant_row_batches_(const uint8_t* wst, uint32_t meta, int r, uint32_t taddr,
+                                                     int row_off, int B0) {
   const uint32_t s2 = (meta & 0xFFFFu) * 0x10001u;
   const uint32_t z2 = (meta >> 16) * 0x10001u;
   constexpr uint32_t K1024 = 0x64006400u, K64 = 0x54005400u;
@@ -93,10 +107,10 @@ __device__ __forceinline__ void dequant_row_batches(const uint8_t* wst, uint32_t
 #pragma unroll
       for (int w = 0; w < 4; ++w) {
         const uint32_t x = wv[w], x8 = x >> 8;
-        o[4 * w + 0] = hsub_fma(lop3_and_or(x, 0x000F000Fu, K1024), K1024, s2, z2);
-        o[4 * w + 1] = hsub_fma(lop3_and_or(x, 0x00F000F0u, K64), K64, s2, z2);
-        o[4 * w + 2] = hsub_fma(lop3_and_or(x8, 0x000F000Fu, K1024), K1024, s2, z2);
-        o[4 * w + 3] = hsub_fma(lop3_and_or(x8, 0x00F000F0u, K64), K64, s2, z2);
+        o[4 * w + 0] = hsub_fma<SAT>(lop3_and_or(x, 0x000F000Fu, K1024), K1024, s2, z2);
+        o[4 * w + 1] = hsub_fma<SAT>(lop3_and_or(x, 0x00F000F0u, K64), K64, s2, z2);
+        o[4 * w + 2] = hsub_fma<SAT>(lop3_and_or(x8, 0x000F000Fu, K1024), K1024, s2, z2);
+        o[4 * w + 3] = hsub_fma<SAT>(lop3_and_or(x8, 0x00F000F0u, K64), K64, s2, z2);
       }
       tmem_st16(taddr + 16 * b, o);
     }
@@ -113,8 +127,8 @@ __device__ __forceinline__ void dequant_row_batches(const uint8_t* wst, uint32_t
         const uint32_t wv[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
         for (int t = 0; t < 4; ++t) {
-          o[8 * h + 2 * t] = hsub_fma(prmt(wv[t], 0x64646464u, 0x4140u), K1024, s2, z2);
-          o[8 * h + 2 * t + 1] = hsub_fma(prmt(wv[t], 0x64646464u, 0x4342u), K1024, s2, z2);
+          o[8 * h + 2 * t] = hsub_fma<SAT>(prmt(wv[t], 0x64646464u, 0x4140u), K1024, s2, z2);
+          o[8 * h + 2 * t + 1] = hsub_fma<SAT>(prmt(wv[t], 0x64646464u, 0x4342u), K1024, s2, z2);
         }
       }
       tmem_st16(taddr + 16 * b, o);
@@ -136,7 +150,7 @@ __device__ __forceinline__ void dequant_row_batches(const uint8_t* wst, uint32_t
           const uint32_t hs = sh >= 0 ? (H >> sh) : (H << (-sh));
           uint32_t t;
           asm("lop3.b32 %0, %1, %2, %3, 0xD8;" : "=r"(t) : "r"(hs), "r"(lo), "r"(0x00030003u));  // mask ? lo : hs
-          o[8 * a + i] = hsub_fma(lop3_and_or(t, 0x00070007u, K1024), K1024, s2, z2);
+          o[8 * a + i] = hsub_fma<SAT>(lop3_and_or(t, 0x00070007u, K1024), K1024, s2, z2);
         }
       }
       tmem_st16(taddr + 16 * bl, o);
@@ -156,6 +170,19 @@ __device__ __forceinline__ void dequant_row_batches(const uint8_t* wst, uint32_t
       }
       tmem_st16(taddr + 16 * b, o);
     }
+  }
+}
+
+template <int BITS, int NB>
+__device__ __forceinline__ void dequant_row_batches(const uint8_t* wst, uint32_t meta, int r, uint32_t taddr,
+                                                    int row_off, int B0) {
+  if constexpr (BITS == 16) {
+    dequant_row_batches_<BITS, NB, false>(wst, meta, r, taddr, row_off, B0);
+  } else {
+    if (__builtin_expect(group_may_overflow<BITS>(meta), 0))
+      dequant_row_batches_<BITS, NB, true>(wst, meta, r, taddr, row_off, B0);
+    else
+      dequant_row_batches_<BITS, NB, false>(wst, meta, r, taddr, row_off, B0);
   }
 }
 

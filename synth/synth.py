@@ -161,3 +161,24 @@ def grid_aligned_weight_f16(seed: int, n: int, k: int, bits: int, group: int = 1
     w16 = w.astype(np.float16)
     assert np.array_equal(w16.astype(np.float64), w), "grid weights must be fp16-exact"
     return w16, c.astype(np.uint8), s.astype(np.float16), z.astype(np.float16)
+
+
+def adversarial_weight_f16(seed: int, n: int = 64, k: int = 512) -> np.ndarray:
+    """Synthetic weight with the edge cases of the quantizer and the dequantizing kernels (no method
+    arithmetic): a constant group, a -0 group, subnormals, +-65504 groups (the dequantized top code
+    overflows fp16 unless saturated, R20) in several rows of one 128-row tile, exact
+    half-step ties, a linear ramp and a large outlier.  Needs n >= 16, k >= 256."""
+    w = weight_f16(seed, n, k).copy()
+    w[0, :128] = np.float16(0.5)                                   # constant group
+    w[1, 128:256] = np.float16(-0.0)                               # -0 group
+    w[1, 130] = np.float16(0.0)
+    w[2, :128] = np.float16(6e-8)                                  # subnormal range
+    w[2, 5] = np.float16(-6e-8)
+    w[3, 0], w[3, 1] = np.float16(65504.0), np.float16(-65504.0)   # extremes (group 0)
+    w[4, :128] = (np.arange(128) % 16).astype(np.float16) * np.float16(0.25)  # exact ties for b = 3
+    w[5, 128:256] = np.linspace(-1, 1, 128).astype(np.float16)
+    w[6, 7] = np.float16(30.0)                                     # outlier
+    for r in range(8, min(n, 12)):                                 # extremes in group 1 of more rows
+        w[r, 128 + r], w[r, 140 + r] = np.float16(65504.0), np.float16(-65504.0)
+    w[12, 200] = np.float16(65504.0)                               # top only: s*qmax + z lands near 65504
+    return w

@@ -39,8 +39,57 @@ def main():
                 err = float(np.abs(dy - ref).max() / np.abs(ref).max())
                 worst = max(worst, err)
                 assert err <= 2e-3, (os.environ.get("SQ_GEMV_PATH"), "accum", bits, n, k, m, err)
+    # adversarial groups (R20: +-65504 spans saturate; constant, -0, subnormal, ties) on the forced kernel
+    for bits in (3, 4, 8):
+        n, k = 256, 512
+        w = synth.adversarial_weight_f16(60 + bits, n, k)
+        qo = O.QWeight(w, bits)
+        qg = sq.QLinear.from_fp16(torch.from_numpy(w).cuda(), bits)
+        keep = np.setdiff1d(np.arange(n), [3, 8, 9, 10, 11, 12])
+        for m in (1, 5, 32):
+            x = synth.act_f16(904 + m, m, k)
+            ref = O.linear(x, qo)
+            y0 = np.zeros((m, n), np.float32)
+            ya = torch.from_numpy(y0).cuda()
+            sq.sq_linear_decode(qg, torch.from_numpy(x).cuda(), ya, sq.SQ_EPI_F32_ACCUM)
+            torch.cuda.synchronize()
+            yy = ya.cpu().numpy().astype(np.float64)
+            assert np.isfinite(yy).all(), ("adv", bits, m)
+            for cols in (slice(None), keep):
+                err = float(np.abs(yy[:, cols] - ref[:, cols]).max() / np.abs(ref[:, cols]).max())
+                worst = max(worst, err)
+                assert err <= 2e-3, (os.environ.get("SQ_GEMV_PATH"), "adv", bits, m, err)
     print("ok worst", worst)
 
 
+def full(bits):
+    """configs[1] OPT-13B fc1 at m = 1 on the forced kernel; sampled rows vs the oracle."""
+    n, k, m = 20480, 5120, 1
+    seed = synth.weight_seed(1, "fc1")
+    wd = torch.empty((n, k), dtype=torch.float16, device="cuda")
+    synth.device_weight_f16(wd.data_ptr(), seed, n, k)
+    qg = sq.QLinear.from_fp16(wd, bits)
+    del wd
+    x = synth.act_f16(17, m, k)
+    y = torch.empty((m, n), dtype=torch.float16, device="cuda")
+    sq.sq_linear_decode(qg, torch.from_numpy(x).cuda(), y, 0)
+    torch.cuda.synchronize()
+    yy = y.float().cpu().numpy().astype(np.float64)
+    rows = np.random.default_rng(bits).choice(n, 64, replace=False)
+    rows[0], rows[1] = 0, n - 1
+    ref = O.linear(x, O.QWeight(synth.weight_f16(seed, n, k, rows=rows), bits))
+    err = float(np.abs(yy[:, rows] - ref).max() / np.abs(ref).max())
+    assert err <= 2e-3, ("full", os.environ.get("SQ_GEMV_PATH"), bits, err)
+    # determinism of the cross-CTA fix-up at the full grid
+    y2 = torch.empty_like(y)
+    sq.sq_linear_decode(qg, torch.from_numpy(x).cuda(), y2, 0)
+    torch.cuda.synchronize()
+    assert torch.equal(y, y2)
+    print("ok full", bits, err)
+
+
 if __name__ == "__main__":
-    main()
+    if len(sys.argv) > 2 and sys.argv[1] == "full":
+        full(int(sys.argv[2]))
+    else:
+        main()

@@ -1,6 +1,6 @@
 """Error budget of the GPU linears vs the fp64 oracle (normwise), per bits / phase / m."""
 import sys, os
-sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__)))))  # repo root (tests/diag/..)
 import numpy as np, torch, synth
 from oracle import oracle as O
 import paper_conf_cluster_zhaowplw25_b200 as sq

@@ -1,12 +1,12 @@
 """Where does the stage error come from?  One OPT-13B layer, GPU stage vs oracle, plus
 teacher-forced per-step errors (each GPU step fed the GPU's own previous output)."""
 import sys, os
-sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__)))))  # repo root (tests/diag/..)
 import numpy as np, torch, synth
 from oracle import oracle as O
 import paper_conf_cluster_zhaowplw25_b200 as sq
 from paper_conf_cluster_zhaowplw25_b200 import runtime as R
-sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tests"))
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))  # tests/
 from test_gpu_stage import oracle_layers
 
 def nw(y, r):

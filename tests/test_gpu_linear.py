@@ -29,17 +29,19 @@ def normwise(y, ref):
 
 
 def adversarial_weight(n=64, k=512, seed=3):
-    w = synth.weight_f16(seed, n, k).copy()
-    w[0, :128] = np.float16(0.5)                      # constant group
-    w[1, 128:256] = np.float16(-0.0)                  # -0 group
-    w[1, 130] = np.float16(0.0)
-    w[2, :128] = np.float16(6e-8)                     # subnormal range
-    w[2, 5] = np.float16(-6e-8)
-    w[3, 0], w[3, 1] = np.float16(65504.0), np.float16(-65504.0)  # extremes
-    w[4, :128] = (np.arange(128) % 16).astype(np.float16) * np.float16(0.25)  # exact ties for b=3
-    w[5, 128:256] = np.linspace(-1, 1, 128).astype(np.float16)
-    w[6, 7] = np.float16(30.0)                        # outlier
-    return w
+    return synth.adversarial_weight_f16(seed, n, k)
+
+
+ADV_ROWS = [3, 8, 9, 10, 11, 12]  # rows holding +-65504 (their outputs dwarf the others)
+
+
+def check_adversarial(y, ref):
+    """Finite outputs; normwise over the tensor (R10), and separately over the ordinary rows, whose
+    magnitudes the +-65504 rows would otherwise hide."""
+    assert np.isfinite(y).all()
+    assert normwise(y, ref) <= TOL, normwise(y, ref)
+    keep = np.setdiff1d(np.arange(ref.shape[1]), ADV_ROWS)
+    assert normwise(y[:, keep], ref[:, keep]) <= TOL, normwise(y[:, keep], ref[:, keep])
 
 
 @pytest.mark.parametrize("bits", [3, 4, 8])
@@ -243,4 +245,53 @@ def test_decode_forced_path(path):
         env["SQ_TC_CLUSTER"] = "0"
     script = os.path.join(os.path.dirname(os.path.abspath(__file__)), "_decode_path_check.py")
     r = subprocess.run([sys.executable, script], env=env, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+
+
+def _adv_case(bits, m, seed):
+    sq = sqm()
+    n, k = 256, 512
+    w = adversarial_weight(n, k, seed=seed)
+    b = synth.bias_f16(seed, n)
+    qo = O.QWeight(w, bits, bias=b)
+    qg = sq.QLinear.from_fp16(torch.from_numpy(w).cuda(), bits, torch.from_numpy(b).cuda())
+    # fp16 outputs: activations scaled by 1/16 (exact) so the +-65504 rows stay inside fp16's range
+    x = (synth.act_f16(seed + 1, m, k) * np.float16(0.0625)).astype(np.float16)
+    x32 = synth.act_f16(seed + 2, m, k)
+    return qo, qg, x, x32
+
+
+@pytest.mark.parametrize("bits", [3, 4, 8])
+@pytest.mark.parametrize("m", [1, 8, 32])
+def test_decode_adversarial(bits, m):
+    """R20: groups spanning +-65504 dequantize to a finite top code on every decode kernel; constant,
+    -0, subnormal and tie groups in the same tile (both the fp16 and the fp32-residual epilogues)."""
+    qo, qg, x, x32 = _adv_case(bits, m, 40 + bits)
+    check_adversarial(_run_linear("decode", qg, x, 0), O.linear(x, qo))
+    y0 = synth.hidden_f32(43, m, qg.n)
+    y = _run_linear("decode", qg, x32, 3, y0)
+    check_adversarial(y - y0, O.linear(x32, qo))
+
+
+@pytest.mark.parametrize("bits", [3, 4, 8])
+@pytest.mark.parametrize("m", [1, 300])
+def test_prefill_adversarial(bits, m):
+    qo, qg, x, x32 = _adv_case(bits, m, 50 + bits)
+    check_adversarial(_run_linear("prefill", qg, x, 0), O.linear(x, qo))
+    y0 = synth.hidden_f32(53, m, qg.n)
+    y = _run_linear("prefill", qg, x32, 3, y0)
+    check_adversarial(y - y0, O.linear(x32, qo))
+
+
+@pytest.mark.parametrize("bits", [3, 4, 8])
+def test_decode_mma_full_grid_sampled(bits):
+    """The mma.sync decode kernel (K2) at its configs[1] launch shape: OPT-13B fc1 (20480 x 5120) at
+    m = 1 (one 16-warp CTA per SM, units split evenly, tiles straddling CTAs -> cross-CTA fix-up),
+    forced with SQ_GEMV_PATH=mma in a subprocess; 64 sampled output rows vs the oracle."""
+    import os
+    import subprocess
+    import sys
+    env = dict(os.environ, SQ_GEMV_PATH="mma")
+    script = os.path.join(os.path.dirname(os.path.abspath(__file__)), "_decode_path_check.py")
+    r = subprocess.run([sys.executable, script, "full", str(bits)], env=env, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]

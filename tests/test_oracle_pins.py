@@ -58,6 +58,43 @@ def test_quantize_matches_bruteforce_argmin(bits):
 
 
 @pytest.mark.parametrize("bits", [3, 4, 8])
+def test_exact_ties_round_half_even(bits):
+    # R1: P:91's rounding function at EXACT ties.  s0 = 2^-6 and the group spans [0, qmax*s0], so the
+    # stored scale is exactly s0 and (w - z)/s = c + 1/2 exactly in fp32: half-to-even must give the
+    # even neighbour (roundf / floor(x + 0.5) give c + 1 at every even c and fail).
+    qmax = (1 << bits) - 1
+    s0 = 2.0 ** -6
+    w = np.zeros((1, 128), np.float64)
+    w[0, 0], w[0, 1] = 0.0, qmax * s0
+    nt = min(qmax, 126)
+    w[0, 2:2 + nt] = (np.arange(nt) + 0.5) * s0
+    codes, s, z = O.quantize_groups(w.astype(np.float16), bits)
+    assert float(s[0, 0]) == s0 and float(z[0, 0]) == 0.0
+    want = np.arange(nt) + (np.arange(nt) % 2)  # c + 1/2 -> c if c even, c + 1 if c odd
+    assert np.array_equal(codes[0, 2:2 + nt].astype(np.int64), want)
+    if bits == 3:  # written out by hand: 0.5, 1.5, ..., 6.5 -> 0, 2, 2, 4, 4, 6, 6
+        assert list(codes[0, 2:9]) == [0, 2, 2, 4, 4, 6, 6]
+
+
+# R20 hand computation for a group holding +-65504 (the rest 0):
+#   INT3: s = fp16(131008/7 = 18715.43) = 18720 (spacing 16); c(65504) = rint(6.998) = 7 -> 65536 -> 65504;
+#         c(0) = rint(65504/18720 = 3.499) = 3 -> 3*18720 - 65504 = -9344
+#   INT4: s = fp16(131008/15 = 8733.87) = 8736 (spacing 8);  c(65504) = 15 -> 65536 -> 65504;
+#         c(0) = rint(7.498) = 7 -> 61152 - 65504 = -4352
+#   INT8: s = fp16(131008/255 = 513.76) = 514 (spacing 0.5); c(65504) = rint(254.88) = 255 -> 65566 -> 65504;
+#         c(0) = rint(127.44) = 127 -> 65278 - 65504 = -226
+@pytest.mark.parametrize("bits,scale,w_zero", [(3, 18720.0, -9344.0), (4, 8736.0, -4352.0), (8, 514.0, -226.0)])
+def test_dequant_saturates_at_fp16_max(bits, scale, w_zero):
+    w = np.zeros((16, 128), np.float16)
+    w[0, 0], w[0, 1] = np.float16(65504.0), np.float16(-65504.0)
+    q = O.QWeight(w, bits)
+    assert float(q.scales[0, 0]) == scale and float(q.zeros[0, 0]) == -65504.0
+    wt = q.dequant()
+    assert wt[0, 0] == 65504.0 and wt[0, 1] == -65504.0 and wt[0, 2] == w_zero
+    assert np.isfinite(wt).all()
+
+
+@pytest.mark.parametrize("bits", [3, 4, 8])
 def test_scale_zero_closed_form(bits):
     # P:91 s = (x_max - x_min)/(2^b - 1), q = x_min (R3), scale stored fp16 (R5).
     w = synth.weight_f16(11, 16, 512)
@@ -162,8 +199,12 @@ def test_pack_unpack_round_trip(bits, shape):
 
 
 def test_tile_placement_t16():
-    # T16: unit (tile t, group g) = rows 16t..16t+15 of group g, contiguous, tile-major/group-minor;
-    # meta[(t*kg + g)*16 + r%16] = scale | zero << 16
+    # T16: the packed bytes are [n/16 tiles][k/128 groups][16 rows][GB] --
+    # written here as a numpy reshape/transpose of the row-major codes (not the oracle's index
+    # arithmetic), plus byte offsets derived by hand from the layout definition:
+    #   n = 32, k = 384, bits 8 (GB = 128, kg = 3): row 17, k 130 -> tile 1, group 1, row-in-tile 1
+    #   -> unit 1*3 + 1 = 4 -> byte (4*16 + 1)*128 + 2 = 8322;  row 0, k 383 -> unit 2 -> 2*16*128 + 127 = 4223;
+    #   meta of (row 31, group 0) -> unit 3, entry 3*16 + 15 = 63.
     rng = np.random.default_rng(3)
     n, k, bits = 32, 384, 8
     c = rng.integers(0, 256, size=(n, k)).astype(np.uint8)
@@ -171,11 +212,16 @@ def test_tile_placement_t16():
     z = rng.standard_normal((n, 3)).astype(np.float16)
     packed, meta = O.pack(c, s, z, bits)
     flat = packed.reshape(-1)
-    for r in (0, 7, 16, 31):
-        for g in range(3):
-            off = ((r // 16) * 3 + g) * 16 + r % 16
-            assert np.array_equal(flat[off * 128:(off + 1) * 128], c[r, 128 * g:128 * (g + 1)])
-            assert meta.reshape(-1)[off] == (int(s[r, g].view(np.uint16)) | (int(z[r, g].view(np.uint16)) << 16))
+    assert np.array_equal(flat, c.reshape(2, 16, 3, 128).transpose(0, 2, 1, 3).reshape(-1))
+    assert flat[8322] == c[17, 130] and flat[4223] == c[0, 383]
+    word = s.view(np.uint16).astype(np.uint32) | (z.view(np.uint16).astype(np.uint32) << 16)
+    assert np.array_equal(meta.reshape(-1), word.reshape(2, 16, 3).transpose(0, 2, 1).reshape(-1))
+    assert meta.reshape(-1)[63] == word[31, 0]
+    # L4 under T16: the same transpose on the nibble-packed rows (2 rows x 1 group = 2 x 64 bytes)
+    c4 = rng.integers(0, 16, size=(16, 256)).astype(np.uint8)
+    p4, _ = O.pack(c4, s[:16, :2], z[:16, :2], 4)
+    one = np.stack([O.pack(c4[:, 128 * g:128 * (g + 1)], s[:16, :1], z[:16, :1], 4)[0] for g in range(2)])
+    assert np.array_equal(p4.reshape(-1), one.reshape(-1))  # group-minor units of 16 rows x 64 B
 
 
 @pytest.mark.parametrize("h1", [768, 5120, 7168, 9216, 14336])
@@ -293,11 +339,26 @@ def test_stage_partition_invariance_and_row_independence():
 
 
 def test_pipeline_loopback_definition():
-    # R13/R14: out[:,0] = last prompt position; e_{t+1} = LN(out[:, t]).
-    layers = _tiny_layers(n_layers=2)
-    x0 = synth.hidden_f32(91, 2 * 3 * 128, 1).reshape(2, 3, 128)
+    # R13/R14 with layers whose stage function is known in closed form: every weight 0 (bits 16) and
+    # only fc2 carrying a bias b, so a stage of L layers maps x -> x + L*b (the stub's v = 0, o = 0,
+    # fc1 = 0 -> ReLU(0) = 0).  Then out[:, 0] = x0[:, s-1] + L b (LAST prompt position) and
+    # out[:, t] = LN(out[:, t-1]) + L b, with LN the textbook numpy formula (eps 1e-5).
+    h1, L = 128, 3
+    rng = np.random.default_rng(5)
+    bvec = rng.standard_normal(h1).astype(np.float16)
+    zero = lambda n, k, bias=None: O.QWeight(np.zeros((n, k), np.float16), 16, bias=bias)
+    layers = [O.Layer(16, 0, zero(3 * h1, h1), zero(h1, h1), zero(4 * h1, h1), zero(h1, 4 * h1, bvec))
+              for _ in range(L)]
+    x0 = synth.hidden_f32(91, 2 * 3 * h1, 1).reshape(2, 3, h1)
     out = O.pipeline(layers, x0, 2)
-    h, _ = O.stage(layers, x0[:, 2].astype(np.float64))
-    assert np.array_equal(out[:, 0], h)
-    h1, _ = O.stage(layers, O.layernorm(h))
-    assert np.array_equal(out[:, 1], h1)
+    lb = L * bvec.astype(np.float64)
+
+    def ln(t):
+        mu = t.mean(-1, keepdims=True)
+        return (t - mu) / np.sqrt(((t - mu) ** 2).mean(-1, keepdims=True) + 1e-5)
+
+    ref0 = x0[:, 2].astype(np.float64) + lb
+    np.testing.assert_allclose(out[:, 0], ref0, rtol=1e-13, atol=1e-13)
+    ref1 = ln(ref0) + lb
+    np.testing.assert_allclose(out[:, 1], ref1, rtol=1e-12, atol=1e-12)
+    np.testing.assert_allclose(out[:, 2], ln(ref1) + lb, rtol=1e-12, atol=1e-12)

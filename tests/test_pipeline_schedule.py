@@ -22,7 +22,7 @@ def plan_for(P, L=8, B=6, eta=4, xi=4, s=3, n_dec=3, h1=128, h2=512, bits=None):
     return R().Plan(bits, sol, h1, h2, B, eta, xi, s, n_dec)
 
 
-@pytest.mark.parametrize("P", [2, 4, 8])
+@pytest.mark.parametrize("P", [2, 3, 4, 5, 8])
 @pytest.mark.parametrize("shape", [(6, 4, 4, 3), (32, 8, 32, 5), (7, 3, 2, 1)])
 def test_sends_match_receives_in_order(P, shape):
     # every link j -> j+1 (mod P) carries the same sequence of message sizes on both ends,
@@ -126,20 +126,22 @@ def oracle_model(plan):
     return layers, x0
 
 
-def test_gloo_world2_executes_schedule_like_the_oracle():
+@pytest.mark.parametrize("world", [2, 3])
+def test_gloo_world_executes_schedule_like_the_oracle(world):
+    """world 2 and an odd stage count (3): the ring's wrap link joins two even ranks."""
     import multiprocessing as mp
     from oracle import oracle as O
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
     for p_ in procs:
         p_.start()
     out = q.get(timeout=600)
     for p_ in procs:
         p_.join(timeout=120)
         assert p_.exitcode == 0
-    plan = plan_for(2)
+    plan = plan_for(world)
     layers, x0 = oracle_model(plan)
     ref = O.pipeline(layers, x0, plan.n_decode)
     assert np.array_equal(out, ref)   # rows are independent: bitwise, whatever the partition
