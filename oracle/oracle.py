@@ -42,6 +42,12 @@ def _lib() -> ctypes.CDLL:
     if _L is None:
         L = ctypes.CDLL(build())
         L.oq_quantize_groups.argtypes = [P, I64, I64, ctypes.c_int, ctypes.c_int, P, P, P]
+        L.oq_quantize_groups_ex.argtypes = [P, I64, I64, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_uint64,
+                                            P, P, P]
+        L.oq_splitmix64.argtypes = [ctypes.c_uint64, ctypes.c_uint64]
+        L.oq_splitmix64.restype = ctypes.c_uint64
+        L.oq_uniform24.argtypes = [ctypes.c_uint64, ctypes.c_uint64]
+        L.oq_uniform24.restype = ctypes.c_float
         L.oq_pack.argtypes = [P, P, P, I64, I64, ctypes.c_int, ctypes.c_int, P, P]
         L.oq_unpack.argtypes = [P, I64, I64, ctypes.c_int, P]
         L.oq_dequant.argtypes = [P, P, I64, I64, ctypes.c_int, ctypes.c_int, P]
@@ -84,10 +90,34 @@ def quantize_groups(w: np.ndarray, bits: int, group: int = 128):
     return codes, s, z
 
 
-def scale_sq_sum(w: np.ndarray, bits: int, group: int = 128) -> float:
+SYMMETRIC, STOCHASTIC = 1, 2
+
+
+def quantize_groups_ex(w: np.ndarray, bits: int, group: int = 128, mode: int = 0, seed: int = 0):
+    """O1 with the variants (P:184 symmetric S_W, R21; Theorem 1 stochastic rounding, R22).
+    mode = SYMMETRIC | STOCHASTIC bits; seed of the counter-based uniform generator."""
+    w = np.ascontiguousarray(w, dtype=np.float16)
+    n, k = w.shape
+    codes = np.empty((n, k), np.uint8)
+    s = np.empty((n, k // group), np.float16)
+    z = np.empty((n, k // group), np.float16)
+    _check(_lib().oq_quantize_groups_ex(_p(w), n, k, bits, group, mode, seed, _p(codes), _p(s), _p(z)), "quantize_ex")
+    return codes, s, z
+
+
+def splitmix64(seed: int, i: int) -> int:
+    return int(_lib().oq_splitmix64(seed, i))
+
+
+def uniform24(seed: int, i: int) -> float:
+    return float(_lib().oq_uniform24(seed, i))
+
+
+def scale_sq_sum(w: np.ndarray, bits: int, group: int = 128, mode: int = 0) -> float:
     """f2, eq. (3) weight term: D_W * S_W(b)^2 with the per-group scale of reading R4
-    (R17) = sum over groups of group * s_g(b)^2, s_g(b) the scale O1 stores.  fp64."""
-    _, s, _ = quantize_groups(w, bits, group)
+    (R17) = sum over groups of group * s_g(b)^2, s_g(b) the scale O1 stores (asymmetric or,
+    mode & SYMMETRIC, P:184's symmetric S_W).  fp64."""
+    _, s, _ = quantize_groups_ex(w, bits, group, mode & SYMMETRIC, 0)
     sd = s.astype(np.float64)
     return float(np.sum(group * sd * sd))
 
@@ -144,7 +174,8 @@ def packed_bytes(n: int, k: int, bits: int) -> int:
 class QWeight:
     """Oracle-side quantized linear: packed codes + meta (or fp16 W at bits 16)."""
 
-    def __init__(self, w16: np.ndarray, bits: int, group: int = 128, bias: np.ndarray | None = None):
+    def __init__(self, w16: np.ndarray, bits: int, group: int = 128, bias: np.ndarray | None = None,
+                 mode: int = 0, seed: int = 0):
         self.n, self.k = w16.shape
         self.bits, self.group = bits, group
         self.bias = None if bias is None else np.ascontiguousarray(bias, np.float16)
@@ -153,7 +184,7 @@ class QWeight:
             self.meta = None
             self.codes = self.scales = self.zeros = None
         else:
-            self.codes, self.scales, self.zeros = quantize_groups(w16, bits, group)
+            self.codes, self.scales, self.zeros = quantize_groups_ex(w16, bits, group, mode, seed)
             self.packed, self.meta = pack(self.codes, self.scales, self.zeros, bits, group)
 
     def dequant(self) -> np.ndarray:

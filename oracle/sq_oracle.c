@@ -15,8 +15,12 @@
  * Functions and what pins them (tests/test_oracle_pins.py):
  *   oq_quantize_groups  P:91 (x^ = round((x - q_x)/s_x), s_x = (x_max - x_min)/(2^b - 1)),
  *                       asymmetric S_W of P:184; readings R1-R6 of DESIGN.md.
- *                       Pinned by brute-force argmin, |w - w~| <= s/2, grid-aligned
+ *                       Pinned by brute-force argmin, exact ties, |w - w~| <= s/2, grid-aligned
  *                       recovery, constant groups, closed-form scale bound.
+ *   oq_quantize_groups_ex  + symmetric S_W (R21) and stochastic rounding (Theorem 1,
+ *                       P:176-180, R22).  Pinned by the published splitmix64 vectors, brute
+ *                       force (symmetric), sign symmetry, unbiasedness, the floor/ceil
+ *                       frequencies and Theorem 1's stochastic variance (tests/test_quant_variants.py).
  *   oq_pack/oq_unpack   Layouts L3/L4/L8 + tiling T16 of DESIGN.md (paper silent).  Pinned by
  *                       hand-derived golden words (tests/golden/pack_words.txt),
  *                       round trip, and the P:160 byte count.
@@ -55,19 +59,47 @@ void oq_set_threads(int n) { omp_set_num_threads(n > 0 ? n : 1); }
 int oq_max_threads(void) { return omp_get_max_threads(); }
 uint16_t oq_f2h(float f) { return f2h(f); }
 
-/* ---------------- O1: round-to-nearest per-group min/max quantization ----------------
+/* ---------------- O1: per-group quantization (S_W variants of P:184; rounding of P:176-180) ----
  * x^ = round((x - q_x) / s_x),  s_x = (x_max - x_min) / (2^b - 1),  x~ = s_x x^ + q_x.
  * Group = `group` contiguous weights of one output row (reading R4).  All arithmetic is
  * IEEE binary32 with one rounding per operation; the code is computed against the
- * fp16-ROUNDED scale that is stored (R5); q_x = group minimum (R3, fp16 exact, -0 -> +0);
- * ties round half to even (R1); s == 0 (constant group or underflow) gives code 0 (R6).
+ * fp16-ROUNDED scale that is stored (R5).
+ *
+ * mode bit 0 (OQ_SYMMETRIC, reading R21): P:184's symmetric scale
+ *   S = max(|W_max|, |W_min|) / (2^(b-1) - 1), signed code c^ = clamp(round(w / S), -(2^(b-1)-1), 2^(b-1)-1),
+ *   stored in the same unsigned (code, scale, zero) form as the asymmetric quantizer:
+ *   c = c^ + 2^(b-1) in [1, 2^b - 1], zero q = -2^(b-1) S (so x~ = S c + q = S c^).  S == 0 -> c^ = 0, q = +0.
+ *   A group whose q overflows fp16 is rejected (return 3).
+ * otherwise (asymmetric, readings R2/R3): q_x = group minimum (fp16 exact, -0 -> +0), c in [0, 2^b - 1].
+ *
+ * mode bit 1 (OQ_STOCHASTIC, reading R22): the stochastic rounding of Theorem 1: with
+ *   d the scaled value, c = floor(d) + [u < d - floor(d)], u = uniform24(seed, i) the i-th output of
+ *   the counter-based generator below for the weight's row-major index i = r*k + col.
+ *   Otherwise round to nearest, ties to even (R1).  s == 0 (constant group / underflow) -> d = 0.
  */
-int oq_quantize_groups(const uint16_t* w, int64_t n, int64_t k, int bits, int group,
-                       uint8_t* codes, uint16_t* scales, uint16_t* zeros) {
-  if (!(bits == 3 || bits == 4 || bits == 8) || group <= 0 || k % group) return 1;
+#define OQ_SYMMETRIC 1
+#define OQ_STOCHASTIC 2
+
+/* splitmix64 (Steele, Lea, Flood 2014): output i of the stream seeded `seed`, i.e. the finalizer of
+ * state seed + (i + 1) * 0x9E3779B97F4A7C15.  uniform24 = top 24 bits / 2^24, exact in fp32. */
+uint64_t oq_splitmix64(uint64_t seed, uint64_t i) {
+  uint64_t z = seed + (i + 1) * 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+float oq_uniform24(uint64_t seed, uint64_t i) { return (float)(oq_splitmix64(seed, i) >> 40) * (1.0f / 16777216.0f); }
+
+int oq_quantize_groups_ex(const uint16_t* w, int64_t n, int64_t k, int bits, int group, int mode, uint64_t seed,
+                          uint8_t* codes, uint16_t* scales, uint16_t* zeros) {
+  if (!(bits == 3 || bits == 4 || bits == 8) || group <= 0 || k % group || mode < 0 || mode > 3) return 1;
   const int64_t ng = k / group;
-  const int qmax_i = (1 << bits) - 1;
-  const float qmax = (float)qmax_i;
+  const int sym = mode & OQ_SYMMETRIC, stoch = mode & OQ_STOCHASTIC;
+  const int half_i = 1 << (bits - 1);
+  const float qmax = (float)((1 << bits) - 1);
+  const float cmin = sym ? -(float)(half_i - 1) : 0.0f;   /* clamp range of the (signed) code */
+  const float cmax = sym ? (float)(half_i - 1) : qmax;
+  const float off = sym ? (float)half_i : 0.0f;           /* stored code = code + off */
   for (int64_t r = 0; r < n; ++r) {
     for (int64_t g = 0; g < ng; ++g) {
       const uint16_t* p = w + r * k + g * group;
@@ -79,25 +111,46 @@ int oq_quantize_groups(const uint16_t* w, int64_t n, int64_t k, int bits, int gr
       }
       mn = mn + 0.0f;                       /* canonical zeros: -0 -> +0 */
       mx = mx + 0.0f;
-      float sf = (mx - mn) / qmax;          /* two single-rounded fp32 ops */
-      uint16_t s16 = f2h(sf);
-      float s = h2f(s16);
+      float sf, z;
+      if (sym) {
+        const float amax = fabsf(mx) > fabsf(mn) ? fabsf(mx) : fabsf(mn);
+        sf = amax / (float)(half_i - 1);
+      } else {
+        sf = (mx - mn) / qmax;              /* two single-rounded fp32 ops */
+      }
+      const uint16_t s16 = f2h(sf);
+      const float s = h2f(s16);
+      if (sym) {
+        z = -(float)half_i * s + 0.0f;      /* exact (power-of-two multiple); +0 when s == 0 */
+        if (fabsf(z) > 65504.0f) return 3;
+      } else {
+        z = mn;
+      }
       scales[r * ng + g] = s16;
-      zeros[r * ng + g] = f2h(mn);          /* exact: mn is an fp16 value */
+      zeros[r * ng + g] = f2h(z);           /* exact */
       for (int j = 0; j < group; ++j) {
-        int c = 0;
-        if (s != 0.0f) {
-          float d = (h2f(p[j]) - mn) / s;   /* fp32 sub, fp32 div */
-          float q = rintf(d);               /* round half to even */
-          if (q < 0.0f) q = 0.0f;
-          if (q > qmax) q = qmax;
-          c = (int)q;
+        float d = 0.0f;
+        if (s != 0.0f) d = sym ? h2f(p[j]) / s : (h2f(p[j]) - mn) / s;  /* fp32 (sub), fp32 div */
+        float q;
+        if (stoch) {
+          const float fl = floorf(d);
+          const float fr = d - fl;          /* fp32 sub */
+          q = fl + (oq_uniform24(seed, (uint64_t)(r * k + g * group + j)) < fr ? 1.0f : 0.0f);
+        } else {
+          q = rintf(d);                     /* round half to even */
         }
-        codes[r * k + g * group + j] = (uint8_t)c;
+        if (q < cmin) q = cmin;
+        if (q > cmax) q = cmax;
+        codes[r * k + g * group + j] = (uint8_t)(int)(q + off);
       }
     }
   }
   return 0;
+}
+
+int oq_quantize_groups(const uint16_t* w, int64_t n, int64_t k, int bits, int group,
+                       uint8_t* codes, uint16_t* scales, uint16_t* zeros) {
+  return oq_quantize_groups_ex(w, n, k, bits, group, 0, 0, codes, scales, zeros);
 }
 
 /* ---------------- O2/O3: bit packing (DESIGN.md layouts L8, L4, L3 + tiling T16) ----------------
