@@ -71,6 +71,23 @@ sq_status sq_quantize_groups(const void* w_dev, int64_t n, int64_t k, int bits, 
                              uint8_t* codes_dev, void* scales_dev, void* zeros_dev,
                              sq_stream_t stream);
 
+/* a1 variants.  mode = OR of:
+ *   SQ_QUANT_SYMMETRIC  P:184's symmetric scale (R21):
+ *       s = fp16(max(|mx|, |mn|) / (2^(bits-1) - 1)), z = -2^(bits-1) * s (exact),
+ *       c = clamp(round(w / s), -(2^(bits-1) - 1), 2^(bits-1) - 1) + 2^(bits-1)  (in [1, 2^bits - 1]),
+ *       stored in the same (codes, scales, zeros) form, so sq_pack and every linear take it as is
+ *       (w~ = s c + z = s c^).  A group whose z overflows fp16 (max|w| close to 65504) sets bit 0 of
+ *       *status_dev (device int32 the caller zeroes and reads after a sync); its outputs are undefined.
+ *   SQ_QUANT_STOCHASTIC Theorem 1's stochastic rounding (R22):
+ *       c = floor(d) + [u_i < d - floor(d)] (then clamped), d the scaled value, u_i the top 24 bits
+ *       of splitmix64 output i (state seed + (i + 1) * 0x9E3779B97F4A7C15, finalizer) / 2^24 for the
+ *       weight's row-major index i = row * k + col.  Bit-exact with the oracle for a given seed.
+ * mode 0 is sq_quantize_groups.  status_dev may be NULL unless SQ_QUANT_SYMMETRIC. */
+enum { SQ_QUANT_SYMMETRIC = 1, SQ_QUANT_STOCHASTIC = 2 };
+sq_status sq_quantize_groups_ex(const void* w_dev, int64_t n, int64_t k, int bits, int group, int mode,
+                                uint64_t seed, uint8_t* codes_dev, void* scales_dev, void* zeros_dev,
+                                int32_t* status_dev, sq_stream_t stream);
+
 /* ------------------------------------------------------------------------
  * a2 — bit packing (layouts L8/L4/L3 + tile placement T16 of DESIGN.md
  *   section 4; the paper is silent on packing; P:160 fixes bits/8 bytes

@@ -82,6 +82,8 @@ _sig("sq_abi_version", ctypes.c_int)
 _sig("sq_packed_bytes", ctypes.c_size_t, I64, I64, ctypes.c_int)
 _sig("sq_meta_bytes", ctypes.c_size_t, I64, I64, ctypes.c_int)
 _sig("sq_quantize_groups", ctypes.c_int, P, I64, I64, ctypes.c_int, ctypes.c_int, P, P, P, P)
+_sig("sq_quantize_groups_ex", ctypes.c_int, P, I64, I64, ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_uint64,
+     P, P, P, P, P)
 _sig("sq_pack", ctypes.c_int, P, P, P, I64, I64, ctypes.c_int, ctypes.c_int, P, P, P)
 _sig("sq_linear_workspace_bytes", ctypes.c_size_t, ctypes.POINTER(sq_qweight), I64)
 _sig("sq_linear_decode", ctypes.c_int, ctypes.POINTER(sq_qweight), P, I64, I64, P, I64, ctypes.c_int, P, P,
@@ -159,6 +161,25 @@ def sq_quantize_groups(w: torch.Tensor, bits: int, group: int = 128, stream=None
     return codes, s, z
 
 
+SQ_QUANT_SYMMETRIC, SQ_QUANT_STOCHASTIC = 1, 2
+
+
+def sq_quantize_groups_ex(w: torch.Tensor, bits: int, group: int = 128, mode: int = 0, seed: int = 0, stream=None):
+    """a1 variants (include/sq.h): mode = SQ_QUANT_SYMMETRIC | SQ_QUANT_STOCHASTIC (Theorem 1).
+    Raises if a symmetric group's zero point overflows fp16 (checked after a stream sync)."""
+    assert w.is_cuda and w.dtype == torch.float16 and w.is_contiguous()
+    n, k = w.shape
+    codes = torch.empty((n, k), dtype=torch.uint8, device=w.device)
+    s = torch.empty((n, k // group), dtype=torch.float16, device=w.device)
+    z = torch.empty_like(s)
+    status = torch.zeros(1, dtype=torch.int32, device=w.device) if mode & SQ_QUANT_SYMMETRIC else None
+    _check(_L.sq_quantize_groups_ex(_ptr(w), n, k, bits, group, mode, seed, _ptr(codes), _ptr(s), _ptr(z),
+                                    _ptr(status), _stream(stream)))
+    if status is not None and int(status.item()) != 0:
+        raise SQError(1, "sq_quantize_groups_ex: a symmetric zero point overflows fp16 (max|w| too close to 65504)")
+    return codes, s, z
+
+
 def sq_pack(codes: torch.Tensor, scales: torch.Tensor, zeros: torch.Tensor, bits: int, group: int = 128, stream=None):
     """a2: codes -> (packed u8 [n, k*bits/8] bytes in placement T16, meta int32 [n/16, k/128, 16] (u32 bits))."""
     n, k = codes.shape
@@ -180,11 +201,15 @@ class QLinear:
                             bias.data_ptr() if bias is not None else None)
 
     @classmethod
-    def from_fp16(cls, w: torch.Tensor, bits: int, bias: torch.Tensor | None = None, group: int = 128, stream=None):
+    def from_fp16(cls, w: torch.Tensor, bits: int, bias: torch.Tensor | None = None, group: int = 128, stream=None,
+                  mode: int = 0, seed: int = 0):
         n, k = w.shape
         if bits == 16:
             return cls(16, n, k, w.contiguous(), None, bias, group)
-        codes, s, z = sq_quantize_groups(w, bits, group, stream)
+        if mode:
+            codes, s, z = sq_quantize_groups_ex(w, bits, group, mode, seed, stream)
+        else:
+            codes, s, z = sq_quantize_groups(w, bits, group, stream)
         packed, meta = sq_pack(codes, s, z, bits, group, stream)
         return cls(bits, n, k, packed, meta, bias, group)
 

@@ -143,18 +143,28 @@ size_t sq_meta_bytes(int64_t n, int64_t k, int group) {
   return (size_t)(n * (k / group) * 4);
 }
 
-sq_status sq_quantize_groups(const void* w_dev, int64_t n, int64_t k, int bits, int group, uint8_t* codes_dev,
-                             void* scales_dev, void* zeros_dev, sq_stream_t stream) {
+sq_status sq_quantize_groups_ex(const void* w_dev, int64_t n, int64_t k, int bits, int group, int mode,
+                                uint64_t seed, uint8_t* codes_dev, void* scales_dev, void* zeros_dev,
+                                int32_t* status_dev, sq_stream_t stream) {
   if (!(bits == 3 || bits == 4 || bits == 8)) return fail(SQ_EINVAL, "sq_quantize_groups: bits=%d not in {3,4,8}", bits);
   if (!(group == 32 || group == 64 || group == 128))
     return fail(SQ_EINVAL, "sq_quantize_groups: group=%d not in {32,64,128}", group);
   if (n <= 0 || k <= 0 || k % group) return fail(SQ_EINVAL, "sq_quantize_groups: bad shape n=%lld k=%lld", (long long)n, (long long)k);
+  if (mode < 0 || mode > (SQ_QUANT_SYMMETRIC | SQ_QUANT_STOCHASTIC))
+    return fail(SQ_EINVAL, "sq_quantize_groups_ex: mode=%d", mode);
   if (!w_dev || !codes_dev || !scales_dev || !zeros_dev) return fail(SQ_EINVAL, "sq_quantize_groups: null pointer");
+  if ((mode & SQ_QUANT_SYMMETRIC) && !status_dev)
+    return fail(SQ_EINVAL, "sq_quantize_groups_ex: the symmetric mode needs status_dev");
   if ((reinterpret_cast<uintptr_t>(w_dev) & 7u) || (reinterpret_cast<uintptr_t>(codes_dev) & 3u))
     return fail(SQ_EINVAL, "sq_quantize_groups: w must be 8-B and codes 4-B aligned");
   return cuda_check(launch_quantize((const __half*)w_dev, n, k, bits, group, codes_dev, (__half*)scales_dev,
-                                    (__half*)zeros_dev, (cudaStream_t)stream),
+                                    (__half*)zeros_dev, mode, seed, (int*)status_dev, (cudaStream_t)stream),
                     "sq_quantize_groups");
+}
+
+sq_status sq_quantize_groups(const void* w_dev, int64_t n, int64_t k, int bits, int group, uint8_t* codes_dev,
+                             void* scales_dev, void* zeros_dev, sq_stream_t stream) {
+  return sq_quantize_groups_ex(w_dev, n, k, bits, group, 0, 0, codes_dev, scales_dev, zeros_dev, nullptr, stream);
 }
 
 sq_status sq_pack(const uint8_t* codes_dev, const void* scales_dev, const void* zeros_dev, int64_t n, int64_t k,

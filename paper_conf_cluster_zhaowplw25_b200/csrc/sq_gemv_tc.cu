@@ -403,6 +403,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       }
       if (tr) trace_ev(p, 2, i);
     }
+    // split panels keep their partials in the weight ring: an explicit CTA barrier with the epilogue
+    // (on top of the mbarrier chain dequant -> MMA -> d_full) orders this warp's last stage reads first
+    if (Z > 1 && p.cl) asm volatile("bar.arrive 2, %0;" :: "r"((DQ_WARPS + 4) * 32) : "memory");
   } else {
     // ---------------- epilogue warps: drain each item's accumulators
     const int sp = warp & 3;
@@ -414,6 +417,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       const int pn = it / Z, pp = tiles_of(pn);
       wait_bar(d_full, n_item & 1);
       tc_fence_after();
+      if (Z > 1 && p.cl) asm volatile("bar.sync 2, %0;" :: "r"((DQ_WARPS + 4) * 32) : "memory");
       for (int t = 0; t < pp; ++t) {
         float v[BT];
         {

@@ -25,7 +25,7 @@ void count_launch(int n = 1);
 
 // ---- kernel launchers (validated arguments) ----
 cudaError_t launch_quantize(const __half* w, int64_t n, int64_t k, int bits, int group, uint8_t* codes,
-                            __half* scales, __half* zeros, cudaStream_t s);
+                            __half* scales, __half* zeros, int mode, uint64_t seed, int* status, cudaStream_t s);
 cudaError_t launch_pack(const uint8_t* codes, const __half* scales, const __half* zeros, int64_t n, int64_t k,
                         int bits, int group, void* packed, uint32_t* meta, cudaStream_t s);
 cudaError_t launch_xsum(const __half* x, int64_t ldx, int64_t m, int64_t k, float2* xsum, cudaStream_t s);

@@ -7,14 +7,29 @@
 namespace sq {
 namespace {
 
+// splitmix64 output i of the stream seeded `seed` (finalizer of seed + (i + 1) * golden) and its top 24
+// bits as a uniform in [0, 1) -- the counter-based generator of the stochastic-rounding variant (R22).
+__device__ __forceinline__ float uniform24(uint64_t seed, uint64_t i) {
+  uint64_t z = seed + (i + 1) * 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  z ^= z >> 31;
+  return (float)(uint32_t)(z >> 40) * (1.0f / 16777216.0f);
+}
+
 // One warp per (row, group).  IEEE fp32 with one rounding per op, identical op
-// sequence to the CPU oracle's definition (R1-R6):
-//   mn, mx (canonical +0); s = fp16(fp32(mx - mn) / (2^b - 1)); z = mn;
-//   c = s == 0 ? 0 : clamp(rint_even(fp32(w - z) / s), 0, 2^b - 1)
-template <int G>
+// sequence to the CPU oracle's definition (R1-R6, R21, R22):
+//   mn, mx (canonical +0);
+//   asymmetric:  s = fp16(fp32(mx - mn) / (2^b - 1)); z = mn; d = fp32(w - z) / s; c in [0, 2^b - 1]
+//   symmetric:  s = fp16(max(|mx|, |mn|) / (2^(b-1) - 1)); z = -2^(b-1) s; d = w / s;
+//                       c = clamp(., -(2^(b-1) - 1), 2^(b-1) - 1) + 2^(b-1)
+//   rounding: rint_even(d), or stochastic floor(d) + [u < d - floor(d)] (Theorem 1)
+//   s == 0 -> d = 0.  A symmetric zero beyond the fp16 range sets *status (the oracle rejects it).
+template <int G, int MODE>
 __global__ void __launch_bounds__(256) k_quantize(const __half* __restrict__ w, int64_t n, int64_t k, int bits,
                                                   uint8_t* __restrict__ codes, __half* __restrict__ scales,
-                                                  __half* __restrict__ zeros) {
+                                                  __half* __restrict__ zeros, uint64_t seed, int* status) {
+  constexpr bool SYM = MODE & SQ_QUANT_SYMMETRIC, STOCH = MODE & SQ_QUANT_STOCHASTIC;
   constexpr int PER = G / 32;  // elements per lane: 4, 2, 1
   const int64_t ng = k / G;
   const int64_t gid = (int64_t)blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5);
@@ -43,25 +58,37 @@ __global__ void __launch_bounds__(256) k_quantize(const __half* __restrict__ w, 
   }
   mn = __fadd_rn(mn, 0.0f);  // canonical zeros: -0 -> +0
   mx = __fadd_rn(mx, 0.0f);
+  const int half_i = 1 << (bits - 1);
   const float qmax = (float)((1 << bits) - 1);
-  const float sf = __fdiv_rn(__fsub_rn(mx, mn), qmax);
+  const float sf = SYM ? __fdiv_rn(fmaxf(fabsf(mx), fabsf(mn)), (float)(half_i - 1)) : __fdiv_rn(__fsub_rn(mx, mn), qmax);
   const __half s16 = __float2half_rn(sf);
   const float s = __half2float(s16);
+  float z = mn;
+  if constexpr (SYM) {
+    z = __fadd_rn(__fmul_rn(-(float)half_i, s), 0.0f);  // exact; +0 when s == 0
+    if (fabsf(z) > 65504.f && lane == 0) atomicOr(status, 1);
+  }
   if (lane == 0) {
     scales[r * ng + g] = s16;
-    zeros[r * ng + g] = __float2half_rn(mn);
+    zeros[r * ng + g] = __float2half_rn(z);
   }
+  const float cmin = SYM ? -(float)(half_i - 1) : 0.0f, cmax = SYM ? (float)(half_i - 1) : qmax;
+  const float off = SYM ? (float)half_i : 0.0f;
   uint32_t packed = 0;
 #pragma unroll
   for (int i = 0; i < PER; ++i) {
-    uint32_t c = 0;
-    if (s != 0.0f) {
-      float d = __fdiv_rn(__fsub_rn(v[i], mn), s);
-      float q = rintf(d);
-      q = fminf(fmaxf(q, 0.0f), qmax);
-      c = (uint32_t)q;
+    float d = 0.0f;
+    if (s != 0.0f) d = SYM ? __fdiv_rn(v[i], s) : __fdiv_rn(__fsub_rn(v[i], mn), s);
+    float q;
+    if constexpr (STOCH) {
+      const float fl = floorf(d);
+      const float fr = __fsub_rn(d, fl);
+      q = fl + (uniform24(seed, (uint64_t)(r * k + g * G + lane * PER + i)) < fr ? 1.0f : 0.0f);
+    } else {
+      q = rintf(d);
     }
-    packed |= c << (8 * i);
+    q = fminf(fmaxf(q, cmin), cmax);
+    packed |= (uint32_t)(int)(q + off) << (8 * i);
   }
   uint8_t* cp = codes + r * k + g * G + lane * PER;
   if constexpr (PER == 4) *reinterpret_cast<uint32_t*>(cp) = packed;
@@ -139,15 +166,26 @@ inline unsigned blocks_for(int64_t n, int t) { return (unsigned)((n + t - 1) / t
 
 }  // namespace
 
+template <int G>
+void launch_quantize_g(dim3 grid, dim3 block, cudaStream_t s, const __half* w, int64_t n, int64_t k, int bits,
+                       uint8_t* codes, __half* scales, __half* zeros, int mode, uint64_t seed, int* status) {
+  switch (mode) {
+    case 0: k_quantize<G, 0><<<grid, block, 0, s>>>(w, n, k, bits, codes, scales, zeros, seed, status); break;
+    case 1: k_quantize<G, 1><<<grid, block, 0, s>>>(w, n, k, bits, codes, scales, zeros, seed, status); break;
+    case 2: k_quantize<G, 2><<<grid, block, 0, s>>>(w, n, k, bits, codes, scales, zeros, seed, status); break;
+    default: k_quantize<G, 3><<<grid, block, 0, s>>>(w, n, k, bits, codes, scales, zeros, seed, status); break;
+  }
+}
+
 cudaError_t launch_quantize(const __half* w, int64_t n, int64_t k, int bits, int group, uint8_t* codes,
-                            __half* scales, __half* zeros, cudaStream_t s) {
+                            __half* scales, __half* zeros, int mode, uint64_t seed, int* status, cudaStream_t s) {
   const int64_t groups = n * (k / group);
   dim3 grid(blocks_for(groups, 8)), block(256);
   auto t = prof_begin(KC_QUANT, (double)n * k * 3 + groups * 4.0, 0, s);
   switch (group) {
-    case 128: k_quantize<128><<<grid, block, 0, s>>>(w, n, k, bits, codes, scales, zeros); break;
-    case 64: k_quantize<64><<<grid, block, 0, s>>>(w, n, k, bits, codes, scales, zeros); break;
-    default: k_quantize<32><<<grid, block, 0, s>>>(w, n, k, bits, codes, scales, zeros); break;
+    case 128: launch_quantize_g<128>(grid, block, s, w, n, k, bits, codes, scales, zeros, mode, seed, status); break;
+    case 64: launch_quantize_g<64>(grid, block, s, w, n, k, bits, codes, scales, zeros, mode, seed, status); break;
+    default: launch_quantize_g<32>(grid, block, s, w, n, k, bits, codes, scales, zeros, mode, seed, status); break;
   }
   prof_end(t, s);
   count_launch();

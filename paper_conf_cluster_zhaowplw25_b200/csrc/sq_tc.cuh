@@ -62,8 +62,9 @@ constexpr uint32_t make_idesc(int M, int N) {
 }
 
 // w~ = s*c + z in one fp16 FMA (c exact after the magic-number subtraction).  SAT: saturate at the fp16
-// maximum (reading R20) -- only a group with s*(2^b - 1) + z >= 65520 can overflow to +inf, and such
-// groups take this variant (one extra HMNMX2 per pair); q = group min keeps the bottom finite.
+// maximum (reading R20) -- only a group with s*(2^b - 1) + z >= 65520 can overflow to +inf, and a warp
+// holding such a group takes this variant (one extra HMNMX2 per pair; saturation is the identity on
+// the other lanes' finite values); q = group min keeps the bottom finite.
 template <bool SAT = false>
 __device__ __forceinline__ uint32_t hsub_fma(uint32_t h, uint32_t off2, uint32_t s2, uint32_t z2) {
   __half2 c = __hsub2(*reinterpret_cast<__half2*>(&h), *reinterpret_cast<__half2*>(&off2));
@@ -179,7 +180,8 @@ __device__ __forceinline__ void dequant_row_batches(const uint8_t* wst, uint32_t
   if constexpr (BITS == 16) {
     dequant_row_batches_<BITS, NB, false>(wst, meta, r, taddr, row_off, B0);
   } else {
-    if (__builtin_expect(group_may_overflow<BITS>(meta), 0))
+    // warp-uniform choice: tcgen05.st is .sync.aligned, so every lane of the warp must take the same path
+    if (__builtin_expect(__any_sync(0xffffffffu, group_may_overflow<BITS>(meta)), 0))
       dequant_row_batches_<BITS, NB, true>(wst, meta, r, taddr, row_off, B0);
     else
       dequant_row_batches_<BITS, NB, false>(wst, meta, r, taddr, row_off, B0);

@@ -191,3 +191,69 @@ def test_indicator_symmetric_scale():
     _, s, _ = O.quantize_groups_ex(w, 4, 128, SYM)
     assert O.scale_sq_sum(w, 4, 128, SYM) == pytest.approx(float((128 * s.astype(np.float64) ** 2).sum()), rel=1e-15)
     assert O.scale_sq_sum(w, 4, 128, SYM) > O.scale_sq_sum(w, 4, 128)  # symmetric grids are coarser
+
+
+# ---------------------------------------------------------------- GPU: bit-exact with the oracle
+def _sq():
+    import paper_conf_cluster_zhaowplw25_b200 as sq
+    return sq
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("mode", [SYM, STO, SYM | STO])
+@pytest.mark.parametrize("bits", [3, 4, 8])
+@pytest.mark.parametrize("group", [128, 64, 32])
+def test_gpu_variants_bit_exact(mode, bits, group):
+    import torch
+    sq = _sq()
+    w = synth.adversarial_weight_f16(70 + bits, 64, 512)
+    if mode & SYM:  # keep every symmetric zero point inside fp16 (the overflow case is tested below)
+        w = (w.astype(np.float32) * np.float32(0.5)).astype(np.float16)
+    codes, s, z = O.quantize_groups_ex(w, bits, group, mode, seed=1234 + bits)
+    gc, gs, gz = sq.sq_quantize_groups_ex(torch.from_numpy(w).cuda(), bits, group, mode, 1234 + bits)
+    assert np.array_equal(gc.cpu().numpy(), codes)
+    assert np.array_equal(gs.cpu().numpy().view(np.uint16), s.view(np.uint16))
+    assert np.array_equal(gz.cpu().numpy().view(np.uint16), z.view(np.uint16))
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("mode", [SYM, STO])
+def test_gpu_variants_bit_exact_opt13b_and_linear(mode):
+    # full OPT-13B 5120 x 5120 (device-generated, same generator); then a decode and a prefill linear
+    # on the variant-quantized weight vs the oracle's (the stored form is the same (code, s, z))
+    import torch
+    sq = _sq()
+    n = k = 5120
+    seed = synth.weight_seed(0, "o")
+    wd = torch.empty((n, k), dtype=torch.float16, device="cuda")
+    synth.device_weight_f16(wd.data_ptr(), seed, n, k)
+    w = synth.weight_f16(seed, n, k)
+    codes, s, z = O.quantize_groups_ex(w, 4, 128, mode, seed=99)
+    gc, gs, gz = sq.sq_quantize_groups_ex(wd, 4, 128, mode, 99)
+    assert np.array_equal(gc.cpu().numpy(), codes)
+    assert np.array_equal(gs.cpu().numpy().view(np.uint16), s.view(np.uint16))
+    rows = np.arange(0, n, 40)
+    qg = sq.QLinear.from_fp16(wd, 4, mode=mode, seed=99)
+    packed, meta = O.pack(codes, s, z, 4)
+    assert np.array_equal(qg.packed.cpu().numpy(), packed)
+    x = synth.act_f16(5, 8, k)
+    y = torch.empty((8, n), dtype=torch.float16, device="cuda")
+    sq.sq_linear_decode(qg, torch.from_numpy(x).cuda(), y, 0)
+    torch.cuda.synchronize()
+    # y = x (s c + z)^T on sampled rows from the oracle's codes (O4/O5 written out in fp64)
+    ref = x.astype(np.float64) @ (codes[rows].astype(np.float64) * s[rows].astype(np.float64).repeat(128, 1)
+                                  + z[rows].astype(np.float64).repeat(128, 1)).T
+    yy = y.float().cpu().numpy()[:, rows]
+    assert np.abs(yy - ref).max() / np.abs(ref).max() <= 2e-3
+
+
+@pytest.mark.gpu
+def test_gpu_symmetric_overflow_flag():
+    import torch
+    sq = _sq()
+    w = np.zeros((16, 128), np.float16)
+    w[3, 9] = np.float16(60000.0)
+    with pytest.raises(RuntimeError):
+        O.quantize_groups_ex(w, 4, 128, SYM)
+    with pytest.raises(sq.SQError):
+        sq.sq_quantize_groups_ex(torch.from_numpy(w).cuda(), 4, 128, SYM)
