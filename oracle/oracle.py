@@ -57,6 +57,8 @@ def _lib() -> ctypes.CDLL:
         L.oq_stage.argtypes = [P, ctypes.c_int, P, I64, I64, P]
         L.oq_packed_bytes.argtypes = [I64, I64, ctypes.c_int]
         L.oq_packed_bytes.restype = ctypes.c_size_t
+        L.oq_attention.argtypes = [P, I64, I64, I64, I64, I64, ctypes.c_int, P, P, I64, P]
+        L.oq_stage_attn.argtypes = [P, ctypes.c_int, P, I64, I64, I64, I64, I64, ctypes.c_int, I64, I64, P, P]
         L.oq_set_threads.argtypes = [ctypes.c_int]
         L.oq_set_threads.restype = None
         L.oq_max_threads.restype = ctypes.c_int
@@ -267,4 +269,54 @@ def pipeline(layers: list[Layer], x0: np.ndarray, n_decode: int) -> np.ndarray:
         e = layernorm(out[:, t - 1])
         h, _ = stage(layers, e)
         out[:, t] = h
+    return out
+
+
+# ---------------------------------------------------------------- O8: attention + KV cache (f3)
+class KVCache:
+    """Oracle-side KV cache of a stage: k, v fp64 [n_layers][B][max_len][h1] (P:162 sizing)."""
+
+    def __init__(self, n_layers: int, B: int, max_len: int, h1: int):
+        self.k = np.zeros((n_layers, B, max_len, h1), np.float64)
+        self.v = np.zeros_like(self.k)
+        self.B, self.max_len, self.h1 = B, max_len, h1
+
+
+def attention(qkv: np.ndarray, nseq: int, length: int, pos0: int, seq0: int, n_heads: int,
+              kc: np.ndarray, vc: np.ndarray) -> np.ndarray:
+    """O8 for one layer: qkv fp64 [nseq*length, 3*h1] (rows = (sequence, position)); kc/vc one layer's
+    cache [B][max_len][h1], updated in place.  Returns the attention output [nseq*length, h1]."""
+    qkv = np.ascontiguousarray(qkv, np.float64)
+    h1 = qkv.shape[1] // 3
+    assert kc.flags.c_contiguous and vc.flags.c_contiguous and kc.dtype == np.float64
+    out = np.empty((nseq * length, h1), np.float64)
+    _check(_lib().oq_attention(_p(qkv), nseq, length, pos0, seq0, h1, n_heads, _p(kc), _p(vc), kc.shape[1], _p(out)),
+           "attention")
+    return out
+
+
+def stage_attn(layers: list[Layer], x: np.ndarray, nseq: int, length: int, pos0: int, seq0: int, n_heads: int,
+               cache: KVCache) -> np.ndarray:
+    """O6 with O8: run the stage's layers on x [nseq*length, h1] (rows = (sequence, position))."""
+    x = np.array(x, dtype=np.float64, order="C", copy=True)
+    h1 = x.shape[1]
+    arr = (_OqLayer * len(layers))(*[L.c_struct() for L in layers])
+    _check(_lib().oq_stage_attn(arr, len(layers), _p(x), nseq, length, pos0, seq0, h1, n_heads, cache.B,
+                                cache.max_len, _p(cache.k), _p(cache.v)), "stage_attn")
+    return x
+
+
+def pipeline_attn(layers: list[Layer], x0: np.ndarray, n_decode: int, n_heads: int) -> np.ndarray:
+    """O7 with attention: every sequence's whole prompt through all layers (positions 0..s-1 fill the
+    cache), out[b, 0] = hidden at the last prompt position, then n_decode steps at positions s + t - 1
+    with e_1 = LN(out[b, 0]), e_{t+1} = LN(out[b, t]) (R14).  Sequences are independent, so micro-batch
+    sizes, chunking and the stage partition cannot change the exact result.  -> [B, 1 + n_decode, h1]."""
+    B, s, h1 = x0.shape
+    cache = KVCache(len(layers), B, s + n_decode, h1)
+    out = np.empty((B, 1 + n_decode, h1), np.float64)
+    h = stage_attn(layers, np.asarray(x0, np.float64).reshape(B * s, h1), B, s, 0, 0, n_heads, cache)
+    out[:, 0] = h.reshape(B, s, h1)[:, -1]
+    for t in range(1, n_decode + 1):
+        e = layernorm(out[:, t - 1])
+        out[:, t] = stage_attn(layers, e, B, 1, s + t - 1, 0, n_heads, cache)
     return out

@@ -369,3 +369,91 @@ int oq_stage(const oq_layer* layers, int n_layers, double* x, int64_t t, int64_t
   free(u);
   return err;
 }
+
+/* ---------------- O8: causal multi-head self-attention with a KV cache ----------------
+ * Readings R23-R25: h1 = n_heads * dh; the fused qkv row holds q = [0, h1), k = [h1, 2h1),
+ * v = [2h1, 3h1) (R11), head j = columns j*dh .. (j+1)*dh - 1; scores q.k / sqrt(dh), causal within
+ * a sequence (query at position p sees cache positions 0..p), softmax, no positional term inside the
+ * layer; the KV cache of a layer holds k, v per (sequence, position): [B][max_len][h1] (P:162 sizes it
+ * 2 v (s + n) h1 elements).
+ * One call = one micro-batch of nseq sequences (cache rows seq0 .. seq0 + nseq - 1), each with `len`
+ * new tokens at positions pos0 .. pos0 + len - 1 (prefill chunk: pos0 = chunk start; decode: len = 1,
+ * pos0 = s + t - 1).  Row i*len + (p - pos0) of qkv/out is (sequence i, position p).  The new k, v rows
+ * are written into the cache first, then every query attends over cache positions 0..p.  fp64.
+ */
+int oq_attention(const double* qkv, int64_t nseq, int64_t len, int64_t pos0, int64_t seq0, int64_t h1,
+                 int n_heads, double* kc, double* vc, int64_t max_len, double* out) {
+  if (n_heads <= 0 || h1 % n_heads || pos0 < 0 || pos0 + len > max_len) return 1;
+  const int64_t dh = h1 / n_heads;
+  const double scale = 1.0 / sqrt((double)dh);
+  for (int64_t i = 0; i < nseq; ++i)
+    for (int64_t p = pos0; p < pos0 + len; ++p) {
+      const double* row = qkv + (i * len + (p - pos0)) * 3 * h1;
+      double* kd = kc + ((seq0 + i) * max_len + p) * h1;
+      double* vd = vc + ((seq0 + i) * max_len + p) * h1;
+      for (int64_t c = 0; c < h1; ++c) { kd[c] = row[h1 + c]; vd[c] = row[2 * h1 + c]; }
+    }
+  double* w = (double*)malloc((size_t)max_len * sizeof(double));
+  if (!w) return 2;
+  for (int64_t i = 0; i < nseq; ++i)
+    for (int64_t p = pos0; p < pos0 + len; ++p) {
+      const double* q = qkv + (i * len + (p - pos0)) * 3 * h1;
+      double* o = out + (i * len + (p - pos0)) * h1;
+      for (int hd = 0; hd < n_heads; ++hd) {
+        double mx = -INFINITY;
+        for (int64_t j = 0; j <= p; ++j) {
+          const double* kj = kc + ((seq0 + i) * max_len + j) * h1 + hd * dh;
+          double sc = 0.0;
+          for (int64_t c = 0; c < dh; ++c) sc += q[hd * dh + c] * kj[c];
+          w[j] = sc * scale;
+          if (w[j] > mx) mx = w[j];
+        }
+        double den = 0.0;
+        for (int64_t j = 0; j <= p; ++j) { w[j] = exp(w[j] - mx); den += w[j]; }
+        for (int64_t c = 0; c < dh; ++c) {
+          double acc = 0.0;
+          for (int64_t j = 0; j <= p; ++j) acc += w[j] * vc[((seq0 + i) * max_len + j) * h1 + hd * dh + c];
+          o[hd * dh + c] = acc / den;
+        }
+      }
+    }
+  free(w);
+  return 0;
+}
+
+/* One stage with real attention (O6 with O8 in place of the R12 stub): for each layer l,
+ *   a = LN(x); [q k v] = a Wqkv^T (+b); att = O8(q, k, v; cache of layer l); h = x + att Wo^T (+b);
+ *   u = act(LN(h) W1^T + b1); x = h + u W2^T (+b2).
+ * kc_all / vc_all: [n_layers][B][max_len][h1] fp64 (this stage's layers). */
+int oq_stage_attn(const oq_layer* layers, int n_layers, double* x, int64_t nseq, int64_t len, int64_t pos0,
+                  int64_t seq0, int64_t h1, int n_heads, int64_t B, int64_t max_len, double* kc_all,
+                  double* vc_all) {
+  const int64_t t = nseq * len;
+  const int64_t h2 = layers[0].fc1.n;
+  double* a = (double*)malloc((size_t)(t * h1) * sizeof(double));
+  double* qkv = (double*)malloc((size_t)(t * 3 * h1) * sizeof(double));
+  double* att = (double*)malloc((size_t)(t * h1) * sizeof(double));
+  double* o = (double*)malloc((size_t)(t * h1) * sizeof(double));
+  double* u = (double*)malloc((size_t)(t * h2) * sizeof(double));
+  int err = (!a || !qkv || !att || !o || !u) ? 2 : 0;
+  const size_t cl = (size_t)(B * max_len * h1);
+  for (int l = 0; l < n_layers && !err; ++l) {
+    const oq_layer* L = &layers[l];
+    oq_layernorm(x, t, h1, 1e-5, a);
+    err |= oq_linear(a, t, h1, L->qkv.packed, L->qkv.meta, 3 * h1, L->qkv.bits, L->qkv.group, L->qkv.bias, qkv);
+    err |= oq_attention(qkv, nseq, len, pos0, seq0, h1, n_heads, kc_all + l * cl, vc_all + l * cl, max_len, att);
+    err |= oq_linear(att, t, h1, L->o.packed, L->o.meta, h1, L->o.bits, L->o.group, L->o.bias, o);
+    for (int64_t i = 0; i < t * h1; ++i) x[i] += o[i];
+    oq_layernorm(x, t, h1, 1e-5, a);
+    err |= oq_linear(a, t, h1, L->fc1.packed, L->fc1.meta, h2, L->fc1.bits, L->fc1.group, L->fc1.bias, u);
+    for (int64_t i = 0; i < t * h2; ++i) u[i] = act_fn(u[i], L->act);
+    err |= oq_linear(u, t, h2, L->fc2.packed, L->fc2.meta, h1, L->fc2.bits, L->fc2.group, L->fc2.bias, o);
+    for (int64_t i = 0; i < t * h1; ++i) x[i] += o[i];
+  }
+  free(a);
+  free(qkv);
+  free(att);
+  free(o);
+  free(u);
+  return err;
+}
