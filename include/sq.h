@@ -45,7 +45,7 @@ typedef enum {
 
 const char* sq_last_error(void);
 const char* sq_version(void);
-int sq_abi_version(void); /* bumped on any incompatible change of this header */
+int sq_abi_version(void); /* bumped on any incompatible change of this header (2: sq_plan.n_heads/kappa) */
 
 /* ------------------------------------------------------------------------
  * Sizes.  P:160: a decoder layer with precision `bit` stores
@@ -202,6 +202,44 @@ sq_status sq_stage_forward(const sq_layer* layers, int n_layers, int phase, cons
                            int64_t tokens, float* x_out_dev, void* qkv_dbg_dev, void* ws_dev,
                            size_t ws_bytes, sq_stream_t stream);
 
+/* ------------------------------------------------------------------------
+ * f3 — causal multi-head self-attention over a per-layer KV cache (DESIGN.md
+ *   R23-R25; cache sized 2 v (s + n) h1 elements per layer; chunked prefill kappa).
+ *   Head j uses columns [j*dh, (j+1)*dh) of q = qkv[:, 0:h1], k = qkv[:, h1:2h1], v = qkv[:, 2h1:3h1]
+ *   (dh = h1 / n_heads in {64, 128}); scores q.k / sqrt(dh); the query at position p attends over
+ *   cache positions 0..p of its own sequence; no positional term inside the layer (R24).
+ *   The KV cache of one layer is K, V fp16 [n_seq_cache][max_len][h1] each (caller-owned, device).
+ * ------------------------------------------------------------------------ */
+
+/* One layer, one micro-batch: nseq sequences (cache rows seq0..seq0+nseq-1), each with `len` new
+ * tokens at positions pos0..pos0+len-1; qkv row i*len + (p - pos0) is (sequence i, position p).
+ * Appends the new k, v rows to the cache, then writes the attention output fp16 [nseq*len, h1]
+ * (row stride ld_out) -- len == 1: the HBM-bound decode kernel, else the prefill kernel.
+ * qkv_dev / caches / out_dev 16-B aligned, ld_qkv >= 3*h1 and ld_out >= h1 multiples of 8. */
+sq_status sq_attention(const void* qkv_dev, int64_t ld_qkv, int64_t nseq, int64_t len, int64_t pos0,
+                       int64_t seq0, int64_t h1, int n_heads, void* k_cache_dev, void* v_cache_dev,
+                       int64_t max_len, int64_t n_seq_cache, void* out_dev, int64_t ld_out,
+                       sq_stream_t stream);
+
+typedef struct {            /* attention context of one stage call (host memory) */
+  int32_t n_heads;          /* h1 / head_dim, head_dim in {64, 128} */
+  int32_t max_len;          /* cache positions per sequence (>= s + n_decode) */
+  int64_t n_seq_cache;      /* sequences each layer's cache holds */
+  void* const* k_cache;     /* [n_layers] device pointers: layer l's K cache fp16 [n_seq_cache][max_len][h1] */
+  void* const* v_cache;     /* [n_layers] device pointers: layer l's V cache */
+  int64_t seq0;             /* cache row of the micro-batch's first sequence */
+  int32_t nseq, seq_len;    /* tokens = nseq * seq_len (decode: seq_len = 1) */
+  int32_t pos0;             /* position of each sequence's first token in this call */
+} sq_attn;
+
+/* a5 with real attention in place of the R12 stub:
+ *   a = LN(x); [q k v] = a Wqkv^T (+b); att = attention(q, k, v; cache) (sq_attention);
+ *   h = x + att Wo^T (+b); u = act(LN(h) W1^T + b1); x = h + u W2^T (+b2).
+ * Same workspace rules as sq_stage_forward (sq_stage_workspace_bytes covers both). */
+sq_status sq_stage_forward_attn(const sq_layer* layers, int n_layers, int phase, const sq_attn* attn,
+                                const float* x_in_dev, int64_t tokens, float* x_out_dev, void* ws_dev,
+                                size_t ws_bytes, sq_stream_t stream);
+
 /* Loop-back glue (R14): out_row = x (fp32 copy) and e = LN(x) for the next decode step. */
 sq_status sq_layernorm_f32(const float* x_dev, int64_t rows, int64_t d, float* y_dev,
                            sq_stream_t stream);
@@ -234,6 +272,11 @@ typedef struct {            /* host memory, identical on every rank */
   int32_t eta, xi;          /* prefill / decode micro-batch sizes (sequences) */
   int32_t prompt_len;       /* s */
   int32_t n_decode;         /* decode steps after the prefill token (R14) */
+  int32_t n_heads;          /* 0: attention stub out = v (R12); > 0: real attention (f3) with a KV
+                               cache of 2 x B x (s + n_decode) x h1 fp16 per layer inside the
+                               pipeline workspace */
+  int32_t kappa;            /* prefill chunks per prompt (0 or 1 = whole prompt); s % kappa == 0;
+                               needs n_heads > 0 when > 1 */
 } sq_plan;
 
 typedef struct {
@@ -256,7 +299,8 @@ sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers,
 sq_status sq_plan_check(const sq_plan* plan);
 
 /* Host-only: the exact op sequence `rank` executes inside sq_pipeline_run (rank -1, or a
- * 1-stage plan: the single-process order).  Items: prefill m = 0..mu_pre-1, then decode
+ * 1-stage plan: the single-process order).  Items: prefill (m, c) for m = 0..mu_pre-1 and chunk
+ * c = 0..kappa-1 (only the last chunk produces OUT / loop-back ops), then decode
  * t = 1..n_decode, m = 0..mu_dec-1 (R13/R14).  Send/recv ops name the peer's global rank;
  * the sequence of SEND ops of rank j to j+1 equals, op for op and size for size, the
  * sequence of RECV ops of rank j+1 from j (tests/test_pipeline_schedule.py).  Returns the

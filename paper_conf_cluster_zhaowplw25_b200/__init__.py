@@ -48,7 +48,12 @@ class sq_layer(ctypes.Structure):
 class sq_plan(ctypes.Structure):
     _fields_ = [("n_layers", I32), ("n_stages", I32), ("hidden", I32), ("ffn", I32), ("group", I32),
                 ("bits", ctypes.POINTER(I32)), ("stage_of_layer", ctypes.POINTER(I32)), ("B", I32), ("eta", I32),
-                ("xi", I32), ("prompt_len", I32), ("n_decode", I32)]
+                ("xi", I32), ("prompt_len", I32), ("n_decode", I32), ("n_heads", I32), ("kappa", I32)]
+
+
+class sq_attn(ctypes.Structure):
+    _fields_ = [("n_heads", I32), ("max_len", I32), ("n_seq_cache", I64), ("k_cache", ctypes.POINTER(P)),
+                ("v_cache", ctypes.POINTER(P)), ("seq0", I64), ("nseq", I32), ("seq_len", I32), ("pos0", I32)]
 
 
 class sq_run_stats(ctypes.Structure):
@@ -101,7 +106,8 @@ EXPORTED = [
     "sq_comm_get_unique_id", "sq_comm_init", "sq_comm_init_local", "sq_comm_destroy",
     "sq_pipeline_workspace_bytes", "sq_pipeline_run", "sq_plan_check", "sq_profile_enable", "sq_profile_read",
     "sq_launch_count", "sq_pipeline_schedule", "sq_scale_sq_sums_workspace_bytes", "sq_scale_sq_sums",
-    "sq_act_moments_workspace_bytes", "sq_act_moments",
+    "sq_act_moments_workspace_bytes", "sq_act_moments", "sq_quantize_groups_ex", "sq_attention",
+    "sq_stage_forward_attn",
 ]
 
 
@@ -114,6 +120,9 @@ _opt("sq_stage_workspace_bytes", ctypes.c_size_t, ctypes.POINTER(sq_layer), ctyp
 _opt("sq_stage_forward", ctypes.c_int, ctypes.POINTER(sq_layer), ctypes.c_int, ctypes.c_int, P, I64, P, P, P,
      ctypes.c_size_t, P)
 _opt("sq_layernorm_f32", ctypes.c_int, P, I64, I64, P, P)
+_opt("sq_attention", ctypes.c_int, P, I64, I64, I64, I64, I64, I64, ctypes.c_int, P, P, I64, I64, P, I64, P)
+_opt("sq_stage_forward_attn", ctypes.c_int, ctypes.POINTER(sq_layer), ctypes.c_int, ctypes.c_int,
+     ctypes.POINTER(sq_attn), P, I64, P, P, ctypes.c_size_t, P)
 _opt("sq_comm_unique_id_bytes", ctypes.c_size_t)
 _opt("sq_comm_get_unique_id", ctypes.c_int, P)
 _opt("sq_comm_init", ctypes.c_int, ctypes.POINTER(P), P, ctypes.c_int, ctypes.c_int)
@@ -289,3 +298,16 @@ def sq_launch_count() -> int:
 
 
 from . import runtime  # noqa: E402,F401  (stage / pipeline wrappers)
+
+
+# ---------------------------------------------------------------- f3: attention + KV cache
+def sq_attention(qkv: torch.Tensor, nseq: int, length: int, pos0: int, seq0: int, n_heads: int,
+                 k_cache: torch.Tensor, v_cache: torch.Tensor, out: torch.Tensor, stream=None) -> torch.Tensor:
+    """One layer's causal attention over its KV cache (include/sq.h sq_attention).  qkv fp16
+    [nseq*length, 3*h1] rows (sequence, position); caches fp16 [n_seq_cache, max_len, h1]; out fp16
+    [nseq*length, h1].  Appends the new k, v to the caches."""
+    h1 = qkv.shape[1] // 3
+    assert k_cache.shape == v_cache.shape and k_cache.shape[2] == h1
+    _check(_L.sq_attention(_ptr(qkv), qkv.stride(0), nseq, length, pos0, seq0, h1, n_heads, _ptr(k_cache),
+                           _ptr(v_cache), k_cache.shape[1], k_cache.shape[0], _ptr(out), out.stride(0), _stream(stream)))
+    return out

@@ -53,8 +53,15 @@ cudaError_t launch_copy_rows(const float* src, int64_t sstride, int64_t rows, in
 // ---- stage forward (sq_stage.cu), used by the pipeline runner ----
 size_t stage_workspace_bytes(const sq_layer* layers, int n_layers, int64_t max_tokens);
 sq_status stage_forward(const sq_layer* layers, int n_layers, int phase, const float* x_in, int64_t tokens,
-                        float* x_out, void* qkv_dbg, void* ws, size_t ws_bytes, cudaStream_t s);
+                        float* x_out, void* qkv_dbg, void* ws, size_t ws_bytes, cudaStream_t s,
+                        const sq_attn* att = nullptr);
 sq_status check_layers(const sq_layer* layers, int n_layers, const char* who);
+sq_status check_attn(const sq_attn* a, const sq_layer* layers, int n_layers, int phase, int64_t tokens, const char* who);
+
+// ---- attention (sq_attn.cu): kv_append + prefill / decode attention for one layer
+cudaError_t launch_attention(const __half* qkv, int64_t ldq, int nseq, int len, int pos0, int64_t seq0, int h1,
+                             int n_heads, __half* kc, __half* vc, int max_len, __half* out, int64_t ldo,
+                             cudaStream_t s);
 
 int num_sms();
 

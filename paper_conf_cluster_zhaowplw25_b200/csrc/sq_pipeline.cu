@@ -43,6 +43,7 @@ sq_status nccl_check(ncclResult_t r, const char* what) {
 struct PlanView {
   int L, P, h1, h2, B, eta, xi, s, n_dec;
   int mu_pre, mu_dec;
+  int heads, kappa, len_pre, max_len;  // attention (f3): heads 0 = stub; prefill chunk = s / kappa tokens
   std::vector<int> first_layer;  // [P+1]
 };
 
@@ -52,6 +53,10 @@ PlanView view(const sq_plan& pl) {
   v.eta = pl.eta; v.xi = pl.xi; v.s = pl.prompt_len; v.n_dec = pl.n_decode;
   v.mu_pre = (pl.B + pl.eta - 1) / pl.eta;
   v.mu_dec = (pl.B + pl.xi - 1) / pl.xi;
+  v.heads = pl.n_heads;
+  v.kappa = pl.kappa > 1 ? pl.kappa : 1;
+  v.len_pre = pl.prompt_len / v.kappa;
+  v.max_len = pl.prompt_len + pl.n_decode;
   v.first_layer.assign(v.P + 1, v.L);
   for (int l = v.L - 1; l >= 0; --l) v.first_layer[pl.stage_of_layer[l]] = l;
   v.first_layer[v.P] = v.L;
@@ -59,19 +64,22 @@ PlanView view(const sq_plan& pl) {
 }
 
 struct Ws {
-  size_t stage, act, decin, lb, total;
+  size_t stage, act, decin, lb, kv, kv_layer, total;
 };
 
 Ws ws_layout(const PlanView& v, const sq_layer* layers, int n_layers, int rank) {
   Ws w{};
   size_t off = 0;
   auto al = [](size_t x) { return (x + 255) / 256 * 256; };
-  const int64_t tmax = std::max<int64_t>((int64_t)v.eta * v.s, v.xi);
+  const int64_t tmax = std::max<int64_t>((int64_t)v.eta * v.len_pre, v.xi);
   w.stage = off; off += al(stage_workspace_bytes(layers, n_layers, tmax));
   w.act = off;   off += 2 * al((size_t)tmax * v.h1 * 4);
   const bool first = rank <= 0, last = rank < 0 || rank == v.P - 1;
   w.decin = off; if (first) off += al((size_t)v.B * v.h1 * 4);
   w.lb = off;    if (last) off += 2 * al((size_t)std::max(v.eta, v.xi) * v.h1 * 4);
+  // KV cache of this rank's layers (f3): K and V fp16 [B][s + n_decode][h1] per layer
+  w.kv_layer = v.heads > 0 ? al((size_t)v.B * v.max_len * v.h1 * 2) : 0;
+  w.kv = off;    off += (size_t)n_layers * 2 * w.kv_layer;
   w.total = off;
   return w;
 }
@@ -91,14 +99,16 @@ std::vector<sq_sched_op> make_schedule(const PlanView& v, int rank) {
   // then decode (t, m) for t = 1..n_dec-1 (the last step's successor input is never used)
   const int n_lb = v.mu_pre + std::max(0, v.n_dec - 1) * v.mu_dec;
   int lb_posted = 0;
-  const int total = v.mu_pre + v.n_dec * v.mu_dec;
+  const int n_pre = v.mu_pre * v.kappa;  // prefill items: (micro-batch m, chunk c)
+  const int total = n_pre + v.n_dec * v.mu_dec;
   for (int it = 0; it < total; ++it) {
-    const bool pre = it < v.mu_pre;
-    const int m = pre ? it : (it - v.mu_pre) % v.mu_dec;
-    const int t = pre ? 0 : 1 + (it - v.mu_pre) / v.mu_dec;
+    const bool pre = it < n_pre;
+    const int m = pre ? it / v.kappa : (it - n_pre) % v.mu_dec;
+    const bool last_chunk = !pre || (it % v.kappa == v.kappa - 1);
+    const int t = pre ? 0 : 1 + (it - n_pre) / v.mu_dec;
     const int64_t seq0 = pre ? (int64_t)m * v.eta : (int64_t)m * v.xi;
     const int64_t nseq = std::min<int64_t>(pre ? v.eta : v.xi, v.B - seq0);
-    const int64_t T = pre ? nseq * v.s : nseq;
+    const int64_t T = pre ? nseq * v.len_pre : nseq;
     const int phase = pre ? SQ_PREFILL : SQ_DECODE;
     const int slot = it & 1;
     if (dist && first && !pre) {
@@ -121,7 +131,7 @@ std::vector<sq_sched_op> make_schedule(const PlanView& v, int rank) {
     op(SQ_OP_COMPUTE, it, phase, t, slot, -1, seq0, nseq, T);
     if (!last) {
       op(SQ_OP_SEND_ACT, it, phase, t, slot, rank + 1, seq0, nseq, T);
-    } else {
+    } else if (last_chunk) {
       op(SQ_OP_OUT, it, phase, t, slot, -1, seq0, nseq, nseq);
       if (t < v.n_dec) op(dist ? SQ_OP_SEND_LB : SQ_OP_LOOPBACK_LOCAL, it, phase, t, slot, dist ? 0 : -1, seq0, nseq, nseq);
     }
@@ -145,6 +155,11 @@ sq_status sq_plan_check(const sq_plan* p) {
   if (!p->bits || !p->stage_of_layer) return fail(SQ_EINVAL, "sq_plan_check: null bits/stage_of_layer");
   if (p->B < 1 || p->eta < 1 || p->xi < 1 || p->xi > 32 || p->prompt_len < 1 || p->n_decode < 0)
     return fail(SQ_EINVAL, "sq_plan_check: need B,eta,s >= 1, 1 <= xi <= 32, n_decode >= 0");
+  if (p->n_heads < 0 || (p->n_heads > 0 && (p->hidden % p->n_heads ||
+                                            (p->hidden / p->n_heads != 64 && p->hidden / p->n_heads != 128))))
+    return fail(SQ_EINVAL, "sq_plan_check: n_heads %d: head_dim hidden/n_heads must be 64 or 128", p->n_heads);
+  if (p->kappa < 0 || (p->kappa > 1 && (p->n_heads == 0 || p->prompt_len % p->kappa)))
+    return fail(SQ_EINVAL, "sq_plan_check: kappa %d needs attention (n_heads > 0) and prompt_len %% kappa == 0", p->kappa);
   // eqs. (15)-(16): u_{1,1} = 1, u_{L,N} = 1, adjacent layers on the same or next stage
   if (p->stage_of_layer[0] != 0 || p->stage_of_layer[p->n_layers - 1] != p->n_stages - 1)
     return fail(SQ_EINVAL, "sq_plan_check: first layer must be on stage 0 and last on stage n_stages-1");
@@ -281,8 +296,16 @@ sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers,
   cudaStream_t S = (cudaStream_t)stream_;
   uint8_t* base = static_cast<uint8_t*>(ws_dev);
   void* stage_ws = base + W.stage;
-  const int64_t tmax = std::max<int64_t>((int64_t)v.eta * v.s, v.xi);
+  const int64_t tmax = std::max<int64_t>((int64_t)v.eta * v.len_pre, v.xi);
   const size_t act_slot = ((size_t)tmax * v.h1 * 4 + 255) / 256 * 256;
+  // attention (f3): per-layer cache pointers of this rank's layers (rank -1: all layers)
+  std::vector<void*> kcp, vcp;
+  if (v.heads > 0) {
+    for (int l = 0; l < n_layers; ++l) {
+      kcp.push_back(base + W.kv + (size_t)(2 * l) * W.kv_layer);
+      vcp.push_back(base + W.kv + (size_t)(2 * l + 1) * W.kv_layer);
+    }
+  }
   float* act[2] = {reinterpret_cast<float*>(base + W.act), reinterpret_cast<float*>(base + W.act + act_slot)};
   float* dec_in = reinterpret_cast<float*>(base + W.decin);
   const size_t lb_slot = ((size_t)std::max(v.eta, v.xi) * v.h1 * 4 + 255) / 256 * 256;
@@ -347,6 +370,17 @@ sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers,
       }
       case SQ_OP_COMPUTE: {
         const float* x_in;
+        const int chunk = pre ? o.item % v.kappa : 0;
+        sq_attn ctx{};
+        if (v.heads > 0) {
+          ctx.n_heads = v.heads;
+          ctx.max_len = v.max_len;
+          ctx.n_seq_cache = v.B;
+          ctx.seq0 = o.seq0;
+          ctx.nseq = (int32_t)o.nseq;
+          ctx.seq_len = pre ? v.len_pre : 1;
+          ctx.pos0 = pre ? chunk * v.len_pre : v.s + o.t - 1;
+        }
         if (is_first) {
           x_in = pre ? x0 + o.seq0 * v.s * h1 : dec_in + o.seq0 * h1;
           if (lb_wait_pending) {
@@ -355,6 +389,13 @@ sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers,
             lb_wait_pending = false;
           }
           if (dist) cudaStreamWaitEvent(S, ev_free[o.slot], 0);  // previous send from this buffer done
+          if (pre && v.kappa > 1) {
+            // gather the chunk's rows (sequence i, positions pos0..pos0+len-1) into the item buffer
+            for (int64_t i = 0; i < o.nseq && !ce; ++i)
+              ce = launch_copy_rows(x0 + ((o.seq0 + i) * v.s + (int64_t)chunk * v.len_pre) * h1, h1, v.len_pre, h1,
+                                    buf + i * v.len_pre * h1, h1, S);
+            x_in = buf;
+          }
         } else {
           x_in = buf;
         }
@@ -362,11 +403,15 @@ sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers,
           const float* xi = x_in;
           for (int r = 0; r < v.P && rs == SQ_OK; ++r) {
             const int f = v.first_layer[r], nl = v.first_layer[r + 1] - f;
-            rs = stage_forward(layers + f, nl, o.phase, xi, o.rows, buf, nullptr, stage_ws, stage_ws_bytes, S);
+            if (v.heads > 0) { ctx.k_cache = kcp.data() + f; ctx.v_cache = vcp.data() + f; }
+            rs = stage_forward(layers + f, nl, o.phase, xi, o.rows, buf, nullptr, stage_ws, stage_ws_bytes, S,
+                               v.heads > 0 ? &ctx : nullptr);
             xi = buf;  // the "transfer" to the next stage is the buffer itself
           }
         } else {
-          rs = stage_forward(layers, n_layers, o.phase, x_in, o.rows, buf, nullptr, stage_ws, stage_ws_bytes, S);
+          if (v.heads > 0) { ctx.k_cache = kcp.data(); ctx.v_cache = vcp.data(); }
+          rs = stage_forward(layers, n_layers, o.phase, x_in, o.rows, buf, nullptr, stage_ws, stage_ws_bytes, S,
+                             v.heads > 0 ? &ctx : nullptr);
         }
         if (is_first && !pre && dist) cudaEventRecord(ev_dec_read, S);
         break;
@@ -381,22 +426,22 @@ sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers,
         break;
       }
       case SQ_OP_OUT: {
-        const float* src = pre ? buf + (int64_t)(v.s - 1) * h1 : buf;
-        const int64_t sstride = pre ? (int64_t)v.s * h1 : h1;
+        const float* src = pre ? buf + (int64_t)(v.len_pre - 1) * h1 : buf;
+        const int64_t sstride = pre ? (int64_t)v.len_pre * h1 : h1;
         ce = launch_copy_rows(src, sstride, o.nseq, h1, out + (o.seq0 * out_rows + o.t) * h1, out_rows * h1, S);
         if (dist) cudaEventRecord(ev_free[o.slot], S);
         break;
       }
       case SQ_OP_LOOPBACK_LOCAL: {
-        const float* src = pre ? buf + (int64_t)(v.s - 1) * h1 : buf;
-        const int64_t sstride = pre ? (int64_t)v.s * h1 : h1;
+        const float* src = pre ? buf + (int64_t)(v.len_pre - 1) * h1 : buf;
+        const int64_t sstride = pre ? (int64_t)v.len_pre * h1 : h1;
         ce = launch_copy_rows(src, sstride, o.nseq, h1, lb[0], h1, S);
         if (!ce) ce = launch_layernorm_f32(lb[0], o.nseq, h1, dec_in + o.seq0 * h1, S);
         break;
       }
       case SQ_OP_SEND_LB: {
-        const float* src = pre ? buf + (int64_t)(v.s - 1) * h1 : buf;
-        const int64_t sstride = pre ? (int64_t)v.s * h1 : h1;
+        const float* src = pre ? buf + (int64_t)(v.len_pre - 1) * h1 : buf;
+        const int64_t sstride = pre ? (int64_t)v.len_pre * h1 : h1;
         cudaStreamWaitEvent(S, ev_lbfree[lbslot], 0);
         ce = launch_copy_rows(src, sstride, o.nseq, h1, lb[lbslot], h1, S);
         if (!ce) ce = launch_layernorm_f32(lb[lbslot], o.nseq, h1, lb[lbslot], S);

@@ -1,6 +1,7 @@
 // a5 — stage forward: the consecutive decoder layers of one pipeline stage, each
 // with its own bit-width from the plan.  Per layer
-// (R11/R12, pre-LN block, attention stub = V):
+// (R11/R12, pre-LN block, attention stub = V; with an sq_attn context the
+// stub is replaced by causal attention over the layer's KV cache, f3 / sq_attn.cu):
 //   a = LN(x) -> fp16 (+ group sums)     [K5]
 //   qkv = a Wqkv^T (+b)                  [K2 decode | K3 prefill]   fp16
 //   x  += v Wo^T (+b)                    [K2 | K3, fused fp32 residual add]
@@ -16,7 +17,7 @@ namespace sq {
 namespace {
 
 struct WsLayout {
-  size_t a16, qkv16, u16, xs, gemv, total;
+  size_t a16, qkv16, u16, att16, xs, gemv, total;
 };
 
 int64_t align_up(int64_t v, int64_t a) { return (v + a - 1) / a * a; }
@@ -40,6 +41,7 @@ WsLayout layout(const sq_layer* layers, int n_layers, int64_t T) {
   L.a16 = off;   off += align_up(T * h1 * 2, 256);
   L.qkv16 = off; off += align_up(T * 3 * h1 * 2, 256);
   L.u16 = off;   off += align_up(T * h2 * 2, 256);
+  L.att16 = off; off += align_up(T * h1 * 2, 256);
   L.xs = off;    off += align_up((int64_t)xsum_bytes(h2 > h1 ? h2 : h1), 256);
   L.total = off;
   return L;
@@ -55,6 +57,21 @@ sq_status check_w(const sq_qweight& w, int64_t n, int64_t k, int bits, const cha
 }
 
 }  // namespace
+
+sq_status check_attn(const sq_attn* a, const sq_layer* layers, int n_layers, int phase, int64_t tokens, const char* who) {
+  if (!a || !a->k_cache || !a->v_cache) return fail(SQ_EINVAL, "%s: null attention context / cache arrays", who);
+  const int64_t h1 = layers[0].o.n;
+  if (a->n_heads <= 0 || h1 % a->n_heads || (h1 / a->n_heads != 64 && h1 / a->n_heads != 128))
+    return fail(SQ_EINVAL, "%s: head_dim h1/n_heads must be 64 or 128", who);
+  if (a->nseq < 1 || a->seq_len < 1 || (int64_t)a->nseq * a->seq_len != tokens || (phase == SQ_DECODE && a->seq_len != 1))
+    return fail(SQ_EINVAL, "%s: tokens %lld != nseq %d x seq_len %d (decode: seq_len 1)", who, (long long)tokens, a->nseq, a->seq_len);
+  if (a->pos0 < 0 || a->pos0 + a->seq_len > a->max_len || a->seq0 < 0 || a->seq0 + a->nseq > a->n_seq_cache)
+    return fail(SQ_EINVAL, "%s: positions / sequences outside the cache", who);
+  for (int l = 0; l < n_layers; ++l)
+    if (!a->k_cache[l] || !a->v_cache[l] || ((reinterpret_cast<uintptr_t>(a->k_cache[l]) | reinterpret_cast<uintptr_t>(a->v_cache[l])) & 15u))
+      return fail(SQ_EINVAL, "%s: layer %d cache null or not 16-B aligned", who, l);
+  return SQ_OK;
+}
 
 sq_status check_layers(const sq_layer* layers, int n_layers, const char* who) {
   if (!layers || n_layers <= 0) return fail(SQ_EINVAL, "%s: no layers", who);
@@ -78,7 +95,7 @@ size_t stage_workspace_bytes(const sq_layer* layers, int n_layers, int64_t max_t
 }
 
 sq_status stage_forward(const sq_layer* layers, int n_layers, int phase, const float* x_in, int64_t T, float* x_out,
-                        void* qkv_dbg, void* ws, size_t ws_bytes, cudaStream_t s) {
+                        void* qkv_dbg, void* ws, size_t ws_bytes, cudaStream_t s, const sq_attn* att) {
   const int64_t h1 = layers[0].o.n, h2 = layers[0].fc1.n;
   const WsLayout W = layout(layers, n_layers, T);
   uint8_t* base = static_cast<uint8_t*>(ws);
@@ -86,6 +103,7 @@ sq_status stage_forward(const sq_layer* layers, int n_layers, int phase, const f
   __half* qkv16 = reinterpret_cast<__half*>(base + W.qkv16);
   __half* u16 = reinterpret_cast<__half*>(base + W.u16);
   float2* xs = reinterpret_cast<float2*>(base + W.xs);
+  __half* att16 = reinterpret_cast<__half*>(base + W.att16);
   void* gws = base + W.gemv;
   const bool dec = phase == SQ_DECODE;
   auto lin = [&](const sq_qweight& w, const __half* x, int64_t ldx, void* y, int64_t ldy, int epi,
@@ -107,13 +125,22 @@ sq_status stage_forward(const sq_layer* layers, int n_layers, int phase, const f
     if (e) break;
     e = lin(L.qkv, a16, h1, qkv16, 3 * h1, SQ_EPI_F16, k2(L.qkv) ? xs : nullptr);
     if (e) break;
-    // attention stub: attn = v = qkv[:, 2h1:3h1] (R12)
+    // attention: the R12 stub attn = v = qkv[:, 2h1:3h1], or causal attention over the KV cache (f3)
     const __half* v = qkv16 + 2 * h1;
+    int64_t ldv = 3 * h1;
+    if (att) {
+      e = launch_attention(qkv16, 3 * h1, att->nseq, att->seq_len, att->pos0, att->seq0, (int)h1, att->n_heads,
+                           static_cast<__half*>(att->k_cache[l]), static_cast<__half*>(att->v_cache[l]), att->max_len,
+                           att16, h1, s);
+      if (e) break;
+      v = att16;
+      ldv = h1;
+    }
     if (k2(L.o)) {
-      e = launch_xsum(v, 3 * h1, T, h1, xs, s);
+      e = launch_xsum(v, ldv, T, h1, xs, s);
       if (e) break;
     }
-    e = lin(L.o, v, 3 * h1, x_out, h1, SQ_EPI_F32_ACCUM, k2(L.o) ? xs : nullptr);
+    e = lin(L.o, v, ldv, x_out, h1, SQ_EPI_F32_ACCUM, k2(L.o) ? xs : nullptr);
     if (e) break;
     e = launch_layernorm_f16(x_out, T, h1, a16, k2(L.fc1) ? xs : nullptr, nullptr, nullptr, s);
     if (e) break;
@@ -159,7 +186,22 @@ sq_status sq_stage_forward(const sq_layer* layers, int n_layers, int phase, cons
   if (!ws_dev || ws_bytes < need || (reinterpret_cast<uintptr_t>(ws_dev) & 255u))
     return fail(SQ_ENOMEM, "sq_stage_forward: workspace %zu < %zu (or null / not 256-B aligned)", ws_bytes, need);
   return stage_forward(layers, n_layers, phase, x_in_dev, tokens, x_out_dev, qkv_dbg_dev, ws_dev, ws_bytes,
-                       (cudaStream_t)stream);
+                       (cudaStream_t)stream, nullptr);
+}
+
+sq_status sq_stage_forward_attn(const sq_layer* layers, int n_layers, int phase, const sq_attn* attn,
+                                const float* x_in_dev, int64_t tokens, float* x_out_dev, void* ws_dev, size_t ws_bytes,
+                                sq_stream_t stream) {
+  sq_status st = check_layers(layers, n_layers, "sq_stage_forward_attn");
+  if (st) return st;
+  if ((st = check_attn(attn, layers, n_layers, phase, tokens, "sq_stage_forward_attn"))) return st;
+  if (!x_in_dev || !x_out_dev || (reinterpret_cast<uintptr_t>(x_in_dev) & 15u) || (reinterpret_cast<uintptr_t>(x_out_dev) & 15u))
+    return fail(SQ_EINVAL, "sq_stage_forward_attn: x_in/x_out null or not 16-B aligned");
+  const size_t need = stage_workspace_bytes(layers, n_layers, tokens);
+  if (!ws_dev || ws_bytes < need || (reinterpret_cast<uintptr_t>(ws_dev) & 255u))
+    return fail(SQ_ENOMEM, "sq_stage_forward_attn: workspace %zu < %zu (or null / not 256-B aligned)", ws_bytes, need);
+  return stage_forward(layers, n_layers, phase, x_in_dev, tokens, x_out_dev, nullptr, ws_dev, ws_bytes,
+                       (cudaStream_t)stream, attn);
 }
 
 sq_status sq_layernorm_f32(const float* x_dev, int64_t rows, int64_t d, float* y_dev, sq_stream_t stream) {

@@ -11,7 +11,7 @@ import ctypes
 
 import torch
 
-from . import (P, QLinear, SQ_DECODE, SQ_PREFILL, _L, _check, _ptr, _stream, sq_layer, sq_plan,
+from . import (P, QLinear, SQ_DECODE, SQ_PREFILL, _L, _check, _ptr, _stream, sq_attn, sq_layer, sq_plan,
                sq_run_stats)
 
 
@@ -83,6 +83,31 @@ def sq_stage_forward(layers: list[Layer], phase: int, x_in: torch.Tensor, x_out:
     return x_out
 
 
+class KVCache:
+    """Device KV cache of a stage (f3): per layer K, V fp16 [n_seq, max_len, h1] (P:162 sizing)."""
+
+    def __init__(self, n_layers: int, n_seq: int, max_len: int, h1: int, device="cuda"):
+        self.k = torch.zeros((n_layers, n_seq, max_len, h1), dtype=torch.float16, device=device)
+        self.v = torch.zeros_like(self.k)
+        self.n_seq, self.max_len, self.h1 = n_seq, max_len, h1
+        self._kp = (P * n_layers)(*[self.k[l].data_ptr() for l in range(n_layers)])
+        self._vp = (P * n_layers)(*[self.v[l].data_ptr() for l in range(n_layers)])
+
+    def ctx(self, n_heads: int, seq0: int, nseq: int, seq_len: int, pos0: int) -> sq_attn:
+        return sq_attn(n_heads, self.max_len, self.n_seq, self._kp, self._vp, seq0, nseq, seq_len, pos0)
+
+
+def sq_stage_forward_attn(layers: list[Layer], phase: int, x_in: torch.Tensor, x_out: torch.Tensor,
+                          ws: StageWorkspace, cache: KVCache, n_heads: int, seq0: int, nseq: int, seq_len: int,
+                          pos0: int, stream=None, arr=None) -> torch.Tensor:
+    """a5 with real attention (f3): rows of x are (sequence, position), tokens = nseq * seq_len."""
+    arr = layer_array(layers) if arr is None else arr
+    ctx = cache.ctx(n_heads, seq0, nseq, seq_len, pos0)
+    _check(_L.sq_stage_forward_attn(arr, len(layers), phase, ctypes.byref(ctx), _ptr(x_in), x_in.shape[0],
+                                    _ptr(x_out), ctypes.c_void_p(ws.ptr), ws.nbytes, _stream(stream)))
+    return x_out
+
+
 def sq_layernorm_f32(x: torch.Tensor, y: torch.Tensor, stream=None) -> torch.Tensor:
     _check(_L.sq_layernorm_f32(_ptr(x), x.shape[0], x.shape[1], _ptr(y), _stream(stream)))
     return y
@@ -93,7 +118,7 @@ class Plan:
     """Host-side plan (per-layer bits, layer->stage partition, micro-batch sizes)."""
 
     def __init__(self, bits: list[int], stage_of_layer: list[int], hidden: int, ffn: int, B: int, eta: int,
-                 xi: int, prompt_len: int, n_decode: int, group: int = 128):
+                 xi: int, prompt_len: int, n_decode: int, group: int = 128, n_heads: int = 0, kappa: int = 1):
         self.bits = [int(b) for b in bits]
         self.stage_of_layer = [int(s) for s in stage_of_layer]
         self.n_layers = len(bits)
@@ -102,8 +127,9 @@ class Plan:
         self.prompt_len, self.n_decode, self.group = prompt_len, n_decode, group
         self._bits = (ctypes.c_int32 * self.n_layers)(*self.bits)
         self._sol = (ctypes.c_int32 * self.n_layers)(*self.stage_of_layer)
+        self.n_heads, self.kappa = n_heads, kappa
         self.c = sq_plan(self.n_layers, self.n_stages, hidden, ffn, group, self._bits, self._sol, B, eta, xi,
-                         prompt_len, n_decode)
+                         prompt_len, n_decode, n_heads, kappa)
 
     def layers_of(self, rank: int) -> list[int]:
         return [l for l, s in enumerate(self.stage_of_layer) if s == rank]

@@ -145,3 +145,39 @@ def test_gloo_world_executes_schedule_like_the_oracle(world):
     layers, x0 = oracle_model(plan)
     ref = O.pipeline(layers, x0, plan.n_decode)
     assert np.array_equal(out, ref)   # rows are independent: bitwise, whatever the partition
+
+
+@pytest.mark.parametrize("P", [1, 2, 3])
+@pytest.mark.parametrize("kappa", [2, 4])
+def test_chunked_prefill_schedule(P, kappa):
+    # P:200 chunked prefill: mu_pre * kappa prefill items of eta sequences x s/kappa tokens; only a
+    # micro-batch's last chunk produces its output row / loop-back; links still pair up one-to-one
+    B, eta, xi, s, n_dec = 7, 3, 4, 8, 2
+    from paper_conf_cluster_zhaowplw25_b200 import plan as PL
+    bits = [4, 8, 3, 16] * 2
+    sol = PL.partition_layers([1.0] * 8, P)
+    plan = R().Plan(bits, sol, 768, 3072, B, eta, xi, s, n_dec, n_heads=12, kappa=kappa)
+    R().sq_plan_check(plan)
+    sched = {r: R().sq_pipeline_schedule(plan, r) for r in range(P)}
+    mu_pre, mu_dec = -(-B // eta), -(-B // xi)
+    comp = [o for o in sched[0] if o["kind"] == "COMPUTE"]
+    assert len(comp) == mu_pre * kappa + n_dec * mu_dec
+    pre = [o for o in comp if o["phase"] == 0]
+    assert all(o["rows"] == o["nseq"] * (s // kappa) for o in pre)
+    outs = [o for o in sched[P - 1] if o["kind"] == "OUT" and o["phase"] == 0]
+    assert [o["item"] % kappa for o in outs] == [kappa - 1] * mu_pre
+    for j in range(P if P > 1 else 0):
+        nxt = (j + 1) % P
+        sends = [o["rows"] for o in sched[j] if o["kind"] in ("SEND_ACT", "SEND_LB") and o["peer"] == nxt]
+        recvs = [o["rows"] for o in sched[nxt] if o["kind"] in ("RECV_ACT", "RECV_LB") and o["peer"] == j]
+        assert sends == recvs
+
+
+def test_plan_check_attention_fields():
+    import paper_conf_cluster_zhaowplw25_b200 as sq
+    bad = [dict(n_heads=0, kappa=2), dict(n_heads=7, kappa=1), dict(n_heads=12, kappa=3), dict(n_heads=-1)]
+    for kw in bad:
+        plan = R().Plan([4, 4], [0, 0], 768, 3072, 2, 1, 2, 8, 2, **kw)
+        with pytest.raises(sq.SQError):
+            R().sq_plan_check(plan)
+    R().sq_plan_check(R().Plan([4, 4], [0, 0], 768, 3072, 2, 1, 2, 8, 2, n_heads=6, kappa=4))  # dh 128
