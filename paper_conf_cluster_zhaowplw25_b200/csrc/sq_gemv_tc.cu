@@ -52,7 +52,11 @@ constexpr int PMAX = 4;     // row tiles per panel (activation reuse), at most
 constexpr int kCnt2 = 2048;  // second per-panel counter (fix-up done) at cnt + kCnt2
 constexpr int XK = 64;
 constexpr int X_BLOCK = BT * XK * 2;  // 4 KB: [32 tokens][64 k] SW128 tile
-constexpr int DQ_WARPS = 16;      // dequant warps, in DQ_GROUPS groups of DQ_PER_GROUP (8 / 24 measured: no gain)
+// Dequant warps: 16, in two alternating groups of 8 (4 lane quadrants x 2 k-halves of a unit).
+// Measured on OPT-13B/66B shapes (INT3/4/8, m = 32): one group of 16 -> 6-18 % slower, 8 warps
+// -> 5-25 % slower, group-granular TMEM A slots with 4 quads of 4 warps -> 5-12 % slower; the
+// warps are issue-bound on the unpack, and two units in flight hide the MMA / slot hand-off best.
+constexpr int DQ_WARPS = 16;      // dequant warps, in DQ_GROUPS groups of DQ_PER_GROUP
 constexpr int DQ_PER_GROUP = 8;   // 4 lane quadrants x KH k-parts of one unit
 constexpr int DQ_KH = DQ_PER_GROUP / 4;
 constexpr int DQ_GROUPS = DQ_WARPS / DQ_PER_GROUP;  // group q dequantizes units i = q (mod DQ_GROUPS)
@@ -145,6 +149,29 @@ __device__ __forceinline__ void trace_cta(const TcP& p, int ev) {
   }
 }
 
+
+// this warp's k-part kh of a unit: batches [kh * NBW, (kh + 1) * NBW) of the unit's 4 * UG 32-k
+// batches, split at 128-k group boundaries (one meta word per group); warp-uniform branches only
+template <int BITS, int UG, int NBW>
+__device__ __forceinline__ void dequant_warp_range(const uint8_t* wst, const uint32_t* mt, int r, uint32_t a_tm, int kh) {
+  constexpr int GB = GCfg<BITS>::GB;
+  int b = kh * NBW;
+  const int e = b + NBW;
+#pragma unroll
+  for (int g = 0; g < UG; ++g) {
+    const int lo = g * 4 > b ? g * 4 : b, hi = (g + 1) * 4 < e ? (g + 1) * 4 : e;
+    if (lo >= hi) continue;
+    const int ru = ((r >> 4) * UG + g) * 16 + (r & 15);  // stage layout [tile][group][16 rows]
+    const uint32_t m = mt[ru];
+    const uint32_t at = a_tm + g * 64;
+    switch (hi - lo) {
+      case 4: dequant_row_batches<BITS, 4>(wst, m, r, at, ru * GB, lo - g * 4); break;
+      case 3: dequant_row_batches<BITS, 3>(wst, m, r, at, ru * GB, lo - g * 4); break;
+      case 2: dequant_row_batches<BITS, 2>(wst, m, r, at, ru * GB, lo - g * 4); break;
+      default: dequant_row_batches<BITS, 1>(wst, m, r, at, ru * GB, lo - g * 4); break;
+    }
+  }
+}
 
 template <int EPI>
 __device__ __forceinline__ void epi_store(const TcP& p, int64_t row, const float (&v)[BT], float bias) {
@@ -358,13 +385,12 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     int nunits = 0;
     if constexpr (BITS != 16)
       for (int it = blockIdx.x; it < I; it += C) nunits += (j1_of(it) - j0_of(it)) * tiles_of(it / Z);
-    constexpr int NBW = 4 * UG / DQ_KH;                      // batches per warp
+    constexpr int NBW = 4 * UG / DQ_KH;                      // 32-k batches per warp (may straddle groups)
+    static_assert(4 * UG % DQ_KH == 0, "a unit's batches split evenly over the k-parts");
     const int sp = warp & 3;
     const int dg = (warp - 2) / DQ_PER_GROUP;
     const int kh = ((warp - 2) >> 2) % DQ_KH;
-    const int gg = (kh * NBW) >> 2, b0 = (kh * NBW) & 3;  // group of the unit and first batch in it
     const int r = sp * 32 + lane;
-    const int ru = ((r >> 4) * UG + gg) * 16 + (r & 15);  // stage layout [tile][group][16 rows]
     const uint32_t lane_base = (uint32_t)(sp * 32) << 16;
     const bool tr = (warp == 2 && lane == 0);
     for (int i = dg; i < nunits; i += DQ_GROUPS) {
@@ -377,22 +403,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       const uint32_t* mt = reinterpret_cast<const uint32_t*>(smem + SM::OFF_META + sw * BN * 4 * UG);
       const uint32_t a_tm = tmem + lane_base + A_COL + sa * DCfg<BITS, UG>::A_SLOT;
       const uint8_t* wst = smem + SM::OFF_W + sw * SM::W_STAGE;
-      if constexpr (BITS != 16 && UG == 3) {
-        // 12 batches over 3 groups, 6 per warp: kh 0 -> group 0 batches 0..3 + group 1 batches 0..1,
-        // kh 1 -> group 1 batches 2..3 + group 2 batches 0..3 (one meta word per group)
-        static_assert(DQ_KH == 2, "UG = 3 splits the unit's k in two warp halves");
-        const int ru1 = ru + 16;  // (gg = 0 here) the row's entry of group 1 / group 2 in the stage
-        if (kh == 0) {
-          dequant_row_batches<BITS, 4>(wst, mt[ru], r, a_tm, ru * GB, 0);
-          dequant_row_batches<BITS, 2>(wst, mt[ru1], r, a_tm + 64, ru1 * GB, 0);
-        } else {
-          const int ru0 = ru - 16 * gg;
-          dequant_row_batches<BITS, 2>(wst, mt[ru0 + 16], r, a_tm + 64, (ru0 + 16) * GB, 2);
-          dequant_row_batches<BITS, 4>(wst, mt[ru0 + 32], r, a_tm + 128, (ru0 + 32) * GB, 0);
-        }
-      } else if constexpr (BITS != 16) {
-        dequant_row_batches<BITS, NBW < 4 ? NBW : 4>(wst, mt[ru], r, a_tm + gg * 64, ru * GB, b0);
-      }
+      if constexpr (BITS != 16) dequant_warp_range<BITS, UG, NBW>(wst, mt, r, a_tm, kh);
       if (tr) trace_ev(p, 12, i);
       tc_wait_st();
       tc_fence_before();

@@ -165,8 +165,9 @@ int main() {
       const uint64_t cols = (256ull << 20) / 4 / ((uint64_t)sms * 8);
       cuuint64_t d[2] = {cols, (cuuint64_t)sms * 8}, stv[1] = {cols * 4};
       cuuint32_t b[2] = {48, 8};
-      enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, mbuf, d, stv, b, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-          CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+      CUresult r = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, mbuf, d, stv, b, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                       CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+      if (r != CUDA_SUCCESS) printf("meta encode failed %d\n", (int)r);
     }
     struct V { const char* name; int meta, x, P, m, rows, SW, SX; };
     const V vs[] = {
@@ -182,8 +183,9 @@ int main() {
       {
         cuuint64_t d[3] = {64, (cuuint64_t)v.m > 0 ? (cuuint64_t)v.m : 1, (cuuint64_t)K / 64}, stv[2] = {(cuuint64_t)K * 2, 128};
         cuuint32_t b[3] = {64, (cuuint32_t)(v.rows > 0 ? v.rows : 32), 6};
-        enc(&tx, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 3, xbuf, d, stv, b, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-            CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        CUresult r = enc(&tx, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 3, xbuf, d, stv, b, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                         CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (r != CUDA_SUCCESS) printf("x encode failed %d\n", (int)r);
       }
       const uint32_t xbytes = 64 * 2 * 6 * (v.rows > 0 ? v.rows : 32);
       const int smem = v.SW * (WST + 1536) + v.SX * XST + 1024;
