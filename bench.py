@@ -456,6 +456,10 @@ def run_ours(args, wl):
                                      "results": gemm_sweep(pk)}
         if not args.no_configs0:
             extra["configs0"] = configs0_latency()
+        if not args.no_attention:
+            del ws
+            torch.cuda.empty_cache()
+            extra["attention"] = attention_run(wl, plan, layers, arr, x0, pk)
         if not args.no_cpu:
             cpu = cpu_baseline(wl, B, args.cpu_tokens, args.cpu_row_frac)
     if rank == 0:
@@ -600,6 +604,60 @@ def configs0_latency(runs: int = 20):
             "note": "one sequence; per-run = prefill 32 tokens + 8 decode steps through sq_pipeline_run (P = 1)"}
 
 
+# ------------------------------------------------------------------ f3: the same run with real attention
+def attention_run(wl: dict, plan0, layers, arr, x0, pk: dict, steps: int = 1):
+    """the configs[3] generation with causal attention over a KV cache (head_dim 128,
+    h1 / 128 heads; KV cache 2 x B x (s + n_dec) x h1 fp16 per layer inside the pipeline workspace)
+    in place of the R12 stub; same layers, plan and inputs.  One warm-up run, `steps` timed runs, then a
+    profiled run for the attention kernels' own rooflines (decode: KV-cache GB/s vs HBM; prefill: causal
+    TFLOP/s)."""
+    import torch
+    import paper_conf_cluster_zhaowplw25_b200 as sq
+    from paper_conf_cluster_zhaowplw25_b200 import runtime as R
+    heads = wl["h1"] // 128
+    plan = R.Plan(plan0.bits, plan0.stage_of_layer, plan0.hidden, plan0.ffn, plan0.B, plan0.eta, plan0.xi,
+                  plan0.prompt_len, plan0.n_decode, n_heads=heads, kappa=1)
+    R.sq_plan_check(plan)
+    ws = R.PipelineWorkspace(plan, layers, 0)
+    out = torch.zeros((plan.B, 1 + plan.n_decode, plan.hidden), dtype=torch.float32, device="cuda")
+    R.sq_pipeline_run(plan, 0, layers, None, x0, out, ws, arr=arr)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    st = None
+    for _ in range(steps):
+        st = R.sq_pipeline_run(plan, 0, layers, None, x0, out, ws, arr=arr)
+    e1.record()
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / steps
+    sq.sq_profile_enable(True)
+    R.sq_pipeline_run(plan, 0, layers, None, x0, out, ws, arr=arr)
+    torch.cuda.synchronize()
+    sq.sq_profile_enable(False)
+    prof = sq.sq_profile_read()
+    ad, ap_ = prof["attn_decode"], prof["attn_prefill"]
+    kv_gb = 2 * plan.B * (plan.prompt_len + plan.n_decode) * plan.hidden * 2 * len(layers) / 1e9
+    res = {"workload": wl["name"] + ", with causal attention over a KV cache (f3)", "n_heads": heads, "head_dim": 128,
+           "kv_cache_GB": round(kv_gb, 2), "ms_per_step": round(ms, 1),
+           "tokens_per_s": round(plan.B * (1 + plan.n_decode) / (ms / 1e3), 1),
+           "phase_ms": {"prefill": round(st["t_prefill_ms"], 1), "decode": round(st["t_decode_ms"], 1)},
+           "gpu_launches_per_step": st["gpu_launches"]}
+    if ad["launches"] and ad["ms"] > 0:
+        gbs = ad["bytes"] / (ad["ms"] / 1e3) / 1e9
+        res["decode_attention"] = {"bound": "hbm", "achieved": round(gbs, 1), "peak": pk["hbm_gbs"], "unit": "GB/s",
+                                   "frac": round(gbs / pk["hbm_gbs"], 3), "launches": ad["launches"],
+                                   "ms_per_step": round(ad["ms"], 1),
+                                   "bytes_per_launch": ad["bytes"] / ad["launches"]}
+    if ap_["launches"] and ap_["ms"] > 0:
+        tf = ap_["flops"] / (ap_["ms"] / 1e3) / 1e12
+        res["prefill_attention"] = {"bound": "tensor", "achieved": round(tf, 1), "unit": "TFLOP/s",
+                                    "peak_mma_sync_note": "mma.sync path; the tcgen05 peak is " + str(pk["tflops"]),
+                                    "launches": ap_["launches"], "ms_per_step": round(ap_["ms"], 1)}
+    del ws
+    torch.cuda.empty_cache()
+    return res
+
+
 def traffic_for(kernel: str, per_launch: float | None = None):
     """DRAM bytes per launch of the dominant kernel from the committed ncu --set full capture
     (profiles/traffic.json): the captured launch's dram/algorithmic ratio applied to this run's
@@ -628,6 +686,7 @@ def main():
     ap.add_argument("--no-gemv-sweep", action="store_true")
     ap.add_argument("--no-gemm-sweep", action="store_true")
     ap.add_argument("--no-configs0", action="store_true")
+    ap.add_argument("--no-attention", action="store_true")
     ap.add_argument("--cpu-tokens", type=int, default=8)
     ap.add_argument("--cpu-row-frac", type=int, default=8)
     args = ap.parse_args()

@@ -325,13 +325,15 @@ int64_t sq_pipeline_schedule(const sq_plan* plan, int rank, sq_sched_op* ops, in
 /* ------------------------------------------------------------------------
  * Measurement hooks (bench.py): per-kernel-class CUDA-event timing of every
  * launch made by the library while enabled, on the launching stream.
- * class 0 = decode GEMV, 1 = prefill GEMM, 2 = glue (LN/xsum), 3 = quantize/pack.
+ * class 0 = decode GEMV, 1 = prefill GEMM, 2 = glue (LN/xsum), 3 = quantize/pack,
+ * 4 = decode attention (KV-cache bytes), 5 = prefill attention (causal flops).
  * ------------------------------------------------------------------------ */
+#define SQ_PROFILE_CLASSES 6
 typedef struct {
-  int64_t launches[4];
-  double ms[4];             /* summed event durations */
-  double bytes[4];          /* algorithmic bytes */
-  double flops[4];          /* algorithmic flops */
+  int64_t launches[SQ_PROFILE_CLASSES];
+  double ms[SQ_PROFILE_CLASSES];      /* summed event durations */
+  double bytes[SQ_PROFILE_CLASSES];   /* algorithmic bytes */
+  double flops[SQ_PROFILE_CLASSES];   /* algorithmic flops */
 } sq_profile;
 sq_status sq_profile_enable(int on);
 sq_status sq_profile_read(sq_profile* out);   /* synchronizes the device */

@@ -70,8 +70,8 @@ SQ_OP_NAMES = ["RECV_LB", "RECV_ACT", "COMPUTE", "SEND_ACT", "OUT", "SEND_LB", "
 
 
 class sq_profile(ctypes.Structure):
-    _fields_ = [("launches", I64 * 4), ("ms", ctypes.c_double * 4), ("bytes", ctypes.c_double * 4),
-                ("flops", ctypes.c_double * 4)]
+    _fields_ = [("launches", I64 * 6), ("ms", ctypes.c_double * 6), ("bytes", ctypes.c_double * 6),
+                ("flops", ctypes.c_double * 6)]
 
 
 def _sig(name, restype, *argtypes):
@@ -288,9 +288,9 @@ def sq_profile_enable(on: bool = True) -> None:
 def sq_profile_read() -> dict:
     p = sq_profile()
     _check(_L.sq_profile_read(ctypes.byref(p)))
-    names = ["gemv", "gemm", "glue", "quant"]
+    names = ["gemv", "gemm", "glue", "quant", "attn_decode", "attn_prefill"]
     return {names[i]: {"launches": p.launches[i], "ms": p.ms[i], "bytes": p.bytes[i], "flops": p.flops[i]}
-            for i in range(4)}
+            for i in range(6)}
 
 
 def sq_launch_count() -> int:

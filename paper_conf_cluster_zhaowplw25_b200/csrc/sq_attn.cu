@@ -329,7 +329,11 @@ cudaError_t launch_attention(const __half* qkv, int64_t ldq, int nseq, int len, 
     count_launch();
   }
   const float qscale = kLog2e / sqrtf((float)dh);
-  auto t = prof_begin(KC_GLUE, (double)nseq * n_heads * 2.0 * (pos0 + len) * dh * 2, 0, s);
+  // algorithmic work: decode reads the K and V rows 0..p of every (sequence, head); prefill does
+  // 2 x 2 dh flops per (query, visible key, head) for S = Q K^T and O = P V
+  const double keys = (double)len * pos0 + (double)len * (len + 1) / 2.0;  // sum over queries of (p + 1)
+  auto t = prof_begin(len == 1 ? KC_ATTN_DEC : KC_ATTN_PRE, (double)nseq * 2.0 * (pos0 + 1) * h1 * 2,
+                      (double)nseq * n_heads * 4.0 * dh * keys, s);
   if (len == 1) {
     dim3 grid(n_heads, nseq);
     if (dh == 128) launch_pdl(k_attn_decode<128>, grid, dim3(128), 0, s, qkv, ldq, pos0, seq0, h1, (const __half*)kc, (const __half*)vc, max_len, out, ldo, qscale);

@@ -15,7 +15,7 @@ sq_status fail(sq_status st, const char* fmt, ...);
 sq_status cuda_check(cudaError_t e, const char* what);
 
 // ---- launch accounting / profiling (sq_profile_*) ----
-enum KClass { KC_GEMV = 0, KC_GEMM = 1, KC_GLUE = 2, KC_QUANT = 3 };
+enum KClass { KC_GEMV = 0, KC_GEMM = 1, KC_GLUE = 2, KC_QUANT = 3, KC_ATTN_DEC = 4, KC_ATTN_PRE = 5 };
 struct ProfTicket {
   int slot = -1;
 };
