@@ -283,14 +283,19 @@ typedef struct {
   double t_total_ms, t_prefill_ms, t_decode_ms;  /* device time (events) on this rank */
   double tokens_per_s;      /* B*(1+n_decode) / t_total */
   int64_t bytes_sent;       /* inter-stage bytes sent by this rank */
-  int64_t gpu_launches;     /* kernels launched by this rank */
+  int64_t gpu_launches;     /* kernels launched by this rank (graph replays count their kernels) */
+  double host_enqueue_ms;   /* host time spent issuing the run's work (before the final sync) */
+  int64_t graph_replays;    /* decode micro-batches replayed from a cached CUDA graph */
 } sq_run_stats;
 
 size_t sq_pipeline_workspace_bytes(const sq_plan* plan, const sq_layer* layers, int rank);
 /* rank >= 0: this process's stage (layers = its layers, in order); rank == -1 with a
  * local comm: all stages (layers = all n_layers).  x0_dev: embeddings fp32 [B, s, h1]
  * (needed on stage 0); out_dev: fp32 [B, 1+n_decode, h1] (written on the last stage).
- * Blocking: returns after the run completed on this rank. */
+ * Blocking: returns after the run completed on this rank.
+ * Decode micro-batches of the attention-stub path (plan.n_heads == 0) are captured once per
+ * (layers, input / output buffer, rows, workspace) into a CUDA graph and replayed (a process-wide
+ * cache of instantiated graphs; SQ_GRAPH=0 disables it, and it is bypassed while sq_profile is on). */
 sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers, int n_layers,
                           sq_comm* comm, const float* x0_dev, float* out_dev, void* ws_dev,
                           size_t ws_bytes, sq_run_stats* stats, sq_stream_t stream);

@@ -58,7 +58,8 @@ class sq_attn(ctypes.Structure):
 
 class sq_run_stats(ctypes.Structure):
     _fields_ = [("t_total_ms", ctypes.c_double), ("t_prefill_ms", ctypes.c_double), ("t_decode_ms", ctypes.c_double),
-                ("tokens_per_s", ctypes.c_double), ("bytes_sent", I64), ("gpu_launches", I64)]
+                ("tokens_per_s", ctypes.c_double), ("bytes_sent", I64), ("gpu_launches", I64),
+                ("host_enqueue_ms", ctypes.c_double), ("graph_replays", I64)]
 
 
 class sq_sched_op(ctypes.Structure):

@@ -88,6 +88,8 @@ void prof_end(ProfTicket t, cudaStream_t s) {
   cudaEventRecord(g_prof[t.slot].e1, s);
 }
 
+bool prof_enabled() { return g_prof_on.load(std::memory_order_relaxed) != 0; }
+
 }  // namespace sq
 
 using namespace sq;

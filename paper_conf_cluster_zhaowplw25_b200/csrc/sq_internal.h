@@ -22,6 +22,7 @@ struct ProfTicket {
 ProfTicket prof_begin(int kclass, double bytes, double flops, cudaStream_t s);
 void prof_end(ProfTicket t, cudaStream_t s);
 void count_launch(int n = 1);
+bool prof_enabled();
 
 // ---- kernel launchers (validated arguments) ----
 cudaError_t launch_quantize(const __half* w, int64_t n, int64_t k, int bits, int group, uint8_t* codes,

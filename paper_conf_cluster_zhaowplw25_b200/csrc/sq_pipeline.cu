@@ -20,7 +20,11 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <chrono>
+#include <cstdlib>
 #include <cstring>
+#include <mutex>
+#include <unordered_map>
 #include <vector>
 
 #include "sq_common.cuh"
@@ -82,6 +86,106 @@ Ws ws_layout(const PlanView& v, const sq_layer* layers, int n_layers, int rank) 
   w.kv = off;    off += (size_t)n_layers * 2 * w.kv_layer;
   w.total = off;
   return w;
+}
+
+// ---- CUDA-graph cache of decode stage calls.  A decode micro-batch re-runs the same kernels with the
+// same pointers every step (stub attention: no position argument), so its launches are captured once
+// (on a private stream: capture executes nothing) and replayed on the run's stream.  The key covers
+// every value the launches bake in: the layers' structs (bits, shapes, pointers), the input/output
+// buffers, the token count and the workspace; replays count their kernels in sq_launch_count.
+struct GraphKey {
+  uint64_t layers_hash;
+  const void* x_in;
+  const void* x_out;
+  const void* ws;
+  int64_t rows;
+  int n_layers, dev;
+  bool operator==(const GraphKey& o) const {
+    return layers_hash == o.layers_hash && x_in == o.x_in && x_out == o.x_out && ws == o.ws && rows == o.rows &&
+           n_layers == o.n_layers && dev == o.dev;
+  }
+};
+struct GraphKeyHash {
+  size_t operator()(const GraphKey& k) const {
+    uint64_t h = k.layers_hash ^ (reinterpret_cast<uint64_t>(k.x_in) * 0x9E3779B97F4A7C15ull);
+    h ^= reinterpret_cast<uint64_t>(k.x_out) + (h << 7) + (reinterpret_cast<uint64_t>(k.ws) >> 3) + (uint64_t)k.rows * 131;
+    return (size_t)(h ^ (uint64_t)k.n_layers ^ ((uint64_t)k.dev << 40));
+  }
+};
+struct CachedGraph {
+  cudaGraphExec_t exec = nullptr;
+  int64_t launches = 0;
+};
+std::mutex g_graph_mu;
+std::unordered_map<GraphKey, CachedGraph, GraphKeyHash>* g_graphs = nullptr;
+constexpr size_t kMaxGraphs = 256;
+
+uint64_t hash_layers(const sq_layer* layers, int n) {
+  const unsigned char* p = reinterpret_cast<const unsigned char*>(layers);
+  uint64_t h = 1469598103934665603ull;
+  for (size_t i = 0; i < (size_t)n * sizeof(sq_layer); ++i) h = (h ^ p[i]) * 1099511628211ull;
+  return h;
+}
+
+bool graphs_enabled() {
+  static int on = -1;
+  if (on < 0) { const char* e = getenv("SQ_GRAPH"); on = (e && e[0] == '0') ? 0 : 1; }
+  return on == 1;
+}
+
+// decode stage call through the graph cache (falls back to direct launches on any capture error)
+sq_status stage_forward_graph(const sq_layer* layers, int n_layers, const float* x_in, int64_t rows, float* x_out,
+                              void* ws, size_t ws_bytes, cudaStream_t S, int64_t* replays) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  const GraphKey key{hash_layers(layers, n_layers), x_in, x_out, ws, rows, n_layers, dev};
+  {
+    std::lock_guard<std::mutex> lk(g_graph_mu);
+    if (!g_graphs) g_graphs = new std::unordered_map<GraphKey, CachedGraph, GraphKeyHash>();
+    auto it = g_graphs->find(key);
+    if (it != g_graphs->end()) {
+      if (cudaGraphLaunch(it->second.exec, S) != cudaSuccess) return cuda_check(cudaGetLastError(), "cudaGraphLaunch");
+      count_launch((int)it->second.launches);
+      ++*replays;
+      return SQ_OK;
+    }
+  }
+  cudaStream_t cs = nullptr;
+  if (cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking) != cudaSuccess) {
+    cudaGetLastError();
+    return stage_forward(layers, n_layers, SQ_DECODE, x_in, rows, x_out, nullptr, ws, ws_bytes, S);
+  }
+  const int64_t l0 = sq_launch_count();
+  cudaGraph_t g = nullptr;
+  cudaGraphExec_t ex = nullptr;
+  sq_status st = SQ_OK;
+  bool ok = cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal) == cudaSuccess;
+  if (ok) {
+    st = stage_forward(layers, n_layers, SQ_DECODE, x_in, rows, x_out, nullptr, ws, ws_bytes, cs);
+    ok = cudaStreamEndCapture(cs, &g) == cudaSuccess && st == SQ_OK;
+  }
+  const int64_t n_launch = sq_launch_count() - l0;
+  count_launch(-(int)n_launch);  // capture launched nothing
+  if (ok) ok = cudaGraphInstantiate(&ex, g, 0) == cudaSuccess;
+  if (g) cudaGraphDestroy(g);
+  cudaStreamDestroy(cs);
+  if (!ok) {
+    cudaGetLastError();
+    if (ex) cudaGraphExecDestroy(ex);
+    return stage_forward(layers, n_layers, SQ_DECODE, x_in, rows, x_out, nullptr, ws, ws_bytes, S);
+  }
+  {
+    std::lock_guard<std::mutex> lk(g_graph_mu);
+    if (g_graphs->size() >= kMaxGraphs) {
+      for (auto& kv : *g_graphs) cudaGraphExecDestroy(kv.second.exec);
+      g_graphs->clear();
+    }
+    (*g_graphs)[key] = CachedGraph{ex, n_launch};
+  }
+  if (cudaGraphLaunch(ex, S) != cudaSuccess) return cuda_check(cudaGetLastError(), "cudaGraphLaunch");
+  count_launch((int)n_launch);
+  ++*replays;
+  return SQ_OK;
 }
 
 // ---- schedule: the op sequence of one rank (also exported as sq_pipeline_schedule)
@@ -333,9 +437,11 @@ sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers,
     cudaStreamWaitEvent(comm->s_send, ev_start, 0);
     cudaStreamWaitEvent(comm->s_recv, ev_start, 0);
   }
-  int64_t bytes_sent = 0;
+  int64_t bytes_sent = 0, replays = 0;
   cudaError_t ce = cudaSuccess;
   sq_status rs = SQ_OK;
+  const auto host_t0 = std::chrono::steady_clock::now();
+  const bool use_graphs = graphs_enabled() && v.heads == 0 && !prof_enabled();
 
   // ---- execute this rank's schedule (sq_pipeline_schedule): one op at a time, compute on S,
   // sends on s_send, receives on s_recv, CUDA events for every cross-stream dependency.
@@ -404,14 +510,20 @@ sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers,
           for (int r = 0; r < v.P && rs == SQ_OK; ++r) {
             const int f = v.first_layer[r], nl = v.first_layer[r + 1] - f;
             if (v.heads > 0) { ctx.k_cache = kcp.data() + f; ctx.v_cache = vcp.data() + f; }
-            rs = stage_forward(layers + f, nl, o.phase, xi, o.rows, buf, nullptr, stage_ws, stage_ws_bytes, S,
-                               v.heads > 0 ? &ctx : nullptr);
+            if (use_graphs && !pre)
+              rs = stage_forward_graph(layers + f, nl, xi, o.rows, buf, stage_ws, stage_ws_bytes, S, &replays);
+            else
+              rs = stage_forward(layers + f, nl, o.phase, xi, o.rows, buf, nullptr, stage_ws, stage_ws_bytes, S,
+                                 v.heads > 0 ? &ctx : nullptr);
             xi = buf;  // the "transfer" to the next stage is the buffer itself
           }
         } else {
           if (v.heads > 0) { ctx.k_cache = kcp.data(); ctx.v_cache = vcp.data(); }
-          rs = stage_forward(layers, n_layers, o.phase, x_in, o.rows, buf, nullptr, stage_ws, stage_ws_bytes, S,
-                             v.heads > 0 ? &ctx : nullptr);
+          if (use_graphs && !pre)
+            rs = stage_forward_graph(layers, n_layers, x_in, o.rows, buf, stage_ws, stage_ws_bytes, S, &replays);
+          else
+            rs = stage_forward(layers, n_layers, o.phase, x_in, o.rows, buf, nullptr, stage_ws, stage_ws_bytes, S,
+                               v.heads > 0 ? &ctx : nullptr);
         }
         if (is_first && !pre && dist) cudaEventRecord(ev_dec_read, S);
         break;
@@ -466,6 +578,7 @@ sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers,
     cudaStreamWaitEvent(S, ev_consumed, 0);
   }
   cudaEventRecord(ev_end, S);
+  const double host_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - host_t0).count();
   cudaError_t se = cudaEventSynchronize(ev_end);
   if (ce == cudaSuccess) ce = se;
   if (ce == cudaSuccess) ce = cudaGetLastError();
@@ -479,6 +592,8 @@ sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers,
     stats->tokens_per_s = tt > 0 ? (double)v.B * (1 + v.n_dec) / (tt * 1e-3) : 0.0;
     stats->bytes_sent = bytes_sent;
     stats->gpu_launches = sq_launch_count() - launches0;
+    stats->host_enqueue_ms = host_ms;
+    stats->graph_replays = replays;
   }
   cudaEventDestroy(ev_start); cudaEventDestroy(ev_pre); cudaEventDestroy(ev_end);
   for (int i = 0; i < 2; ++i) {

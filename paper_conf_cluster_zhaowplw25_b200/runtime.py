@@ -201,4 +201,5 @@ def sq_pipeline_run(plan: Plan, rank: int, layers: list[Layer], comm: Comm | Non
     _check(_L.sq_pipeline_run(ctypes.byref(plan.c), rank, arr, len(layers), comm.h if comm else None, _ptr(x0),
                               _ptr(out), ctypes.c_void_p(ws.ptr), ws.nbytes, ctypes.byref(st), _stream(stream)))
     return {"t_total_ms": st.t_total_ms, "t_prefill_ms": st.t_prefill_ms, "t_decode_ms": st.t_decode_ms,
-            "tokens_per_s": st.tokens_per_s, "bytes_sent": st.bytes_sent, "gpu_launches": st.gpu_launches}
+            "tokens_per_s": st.tokens_per_s, "bytes_sent": st.bytes_sent, "gpu_launches": st.gpu_launches,
+            "host_enqueue_ms": st.host_enqueue_ms, "graph_replays": st.graph_replays}

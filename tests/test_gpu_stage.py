@@ -153,6 +153,52 @@ def test_pipeline_configs0_end_to_end(opt125m):
     assert st["gpu_launches"] > 0 and st["t_total_ms"] > 0
 
 
+def test_decode_graph_replay_bitwise_equals_eager(opt125m, tmp_path):
+    """sq_pipeline_run replays cached CUDA graphs of the decode micro-batches (stub path): a second run
+    replays them (graph_replays > 0), and the output equals a run with SQ_GRAPH=0 (eager launches,
+    subprocess) bit for bit."""
+    import os
+    import subprocess
+    import sys
+    sq, R = rt()
+    bits, g, o = opt125m
+    B, eta, xi, s, n_dec = 3, 2, 2, 16, 4
+    x0 = torch.from_numpy(synth.hidden_f32(9, B * s, H1).reshape(B, s, H1)).cuda()
+    plan = R.Plan(bits, [0] * 6 + [1] * 6, H1, H2, B, eta, xi, s, n_dec)
+    comm = R.Comm.local(2)
+    ws = R.PipelineWorkspace(plan, g, -1)
+    out = torch.zeros((B, 1 + n_dec, H1), dtype=torch.float32, device="cuda")
+    R.sq_pipeline_run(plan, -1, g, comm, x0, out, ws)      # captures
+    a = out.cpu().numpy()
+    out.zero_()
+    st = R.sq_pipeline_run(plan, -1, g, comm, x0, out, ws)  # replays
+    comm.destroy()
+    b = out.cpu().numpy()
+    assert np.array_equal(a, b) and st["graph_replays"] > 0
+    assert st["host_enqueue_ms"] > 0
+    np.save(tmp_path / "graph.npy", b)
+    code = f"""
+import sys; sys.path.insert(0, {os.path.dirname(os.path.dirname(os.path.abspath(__file__)))!r})
+import numpy as np, torch, synth
+from paper_conf_cluster_zhaowplw25_b200 import runtime as R
+H1, H2, L = {H1}, {H2}, {L}
+bits = synth.bits_plan(2, L)
+g = R.build_layers(L, H1, H2, bits)
+plan = R.Plan(bits, [0] * 6 + [1] * 6, H1, H2, {B}, {eta}, {xi}, {s}, {n_dec})
+comm = R.Comm.local(2)
+ws = R.PipelineWorkspace(plan, g, -1)
+x0 = torch.from_numpy(synth.hidden_f32(9, {B} * {s}, H1).reshape({B}, {s}, H1)).cuda()
+out = torch.zeros(({B}, 1 + {n_dec}, H1), dtype=torch.float32, device="cuda")
+st = R.sq_pipeline_run(plan, -1, g, comm, x0, out, ws)
+assert st["graph_replays"] == 0
+np.save({str(tmp_path / "eager.npy")!r}, out.cpu().numpy())
+"""
+    r = subprocess.run([sys.executable, "-c", code], env=dict(os.environ, SQ_GRAPH="0"), capture_output=True,
+                       text=True, timeout=600)
+    assert r.returncode == 0, r.stderr[-2000:]
+    assert np.array_equal(np.load(tmp_path / "eager.npy"), b)
+
+
 def test_virtual_pipeline_partition_invariance(opt125m):
     # eqs. (15)-(16) contiguous uneven partitions must not change a single bit
     sq, R = rt()
