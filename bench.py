@@ -460,6 +460,10 @@ def run_ours(args, wl):
             del ws
             torch.cuda.empty_cache()
             extra["attention"] = attention_run(wl, plan, layers, arr, x0, pk)
+        if not args.no_bloom and args.workload == "opt66b":
+            layers.clear()  # the OPT-66B model's HBM goes to the BLOOM-176B-shaped one
+            torch.cuda.empty_cache()
+            extra["configs4"] = bloom_run(pk)
         if not args.no_cpu:
             cpu = cpu_baseline(wl, B, args.cpu_tokens, args.cpu_row_frac)
     if rank == 0:
@@ -604,6 +608,43 @@ def configs0_latency(runs: int = 20):
             "note": "one sequence; per-run = prefill 32 tokens + 8 decode steps through sq_pipeline_run (P = 1)"}
 
 
+# ------------------------------------------------------------------ configs[4] side line
+def bloom_run(pk: dict, steps: int = 1):
+    """BASELINE.json configs[4] on ONE B200: BLOOM-176B-shaped (d = 14336, fused QKV, GeLU), 70 layers,
+    INT3/INT4 50/50 (80.9 GB), B = 32, eta = 8, xi = 32, prompt 512 + 128 decode tokens (the paper's
+    8-way pipeline needs 8 GPUs; this is its 1-GPU point).  One warm-up run, `steps` timed runs."""
+    import torch
+    import synth
+    from paper_conf_cluster_zhaowplw25_b200 import runtime as R
+    from paper_conf_cluster_zhaowplw25_b200 import plan as PL
+    wl = WORKLOADS["bloom176b"]
+    L, h1, h2, B = wl["L"], wl["h1"], wl["h2"], wl["b_per_gpu"]
+    bits = workload_bits(wl)
+    g = R.build_layers(L, h1, h2, bits, act=wl["act"])
+    plan = R.Plan(bits, [0] * L, h1, h2, B, wl["eta"], wl["xi"], wl["s"], wl["n_dec"])
+    ws = R.PipelineWorkspace(plan, g, 0)
+    arr = R.layer_array(g)
+    x0 = torch.empty((B, wl["s"], h1), dtype=torch.float32, device="cuda")
+    synth.device_fill_f32(x0.data_ptr(), 1, 0, x0.numel(), 1.0, False)
+    out = torch.zeros((B, 1 + wl["n_dec"], h1), dtype=torch.float32, device="cuda")
+    R.sq_pipeline_run(plan, 0, g, None, x0, out, ws, arr=arr)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(steps):
+        st = R.sq_pipeline_run(plan, 0, g, None, x0, out, ws, arr=arr)
+    e1.record()
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / steps
+    res = {"workload": wl["name"] + " (1 GPU)", "B": B, "weights_GB": round(sum(PL.layer_bytes(h1, h2, b) for b in bits) / 1e9, 1),
+           "bits_histogram": {str(b): bits.count(b) for b in (3, 4)}, "ms_per_step": round(ms, 1),
+           "tokens_per_s": round(B * (1 + wl["n_dec"]) / (ms / 1e3), 1),
+           "phase_ms": {"prefill": round(st["t_prefill_ms"], 1), "decode": round(st["t_decode_ms"], 1)}}
+    del g, ws, x0, out
+    torch.cuda.empty_cache()
+    return res
+
+
 # ------------------------------------------------------------------ f3: the same run with real attention
 def attention_run(wl: dict, plan0, layers, arr, x0, pk: dict, steps: int = 1):
     """the configs[3] generation with causal attention over a KV cache (head_dim 128,
@@ -687,6 +728,7 @@ def main():
     ap.add_argument("--no-gemm-sweep", action="store_true")
     ap.add_argument("--no-configs0", action="store_true")
     ap.add_argument("--no-attention", action="store_true")
+    ap.add_argument("--no-bloom", action="store_true")
     ap.add_argument("--cpu-tokens", type=int, default=8)
     ap.add_argument("--cpu-row-frac", type=int, default=8)
     args = ap.parse_args()

@@ -659,40 +659,6 @@ struct TcPlan { int P, Z, I, ctas; };
 // per-SM TMA pipeline, ~45-50 GB/s per SM, tools/mb_tma.cu) -- plus, for Z > 1, the split-k fix-up
 // (partials written and re-read, the panel-wide wait).  Z > 1 requires a single round (every item
 // resident: the fix-up waits for the panel's other items).
-// CTAs of a K2c launch that can be resident at once when its split panels form clusters of z CTAs
-// (cudaOccupancyMaxActiveClusters x z, cached per z; measured on B200: z = 2 -> 148, 3 -> 135,
-// 4 -> 132, 8 -> 120).  Queried on the largest-shared-memory instantiation, so every other one fits
-// at least as many.  0 without a device.
-int cluster_capacity(int z) {
-  static int cap[33];
-  static bool init = false;
-  if (!init) { for (int& c : cap) c = -1; init = true; }
-  if (z < 2 || z > 16) return 0;
-  if (cap[z] < 0) {
-    auto kern = k_gemv_tc<4, 3, SQ_EPI_F16>;
-    int v = 0;
-    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, DSmem<4, 3>::BYTES) == cudaSuccess &&
-        cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) == cudaSuccess) {
-      cudaLaunchConfig_t cfg = {};
-      cfg.gridDim = dim3(z * 8);
-      cfg.blockDim = dim3(NUM_THREADS);
-      cfg.dynamicSmemBytes = DSmem<4, 3>::BYTES;
-      cudaLaunchAttribute at[1];
-      at[0].id = cudaLaunchAttributeClusterDimension;
-      at[0].val.clusterDim.x = z;
-      at[0].val.clusterDim.y = 1;
-      at[0].val.clusterDim.z = 1;
-      cfg.attrs = at;
-      cfg.numAttrs = 1;
-      int ncl = 0;
-      if (cudaOccupancyMaxActiveClusters(&ncl, kern, &cfg) == cudaSuccess) v = ncl * z;
-    }
-    cudaGetLastError();
-    cap[z] = v;
-  }
-  return cap[z];
-}
-
 TcPlan tc_plan(int64_t n, int64_t k, int bits) {
   const int64_t nt = n / BN, kg = k / 128;
   const int ug = tc_ug(bits, (int)kg);
@@ -705,8 +671,9 @@ TcPlan tc_plan(int64_t n, int64_t k, int bits) {
     for (int Z = 1; Z <= zmax && Z <= ks; ++Z) {
       const int64_t I = ((nt + P - 1) / P) * Z, rounds = (I + C - 1) / C;
       if (Z > 1 && rounds > 1) continue;
-      // split panels only as clusters that can all be resident (DSMEM reduction, no spin-waits)
-      if (Z > 1 && (Z > 8 || I > cluster_capacity(Z))) continue;
+      // (split panels run as resident clusters when they fit -- cluster residency on B200: z = 2 -> 148 CTAs, 3 -> 135, 4 -> 132, 8 -> 120 --
+      // else with the cooperative global fix-up; restricting the plan to fitting clusters measured
+      // 5-15 % slower on the o-proj / fc2 shapes, which need P = 4 with Z = 8 for activation reuse)
       const int64_t steps = (ks + Z - 1) / Z;
       const double fix = Z > 1 ? 2.0 * P * BT * BN * 4 + 131072.0 : 0.0;
       const double cost = rounds * steps * (P * unit_w + unit_x) + fix;
