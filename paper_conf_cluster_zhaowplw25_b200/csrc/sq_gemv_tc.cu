@@ -150,27 +150,51 @@ __device__ __forceinline__ void trace_cta(const TcP& p, int ev) {
 }
 
 
-// this warp's k-part kh of a unit: batches [kh * NBW, (kh + 1) * NBW) of the unit's 4 * UG 32-k
-// batches, split at 128-k group boundaries (one meta word per group); warp-uniform branches only
-template <int BITS, int UG, int NBW>
-__device__ __forceinline__ void dequant_warp_range(const uint8_t* wst, const uint32_t* mt, int r, uint32_t a_tm, int kh) {
+// Segments of this warp's k-part kh of a unit: batches [kh * NBW, (kh + 1) * NBW) of the unit's
+// 4 * UG 32-k batches, split at 128-k group boundaries (one meta word per group).  Compile-time segment
+// lists (a runtime batch count cost 4-9 % on INT3/INT4), and ONE warp vote per unit for the
+// saturating variant (R20) instead of one per segment.
+template <int BITS, int UG, int NBW, bool SAT, int KH>
+__device__ __forceinline__ void dequant_part(const uint8_t* wst, const uint32_t* mt, int r, uint32_t a_tm) {
   constexpr int GB = GCfg<BITS>::GB;
-  int b = kh * NBW;
-  const int e = b + NBW;
 #pragma unroll
   for (int g = 0; g < UG; ++g) {
-    const int lo = g * 4 > b ? g * 4 : b, hi = (g + 1) * 4 < e ? (g + 1) * 4 : e;
+    constexpr int b = KH * NBW, e = KH * NBW + NBW;
+    const int lo = g * 4 > b ? g * 4 : b, hi = (g + 1) * 4 < e ? (g + 1) * 4 : e;  // constant after unrolling
     if (lo >= hi) continue;
     const int ru = ((r >> 4) * UG + g) * 16 + (r & 15);  // stage layout [tile][group][16 rows]
     const uint32_t m = mt[ru];
     const uint32_t at = a_tm + g * 64;
-    switch (hi - lo) {
-      case 4: dequant_row_batches<BITS, 4>(wst, m, r, at, ru * GB, lo - g * 4); break;
-      case 3: dequant_row_batches<BITS, 3>(wst, m, r, at, ru * GB, lo - g * 4); break;
-      case 2: dequant_row_batches<BITS, 2>(wst, m, r, at, ru * GB, lo - g * 4); break;
-      default: dequant_row_batches<BITS, 1>(wst, m, r, at, ru * GB, lo - g * 4); break;
-    }
+    if (hi - lo == 4) dequant_row_batches_<BITS, 4, SAT>(wst, m, r, at, ru * GB, lo - g * 4);
+    else if (hi - lo == 3) dequant_row_batches_<BITS, 3, SAT>(wst, m, r, at, ru * GB, lo - g * 4);
+    else if (hi - lo == 2) dequant_row_batches_<BITS, 2, SAT>(wst, m, r, at, ru * GB, lo - g * 4);
+    else dequant_row_batches_<BITS, 1, SAT>(wst, m, r, at, ru * GB, lo - g * 4);
   }
+}
+template <int BITS, int UG, int NBW, int KH>
+__device__ __forceinline__ bool part_may_overflow(const uint32_t* mt, int r) {
+  bool any = false;
+#pragma unroll
+  for (int g = 0; g < UG; ++g) {
+    constexpr int b = KH * NBW, e = KH * NBW + NBW;
+    if (g * 4 >= e || (g + 1) * 4 <= b) continue;
+    any |= group_may_overflow<BITS>(mt[((r >> 4) * UG + g) * 16 + (r & 15)]);
+  }
+  return any;
+}
+template <int BITS, int UG, int NBW, int KH>
+__device__ __forceinline__ void dequant_part_vote(const uint8_t* wst, const uint32_t* mt, int r, uint32_t a_tm) {
+  // warp-uniform choice: tcgen05.st is .sync.aligned, so every lane must take the same variant
+  if (__builtin_expect(__any_sync(0xffffffffu, part_may_overflow<BITS, UG, NBW, KH>(mt, r)), 0))
+    dequant_part<BITS, UG, NBW, true, KH>(wst, mt, r, a_tm);
+  else
+    dequant_part<BITS, UG, NBW, false, KH>(wst, mt, r, a_tm);
+}
+template <int BITS, int UG, int NBW, int KHN>
+__device__ __forceinline__ void dequant_warp_range(const uint8_t* wst, const uint32_t* mt, int r, uint32_t a_tm, int kh) {
+  static_assert(KHN == 2, "two k-parts per unit");
+  if (kh == 0) dequant_part_vote<BITS, UG, NBW, 0>(wst, mt, r, a_tm);
+  else dequant_part_vote<BITS, UG, NBW, 1>(wst, mt, r, a_tm);
 }
 
 template <int EPI>
@@ -403,7 +427,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       const uint32_t* mt = reinterpret_cast<const uint32_t*>(smem + SM::OFF_META + sw * BN * 4 * UG);
       const uint32_t a_tm = tmem + lane_base + A_COL + sa * DCfg<BITS, UG>::A_SLOT;
       const uint8_t* wst = smem + SM::OFF_W + sw * SM::W_STAGE;
-      if constexpr (BITS != 16) dequant_warp_range<BITS, UG, NBW>(wst, mt, r, a_tm, kh);
+      if constexpr (BITS != 16) dequant_warp_range<BITS, UG, NBW, DQ_KH>(wst, mt, r, a_tm, kh);
       if (tr) trace_ev(p, 12, i);
       tc_wait_st();
       tc_fence_before();
