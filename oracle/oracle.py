@@ -59,6 +59,9 @@ def _lib() -> ctypes.CDLL:
         L.oq_packed_bytes.restype = ctypes.c_size_t
         L.oq_attention.argtypes = [P, I64, I64, I64, I64, I64, ctypes.c_int, P, P, I64, P]
         L.oq_stage_attn.argtypes = [P, ctypes.c_int, P, I64, I64, I64, I64, I64, ctypes.c_int, I64, I64, P, P]
+        L.oq_quantize_w8_channel.argtypes = [P, I64, I64, P, P]
+        L.oq_quantize_act8.argtypes = [P, I64, I64, P, P]
+        L.oq_linear_w8a8.argtypes = [P, P, I64, I64, P, P, I64, P, P, P]
         L.oq_set_threads.argtypes = [ctypes.c_int]
         L.oq_set_threads.restype = None
         L.oq_max_threads.restype = ctypes.c_int
@@ -320,3 +323,38 @@ def pipeline_attn(layers: list[Layer], x0: np.ndarray, n_decode: int, n_heads: i
         e = layernorm(out[:, t - 1])
         out[:, t] = stage_attn(layers, e, B, 1, s + t - 1, 0, n_heads, cache)
     return out
+
+
+# ---------------------------------------------------------------- O9: W8A8 (f4)
+def quantize_w8_channel(w: np.ndarray):
+    """R26: symmetric per-output-channel INT8 weights -> (codes int8 [n,k], scales fp16 [n])."""
+    w = np.ascontiguousarray(w, np.float16)
+    n, k = w.shape
+    q = np.empty((n, k), np.int8)
+    s = np.empty(n, np.float16)
+    _check(_lib().oq_quantize_w8_channel(_p(w), n, k, _p(q), _p(s)), "quantize_w8")
+    return q, s
+
+
+def quantize_act8(x: np.ndarray):
+    """R26: symmetric per-token INT8 activations -> (codes int8 [m,k], scales fp32 [m])."""
+    x = np.ascontiguousarray(x, np.float16)
+    m, k = x.shape
+    q = np.empty((m, k), np.int8)
+    s = np.empty(m, np.float32)
+    _check(_lib().oq_quantize_act8(_p(x), m, k, _p(q), _p(s)), "quantize_act8")
+    return q, s
+
+
+def linear_w8a8(xq, sx, wq, sw, bias=None):
+    """O9: exact integer accumulation, y = acc * s_x * s_w (+ bias) in fp64 -> (y [m,n] fp64, acc int64)."""
+    xq = np.ascontiguousarray(xq, np.int8)
+    wq = np.ascontiguousarray(wq, np.int8)
+    m, k = xq.shape
+    n = wq.shape[0]
+    acc = np.empty((m, n), np.int64)
+    y = np.empty((m, n), np.float64)
+    b = None if bias is None else np.ascontiguousarray(bias, np.float16)
+    _check(_lib().oq_linear_w8a8(_p(xq), _p(np.ascontiguousarray(sx, np.float32)), m, k, _p(wq),
+                                 _p(np.ascontiguousarray(sw, np.float16)), n, _p(b), _p(acc), _p(y)), "linear_w8a8")
+    return y, acc

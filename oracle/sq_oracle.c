@@ -457,3 +457,60 @@ int oq_stage_attn(const oq_layer* layers, int n_layers, double* x, int64_t nseq,
   free(u);
   return err;
 }
+
+/* ---------------- O9: W8A8 (weight-activation INT8; P:93 SmoothQuant / bitsandbytes) ------------
+ * Reading R26: weights symmetric per output channel, activations symmetric per token (dynamic),
+ * no smoothing factor; codes against the stored scale, fp32 single-rounded ops, ties to even:
+ *   s_w[n] = fp16(fp32(max_k |W[n,k]|) / 127),  q_w = clamp(rint(fp32(W) / s_w), -127, 127)   (s_w == 0 -> 0)
+ *   s_x[t] = fp32(max_k |x[t,k]|) / 127 (kept fp32),  q_x = clamp(rint(fp32(x) / s_x), -127, 127)
+ *   acc[t,n] = sum_k q_x q_w (exact integer),  y = acc * s_x[t] * s_w[n] (+ bias) in fp64.
+ */
+static float rint_clamp127(float d) {
+  float q = rintf(d);
+  if (q < -127.0f) q = -127.0f;
+  if (q > 127.0f) q = 127.0f;
+  return q;
+}
+
+int oq_quantize_w8_channel(const uint16_t* w, int64_t n, int64_t k, int8_t* codes, uint16_t* scales) {
+  for (int64_t r = 0; r < n; ++r) {
+    float amax = 0.0f;
+    for (int64_t j = 0; j < k; ++j) {
+      const float a = fabsf(h2f(w[r * k + j]));
+      if (a > amax) amax = a;
+    }
+    const uint16_t s16 = f2h(amax / 127.0f);
+    const float s = h2f(s16);
+    scales[r] = s16;
+    for (int64_t j = 0; j < k; ++j) codes[r * k + j] = (int8_t)(s == 0.0f ? 0 : (int)rint_clamp127(h2f(w[r * k + j]) / s));
+  }
+  return 0;
+}
+
+int oq_quantize_act8(const uint16_t* x, int64_t m, int64_t k, int8_t* codes, float* scales) {
+  for (int64_t t = 0; t < m; ++t) {
+    float amax = 0.0f;
+    for (int64_t j = 0; j < k; ++j) {
+      const float a = fabsf(h2f(x[t * k + j]));
+      if (a > amax) amax = a;
+    }
+    const float s = amax / 127.0f;
+    scales[t] = s;
+    for (int64_t j = 0; j < k; ++j) codes[t * k + j] = (int8_t)(s == 0.0f ? 0 : (int)rint_clamp127(h2f(x[t * k + j]) / s));
+  }
+  return 0;
+}
+
+int oq_linear_w8a8(const int8_t* xq, const float* sx, int64_t m, int64_t k, const int8_t* wq, const uint16_t* sw,
+                   int64_t n, const uint16_t* bias, int64_t* acc_out, double* y) {
+#pragma omp parallel for schedule(static)
+  for (int64_t j = 0; j < n; ++j) {
+    for (int64_t t = 0; t < m; ++t) {
+      int64_t acc = 0;
+      for (int64_t kk = 0; kk < k; ++kk) acc += (int64_t)xq[t * k + kk] * (int64_t)wq[j * k + kk];
+      if (acc_out) acc_out[t * n + j] = acc;
+      y[t * n + j] = (double)acc * (double)sx[t] * (double)h2f(sw[j]) + (bias ? (double)h2f(bias[j]) : 0.0);
+    }
+  }
+  return 0;
+}
