@@ -240,6 +240,28 @@ sq_status sq_stage_forward_attn(const sq_layer* layers, int n_layers, int phase,
                                 const float* x_in_dev, int64_t tokens, float* x_out_dev, void* ws_dev,
                                 size_t ws_bytes, sq_stream_t stream);
 
+/* ------------------------------------------------------------------------
+ * f4 — W8A8 linear (weight-activation INT8, P:93 SmoothQuant / bitsandbytes; R26):
+ *   weights symmetric per output channel: s_w[n] = fp16(max_k |W[n,k]| / 127),
+ *     q_w = clamp(rint(W / s_w), -127, 127) int8;
+ *   activations symmetric per token (dynamic): s_x[t] = max_k |x[t,k]| / 127 (fp32),
+ *     q_x = clamp(rint(x / s_x), -127, 127) int8;     (fp32 single-rounded ops, ties to even)
+ *   acc = sum_k q_x q_w (exact int32 on tcgen05 kind::i8),  y = acc * s_x[t] * s_w[n] (+ bias).
+ * Codes and scales are bit-exact with the oracle; acc is exact (mode SQ_W8A8_I32 returns it).
+ * ------------------------------------------------------------------------ */
+enum { SQ_W8A8_I32 = 4 };   /* mode: raw int32 accumulator y_dev [m][n] (epilogue modes 0..3 as SQ_EPI_*) */
+sq_status sq_quantize_w8(const void* w_dev /* fp16 [n,k] */, int64_t n, int64_t k, int8_t* codes_dev /* [n,k] */,
+                         void* scales_f16_dev /* [n] */, sq_stream_t stream);
+sq_status sq_quantize_act8(const void* x_dev /* fp16 [m, ldx] */, int64_t m, int64_t k, int64_t ldx,
+                           int8_t* codes_dev /* [m,k] */, float* scales_dev /* [m] */, sq_stream_t stream);
+size_t sq_linear_w8a8_workspace_bytes(int64_t n, int64_t k, int64_t m);   /* split-k int32 partials (0: none) */
+/* n, k multiples of 128; codes 16-B aligned; y fp16 / fp32 [m, ldy] by mode (SQ_EPI_F16, _RELU, _GELU,
+ * _F32_ACCUM) or int32 [m, n] (SQ_W8A8_I32).  Narrow grids (decode) split k over Z CTAs whose exact int32
+ * partials a second kernel sums (order-independent: deterministic). */
+sq_status sq_linear_w8a8(const int8_t* wq_dev, const void* sw_f16_dev, const void* bias_f16_dev, int64_t n, int64_t k,
+                         const int8_t* xq_dev, const float* sx_dev, int64_t m, void* y_dev, int64_t ldy, int mode,
+                         void* ws_dev, size_t ws_bytes, sq_stream_t stream);
+
 /* Loop-back glue (R14): out_row = x (fp32 copy) and e = LN(x) for the next decode step. */
 sq_status sq_layernorm_f32(const float* x_dev, int64_t rows, int64_t d, float* y_dev,
                            sq_stream_t stream);

@@ -108,7 +108,8 @@ EXPORTED = [
     "sq_pipeline_workspace_bytes", "sq_pipeline_run", "sq_plan_check", "sq_profile_enable", "sq_profile_read",
     "sq_launch_count", "sq_pipeline_schedule", "sq_scale_sq_sums_workspace_bytes", "sq_scale_sq_sums",
     "sq_act_moments_workspace_bytes", "sq_act_moments", "sq_quantize_groups_ex", "sq_attention",
-    "sq_stage_forward_attn",
+    "sq_stage_forward_attn", "sq_quantize_w8", "sq_quantize_act8", "sq_linear_w8a8_workspace_bytes",
+    "sq_linear_w8a8",
 ]
 
 
@@ -121,6 +122,10 @@ _opt("sq_stage_workspace_bytes", ctypes.c_size_t, ctypes.POINTER(sq_layer), ctyp
 _opt("sq_stage_forward", ctypes.c_int, ctypes.POINTER(sq_layer), ctypes.c_int, ctypes.c_int, P, I64, P, P, P,
      ctypes.c_size_t, P)
 _opt("sq_layernorm_f32", ctypes.c_int, P, I64, I64, P, P)
+_opt("sq_quantize_w8", ctypes.c_int, P, I64, I64, P, P, P)
+_opt("sq_quantize_act8", ctypes.c_int, P, I64, I64, I64, P, P, P)
+_opt("sq_linear_w8a8_workspace_bytes", ctypes.c_size_t, I64, I64, I64)
+_opt("sq_linear_w8a8", ctypes.c_int, P, P, P, I64, I64, P, P, I64, P, I64, ctypes.c_int, P, ctypes.c_size_t, P)
 _opt("sq_attention", ctypes.c_int, P, I64, I64, I64, I64, I64, I64, ctypes.c_int, P, P, I64, I64, P, I64, P)
 _opt("sq_stage_forward_attn", ctypes.c_int, ctypes.POINTER(sq_layer), ctypes.c_int, ctypes.c_int,
      ctypes.POINTER(sq_attn), P, I64, P, P, ctypes.c_size_t, P)
@@ -312,3 +317,44 @@ def sq_attention(qkv: torch.Tensor, nseq: int, length: int, pos0: int, seq0: int
     _check(_L.sq_attention(_ptr(qkv), qkv.stride(0), nseq, length, pos0, seq0, h1, n_heads, _ptr(k_cache),
                            _ptr(v_cache), k_cache.shape[1], k_cache.shape[0], _ptr(out), out.stride(0), _stream(stream)))
     return out
+
+
+# ---------------------------------------------------------------- f4: W8A8
+SQ_W8A8_I32 = 4
+
+
+class W8Linear:
+    """W8A8 linear (include/sq.h): int8 codes [n, k] + fp16 per-channel scales (+ fp16 bias)."""
+
+    def __init__(self, codes: torch.Tensor, scales: torch.Tensor, bias: torch.Tensor | None = None):
+        self.codes, self.scales, self.bias = codes, scales, bias
+        self.n, self.k = codes.shape
+
+    @classmethod
+    def from_fp16(cls, w: torch.Tensor, bias: torch.Tensor | None = None, stream=None) -> "W8Linear":
+        assert w.is_cuda and w.dtype == torch.float16 and w.is_contiguous()
+        n, k = w.shape
+        q = torch.empty((n, k), dtype=torch.int8, device=w.device)
+        s = torch.empty(n, dtype=torch.float16, device=w.device)
+        _check(_L.sq_quantize_w8(_ptr(w), n, k, _ptr(q), _ptr(s), _stream(stream)))
+        return cls(q, s, bias)
+
+
+def sq_quantize_act8(x: torch.Tensor, stream=None):
+    m, k = x.shape
+    q = torch.empty((m, k), dtype=torch.int8, device=x.device)
+    s = torch.empty(m, dtype=torch.float32, device=x.device)
+    _check(_L.sq_quantize_act8(_ptr(x), m, k, x.stride(0), _ptr(q), _ptr(s), _stream(stream)))
+    return q, s
+
+
+def sq_linear_w8a8(w: W8Linear, xq: torch.Tensor, sx: torch.Tensor, y: torch.Tensor, mode: int = SQ_EPI_F16,
+                   ws: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    m = xq.shape[0]
+    need = int(_L.sq_linear_w8a8_workspace_bytes(w.n, w.k, m))
+    if need and (ws is None or ws.numel() < need):
+        ws = torch.empty(need, dtype=torch.uint8, device=xq.device)
+    _check(_L.sq_linear_w8a8(_ptr(w.codes), _ptr(w.scales), _ptr(w.bias), w.n, w.k, _ptr(xq), _ptr(sx), m, _ptr(y),
+                             y.stride(0) if mode != SQ_W8A8_I32 else w.n, mode, _ptr(ws) if need else None,
+                             need, _stream(stream)))
+    return y

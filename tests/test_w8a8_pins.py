@@ -107,3 +107,77 @@ def test_grid_aligned_is_exact_and_error_bound():
     bound = (np.abs(X).sum(1)[:, None] * SW[None, :] / 2 + SX[:, None] * np.abs(W).sum(1)[None, :] / 2
              + 384 * SX[:, None] * SW[None, :] / 4)
     assert (np.abs(y - X @ W.T) <= bound * (1 + 1e-9)).all()
+
+
+# ---------------------------------------------------------------- GPU parity (kind::i8 tensor cores)
+def _sq():
+    import paper_conf_cluster_zhaowplw25_b200 as sq
+    return sq
+
+
+@pytest.mark.gpu
+def test_gpu_w8a8_codes_bit_exact():
+    import torch
+    sq = _sq()
+    w = synth.adversarial_weight_f16(9, 256, 640)
+    x = synth.act_f16(10, 37, 640)
+    x[5] = np.float16(0.0)
+    qw, sw = O.quantize_w8_channel(w)
+    qx, sx = O.quantize_act8(x)
+    g = sq.W8Linear.from_fp16(torch.from_numpy(w).cuda())
+    gx, gs = sq.sq_quantize_act8(torch.from_numpy(x).cuda())
+    assert np.array_equal(g.codes.cpu().numpy(), qw) and np.array_equal(g.scales.cpu().numpy().view(np.uint16), sw.view(np.uint16))
+    assert np.array_equal(gx.cpu().numpy(), qx) and np.array_equal(gs.cpu().numpy().view(np.uint32), sx.view(np.uint32))
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("m", [1, 5, 32, 33, 100, 300])
+@pytest.mark.parametrize("n,k", [(256, 640), (1024, 4096), (128, 128)])
+def test_gpu_w8a8_accumulator_exact(m, n, k):
+    """the int32 accumulator of tcgen05 kind::i8 equals the oracle's integer sum exactly (every tile
+    size BT = 32..256, split-k for narrow grids, ragged token tiles)"""
+    import torch
+    sq = _sq()
+    rng = np.random.default_rng(m * 7 + n)
+    qx = rng.integers(-127, 128, size=(m, k)).astype(np.int8)
+    qw = rng.integers(-127, 128, size=(n, k)).astype(np.int8)
+    sx = np.ones(m, np.float32)
+    sw = np.ones(n, np.float16)
+    _, acc = O.linear_w8a8(qx, sx, qw, sw)
+    g = sq.W8Linear(torch.from_numpy(qw).cuda(), torch.from_numpy(sw).cuda())
+    y = torch.empty((m, n), dtype=torch.int32, device="cuda")
+    sq.sq_linear_w8a8(g, torch.from_numpy(qx).cuda(), torch.from_numpy(sx).cuda(), y, sq.SQ_W8A8_I32)
+    torch.cuda.synchronize()
+    assert np.array_equal(y.cpu().numpy().astype(np.int64), acc)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("mode", [0, 1, 2, 3])
+@pytest.mark.parametrize("m", [3, 32, 300])
+def test_gpu_w8a8_linear_epilogues(mode, m):
+    import torch
+    sq = _sq()
+    n, k = 384, 1280
+    w = synth.weight_f16(20, n, k)
+    b = synth.bias_f16(21, n)
+    x = synth.act_f16(22 + m, m, k)
+    qw, sw = O.quantize_w8_channel(w)
+    qx, sx = O.quantize_act8(x)
+    ref, _ = O.linear_w8a8(qx, sx, qw, sw, b)
+    if mode == 1:
+        ref = np.maximum(ref, 0)
+    elif mode == 2:
+        ref = 0.5 * ref * (1 + np.tanh(np.sqrt(2 / np.pi) * (ref + 0.044715 * ref ** 3)))
+    g = sq.W8Linear.from_fp16(torch.from_numpy(w).cuda(), torch.from_numpy(b).cuda())
+    gx, gs = sq.sq_quantize_act8(torch.from_numpy(x).cuda())
+    if mode == 3:
+        y0 = synth.hidden_f32(23, m, n)
+        y = torch.from_numpy(y0.copy()).cuda()
+        sq.sq_linear_w8a8(g, gx, gs, y, mode)
+        got = y.cpu().numpy().astype(np.float64) - y0
+    else:
+        y = torch.empty((m, n), dtype=torch.float16, device="cuda")
+        sq.sq_linear_w8a8(g, gx, gs, y, mode)
+        got = y.float().cpu().numpy()
+    torch.cuda.synchronize()
+    assert np.abs(got - ref).max() / np.abs(ref).max() <= 2e-3
