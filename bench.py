@@ -277,6 +277,55 @@ def gemv_sweep(n_launch=40, ms=(1, 2, 4, 8, 16, 32), bit_list=(3, 4, 8, 16)):
     return out
 
 
+def w8a8_decode_sweep(n_launch=40, ms=(1, 32)):
+    """f4 W8A8 at configs[1] shapes: per launch the per-token activation quantization + the kind::i8
+    linear (split-k + integer reduce for narrow grids), R weight copies > 2 x L2, one CUDA graph of
+    n_launch launches, best of 3.  GB/s = weight bytes (n k codes + 2 n scales) / time per launch."""
+    import torch
+    import synth
+    import paper_conf_cluster_zhaowplw25_b200 as sq
+    pk = peaks()
+    l2 = torch.cuda.get_device_properties(0).L2_cache_size
+    out = []
+    for (n, k) in ((5120, 5120), (20480, 5120), (5120, 20480)):
+        wd = torch.empty((n, k), dtype=torch.float16, device="cuda")
+        synth.device_weight_f16(wd.data_ptr(), 4243, n, k)
+        w0 = sq.W8Linear.from_fp16(wd)
+        nbytes = n * k + 2 * n
+        R = max(2, int(2 * l2 // nbytes) + 2)
+        ws = [w0] + [sq.W8Linear(w0.codes.clone(), w0.scales.clone()) for _ in range(R - 1)]
+        for m in ms:
+            x = torch.randn(m, k, device="cuda").half()
+            y = torch.empty(m, n, device="cuda", dtype=torch.float16)
+            wsb = torch.empty(max(1, int(sq.lib().sq_linear_w8a8_workspace_bytes(n, k, m))), dtype=torch.uint8, device="cuda")
+            for i in range(R):
+                xq, sx = sq.sq_quantize_act8(x)
+                sq.sq_linear_w8a8(ws[i], xq, sx, y, 0, ws=wsb)
+            torch.cuda.synchronize()
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g):
+                for i in range(n_launch):
+                    xq, sx = sq.sq_quantize_act8(x)
+                    sq.sq_linear_w8a8(ws[i % R], xq, sx, y, 0, ws=wsb)
+            g.replay()
+            torch.cuda.synchronize()
+            best = float("inf")
+            for _ in range(3):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                g.replay()
+                e1.record()
+                torch.cuda.synchronize()
+                best = min(best, e0.elapsed_time(e1))
+            us = best * 1e3 / n_launch
+            gbs = nbytes / us / 1e3
+            out.append({"n": n, "k": k, "bits": "w8a8", "m": m, "us": round(us, 2), "GBps": round(gbs, 1),
+                        "frac": round(gbs / pk["hbm_gbs"], 3)})
+            del g
+        del ws, w0, wd
+    return out
+
+
 # ------------------------------------------------------------------ our arm
 def run_ours(args, wl):
     import torch
@@ -450,7 +499,7 @@ def run_ours(args, wl):
     if rank == 0 and P == 1:
         if not args.no_gemv_sweep:
             extra["decode_gemv"] = {"workload": "configs[1] OPT-13B linear shapes, m = 1..32, bits 3/4/8 (+16); 40 back-to-back launches over > 2 x L2 of distinct weight copies in one CUDA graph, best of 3",
-                                    "results": gemv_sweep()}
+                                    "results": gemv_sweep(), "w8a8": w8a8_decode_sweep()}
         if not args.no_gemm_sweep:
             extra["prefill_gemm"] = {"workload": "configs[2] OPT-30B linear shapes (fused qkv 21504x7168, o 7168^2, fc1 28672x7168, fc2 7168x28672) at M = 8 x 512 = 4096 tokens, bits 3/4/8/16; median of 5 event-timed launches after 2 warm-up",
                                      "results": gemm_sweep(pk)}
@@ -549,6 +598,24 @@ def gemm_sweep(pk: dict, reps: int = 5):
                         "TFLOPs": round(tf, 1), "frac_burst": round(tf / pk["tflops"], 3),
                         "frac_sustained": round(tf / pk["tflops_sustained"], 3)})
             del q
+        # f4 W8A8 (kind::i8 tensor cores, per-token activation quantization included in the timing);
+        # INT8 dense peak = the measured bf16 peak x 2 (the guide's nominal ratio)
+        w8 = sq.W8Linear.from_fp16(wd)
+        ts = []
+        for r in range(2 + reps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            xq, sx = sq.sq_quantize_act8(xk)
+            sq.sq_linear_w8a8(w8, xq, sx, y, 0)
+            e1.record()
+            torch.cuda.synchronize()
+            if r >= 2:
+                ts.append(e0.elapsed_time(e1))
+        ms = statistics.median(ts)
+        tf = 2.0 * M * n * k / (ms / 1e3) / 1e12
+        out.append({"linear": name, "n": n, "k": k, "bits": "w8a8", "m": M, "us": round(ms * 1e3, 1), "TFLOPs": round(tf, 1),
+                    "frac_int8_peak": round(tf / (2 * pk["tflops"]), 3), "peak_note": "int8 dense = 2 x measured bf16 (burst)"})
+        del w8
         del wd, xk, y
     return out
 
