@@ -3,7 +3,7 @@
 //
 //   K6  kv_append   new tokens' k, v (columns [h1, 3 h1) of the fused qkv rows) -> the layer's cache
 //                   K / V [n_seq][max_len][h1] fp16 at (seq0 + i, pos0 + j).  HBM-bound copy.
-//   K7  attn_prefill  FlashAttention-2 style, one CTA per (sequence, head, 64-query block): Q in
+//   K7  attn_prefill  FlashAttention-2 style, one CTA per (sequence, head, 128-query block): Q in
 //                   registers, 64-key K / V blocks of the cache double-buffered in shared memory
 //                   (cp.async, zero-filled beyond the last visible key), S = Q K^T and O += P V on
 //                   mma.sync m16n8k16 (fp16 in, fp32 accumulate), online softmax in fp32 (exp2).
@@ -56,13 +56,24 @@ __device__ __forceinline__ uint32_t pack_h2(float a, float b) {
 
 template <int DH>
 struct PreCfg {
-  static constexpr int BQ = 64, BK = 64, LD = DH + 8;  // padded rows: conflict-free fragment loads
+  static constexpr int BQ = 128, BK = 64, LD = DH + 8;  // padded rows: conflict-free fragment loads
+  static constexpr int THREADS = 32 * (BQ / 16);        // one warp per 16 query rows
   static constexpr int BLK = BK * LD;                   // halves per K or V block
   static constexpr int SMEM = 2 * 2 * BLK * 2;          // 2 stages x (K + V) x fp16
 };
 
+__device__ __forceinline__ float ex2(float x) {
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+__device__ __forceinline__ void ldsm_x4(uint32_t& r0, uint32_t& r1, uint32_t& r2, uint32_t& r3, const void* p) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x4.shared.b16 {%0, %1, %2, %3}, [%4];"
+               : "=r"(r0), "=r"(r1), "=r"(r2), "=r"(r3) : "r"(smem_u32(p)));
+}
+
 template <int DH>
-__global__ void __launch_bounds__(128) k_attn_prefill(const __half* __restrict__ qkv, int64_t ldq, int len, int pos0,
+__global__ void __launch_bounds__(PreCfg<DH>::THREADS) k_attn_prefill(const __half* __restrict__ qkv, int64_t ldq, int len, int pos0,
                                                       int64_t seq0, int h1, const __half* __restrict__ kc,
                                                       const __half* __restrict__ vc, int max_len,
                                                       __half* __restrict__ out, int64_t ldo, float qscale) {
@@ -80,7 +91,7 @@ __global__ void __launch_bounds__(128) k_attn_prefill(const __half* __restrict__
     __half* ks = sm + st * 2 * C::BLK;
     __half* vs = ks + C::BLK;
     constexpr int CH = DH / 8;  // 16-B chunks per row
-    for (int c = threadIdx.x; c < C::BK * CH; c += 128) {
+    for (int c = threadIdx.x; c < C::BK * CH; c += C::THREADS) {
       const int r = c / CH, cc = (c % CH) * 8, j = kb * C::BK + r;
       const bool ok = j <= last_key;
       const int64_t off = (int64_t)(ok ? j : 0) * h1 + cc;
@@ -121,14 +132,18 @@ __global__ void __launch_bounds__(128) k_attn_prefill(const __half* __restrict__
     // S = Q K^T: 16 x 64 per warp (8 n-tiles of 8 keys)
     float s[8][4];
 #pragma unroll
-    for (int n = 0; n < 8; ++n) {
-      s[n][0] = s[n][1] = s[n][2] = s[n][3] = 0.f;
-      const __half* kr = ks + (n * 8 + g) * C::LD + 2 * t;
+    for (int n = 0; n < 8; ++n) s[n][0] = s[n][1] = s[n][2] = s[n][3] = 0.f;
+    // B fragments of two 8-key n-tiles per ldmatrix.x4: matrices (keys n0..+7 | k 0-7), (n0 | k 8-15),
+    // (n0+8 | k 0-7), (n0+8 | k 8-15) -> b0/b1 of tile n, b0/b1 of tile n+1
+    const __half* kbl = ks + ((lane & 7) + ((lane >> 4) & 1) * 8) * C::LD + ((lane >> 3) & 1) * 8;
+#pragma unroll
+    for (int n = 0; n < 8; n += 2) {
 #pragma unroll
       for (int kk = 0; kk < DH / 16; ++kk) {
-        const uint32_t b0 = *reinterpret_cast<const uint32_t*>(kr + kk * 16);
-        const uint32_t b1 = *reinterpret_cast<const uint32_t*>(kr + kk * 16 + 8);
+        uint32_t b0, b1, b2, b3;
+        ldsm_x4(b0, b1, b2, b3, kbl + n * 8 * C::LD + kk * 16);
         mma_16816(s[n], qa[kk], b0, b1, s[n]);
+        mma_16816(s[n + 1], qa[kk], b2, b3, s[n + 1]);
       }
     }
     // scale (log2 domain), causal mask, online softmax per row
@@ -149,15 +164,15 @@ __global__ void __launch_bounds__(128) k_attn_prefill(const __half* __restrict__
     mx_hi = fmaxf(mx_hi, __shfl_xor_sync(0xffffffffu, mx_hi, 2));
     // rows with no visible key yet keep -inf: use 0 as the reference so exp2 gives 0, not NaN
     const float ref_lo = mx_lo == -INFINITY ? 0.f : mx_lo, ref_hi = mx_hi == -INFINITY ? 0.f : mx_hi;
-    const float corr_lo = exp2f(m_lo - ref_lo), corr_hi = exp2f(m_hi - ref_hi);
+    const float corr_lo = ex2(m_lo - ref_lo), corr_hi = ex2(m_hi - ref_hi);
     m_lo = mx_lo;
     m_hi = mx_hi;
     float sum_lo = 0.f, sum_hi = 0.f;
     uint32_t pa[4][4];  // P as A fragments: keys 16 kk .. 16 kk + 15
 #pragma unroll
     for (int n = 0; n < 8; ++n) {
-      const float e0 = exp2f(s[n][0] - ref_lo), e1 = exp2f(s[n][1] - ref_lo);
-      const float e2 = exp2f(s[n][2] - ref_hi), e3 = exp2f(s[n][3] - ref_hi);
+      const float e0 = ex2(s[n][0] - ref_lo), e1 = ex2(s[n][1] - ref_lo);
+      const float e2 = ex2(s[n][2] - ref_hi), e3 = ex2(s[n][3] - ref_hi);
       sum_lo += e0 + e1;
       sum_hi += e2 + e3;
       const int kk = n >> 1, hi = n & 1;
@@ -339,13 +354,18 @@ cudaError_t launch_attention(const __half* qkv, int64_t ldq, int nseq, int len, 
     if (dh == 128) launch_pdl(k_attn_decode<128>, grid, dim3(128), 0, s, qkv, ldq, pos0, seq0, h1, (const __half*)kc, (const __half*)vc, max_len, out, ldo, qscale);
     else launch_pdl(k_attn_decode<64>, grid, dim3(128), 0, s, qkv, ldq, pos0, seq0, h1, (const __half*)kc, (const __half*)vc, max_len, out, ldo, qscale);
   } else {
-    dim3 grid((len + 63) / 64, n_heads, nseq);
     if (dh == 128) {
+      using C = PreCfg<128>;
       static bool set = false;
-      if (!set) { cudaFuncSetAttribute(k_attn_prefill<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, PreCfg<128>::SMEM); set = true; }
-      k_attn_prefill<128><<<grid, 128, PreCfg<128>::SMEM, s>>>(qkv, ldq, len, pos0, seq0, h1, kc, vc, max_len, out, ldo, qscale);
+      if (!set) { cudaFuncSetAttribute(k_attn_prefill<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM); set = true; }
+      dim3 grid((len + C::BQ - 1) / C::BQ, n_heads, nseq);
+      k_attn_prefill<128><<<grid, C::THREADS, C::SMEM, s>>>(qkv, ldq, len, pos0, seq0, h1, kc, vc, max_len, out, ldo, qscale);
     } else {
-      k_attn_prefill<64><<<grid, 128, PreCfg<64>::SMEM, s>>>(qkv, ldq, len, pos0, seq0, h1, kc, vc, max_len, out, ldo, qscale);
+      using C = PreCfg<64>;
+      static bool set = false;
+      if (!set) { cudaFuncSetAttribute(k_attn_prefill<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM); set = true; }
+      dim3 grid((len + C::BQ - 1) / C::BQ, n_heads, nseq);
+      k_attn_prefill<64><<<grid, C::THREADS, C::SMEM, s>>>(qkv, ldq, len, pos0, seq0, h1, kc, vc, max_len, out, ldo, qscale);
     }
   }
   prof_end(t, s);
