@@ -158,9 +158,10 @@ int oq_quantize_groups(const uint16_t* w, int64_t n, int64_t k, int bits, int gr
  * L8: byte j = c_j.
  * L4: 32-bit little-endian word j/8, nibble (j%8)/2 + 4*(j%2)   (even j in the low
  *     four nibbles, odd j in the high four).
- * L3: blocks of 32 codes = 3 words [L0, L1, H]; for j' = j%32: a = j'/16,
- *     i = (j'%16)/2, e = j'%2; low two bits at word La, bits 2i + 16e;
- *     high bit at word H, bit i + 8a + 16e.
+ * L3 (reading R8, round 2): blocks of 32 codes = 3 words W0..W2; for j' = j%32: pair i = j'/2,
+ *     half e = j'%2 (even k in the low 16 bits, odd k in the high 16 bits).  Pairs i < 15: word
+ *     W_{i/5}, bits 16e + 3(i%5) .. +2 (five 3-bit codes per half).  Pair 15 (j' = 30, 31): code
+ *     bit b at bit 15 + 16e of word W_b (the three spare bits of each half).
  * T16 (placement): rows are grouped in tiles of 16; the 16 rows' bytes of group g of
  *     tile t form one contiguous chunk ("unit") at byte ((t*kg + g)*16 + r%16)*GB,
  *     kg = k/128, units ordered tile-major / group-minor.
@@ -192,14 +193,16 @@ int oq_pack(const uint8_t* codes, const uint16_t* scales, const uint16_t* zeros,
         memcpy(grp + 4 * wi, &word, 4);
       } else {
         int64_t blk = j / 32;
-        int kp = (int)(j % 32), a = kp / 16, i = (kp % 16) / 2, e = kp % 2;
-        uint32_t lw, hw;
-        memcpy(&lw, grp + 4 * (3 * blk + a), 4);
-        memcpy(&hw, grp + 4 * (3 * blk + 2), 4);
-        lw |= (c & 3u) << (2 * i + 16 * e);
-        hw |= ((c >> 2) & 1u) << (i + 8 * a + 16 * e);
-        memcpy(grp + 4 * (3 * blk + a), &lw, 4);
-        memcpy(grp + 4 * (3 * blk + 2), &hw, 4);
+        int kp = (int)(j % 32), i = kp / 2, e = kp % 2;
+        for (int b = 0; b < 3; ++b) {
+          int wi, bit;
+          if (i < 15) { wi = i / 5; bit = 16 * e + 3 * (i % 5) + b; }
+          else { wi = b; bit = 15 + 16 * e; }
+          uint32_t word;
+          memcpy(&word, grp + 4 * (3 * blk + wi), 4);
+          word |= ((c >> b) & 1u) << bit;
+          memcpy(grp + 4 * (3 * blk + wi), &word, 4);
+        }
       }
     }
   }
@@ -221,11 +224,17 @@ static uint32_t code_at(const uint8_t* packed, int64_t r, int64_t kk, int64_t kg
     return (word >> (4 * nib)) & 0xF;
   }
   int64_t blk = j / 32;
-  int kp = (int)(j % 32), a = kp / 16, i = (kp % 16) / 2, e = kp % 2;
-  uint32_t lw, hw;
-  memcpy(&lw, grp + 4 * (3 * blk + a), 4);
-  memcpy(&hw, grp + 4 * (3 * blk + 2), 4);
-  return ((lw >> (2 * i + 16 * e)) & 3u) | (((hw >> (i + 8 * a + 16 * e)) & 1u) << 2);
+  int kp = (int)(j % 32), i = kp / 2, e = kp % 2;
+  uint32_t c = 0;
+  for (int b = 0; b < 3; ++b) {
+    int wi, bit;
+    if (i < 15) { wi = i / 5; bit = 16 * e + 3 * (i % 5) + b; }
+    else { wi = b; bit = 15 + 16 * e; }
+    uint32_t word;
+    memcpy(&word, grp + 4 * (3 * blk + wi), 4);
+    c |= ((word >> bit) & 1u) << b;
+  }
+  return c;
 }
 
 int oq_unpack(const uint8_t* packed, int64_t n, int64_t k, int bits, uint8_t* codes) {

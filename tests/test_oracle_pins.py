@@ -164,8 +164,8 @@ def _example_codes(bits, name):
         c[0] = np.arange(128) % (1 << bits)
     elif name == "single13":
         c[0, 13] = 0xA
-    elif name == "single13_22_100":
-        c[0, 13], c[0, 22], c[0, 100] = 5, 6, 7
+    elif name == "single3":
+        c[0, 13], c[0, 22], c[0, 30], c[0, 63], c[0, 100] = 5, 6, 5, 3, 7
     elif name == "single5":
         c[0, 5] = 200
     return c
