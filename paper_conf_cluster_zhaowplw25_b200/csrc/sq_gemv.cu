@@ -103,23 +103,23 @@ __device__ __forceinline__ void frag(const uint32_t* c, int t, uint32_t& lo, uin
     lo = prmt(c[t], 0x64646464u, 0x4140u);
     hi = prmt(c[t], 0x64646464u, 0x4342u);
   } else if constexpr (BITS == 3) {
-    // L3: pair (a, i) = k' 16a + 2i (+1): low bits at La bits 2i(+16), high bit at H bit i+8a(+16).
-    // The code is assembled at mantissa bits 7..9 under exponent 2^3: half2(8 + c), exact, and
-    // the offset 8 (not 1024) keeps the per-group correction D - xoff free of cancellation.
-    const int a = t >> 2;
-    const uint32_t La = c[a], H = c[2];
-#pragma unroll
-    for (int e = 0; e < 2; ++e) {
-      const int i = 2 * (t & 3) + e;
-      const int sl = 7 - 2 * i;              // low two bits -> bits 7..8
-      const uint32_t l = sl >= 0 ? (La << sl) : (La >> (-sl));
-      const int sh = i + 8 * a - 9;          // high bit -> bit 9
-      const uint32_t hs = sh >= 0 ? (H >> sh) : (H << (-sh));
-      uint32_t s;
-      asm("lop3.b32 %0, %1, %2, %3, 0xD8;" : "=r"(s) : "r"(hs), "r"(l), "r"(0x01800180u));  // mask ? l : hs
-      const uint32_t r = lop3_and_or(s, 0x03800380u, 0x48004800u);
-      if (e == 0) lo = r; else hi = r;
-    }
+    // L3: pair i < 15 at word i/5, bits 3(i%5) (+16 for the odd code); pair 15
+    // in the spare bits 15 / 31 of the three words.  Each code is moved to mantissa bits 7..9 under
+    // exponent 2^3: half2(8 + c), exact; the offset 8 (not 1024) keeps the per-group correction
+    // D - xoff free of cancellation (ReLU inputs, measured).
+    auto pairv = [&](int i) -> uint32_t {
+      if (i < 15) {
+        const uint32_t x = c[i / 5];
+        const int sh = 7 - 3 * (i % 5);
+        return lop3_and_or(sh >= 0 ? (x << sh) : (x >> (-sh)), 0x03800380u, 0x48004800u);
+      }
+      uint32_t u;
+      asm("lop3.b32 %0, %1, %2, %3, 0xCA;" : "=r"(u) : "r"(0x00010001u), "r"(c[0] >> 15), "r"(c[1] >> 14));
+      asm("lop3.b32 %0, %1, %2, %3, 0xCA;" : "=r"(u) : "r"(0x00030003u), "r"(u), "r"(c[2] >> 13));
+      return lop3_and_or(u << 7, 0x03800380u, 0x48004800u);
+    };
+    lo = pairv(2 * t);
+    hi = pairv(2 * t + 1);
   } else {
     lo = c[2 * t];
     hi = c[2 * t + 1];

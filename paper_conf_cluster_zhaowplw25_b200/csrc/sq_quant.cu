@@ -119,7 +119,8 @@ __global__ void k_pack4(const uint8_t* __restrict__ codes, int64_t nwords, int k
   out[i] = w;
 }
 
-// L3: one thread per 32-code block -> words [L0, L1, H].
+// L3: one thread per 32-code block -> words W0..W2; code k' = 2i + e: pairs
+// i < 15 at W_{i/5} bits 16e + 3(i%5); pair 15 bit b at W_b bit 15 + 16e.
 __global__ void k_pack3(const uint8_t* __restrict__ codes, int64_t nblocks, int kg, int64_t k, uint32_t* __restrict__ out) {
   int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= nblocks) return;
@@ -128,17 +129,22 @@ __global__ void k_pack3(const uint8_t* __restrict__ codes, int64_t nblocks, int 
   const uint4* src = reinterpret_cast<const uint4*>(codes + src_row_col(unit, rr, kg, k, 32 * bl));
   uint4 a = src[0], b = src[1];
   uint32_t wv[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
-  uint32_t L[2] = {0, 0}, H = 0;
+  uint32_t W[3] = {0, 0, 0};
 #pragma unroll
-  for (int kp = 0; kp < 32; ++kp) {
-    uint32_t c = (wv[kp >> 2] >> (8 * (kp & 3))) & 0x7;
-    int aa = kp >> 4, ii = (kp & 15) >> 1, e = kp & 1;
-    L[aa] |= (c & 3u) << (2 * ii + 16 * e);
-    H |= ((c >> 2) & 1u) << (ii + 8 * aa + 16 * e);
+  for (int kp = 0; kp < 30; ++kp) {
+    const uint32_t c = (wv[kp >> 2] >> (8 * (kp & 3))) & 0x7;
+    const int pi = kp >> 1, e = kp & 1;
+    W[pi / 5] |= c << (16 * e + 3 * (pi % 5));
   }
-  out[3 * i + 0] = L[0];
-  out[3 * i + 1] = L[1];
-  out[3 * i + 2] = H;
+#pragma unroll
+  for (int e = 0; e < 2; ++e) {
+    const uint32_t c = (wv[7] >> (8 * (2 + e))) & 0x7;  // codes 30 (e = 0) and 31 (e = 1)
+#pragma unroll
+    for (int bb = 0; bb < 3; ++bb) W[bb] |= ((c >> bb) & 1u) << (15 + 16 * e);
+  }
+  out[3 * i + 0] = W[0];
+  out[3 * i + 1] = W[1];
+  out[3 * i + 2] = W[2];
 }
 
 // L8: one thread per output word (4 codes).

@@ -135,25 +135,29 @@ __device__ __forceinline__ void dequant_row_batches_(const uint8_t* wst, uint32_
       tmem_st16(taddr + 16 * b, o);
     }
   } else if constexpr (BITS == 3) {
+    // L3: per 32-code block three words; pair q of word w (q < 5) at bits 3q (q >= 3: of w >> 9, bits
+    // 3(q-3)); under magic 1024 / 128 / 16 a 3-bit field at bit 0 / 3 / 6 reads as off + c exactly;
+    // pair 15 gathered from the spare bits 15 / 31 of the three words
+    constexpr uint32_t K128 = 0x58005800u, K16 = 0x4C004C00u;
     const uint32_t* row = reinterpret_cast<const uint32_t*>(wst + (row_off >= 0 ? row_off : r * 48));
 #pragma unroll
     for (int bi = 0; bi < NB; ++bi) {
       const int bl = B0 + bi;
-      const uint32_t L0 = row[3 * bl], L1 = row[3 * bl + 1], H = row[3 * bl + 2];
+      const uint32_t W[3] = {row[3 * bl], row[3 * bl + 1], row[3 * bl + 2]};
       uint32_t o[16];
 #pragma unroll
-      for (int a = 0; a < 2; ++a) {
-        const uint32_t La = a ? L1 : L0;
-#pragma unroll
-        for (int i = 0; i < 8; ++i) {
-          const uint32_t lo = La >> (2 * i);
-          const int sh = i + 8 * a - 2;
-          const uint32_t hs = sh >= 0 ? (H >> sh) : (H << (-sh));
-          uint32_t t;
-          asm("lop3.b32 %0, %1, %2, %3, 0xD8;" : "=r"(t) : "r"(hs), "r"(lo), "r"(0x00030003u));  // mask ? lo : hs
-          o[8 * a + i] = hsub_fma<SAT>(lop3_and_or(t, 0x00070007u, K1024), K1024, s2, z2);
-        }
+      for (int w = 0; w < 3; ++w) {
+        const uint32_t x = W[w], x9 = x >> 9;
+        o[5 * w + 0] = hsub_fma<SAT>(lop3_and_or(x, 0x00070007u, K1024), K1024, s2, z2);
+        o[5 * w + 1] = hsub_fma<SAT>(lop3_and_or(x, 0x00380038u, K128), K128, s2, z2);
+        o[5 * w + 2] = hsub_fma<SAT>(lop3_and_or(x, 0x01C001C0u, K16), K16, s2, z2);
+        o[5 * w + 3] = hsub_fma<SAT>(lop3_and_or(x9, 0x00070007u, K1024), K1024, s2, z2);
+        o[5 * w + 4] = hsub_fma<SAT>(lop3_and_or(x9, 0x00380038u, K128), K128, s2, z2);
       }
+      uint32_t t;
+      asm("lop3.b32 %0, %1, %2, %3, 0xCA;" : "=r"(t) : "r"(0x00010001u), "r"(W[0] >> 15), "r"(W[1] >> 14));  // a ? b : c (bitwise)
+      asm("lop3.b32 %0, %1, %2, %3, 0xCA;" : "=r"(t) : "r"(0x00030003u), "r"(t), "r"(W[2] >> 13));
+      o[15] = hsub_fma<SAT>(lop3_and_or(t, 0x00070007u, K1024), K1024, s2, z2);
       tmem_st16(taddr + 16 * bl, o);
     }
   } else {
