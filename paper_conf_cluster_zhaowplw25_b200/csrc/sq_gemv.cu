@@ -740,9 +740,12 @@ int gemv_path(int64_t n, int64_t k, int m, int bits) {
   // has the shorter ramp -- it wins on OPT-13B-sized linears at m <= 4 (and m <= 8 off INT4),
   // the tcgen05 kernel everywhere else, and always for fp16 weights
   (void)k;
+  // (round 2, INT3 re-laid with a one-LOP3 unpack: the tcgen05 kernel wins INT3 linears from ~80 MB
+  // at every m, e.g. 36864 x 9216 at m = 1: 3.34 vs 2.89 TB/s; the mma.sync kernel keeps the OPT-13B
+  // sizes at m <= 8, e.g. 20480 x 5120: 2.24 vs 2.05 TB/s)
   if (bits == 16 || m > 8) return 1;
   const double bytes = (double)n * k * bits / 8.0;
-  if (bytes >= 120e6) return (bits == 3 && m < 8) ? 0 : 1;
+  if (bytes >= 120e6 || (bits == 3 && bytes >= 80e6)) return 1;
   return (bits == 4 && m > 4) ? 1 : 0;
 }
 
