@@ -358,3 +358,61 @@ def linear_w8a8(xq, sx, wq, sw, bias=None):
     _check(_lib().oq_linear_w8a8(_p(xq), _p(np.ascontiguousarray(sx, np.float32)), m, k, _p(wq),
                                  _p(np.ascontiguousarray(sw, np.float16)), n, _p(b), _p(acc), _p(y)), "linear_w8a8")
     return y, acc
+
+
+# ---------------------------------------------------------------- O10: tensor-parallel stage (f4)
+def tp_shard(name: str, w16: np.ndarray, bias: np.ndarray | None, r: int, T: int):
+    """R27 (P:63 intra-node TP, Megatron split): shard r of T of one fp16 linear -> (w16, bias).
+    qkv: rows [r h/T, (r+1) h/T) of each of the q, k, v blocks (h = n / 3); fc1: output rows
+    [r n/T, (r+1) n/T); o, fc2: input columns [r k/T, (r+1) k/T), bias kept by rank 0 only."""
+    n, k = w16.shape
+    if name == "qkv":
+        h = n // 3
+        s = h // T
+        rows = [np.arange(j * h + r * s, j * h + (r + 1) * s) for j in range(3)]
+        idx = np.concatenate(rows)
+        return np.ascontiguousarray(w16[idx]), None if bias is None else np.ascontiguousarray(bias[idx])
+    if name == "fc1":
+        s = n // T
+        return np.ascontiguousarray(w16[r * s:(r + 1) * s]), None if bias is None else bias[r * s:(r + 1) * s].copy()
+    s = k // T
+    return np.ascontiguousarray(w16[:, r * s:(r + 1) * s]), (None if bias is None or r != 0 else bias.copy())
+
+
+def _act(u: np.ndarray, act: int) -> np.ndarray:
+    if act == 0:
+        return np.maximum(u, 0.0)
+    return 0.5 * u * (1.0 + np.tanh(0.7978845608028654 * (u + 0.044715 * u * u * u)))
+
+
+def stage_tp(shards: list[list[Layer]], x: np.ndarray, n_heads: int = 0, nseq: int = 0, length: int = 0,
+             pos0: int = 0, seq0: int = 0, caches: list[KVCache] | None = None) -> np.ndarray:
+    """O10: one stage (the O6 layer, R11/R12) computed shard by shard under T-way TP, fp64.
+    shards[r][l] = rank r's layer l (tp_shard of every linear).  Per layer: a = LN(x); every rank
+    computes its q/k/v columns (and, with caches, attention over its n_heads / T heads and its cache of
+    width h1 / T), then its partial o-projection p_r = v_r W_o,r^T (+ bias on rank 0); x <- x + sum_r p_r;
+    a = LN(x); u_r = act(a W_1,r^T + b_1,r); x <- x + sum_r u_r W_2,r^T (+ bias on rank 0).
+    In exact arithmetic this equals O6 on the unsharded layer (the sum over r of the column blocks is the
+    full product), which is what pins it (tests/test_tp_pins.py)."""
+    T = len(shards)
+    x = np.array(x, dtype=np.float64, order="C", copy=True)
+    for l in range(len(shards[0])):
+        a = layernorm(x)
+        p = np.zeros_like(x)
+        for r in range(T):
+            L = shards[r][l]
+            qkv = linear(a, L.qkv)
+            hs = L.o.k
+            if caches is not None:
+                v = attention(qkv, nseq, length, pos0, seq0, n_heads // T, caches[r].k[l], caches[r].v[l])
+            else:
+                v = qkv[:, 2 * hs:3 * hs]
+            p += linear(v, L.o)
+        x = x + p
+        a = layernorm(x)
+        p = np.zeros_like(x)
+        for r in range(T):
+            L = shards[r][l]
+            p += linear(_act(linear(a, L.fc1), L.act), L.fc2)
+        x = x + p
+    return x
