@@ -350,6 +350,38 @@ typedef struct {
 int64_t sq_pipeline_schedule(const sq_plan* plan, int rank, sq_sched_op* ops, int64_t max_ops);
 
 /* ------------------------------------------------------------------------
+ * f4 — intra-node tensor-parallel (TP) stage ("we force intra-node TP", P:236 2-D device
+ *   meshes such as TP2+PP2, P:318 TP4 / TP2+PP2 winning on homogeneous clusters).
+ * The TP split of one decoder layer over T ranks (R27):
+ *   qkv, fc1  column-parallel: shard r holds output rows [r n/T, (r+1) n/T) of each of q, k, v
+ *             (resp. of fc1) with that bias slice -> qkv [3 h1/T, h1], fc1 [h2/T, h1];
+ *   o, fc2    row-parallel: shard r holds input columns [r k/T, (r+1) k/T) -> o [h1, h1/T],
+ *             fc2 [h1, h2/T]; the bias sits in tp rank 0's shard only (other ranks: bias NULL);
+ *   attention (attn != NULL) head-parallel: rank r owns heads [r H/T, (r+1) H/T) and a KV cache of
+ *             width h1/T (its sq_attn.n_heads = H/T).
+ * Every shard is quantized on its own; groups run along k and h1/T, h2/T are multiples of 128, so the
+ * shard codes are exactly the matching codes of the unsharded weight.
+ * Per layer on each rank: a = LN(x) (x replicated), the q/k/v and u shards, then the partial o / fc2
+ * products summed over the T ranks in place on the fp32 residual: rank 0 accumulates x + p_0 (the
+ * fused residual epilogue), ranks r > 0 write p_r into a zeroed x, and one NCCL all-reduce (sum)
+ * returns x + sum_r p_r on every rank, so the residual add costs no extra pass.
+ *   tp_rank >= 0: one rank of a T-rank NCCL group; comm from sq_comm_init(nranks = T, rank = tp_rank)
+ *                 (its world communicator carries the all-reduce); shards = this rank's n_layers
+ *                 layers; attn NULL or one context.
+ *   tp_rank == -1: virtual TP on the current device (tests, single-GPU runs of a TP plan): comm
+ *                 ignored (may be NULL); shards = [T][n_layers] rank-major; attn NULL or [T]
+ *                 contexts; the partial products accumulate into x in rank order 0..T-1
+ *                 (deterministic).
+ * x_in, x_out fp32 [tokens, h1] device (may alias); decode: tokens <= 32.  Workspace (256-B aligned)
+ * from sq_stage_tp_workspace_bytes over all the shard layers passed (n_layers * T for virtual TP).
+ * Errors: SQ_EINVAL (shard shapes inconsistent, h1 or h2 not a multiple of 128 T, heads % T, bad
+ * phase / tokens / pointers), SQ_ENOMEM (workspace), SQ_ENCCL, SQ_ECUDA. */
+size_t sq_stage_tp_workspace_bytes(const sq_layer* shards, int n_shard_layers, int64_t max_tokens);
+sq_status sq_stage_forward_tp(const sq_layer* shards, int n_layers, int tp, int tp_rank, sq_comm* comm,
+                              int phase, const sq_attn* attn, const float* x_in_dev, int64_t tokens,
+                              float* x_out_dev, void* ws_dev, size_t ws_bytes, sq_stream_t stream);
+
+/* ------------------------------------------------------------------------
  * Measurement hooks (bench.py): per-kernel-class CUDA-event timing of every
  * launch made by the library while enabled, on the launching stream.
  * class 0 = decode GEMV, 1 = prefill GEMM, 2 = glue (LN/xsum), 3 = quantize/pack,

@@ -109,7 +109,7 @@ EXPORTED = [
     "sq_launch_count", "sq_pipeline_schedule", "sq_scale_sq_sums_workspace_bytes", "sq_scale_sq_sums",
     "sq_act_moments_workspace_bytes", "sq_act_moments", "sq_quantize_groups_ex", "sq_attention",
     "sq_stage_forward_attn", "sq_quantize_w8", "sq_quantize_act8", "sq_linear_w8a8_workspace_bytes",
-    "sq_linear_w8a8",
+    "sq_linear_w8a8", "sq_stage_tp_workspace_bytes", "sq_stage_forward_tp",
 ]
 
 
@@ -129,6 +129,9 @@ _opt("sq_linear_w8a8", ctypes.c_int, P, P, P, I64, I64, P, P, I64, P, I64, ctype
 _opt("sq_attention", ctypes.c_int, P, I64, I64, I64, I64, I64, I64, ctypes.c_int, P, P, I64, I64, P, I64, P)
 _opt("sq_stage_forward_attn", ctypes.c_int, ctypes.POINTER(sq_layer), ctypes.c_int, ctypes.c_int,
      ctypes.POINTER(sq_attn), P, I64, P, P, ctypes.c_size_t, P)
+_opt("sq_stage_tp_workspace_bytes", ctypes.c_size_t, ctypes.POINTER(sq_layer), ctypes.c_int, I64)
+_opt("sq_stage_forward_tp", ctypes.c_int, ctypes.POINTER(sq_layer), ctypes.c_int, ctypes.c_int, ctypes.c_int, P,
+     ctypes.c_int, ctypes.POINTER(sq_attn), P, I64, P, P, ctypes.c_size_t, P)
 _opt("sq_comm_unique_id_bytes", ctypes.c_size_t)
 _opt("sq_comm_get_unique_id", ctypes.c_int, P)
 _opt("sq_comm_init", ctypes.c_int, ctypes.POINTER(P), P, ctypes.c_int, ctypes.c_int)

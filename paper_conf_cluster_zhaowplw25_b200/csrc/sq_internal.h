@@ -57,7 +57,13 @@ sq_status stage_forward(const sq_layer* layers, int n_layers, int phase, const f
                         float* x_out, void* qkv_dbg, void* ws, size_t ws_bytes, cudaStream_t s,
                         const sq_attn* att = nullptr);
 sq_status check_layers(const sq_layer* layers, int n_layers, const char* who);
-sq_status check_attn(const sq_attn* a, const sq_layer* layers, int n_layers, int phase, int64_t tokens, const char* who);
+sq_status check_attn(const sq_attn* a, int64_t h1, int n_layers, int phase, int64_t tokens, const char* who);
+
+// ---- TP all-reduce (sq_pipeline.cu): in-place fp32 sum over the comm's world communicator
+sq_status comm_allreduce_sum_f32(sq_comm* c, float* buf, size_t count, cudaStream_t s);
+int comm_size(const sq_comm* c);
+int comm_rank(const sq_comm* c);
+bool comm_is_local(const sq_comm* c);
 
 // ---- attention (sq_attn.cu): kv_append + prefill / decode attention for one layer
 cudaError_t launch_attention(const __half* qkv, int64_t ldq, int nseq, int len, int pos0, int64_t seq0, int h1,

@@ -244,6 +244,16 @@ std::vector<sq_sched_op> make_schedule(const PlanView& v, int rank) {
 }
 
 }  // namespace
+
+sq_status comm_allreduce_sum_f32(sq_comm* c, float* buf, size_t count, cudaStream_t s) {
+  if (!c || c->local) return fail(SQ_EINVAL, "allreduce: needs an NCCL communicator (sq_comm_init)");
+  if (c->nranks == 1) return SQ_OK;
+  return nccl_check(ncclAllReduce(buf, buf, count, ncclFloat, ncclSum, c->world, s), "ncclAllReduce");
+}
+int comm_size(const sq_comm* c) { return c ? c->nranks : 0; }
+int comm_rank(const sq_comm* c) { return c ? c->rank : -1; }
+bool comm_is_local(const sq_comm* c) { return c && c->local; }
+
 }  // namespace sq
 
 using namespace sq;

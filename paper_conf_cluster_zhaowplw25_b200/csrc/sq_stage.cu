@@ -58,9 +58,9 @@ sq_status check_w(const sq_qweight& w, int64_t n, int64_t k, int bits, const cha
 
 }  // namespace
 
-sq_status check_attn(const sq_attn* a, const sq_layer* layers, int n_layers, int phase, int64_t tokens, const char* who) {
+// h1: the width this context's heads and cache cover (the hidden size, or h1/T for a TP rank)
+sq_status check_attn(const sq_attn* a, int64_t h1, int n_layers, int phase, int64_t tokens, const char* who) {
   if (!a || !a->k_cache || !a->v_cache) return fail(SQ_EINVAL, "%s: null attention context / cache arrays", who);
-  const int64_t h1 = layers[0].o.n;
   if (a->n_heads <= 0 || h1 % a->n_heads || (h1 / a->n_heads != 64 && h1 / a->n_heads != 128))
     return fail(SQ_EINVAL, "%s: head_dim h1/n_heads must be 64 or 128", who);
   if (a->nseq < 1 || a->seq_len < 1 || (int64_t)a->nseq * a->seq_len != tokens || (phase == SQ_DECODE && a->seq_len != 1))
@@ -158,6 +158,131 @@ sq_status stage_forward(const sq_layer* layers, int n_layers, int phase, const f
   return cuda_check(e, "sq_stage_forward");
 }
 
+// ---------------------------------------------------------------- f4: tensor-parallel stage (R27)
+namespace {
+
+struct TpLayout {
+  size_t gemv, a16, qkv16, u16, att16, xsa, xsb, total;
+};
+
+// shard shapes: o [h1, h1s], qkv [3 h1s, h1], fc1 [h2s, h1], fc2 [h1, h2s]
+TpLayout tp_layout(const sq_layer* sh, int n, int64_t T) {
+  const int64_t h1 = sh[0].o.n, h1s = sh[0].o.k, h2s = sh[0].fc1.n;
+  size_t g = 0;
+  for (int l = 0; l < n; ++l) {
+    const sq_qweight* ws[4] = {&sh[l].qkv, &sh[l].o, &sh[l].fc1, &sh[l].fc2};
+    for (auto* w : ws) {
+      size_t b = gemv_workspace_bytes(w->n, w->k, 32);
+      if (b > g) g = b;
+    }
+  }
+  TpLayout L{};
+  size_t off = 0;
+  L.gemv = off;  off += align_up((int64_t)g, 256);  // fixed offset 0: self-resetting counters (see layout())
+  L.a16 = off;   off += align_up(T * h1 * 2, 256);
+  L.qkv16 = off; off += align_up(T * 3 * h1s * 2, 256);
+  L.u16 = off;   off += align_up(T * h2s * 2, 256);
+  L.att16 = off; off += align_up(T * h1s * 2, 256);
+  L.xsa = off;   off += align_up((int64_t)xsum_bytes(h1), 256);                     // LN(x) group sums
+  L.xsb = off;   off += align_up((int64_t)xsum_bytes(h2s > h1s ? h2s : h1s), 256);  // v / u group sums
+  L.total = off;
+  return L;
+}
+
+sq_status check_tp(const sq_layer* sh, int n_layers, int tp, int n_sets, const char* who) {
+  if (!sh || n_layers <= 0 || tp < 1) return fail(SQ_EINVAL, "%s: no shards / tp < 1", who);
+  const int64_t h1 = sh[0].o.n, h1s = sh[0].o.k, h2s = sh[0].fc1.n;
+  if (h1 <= 0 || h1 > 14336 || h1s * tp != h1 || h1s % 128 || h2s <= 0 || h2s % 128)
+    return fail(SQ_EINVAL, "%s: hidden %lld must equal tp %d x shard width %lld, both multiples of 128 (ffn shard %lld)",
+                who, (long long)h1, tp, (long long)h1s, (long long)h2s);
+  for (int i = 0; i < n_layers * n_sets; ++i) {
+    const sq_layer& L = sh[i];
+    const int l = i % n_layers;
+    if (L.act != 0 && L.act != 1) return fail(SQ_EINVAL, "%s: layer %d act %d", who, l, L.act);
+    if (L.bits != sh[l].bits || L.act != sh[l].act)
+      return fail(SQ_EINVAL, "%s: layer %d bits / act differ between tp ranks", who, l);
+    sq_status st;
+    if ((st = check_w(L.qkv, 3 * h1s, h1, L.bits, who, l, "qkv"))) return st;
+    if ((st = check_w(L.o, h1, h1s, L.bits, who, l, "o"))) return st;
+    if ((st = check_w(L.fc1, h2s, h1, L.bits, who, l, "fc1"))) return st;
+    if ((st = check_w(L.fc2, h1, h2s, L.bits, who, l, "fc2"))) return st;
+  }
+  return SQ_OK;
+}
+
+// Ranks `r0 .. r1-1` of the shard sets in `sh` ([set][n_layers]) run on this device; `comm` != NULL
+// means one real TP rank (r1 = r0 + 1 = 1 set passed) whose partial sums go through the all-reduce.
+sq_status stage_forward_tp(const sq_layer* sh, int n_layers, int n_sets, sq_comm* comm, int tp_rank, int phase,
+                           const sq_attn* att, const float* x_in, int64_t T, float* x_out, void* ws, cudaStream_t s) {
+  const int64_t h1 = sh[0].o.n, h1s = sh[0].o.k, h2s = sh[0].fc1.n;
+  const TpLayout W = tp_layout(sh, n_layers * n_sets, T);
+  uint8_t* base = static_cast<uint8_t*>(ws);
+  __half* a16 = reinterpret_cast<__half*>(base + W.a16);
+  __half* qkv16 = reinterpret_cast<__half*>(base + W.qkv16);
+  __half* u16 = reinterpret_cast<__half*>(base + W.u16);
+  __half* att16 = reinterpret_cast<__half*>(base + W.att16);
+  float2* xsa = reinterpret_cast<float2*>(base + W.xsa);
+  float2* xsb = reinterpret_cast<float2*>(base + W.xsb);
+  void* gws = base + W.gemv;
+  const bool dec = phase == SQ_DECODE;
+  const bool zero_first = comm && tp_rank > 0;  // ranks r > 0 contribute p_r only (x comes from rank 0)
+  auto lin = [&](const sq_qweight& w, const __half* x, int64_t ldx, void* y, int64_t ldy, int epi,
+                 const float2* xsum) -> cudaError_t {
+    if (dec) return launch_gemv(w, x, ldx, (int)T, y, ldy, epi, xsum, gws, s);
+    return launch_gemm(w, x, ldx, T, y, ldy, epi, s);
+  };
+  auto reduce = [&]() -> sq_status {
+    if (!comm) return SQ_OK;
+    return comm_allreduce_sum_f32(comm, x_out, (size_t)T * h1, s);
+  };
+  cudaError_t e = cudaSuccess;
+  sq_status st = SQ_OK;
+  for (int l = 0; l < n_layers && e == cudaSuccess && st == SQ_OK; ++l) {
+    const sq_layer& L0 = sh[l];
+    const bool q = L0.bits != 16;
+    auto k2 = [&](const sq_qweight& w) { return dec && q && gemv_path(w.n, w.k, (int)T, w.bits) == 0; };
+    const float* xr = (l == 0) ? x_in : x_out;
+    const bool copy = (l == 0 && x_in != x_out);
+    e = launch_layernorm_f16(xr, T, h1, a16, k2(L0.qkv) ? xsa : nullptr, copy ? x_in : nullptr, copy ? x_out : nullptr, s);
+    if (e) break;
+    for (int r = 0; r < n_sets && !e; ++r) {
+      const sq_layer& L = sh[r * n_layers + l];
+      e = lin(L.qkv, a16, h1, qkv16, 3 * h1s, SQ_EPI_F16, k2(L.qkv) ? xsa : nullptr);
+      if (e) break;
+      const __half* v = qkv16 + 2 * h1s;
+      int64_t ldv = 3 * h1s;
+      if (att) {
+        const sq_attn& A = att[r];
+        e = launch_attention(qkv16, 3 * h1s, A.nseq, A.seq_len, A.pos0, A.seq0, (int)h1s, A.n_heads,
+                             static_cast<__half*>(A.k_cache[l]), static_cast<__half*>(A.v_cache[l]), A.max_len,
+                             att16, h1s, s);
+        if (e) break;
+        v = att16;
+        ldv = h1s;
+      }
+      if (k2(L.o) && (e = launch_xsum(v, ldv, T, h1s, xsb, s))) break;
+      if (zero_first && (e = cudaMemsetAsync(x_out, 0, (size_t)T * h1 * sizeof(float), s))) break;
+      e = lin(L.o, v, ldv, x_out, h1, SQ_EPI_F32_ACCUM, k2(L.o) ? xsb : nullptr);
+    }
+    if (e || (st = reduce())) break;
+    e = launch_layernorm_f16(x_out, T, h1, a16, k2(L0.fc1) ? xsa : nullptr, nullptr, nullptr, s);
+    if (e) break;
+    for (int r = 0; r < n_sets && !e; ++r) {
+      const sq_layer& L = sh[r * n_layers + l];
+      e = lin(L.fc1, a16, h1, u16, h2s, L.act == 0 ? SQ_EPI_F16_RELU : SQ_EPI_F16_GELU, k2(L.fc1) ? xsa : nullptr);
+      if (e) break;
+      if (k2(L.fc2) && (e = launch_xsum(u16, h2s, T, h2s, xsb, s))) break;
+      if (zero_first && (e = cudaMemsetAsync(x_out, 0, (size_t)T * h1 * sizeof(float), s))) break;
+      e = lin(L.fc2, u16, h2s, x_out, h1, SQ_EPI_F32_ACCUM, k2(L.fc2) ? xsb : nullptr);
+    }
+    if (e) break;
+    st = reduce();
+  }
+  if (st) return st;
+  return cuda_check(e, "sq_stage_forward_tp");
+}
+
+}  // namespace
 }  // namespace sq
 
 using namespace sq;
@@ -194,7 +319,7 @@ sq_status sq_stage_forward_attn(const sq_layer* layers, int n_layers, int phase,
                                 sq_stream_t stream) {
   sq_status st = check_layers(layers, n_layers, "sq_stage_forward_attn");
   if (st) return st;
-  if ((st = check_attn(attn, layers, n_layers, phase, tokens, "sq_stage_forward_attn"))) return st;
+  if ((st = check_attn(attn, layers[0].o.n, n_layers, phase, tokens, "sq_stage_forward_attn"))) return st;
   if (!x_in_dev || !x_out_dev || (reinterpret_cast<uintptr_t>(x_in_dev) & 15u) || (reinterpret_cast<uintptr_t>(x_out_dev) & 15u))
     return fail(SQ_EINVAL, "sq_stage_forward_attn: x_in/x_out null or not 16-B aligned");
   const size_t need = stage_workspace_bytes(layers, n_layers, tokens);
@@ -202,6 +327,39 @@ sq_status sq_stage_forward_attn(const sq_layer* layers, int n_layers, int phase,
     return fail(SQ_ENOMEM, "sq_stage_forward_attn: workspace %zu < %zu (or null / not 256-B aligned)", ws_bytes, need);
   return stage_forward(layers, n_layers, phase, x_in_dev, tokens, x_out_dev, nullptr, ws_dev, ws_bytes,
                        (cudaStream_t)stream, attn);
+}
+
+size_t sq_stage_tp_workspace_bytes(const sq_layer* shards, int n_shard_layers, int64_t max_tokens) {
+  if (!shards || n_shard_layers <= 0 || max_tokens <= 0) return 0;
+  return tp_layout(shards, n_shard_layers, max_tokens).total;
+}
+
+sq_status sq_stage_forward_tp(const sq_layer* shards, int n_layers, int tp, int tp_rank, sq_comm* comm, int phase,
+                              const sq_attn* attn, const float* x_in_dev, int64_t tokens, float* x_out_dev,
+                              void* ws_dev, size_t ws_bytes, sq_stream_t stream) {
+  const char* who = "sq_stage_forward_tp";
+  if (tp < 1 || tp_rank < -1 || tp_rank >= tp) return fail(SQ_EINVAL, "%s: tp %d, tp_rank %d", who, tp, tp_rank);
+  const int n_sets = tp_rank < 0 ? tp : 1;
+  sq_status st = check_tp(shards, n_layers, tp, n_sets, who);
+  if (st) return st;
+  if (tp_rank >= 0 && tp > 1) {
+    if (!comm || comm_is_local(comm) || comm_size(comm) != tp || comm_rank(comm) != tp_rank)
+      return fail(SQ_EINVAL, "%s: tp_rank %d needs an NCCL comm of %d ranks with that rank", who, tp_rank, tp);
+  }
+  if (phase != SQ_PREFILL && phase != SQ_DECODE) return fail(SQ_EINVAL, "%s: bad phase %d", who, phase);
+  if (tokens < 1 || (phase == SQ_DECODE && tokens > 32))
+    return fail(SQ_EINVAL, "%s: tokens=%lld (decode needs 1..32)", who, (long long)tokens);
+  if (attn) {
+    for (int r = 0; r < n_sets; ++r)
+      if ((st = check_attn(&attn[r], shards[0].o.k, n_layers, phase, tokens, who))) return st;
+  }
+  if (!x_in_dev || !x_out_dev || (reinterpret_cast<uintptr_t>(x_in_dev) & 15u) || (reinterpret_cast<uintptr_t>(x_out_dev) & 15u))
+    return fail(SQ_EINVAL, "%s: x_in/x_out null or not 16-B aligned", who);
+  const size_t need = tp_layout(shards, n_layers * n_sets, tokens).total;
+  if (!ws_dev || ws_bytes < need || (reinterpret_cast<uintptr_t>(ws_dev) & 255u))
+    return fail(SQ_ENOMEM, "%s: workspace %zu < %zu (or null / not 256-B aligned)", who, ws_bytes, need);
+  return stage_forward_tp(shards, n_layers, n_sets, (tp_rank >= 0 && tp > 1) ? comm : nullptr, tp_rank, phase,
+                          attn, x_in_dev, tokens, x_out_dev, ws_dev, (cudaStream_t)stream);
 }
 
 sq_status sq_layernorm_f32(const float* x_dev, int64_t rows, int64_t d, float* y_dev, sq_stream_t stream) {

@@ -203,3 +203,80 @@ def sq_pipeline_run(plan: Plan, rank: int, layers: list[Layer], comm: Comm | Non
     return {"t_total_ms": st.t_total_ms, "t_prefill_ms": st.t_prefill_ms, "t_decode_ms": st.t_decode_ms,
             "tokens_per_s": st.tokens_per_s, "bytes_sent": st.bytes_sent, "gpu_launches": st.gpu_launches,
             "host_enqueue_ms": st.host_enqueue_ms, "graph_replays": st.graph_replays}
+
+
+# ---------------------------------------------------------------- f4: tensor-parallel stage (R27)
+def tp_shard_fp16(name: str, w: torch.Tensor, bias: torch.Tensor | None, r: int, T: int):
+    """Shard r of T of one linear (sq.h f4 split): qkv / fc1 by output rows (qkv: the same row slice of
+    each of q, k, v), o / fc2 by input columns with the bias on rank 0 only.  -> (w fp16, bias)."""
+    n, k = w.shape
+    if name == "qkv":
+        h = n // 3
+        s = h // T
+        idx = [slice(j * h + r * s, j * h + (r + 1) * s) for j in range(3)]
+        ws = torch.cat([w[i] for i in idx])
+        b = None if bias is None else torch.cat([bias[i] for i in idx])
+    elif name == "fc1":
+        s = n // T
+        ws, b = w[r * s:(r + 1) * s], None if bias is None else bias[r * s:(r + 1) * s]
+    else:
+        s = k // T
+        ws, b = w[:, r * s:(r + 1) * s], (bias if r == 0 else None)
+    return ws.contiguous(), None if b is None else b.contiguous()
+
+
+def build_tp_layers(n_layers: int, h1: int, h2: int, bits: list[int], T: int, act: int = 0, bias: bool = True,
+                    layer_offset: int = 0, device: str = "cuda", ranks=None) -> list[list[Layer]]:
+    """The synthetic layers of build_layers split into T tensor-parallel shards: [rank][layer] for the
+    ranks in `ranks` (default all; a real TP rank builds only its own)."""
+    import synth
+    ranks = list(range(T)) if ranks is None else list(ranks)
+    dims = {"qkv": (3 * h1, h1), "o": (h1, h1), "fc1": (h2, h1), "fc2": (h1, h2)}
+    s = torch.cuda.current_stream()
+    out = [[] for _ in ranks]
+    for i in range(n_layers):
+        l = layer_offset + i
+        b = int(bits[i])
+        lins = [{} for _ in ranks]
+        for name, (n, k) in dims.items():
+            seed = synth.weight_seed(l, name)
+            w = torch.empty((n, k), dtype=torch.float16, device=device)
+            synth.device_weight_f16(w.data_ptr(), seed, n, k, s.cuda_stream)
+            bvec = torch.from_numpy(synth.bias_f16(seed, n)).to(device) if bias else None
+            for j, r in enumerate(ranks):
+                ws, bs = tp_shard_fp16(name, w, bvec, r, T)
+                lins[j][name] = QLinear.from_fp16(ws, b, bs, stream=s)
+        for j in range(len(ranks)):
+            out[j].append(Layer(b, act, lins[j]["qkv"], lins[j]["o"], lins[j]["fc1"], lins[j]["fc2"]))
+    torch.cuda.synchronize()
+    return out
+
+
+class TpWorkspace:
+    def __init__(self, shard_sets: list[list[Layer]], max_tokens: int, device="cuda"):
+        arr = layer_array([l for s in shard_sets for l in s])
+        n = int(_L.sq_stage_tp_workspace_bytes(arr, sum(len(s) for s in shard_sets), max_tokens))
+        if n == 0:
+            raise ValueError("invalid shards for workspace query")
+        self.buf = torch.zeros(n + 256, dtype=torch.uint8, device=device)
+        off = (-self.buf.data_ptr()) % 256
+        self.ptr = self.buf.data_ptr() + off
+        self.nbytes = n
+
+
+def sq_stage_forward_tp(shard_sets: list[list[Layer]], phase: int, x_in: torch.Tensor, x_out: torch.Tensor,
+                        ws: TpWorkspace, T: int, tp_rank: int = -1, comm: Comm | None = None,
+                        caches: list[KVCache] | None = None, n_heads: int = 0, seq0: int = 0, nseq: int = 0,
+                        seq_len: int = 0, pos0: int = 0, stream=None) -> torch.Tensor:
+    """f4: one stage under T-way TP.  tp_rank -1: virtual TP (shard_sets = all T ranks' layers on this
+    device); tp_rank >= 0: this rank's single shard set, partial sums all-reduced over `comm`.  With
+    `caches` (one KVCache of width h1/T per shard set) the layers run causal attention over n_heads
+    heads (n_heads / T per rank)."""
+    n_layers = len(shard_sets[0])
+    arr = layer_array([l for s in shard_sets for l in s])
+    ctx = None
+    if caches is not None:
+        ctx = (sq_attn * len(caches))(*[c.ctx(n_heads // T, seq0, nseq, seq_len, pos0) for c in caches])
+    _check(_L.sq_stage_forward_tp(arr, n_layers, T, tp_rank, comm.h if comm else None, phase, ctx, _ptr(x_in),
+                                  x_in.shape[0], _ptr(x_out), ctypes.c_void_p(ws.ptr), ws.nbytes, _stream(stream)))
+    return x_out
