@@ -45,7 +45,7 @@ typedef enum {
 
 const char* sq_last_error(void);
 const char* sq_version(void);
-int sq_abi_version(void); /* bumped on any incompatible change of this header (2: sq_plan.n_heads/kappa) */
+int sq_abi_version(void); /* bumped on any incompatible change of this header (2: sq_plan.n_heads/kappa; 3: sq_plan.tp) */
 
 /* ------------------------------------------------------------------------
  * Sizes.  P:160: a decoder layer with precision `bit` stores
@@ -281,6 +281,11 @@ sq_status sq_comm_init(sq_comm** out, const uint8_t* id_host, int nranks, int ra
 /* Single-process "virtual pipeline": every stage on the current device, transfers
  * are device copies.  Bitwise reference for the multi-GPU run. */
 sq_status sq_comm_init_local(sq_comm** out, int nstages);
+/* P x T mesh (f4: TP inside every pipeline stage): nranks = n_stages * tp, global rank
+ * g = stage * tp + j.  Builds the T independent stage rings (link (p, j) -> (p+1 mod P, j), the same
+ * three-split scheme as sq_comm_init per ring) plus one tp-rank communicator per stage (ncclCommSplit
+ * colour = stage, key = j) that carries sq_stage_forward_tp's all-reduce.  Collective over all ranks. */
+sq_status sq_comm_init_mesh(sq_comm** out, const uint8_t* id_host, int n_stages, int tp, int rank);
 sq_status sq_comm_destroy(sq_comm* comm);
 
 typedef struct {            /* host memory, identical on every rank */
@@ -299,6 +304,10 @@ typedef struct {            /* host memory, identical on every rank */
                                pipeline workspace */
   int32_t kappa;            /* prefill chunks per prompt (0 or 1 = whole prompt); s % kappa == 0;
                                needs n_heads > 0 when > 1 */
+  int32_t tp;               /* intra-node tensor parallelism per stage (f4, P:63 / P:236; 0 or 1 = none):
+                               every stage spans tp ranks (a P x tp mesh, e.g. TP2+PP2 of P:318), each
+                               holding the sq_stage_forward_tp shard of its stage's layers; hidden and
+                               ffn multiples of 128 tp, n_heads % tp == 0 */
 } sq_plan;
 
 typedef struct {
@@ -314,10 +323,16 @@ size_t sq_pipeline_workspace_bytes(const sq_plan* plan, const sq_layer* layers, 
 /* rank >= 0: this process's stage (layers = its layers, in order); rank == -1 with a
  * local comm: all stages (layers = all n_layers).  x0_dev: embeddings fp32 [B, s, h1]
  * (needed on stage 0); out_dev: fp32 [B, 1+n_decode, h1] (written on the last stage).
+ * With plan.tp = T > 1 the global rank is g = stage * T + j (j = TP index), comm comes from
+ * sq_comm_init_mesh, layers = this rank's TP shards of its stage's layers (n_layers = the stage's
+ * layer count), and hidden states travel (stage p, j) -> (stage p+1, j), loop-back (P-1, j) -> (0, j)
+ * (the residual is replicated over a TP group).  rank == -1 runs the whole mesh on one device:
+ * layers = [T][n_layers] (TP index major), n_layers = plan.n_layers.
  * Blocking: returns after the run completed on this rank.
  * Decode micro-batches of the attention-stub path (plan.n_heads == 0) are captured once per
  * (layers, input / output buffer, rows, workspace) into a CUDA graph and replayed (a process-wide
- * cache of instantiated graphs; SQ_GRAPH=0 disables it, and it is bypassed while sq_profile is on). */
+ * cache of instantiated graphs; SQ_GRAPH=0 disables it, and it is bypassed while sq_profile is on and
+ * around a real TP rank's NCCL all-reduce). */
 sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers, int n_layers,
                           sq_comm* comm, const float* x0_dev, float* out_dev, void* ws_dev,
                           size_t ws_bytes, sq_run_stats* stats, sq_stream_t stream);
@@ -366,7 +381,8 @@ int64_t sq_pipeline_schedule(const sq_plan* plan, int rank, sq_sched_op* ops, in
  * fused residual epilogue), ranks r > 0 write p_r into a zeroed x, and one NCCL all-reduce (sum)
  * returns x + sum_r p_r on every rank, so the residual add costs no extra pass.
  *   tp_rank >= 0: one rank of a T-rank NCCL group; comm from sq_comm_init(nranks = T, rank = tp_rank)
- *                 (its world communicator carries the all-reduce); shards = this rank's n_layers
+ *                 (its world communicator carries the all-reduce) or from sq_comm_init_mesh (its
+ *                 stage's TP communicator); shards = this rank's n_layers
  *                 layers; attn NULL or one context.
  *   tp_rank == -1: virtual TP on the current device (tests, single-GPU runs of a TP plan): comm
  *                 ignored (may be NULL); shards = [T][n_layers] rank-major; attn NULL or [T]

@@ -48,7 +48,7 @@ class sq_layer(ctypes.Structure):
 class sq_plan(ctypes.Structure):
     _fields_ = [("n_layers", I32), ("n_stages", I32), ("hidden", I32), ("ffn", I32), ("group", I32),
                 ("bits", ctypes.POINTER(I32)), ("stage_of_layer", ctypes.POINTER(I32)), ("B", I32), ("eta", I32),
-                ("xi", I32), ("prompt_len", I32), ("n_decode", I32), ("n_heads", I32), ("kappa", I32)]
+                ("xi", I32), ("prompt_len", I32), ("n_decode", I32), ("n_heads", I32), ("kappa", I32), ("tp", I32)]
 
 
 class sq_attn(ctypes.Structure):
@@ -109,7 +109,7 @@ EXPORTED = [
     "sq_launch_count", "sq_pipeline_schedule", "sq_scale_sq_sums_workspace_bytes", "sq_scale_sq_sums",
     "sq_act_moments_workspace_bytes", "sq_act_moments", "sq_quantize_groups_ex", "sq_attention",
     "sq_stage_forward_attn", "sq_quantize_w8", "sq_quantize_act8", "sq_linear_w8a8_workspace_bytes",
-    "sq_linear_w8a8", "sq_stage_tp_workspace_bytes", "sq_stage_forward_tp",
+    "sq_linear_w8a8", "sq_stage_tp_workspace_bytes", "sq_stage_forward_tp", "sq_comm_init_mesh",
 ]
 
 
@@ -136,6 +136,7 @@ _opt("sq_comm_unique_id_bytes", ctypes.c_size_t)
 _opt("sq_comm_get_unique_id", ctypes.c_int, P)
 _opt("sq_comm_init", ctypes.c_int, ctypes.POINTER(P), P, ctypes.c_int, ctypes.c_int)
 _opt("sq_comm_init_local", ctypes.c_int, ctypes.POINTER(P), ctypes.c_int)
+_opt("sq_comm_init_mesh", ctypes.c_int, ctypes.POINTER(P), P, ctypes.c_int, ctypes.c_int, ctypes.c_int)
 _opt("sq_comm_destroy", ctypes.c_int, P)
 _opt("sq_pipeline_workspace_bytes", ctypes.c_size_t, ctypes.POINTER(sq_plan), ctypes.POINTER(sq_layer), ctypes.c_int)
 _opt("sq_pipeline_run", ctypes.c_int, ctypes.POINTER(sq_plan), ctypes.c_int, ctypes.POINTER(sq_layer), ctypes.c_int,

@@ -133,7 +133,7 @@ extern "C" {
 
 const char* sq_last_error(void) { return g_err; }
 const char* sq_version(void) { return "libsq 0.1 (sm_100a)"; }
-int sq_abi_version(void) { return 2; }
+int sq_abi_version(void) { return 3; }
 
 size_t sq_packed_bytes(int64_t n, int64_t k, int bits) {
   if (n <= 0 || k <= 0 || !valid_bits(bits) || (n * k * bits) % 8) return 0;

@@ -59,6 +59,12 @@ sq_status stage_forward(const sq_layer* layers, int n_layers, int phase, const f
 sq_status check_layers(const sq_layer* layers, int n_layers, const char* who);
 sq_status check_attn(const sq_attn* a, int64_t h1, int n_layers, int phase, int64_t tokens, const char* who);
 
+// ---- tensor-parallel stage (sq_stage.cu, f4)
+size_t stage_tp_workspace_bytes(const sq_layer* sh, int n_shard_layers, int64_t max_tokens);
+sq_status check_tp(const sq_layer* sh, int n_layers, int tp, int n_sets, const char* who);
+sq_status stage_forward_tp(const sq_layer* sh, int n_layers, int n_sets, sq_comm* comm, int tp_rank, int phase,
+                           const sq_attn* att, const float* x_in, int64_t T, float* x_out, void* ws, cudaStream_t s);
+
 // ---- TP all-reduce (sq_pipeline.cu): in-place fp32 sum over the comm's world communicator
 sq_status comm_allreduce_sum_f32(sq_comm* c, float* buf, size_t count, cudaStream_t s);
 int comm_size(const sq_comm* c);

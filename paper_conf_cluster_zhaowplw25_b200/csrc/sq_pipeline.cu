@@ -13,6 +13,10 @@
 // Compute of micro-batch m+1 overlaps the transfer of micro-batch m
 // (double-buffered activations, CUDA events for the dependencies).
 //
+// Intra-node TP (f4, P:63 / P:236): with plan.tp = T every stage is a group of T ranks running
+// sq_stage_forward_tp on its shards; ring j (the ranks with TP index j) carries the replicated hidden
+// states and loop-backs exactly as a plain pipeline does.
+//
 // Items (identical order on every rank): prefill m = 0..mu_pre-1, then decode
 // t = 1..n_decode, m = 0..mu_dec-1.  The last stage writes out[b, 0] (hidden at
 // the last prompt position) / out[b, t] and loops LN(hidden) back to stage 0
@@ -31,8 +35,10 @@
 
 struct sq_comm {
   int nranks = 1, rank = 0;
+  int tp = 1;               // mesh (sq_comm_init_mesh): ranks per stage; global rank = stage * tp + j
   bool local = false;
   ncclComm_t world = nullptr, send_comm = nullptr, recv_comm = nullptr;
+  ncclComm_t tp_comm = nullptr;  // mesh: the tp ranks of this rank's stage (all-reduce of the TP stage)
   cudaStream_t s_send = nullptr, s_recv = nullptr;
 };
 
@@ -48,6 +54,7 @@ struct PlanView {
   int L, P, h1, h2, B, eta, xi, s, n_dec;
   int mu_pre, mu_dec;
   int heads, kappa, len_pre, max_len;  // attention (f3): heads 0 = stub; prefill chunk = s / kappa tokens
+  int tp;                              // ranks per stage (f4)
   std::vector<int> first_layer;  // [P+1]
 };
 
@@ -61,6 +68,7 @@ PlanView view(const sq_plan& pl) {
   v.kappa = pl.kappa > 1 ? pl.kappa : 1;
   v.len_pre = pl.prompt_len / v.kappa;
   v.max_len = pl.prompt_len + pl.n_decode;
+  v.tp = pl.tp > 1 ? pl.tp : 1;
   v.first_layer.assign(v.P + 1, v.L);
   for (int l = v.L - 1; l >= 0; --l) v.first_layer[pl.stage_of_layer[l]] = l;
   v.first_layer[v.P] = v.L;
@@ -71,18 +79,21 @@ struct Ws {
   size_t stage, act, decin, lb, kv, kv_layer, total;
 };
 
+// n_layers: the layers passed (rank -1 with tp > 1: all tp shard sets, tp * n_layers entries)
 Ws ws_layout(const PlanView& v, const sq_layer* layers, int n_layers, int rank) {
   Ws w{};
   size_t off = 0;
   auto al = [](size_t x) { return (x + 255) / 256 * 256; };
   const int64_t tmax = std::max<int64_t>((int64_t)v.eta * v.len_pre, v.xi);
-  w.stage = off; off += al(stage_workspace_bytes(layers, n_layers, tmax));
+  w.stage = off; off += al(v.tp > 1 ? stage_tp_workspace_bytes(layers, n_layers, tmax)
+                                   : stage_workspace_bytes(layers, n_layers, tmax));
   w.act = off;   off += 2 * al((size_t)tmax * v.h1 * 4);
-  const bool first = rank <= 0, last = rank < 0 || rank == v.P - 1;
+  const int stage = rank < 0 ? -1 : rank / v.tp;
+  const bool first = stage <= 0, last = stage < 0 || stage == v.P - 1;
   w.decin = off; if (first) off += al((size_t)v.B * v.h1 * 4);
   w.lb = off;    if (last) off += 2 * al((size_t)std::max(v.eta, v.xi) * v.h1 * 4);
-  // KV cache of this rank's layers (f3): K and V fp16 [B][s + n_decode][h1] per layer
-  w.kv_layer = v.heads > 0 ? al((size_t)v.B * v.max_len * v.h1 * 2) : 0;
+  // KV cache of this rank's layers (f3): K and V fp16 [B][s + n_decode][h1 / tp] per layer
+  w.kv_layer = v.heads > 0 ? al((size_t)v.B * v.max_len * (v.h1 / v.tp) * 2) : 0;
   w.kv = off;    off += (size_t)n_layers * 2 * w.kv_layer;
   w.total = off;
   return w;
@@ -133,9 +144,11 @@ bool graphs_enabled() {
   return on == 1;
 }
 
-// decode stage call through the graph cache (falls back to direct launches on any capture error)
+// decode stage call through the graph cache (falls back to direct launches on any capture error);
+// body(stream) issues the stage's launches, layers[0..n_layers) is everything they bake in
+template <class Body>
 sq_status stage_forward_graph(const sq_layer* layers, int n_layers, const float* x_in, int64_t rows, float* x_out,
-                              void* ws, size_t ws_bytes, cudaStream_t S, int64_t* replays) {
+                              void* ws, cudaStream_t S, int64_t* replays, Body body) {
   int dev = 0;
   cudaGetDevice(&dev);
   const GraphKey key{hash_layers(layers, n_layers), x_in, x_out, ws, rows, n_layers, dev};
@@ -153,7 +166,7 @@ sq_status stage_forward_graph(const sq_layer* layers, int n_layers, const float*
   cudaStream_t cs = nullptr;
   if (cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking) != cudaSuccess) {
     cudaGetLastError();
-    return stage_forward(layers, n_layers, SQ_DECODE, x_in, rows, x_out, nullptr, ws, ws_bytes, S);
+    return body(S);
   }
   const int64_t l0 = sq_launch_count();
   cudaGraph_t g = nullptr;
@@ -161,7 +174,7 @@ sq_status stage_forward_graph(const sq_layer* layers, int n_layers, const float*
   sq_status st = SQ_OK;
   bool ok = cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal) == cudaSuccess;
   if (ok) {
-    st = stage_forward(layers, n_layers, SQ_DECODE, x_in, rows, x_out, nullptr, ws, ws_bytes, cs);
+    st = body(cs);
     ok = cudaStreamEndCapture(cs, &g) == cudaSuccess && st == SQ_OK;
   }
   const int64_t n_launch = sq_launch_count() - l0;
@@ -172,7 +185,7 @@ sq_status stage_forward_graph(const sq_layer* layers, int n_layers, const float*
   if (!ok) {
     cudaGetLastError();
     if (ex) cudaGraphExecDestroy(ex);
-    return stage_forward(layers, n_layers, SQ_DECODE, x_in, rows, x_out, nullptr, ws, ws_bytes, S);
+    return body(S);
   }
   {
     std::lock_guard<std::mutex> lk(g_graph_mu);
@@ -190,8 +203,11 @@ sq_status stage_forward_graph(const sq_layer* layers, int n_layers, const float*
 
 // ---- schedule: the op sequence of one rank (also exported as sq_pipeline_schedule)
 std::vector<sq_sched_op> make_schedule(const PlanView& v, int rank) {
+  // global rank = stage * tp + j; the ring of TP index j links (p, j) -> (p + 1, j)
+  const int stage = rank < 0 ? -1 : rank / v.tp, j = rank < 0 ? 0 : rank % v.tp;
+  auto g = [&](int q) { return q * v.tp + j; };
   const bool dist = rank >= 0 && v.P > 1;
-  const bool first = !dist || rank == 0, last = !dist || rank == v.P - 1;
+  const bool first = !dist || stage == 0, last = !dist || stage == v.P - 1;
   std::vector<sq_sched_op> ops;
   auto op = [&](int kind, int item, int phase, int t, int slot, int peer, int64_t seq0, int64_t nseq, int64_t rows) {
     sq_sched_op o;
@@ -228,16 +244,16 @@ std::vector<sq_sched_op> make_schedule(const PlanView& v, int rank) {
           r0 = (int64_t)mm * v.xi;
           nr = std::min<int64_t>(v.xi, v.B - r0);
         }
-        op(SQ_OP_RECV_LB, lb_posted, phase, t, 0, v.P - 1, r0, nr, nr);
+        op(SQ_OP_RECV_LB, lb_posted, phase, t, 0, g(v.P - 1), r0, nr, nr);
       }
     }
-    if (dist && !first) op(SQ_OP_RECV_ACT, it, phase, t, slot, rank - 1, seq0, nseq, T);
+    if (dist && !first) op(SQ_OP_RECV_ACT, it, phase, t, slot, g(stage - 1), seq0, nseq, T);
     op(SQ_OP_COMPUTE, it, phase, t, slot, -1, seq0, nseq, T);
     if (!last) {
-      op(SQ_OP_SEND_ACT, it, phase, t, slot, rank + 1, seq0, nseq, T);
+      op(SQ_OP_SEND_ACT, it, phase, t, slot, g(stage + 1), seq0, nseq, T);
     } else if (last_chunk) {
       op(SQ_OP_OUT, it, phase, t, slot, -1, seq0, nseq, nseq);
-      if (t < v.n_dec) op(dist ? SQ_OP_SEND_LB : SQ_OP_LOOPBACK_LOCAL, it, phase, t, slot, dist ? 0 : -1, seq0, nseq, nseq);
+      if (t < v.n_dec) op(dist ? SQ_OP_SEND_LB : SQ_OP_LOOPBACK_LOCAL, it, phase, t, slot, dist ? g(0) : -1, seq0, nseq, nseq);
     }
   }
   return ops;
@@ -247,11 +263,13 @@ std::vector<sq_sched_op> make_schedule(const PlanView& v, int rank) {
 
 sq_status comm_allreduce_sum_f32(sq_comm* c, float* buf, size_t count, cudaStream_t s) {
   if (!c || c->local) return fail(SQ_EINVAL, "allreduce: needs an NCCL communicator (sq_comm_init)");
-  if (c->nranks == 1) return SQ_OK;
-  return nccl_check(ncclAllReduce(buf, buf, count, ncclFloat, ncclSum, c->world, s), "ncclAllReduce");
+  ncclComm_t cm = c->tp_comm ? c->tp_comm : c->world;
+  if (!cm) return SQ_OK;  // a single rank
+  return nccl_check(ncclAllReduce(buf, buf, count, ncclFloat, ncclSum, cm, s), "ncclAllReduce");
 }
-int comm_size(const sq_comm* c) { return c ? c->nranks : 0; }
-int comm_rank(const sq_comm* c) { return c ? c->rank : -1; }
+// size / rank of the TP group the comm's all-reduce spans (the stage's group for a mesh comm)
+int comm_size(const sq_comm* c) { return !c ? 0 : c->tp_comm ? c->tp : c->nranks; }
+int comm_rank(const sq_comm* c) { return !c ? -1 : c->tp_comm ? c->rank % c->tp : c->rank; }
 bool comm_is_local(const sq_comm* c) { return c && c->local; }
 
 }  // namespace sq
@@ -274,6 +292,8 @@ sq_status sq_plan_check(const sq_plan* p) {
     return fail(SQ_EINVAL, "sq_plan_check: n_heads %d: head_dim hidden/n_heads must be 64 or 128", p->n_heads);
   if (p->kappa < 0 || (p->kappa > 1 && (p->n_heads == 0 || p->prompt_len % p->kappa)))
     return fail(SQ_EINVAL, "sq_plan_check: kappa %d needs attention (n_heads > 0) and prompt_len %% kappa == 0", p->kappa);
+  if (p->tp < 0 || (p->tp > 1 && (p->hidden % (128 * p->tp) || p->ffn % (128 * p->tp) || p->n_heads % p->tp)))
+    return fail(SQ_EINVAL, "sq_plan_check: tp %d needs hidden, ffn multiples of 128 tp and n_heads %% tp == 0", p->tp);
   // eqs. (15)-(16): u_{1,1} = 1, u_{L,N} = 1, adjacent layers on the same or next stage
   if (p->stage_of_layer[0] != 0 || p->stage_of_layer[p->n_layers - 1] != p->n_stages - 1)
     return fail(SQ_EINVAL, "sq_plan_check: first layer must be on stage 0 and last on stage n_stages-1");
@@ -289,7 +309,7 @@ sq_status sq_plan_check(const sq_plan* p) {
 }
 
 int64_t sq_pipeline_schedule(const sq_plan* plan, int rank, sq_sched_op* ops, int64_t max_ops) {
-  if (sq_plan_check(plan) != SQ_OK || rank >= plan->n_stages || rank < -1) return -1;
+  if (sq_plan_check(plan) != SQ_OK || rank >= plan->n_stages * (plan->tp > 1 ? plan->tp : 1) || rank < -1) return -1;
   const std::vector<sq_sched_op> v = make_schedule(view(*plan), rank);
   if (ops) {
     const int64_t n = std::min<int64_t>(max_ops, (int64_t)v.size());
@@ -309,45 +329,64 @@ sq_status sq_comm_get_unique_id(uint8_t* id_host) {
   return SQ_OK;
 }
 
-sq_status sq_comm_init(sq_comm** out, const uint8_t* id_host, int nranks, int rank) {
-  if (!out || !id_host || nranks < 1 || rank < 0 || rank >= nranks)
-    return fail(SQ_EINVAL, "sq_comm_init: bad arguments");
+namespace {
+// P stage rings of tp ranks each (tp = 1: the plain pipeline), global rank = stage * tp + j
+sq_status comm_init(sq_comm** out, const uint8_t* id_host, int P, int tp, int rank, const char* who) {
+  const int nranks = P * tp;
+  if (!out || !id_host || P < 1 || tp < 1 || rank < 0 || rank >= nranks) return fail(SQ_EINVAL, "%s: bad arguments", who);
   sq_comm* c = new sq_comm();
   c->nranks = nranks;
   c->rank = rank;
+  c->tp = tp;
   if (nranks > 1) {
     ncclUniqueId id;
     memcpy(&id, id_host, sizeof(id));
     sq_status st = nccl_check(ncclCommInitRank(&c->world, nranks, id, rank), "ncclCommInitRank");
     if (st) { delete c; return st; }
-    // One 2-rank communicator per link L_j = (j -> j+1 mod P), sender comm-rank 0 (key 0), receiver
-    // comm-rank 1.  ncclCommSplit gives each rank one colour per call, and every rank sits on two links
-    // (it sends on L_r and receives on L_{r-1}), so the links are spread over three split calls with no
-    // rank twice in one call: A = even j < P-1, B = odd j, C = the wrap link L_{P-1} when P is odd
-    // (for even P it is odd and lands in B).  Ranks outside a call's links pass NCCL_SPLIT_NOCOLOR.
-    const int P = nranks, r = rank;
-    auto call_of = [P](int j) { return (j == P - 1 && P % 2) ? 2 : (j % 2); };
-    const int send_link = r, recv_link = (r - 1 + P) % P;
-    ncclComm_t got[3] = {nullptr, nullptr, nullptr};
-    for (int call = 0; call < 3; ++call) {
-      int color = NCCL_SPLIT_NOCOLOR, key = 0;
-      if (call_of(send_link) == call) { color = send_link; key = 0; }
-      else if (call_of(recv_link) == call) { color = recv_link; key = 1; }
-      if (call == 2 && P % 2 == 0) continue;  // no third call for even P (identical on every rank)
-      st = nccl_check(ncclCommSplit(c->world, color, key, &got[call], nullptr), "ncclCommSplit");
-      if (st) {
-        for (ncclComm_t g : got) if (g) ncclCommDestroy(g);
-        sq_comm_destroy(c);
-        return st;
+    // One 2-rank communicator per link L_{p,j} = ((p, j) -> (p+1 mod P, j)), sender comm-rank 0 (key 0),
+    // receiver comm-rank 1.  ncclCommSplit gives each rank one colour per call, and every rank sits on two
+    // links of its ring (it sends on L_{p,j} and receives on L_{p-1,j}), so the links are spread over three
+    // split calls with no rank twice in one call: A = even p < P-1, B = odd p, C = the wrap link L_{P-1,j}
+    // when P is odd (for even P it is odd and lands in B).  Colour = j * P + p keeps the rings apart.
+    // Ranks outside a call's links pass NCCL_SPLIT_NOCOLOR.
+    const int p = rank / tp, j = rank % tp;
+    if (P > 1) {
+      auto call_of = [P](int l) { return (l == P - 1 && P % 2) ? 2 : (l % 2); };
+      const int send_link = p, recv_link = (p - 1 + P) % P;
+      ncclComm_t got[3] = {nullptr, nullptr, nullptr};
+      for (int call = 0; call < 3; ++call) {
+        int color = NCCL_SPLIT_NOCOLOR, key = 0;
+        if (call_of(send_link) == call) { color = j * P + send_link; key = 0; }
+        else if (call_of(recv_link) == call) { color = j * P + recv_link; key = 1; }
+        if (call == 2 && P % 2 == 0) continue;  // no third call for even P (identical on every rank)
+        st = nccl_check(ncclCommSplit(c->world, color, key, &got[call], nullptr), "ncclCommSplit");
+        if (st) {
+          for (ncclComm_t g : got) if (g) ncclCommDestroy(g);
+          sq_comm_destroy(c);
+          return st;
+        }
       }
+      c->send_comm = got[call_of(send_link)];
+      c->recv_comm = got[call_of(recv_link)];
     }
-    c->send_comm = got[call_of(send_link)];
-    c->recv_comm = got[call_of(recv_link)];
+    if (tp > 1) {  // the stage's TP group: colour = stage, comm-rank = TP index
+      st = nccl_check(ncclCommSplit(c->world, p, j, &c->tp_comm, nullptr), "ncclCommSplit(tp)");
+      if (st) { sq_comm_destroy(c); return st; }
+    }
   }
   cudaStreamCreateWithFlags(&c->s_send, cudaStreamNonBlocking);
   cudaStreamCreateWithFlags(&c->s_recv, cudaStreamNonBlocking);
   *out = c;
   return SQ_OK;
+}
+}  // namespace
+
+sq_status sq_comm_init(sq_comm** out, const uint8_t* id_host, int nranks, int rank) {
+  return comm_init(out, id_host, nranks, 1, rank, "sq_comm_init");
+}
+
+sq_status sq_comm_init_mesh(sq_comm** out, const uint8_t* id_host, int n_stages, int tp, int rank) {
+  return comm_init(out, id_host, n_stages, tp, rank, "sq_comm_init_mesh");
 }
 
 sq_status sq_comm_init_local(sq_comm** out, int nstages) {
@@ -364,6 +403,7 @@ sq_status sq_comm_destroy(sq_comm* c) {
   if (!c) return SQ_OK;
   if (c->send_comm) ncclCommDestroy(c->send_comm);
   if (c->recv_comm) ncclCommDestroy(c->recv_comm);
+  if (c->tp_comm) ncclCommDestroy(c->tp_comm);
   if (c->world) ncclCommDestroy(c->world);
   if (c->s_send) cudaStreamDestroy(c->s_send);
   if (c->s_recv) cudaStreamDestroy(c->s_recv);
@@ -374,7 +414,9 @@ sq_status sq_comm_destroy(sq_comm* c) {
 size_t sq_pipeline_workspace_bytes(const sq_plan* plan, const sq_layer* layers, int rank) {
   if (sq_plan_check(plan) != SQ_OK || !layers) return 0;
   PlanView v = view(*plan);
-  const int n = rank < 0 ? v.L : v.first_layer[rank + 1] - v.first_layer[rank];
+  if (rank >= v.P * v.tp || rank < -1) return 0;
+  const int stage = rank < 0 ? -1 : rank / v.tp;
+  const int n = rank < 0 ? v.L * v.tp : v.first_layer[stage + 1] - v.first_layer[stage];
   return ws_layout(v, layers, n, rank).total;
 }
 
@@ -386,24 +428,31 @@ sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers,
   const PlanView v = view(*plan);
   const bool local = (rank < 0);
   if (local && comm && !comm->local) return fail(SQ_EINVAL, "sq_pipeline_run: rank -1 needs a local comm (or NULL)");
+  const int TP = v.tp;
+  const int stage = local ? -1 : rank / TP, tp_j = local ? -1 : rank % TP;
   if (!local) {
-    if (rank >= v.P) return fail(SQ_EINVAL, "sq_pipeline_run: rank %d >= n_stages %d", rank, v.P);
-    if (v.P > 1 && (!comm || comm->local || comm->nranks != v.P || comm->rank != rank))
-      return fail(SQ_EINVAL, "sq_pipeline_run: comm does not match (nranks %d, rank %d)", comm ? comm->nranks : -1,
-                  comm ? comm->rank : -1);
+    if (rank >= v.P * TP) return fail(SQ_EINVAL, "sq_pipeline_run: rank %d >= n_stages %d x tp %d", rank, v.P, TP);
+    if (v.P * TP > 1 && (!comm || comm->local || comm->nranks != v.P * TP || comm->rank != rank ||
+                         comm->tp != TP || (TP > 1 && !comm->tp_comm)))
+      return fail(SQ_EINVAL, "sq_pipeline_run: comm does not match (nranks %d, rank %d, tp %d)", comm ? comm->nranks : -1,
+                  comm ? comm->rank : -1, comm ? comm->tp : -1);
   }
-  const int my_first = local ? 0 : v.first_layer[rank];
-  const int my_n = local ? v.L : v.first_layer[rank + 1] - v.first_layer[rank];
+  const int my_first = local ? 0 : v.first_layer[stage];
+  const int my_n = local ? v.L : v.first_layer[stage + 1] - v.first_layer[stage];
+  const int n_sets = (local && TP > 1) ? TP : 1;  // shard sets passed (rank -1 of a TP plan: all of them)
   if (n_layers != my_n) return fail(SQ_EINVAL, "sq_pipeline_run: got %d layers, plan assigns %d to rank %d", n_layers, my_n, rank);
-  if ((st = check_layers(layers, n_layers, "sq_pipeline_run"))) return st;
-  for (int i = 0; i < n_layers; ++i) {
-    if (layers[i].bits != plan->bits[my_first + i]) return fail(SQ_EINVAL, "sq_pipeline_run: layer %d bits differ from plan", my_first + i);
-    if (layers[i].o.n != v.h1 || layers[i].fc1.n != v.h2) return fail(SQ_EINVAL, "sq_pipeline_run: layer shapes differ from plan");
+  if ((st = TP > 1 ? check_tp(layers, n_layers, TP, n_sets, "sq_pipeline_run") : check_layers(layers, n_layers, "sq_pipeline_run")))
+    return st;
+  for (int i = 0; i < n_layers * n_sets; ++i) {
+    const int l = my_first + i % n_layers;
+    if (layers[i].bits != plan->bits[l]) return fail(SQ_EINVAL, "sq_pipeline_run: layer %d bits differ from plan", l);
+    if (layers[i].o.n != v.h1 || layers[i].o.k != v.h1 / TP || layers[i].fc1.n != v.h2 / TP)
+      return fail(SQ_EINVAL, "sq_pipeline_run: layer shapes differ from plan (tp %d)", TP);
   }
-  const bool is_first = local || rank == 0, is_last = local || rank == v.P - 1;
+  const bool is_first = local || stage == 0, is_last = local || stage == v.P - 1;
   if (is_first && !x0) return fail(SQ_EINVAL, "sq_pipeline_run: stage 0 needs x0");
   if (is_last && !out) return fail(SQ_EINVAL, "sq_pipeline_run: last stage needs out");
-  const Ws W = ws_layout(v, layers, n_layers, rank);
+  const Ws W = ws_layout(v, layers, n_layers * n_sets, rank);
   if (!ws_dev || ws_bytes < W.total || (reinterpret_cast<uintptr_t>(ws_dev) & 255u))
     return fail(SQ_ENOMEM, "sq_pipeline_run: workspace %zu < %zu (or null / not 256-B aligned)", ws_bytes, W.total);
 
@@ -413,9 +462,10 @@ sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers,
   const int64_t tmax = std::max<int64_t>((int64_t)v.eta * v.len_pre, v.xi);
   const size_t act_slot = ((size_t)tmax * v.h1 * 4 + 255) / 256 * 256;
   // attention (f3): per-layer cache pointers of this rank's layers (rank -1: all layers)
+  // (TP, rank -1: set-major, entry r * n_layers + l)
   std::vector<void*> kcp, vcp;
   if (v.heads > 0) {
-    for (int l = 0; l < n_layers; ++l) {
+    for (int l = 0; l < n_layers * n_sets; ++l) {
       kcp.push_back(base + W.kv + (size_t)(2 * l) * W.kv_layer);
       vcp.push_back(base + W.kv + (size_t)(2 * l + 1) * W.kv_layer);
     }
@@ -428,6 +478,9 @@ sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers,
   const int64_t h1 = v.h1;
   const size_t stage_ws_bytes = W.act - W.stage;
   const bool dist = !local && v.P > 1;
+  sq_comm* tp_comm = (!local && TP > 1) ? comm : nullptr;  // its stage's all-reduce group
+  std::vector<sq_layer> tp_sets;                            // rank -1 of a TP plan: one stage's shard sets
+  std::vector<sq_attn> tp_ctx(n_sets);
 
   const int64_t launches0 = sq_launch_count();
   cudaEvent_t ev_start, ev_pre, ev_end;
@@ -451,7 +504,8 @@ sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers,
   cudaError_t ce = cudaSuccess;
   sq_status rs = SQ_OK;
   const auto host_t0 = std::chrono::steady_clock::now();
-  const bool use_graphs = graphs_enabled() && v.heads == 0 && !prof_enabled();
+  // (no graphs around the NCCL all-reduce of a real TP rank)
+  const bool use_graphs = graphs_enabled() && v.heads == 0 && !prof_enabled() && !tp_comm;
 
   // ---- execute this rank's schedule (sq_pipeline_schedule): one op at a time, compute on S,
   // sends on s_send, receives on s_recv, CUDA events for every cross-stream dependency.
@@ -515,25 +569,46 @@ sq_status sq_pipeline_run(const sq_plan* plan, int rank, const sq_layer* layers,
         } else {
           x_in = buf;
         }
+        // one stage's layers [f, f + nl) on the item: plain, or TP (all shard sets of the stage for
+        // rank -1, this rank's shards + the stage's all-reduce otherwise)
+        auto run_stage = [&](int f, int nl, const float* xi) -> sq_status {
+          if (TP == 1) {
+            if (v.heads > 0) { ctx.k_cache = kcp.data() + f; ctx.v_cache = vcp.data() + f; }
+            auto body = [&](cudaStream_t cs) {
+              return stage_forward(layers + f, nl, o.phase, xi, o.rows, buf, nullptr, stage_ws, stage_ws_bytes, cs,
+                                   v.heads > 0 ? &ctx : nullptr);
+            };
+            if (use_graphs && !pre) return stage_forward_graph(layers + f, nl, xi, o.rows, buf, stage_ws, S, &replays, body);
+            return body(S);
+          }
+          const sq_layer* sets = layers + f;
+          if (local) {
+            tp_sets.resize((size_t)n_sets * nl);
+            for (int r = 0; r < n_sets; ++r)
+              for (int i = 0; i < nl; ++i) tp_sets[(size_t)r * nl + i] = layers[(size_t)r * n_layers + f + i];
+            sets = tp_sets.data();
+          }
+          for (int r = 0; r < n_sets && v.heads > 0; ++r) {
+            tp_ctx[r] = ctx;
+            tp_ctx[r].n_heads = v.heads / TP;
+            tp_ctx[r].k_cache = kcp.data() + (size_t)r * n_layers + f;
+            tp_ctx[r].v_cache = vcp.data() + (size_t)r * n_layers + f;
+          }
+          auto body = [&](cudaStream_t cs) {
+            return stage_forward_tp(sets, nl, n_sets, tp_comm, tp_j, o.phase, v.heads > 0 ? tp_ctx.data() : nullptr, xi,
+                                    o.rows, buf, stage_ws, cs);
+          };
+          if (use_graphs && !pre) return stage_forward_graph(sets, nl * n_sets, xi, o.rows, buf, stage_ws, S, &replays, body);
+          return body(S);
+        };
         if (local) {
           const float* xi = x_in;
           for (int r = 0; r < v.P && rs == SQ_OK; ++r) {
-            const int f = v.first_layer[r], nl = v.first_layer[r + 1] - f;
-            if (v.heads > 0) { ctx.k_cache = kcp.data() + f; ctx.v_cache = vcp.data() + f; }
-            if (use_graphs && !pre)
-              rs = stage_forward_graph(layers + f, nl, xi, o.rows, buf, stage_ws, stage_ws_bytes, S, &replays);
-            else
-              rs = stage_forward(layers + f, nl, o.phase, xi, o.rows, buf, nullptr, stage_ws, stage_ws_bytes, S,
-                                 v.heads > 0 ? &ctx : nullptr);
+            rs = run_stage(v.first_layer[r], v.first_layer[r + 1] - v.first_layer[r], xi);
             xi = buf;  // the "transfer" to the next stage is the buffer itself
           }
         } else {
-          if (v.heads > 0) { ctx.k_cache = kcp.data(); ctx.v_cache = vcp.data(); }
-          if (use_graphs && !pre)
-            rs = stage_forward_graph(layers, n_layers, x_in, o.rows, buf, stage_ws, stage_ws_bytes, S, &replays);
-          else
-            rs = stage_forward(layers, n_layers, o.phase, x_in, o.rows, buf, nullptr, stage_ws, stage_ws_bytes, S,
-                               v.heads > 0 ? &ctx : nullptr);
+          rs = run_stage(0, n_layers, x_in);
         }
         if (is_first && !pre && dist) cudaEventRecord(ev_dec_read, S);
         break;

@@ -189,6 +189,8 @@ TpLayout tp_layout(const sq_layer* sh, int n, int64_t T) {
   return L;
 }
 
+}  // namespace
+
 sq_status check_tp(const sq_layer* sh, int n_layers, int tp, int n_sets, const char* who) {
   if (!sh || n_layers <= 0 || tp < 1) return fail(SQ_EINVAL, "%s: no shards / tp < 1", who);
   const int64_t h1 = sh[0].o.n, h1s = sh[0].o.k, h2s = sh[0].fc1.n;
@@ -210,8 +212,13 @@ sq_status check_tp(const sq_layer* sh, int n_layers, int tp, int n_sets, const c
   return SQ_OK;
 }
 
-// Ranks `r0 .. r1-1` of the shard sets in `sh` ([set][n_layers]) run on this device; `comm` != NULL
-// means one real TP rank (r1 = r0 + 1 = 1 set passed) whose partial sums go through the all-reduce.
+size_t stage_tp_workspace_bytes(const sq_layer* sh, int n_shard_layers, int64_t max_tokens) {
+  return tp_layout(sh, n_shard_layers, max_tokens).total;
+}
+
+// The n_sets shard sets in `sh` ([set][n_layers], rank-major) run on this device one after the other
+// (virtual TP); `comm` != NULL means one real TP rank (n_sets = 1) whose partial sums go through the
+// in-place all-reduce.
 sq_status stage_forward_tp(const sq_layer* sh, int n_layers, int n_sets, sq_comm* comm, int tp_rank, int phase,
                            const sq_attn* att, const float* x_in, int64_t T, float* x_out, void* ws, cudaStream_t s) {
   const int64_t h1 = sh[0].o.n, h1s = sh[0].o.k, h2s = sh[0].fc1.n;
@@ -282,7 +289,6 @@ sq_status stage_forward_tp(const sq_layer* sh, int n_layers, int n_sets, sq_comm
   return cuda_check(e, "sq_stage_forward_tp");
 }
 
-}  // namespace
 }  // namespace sq
 
 using namespace sq;

@@ -118,7 +118,8 @@ class Plan:
     """Host-side plan (per-layer bits, layer->stage partition, micro-batch sizes)."""
 
     def __init__(self, bits: list[int], stage_of_layer: list[int], hidden: int, ffn: int, B: int, eta: int,
-                 xi: int, prompt_len: int, n_decode: int, group: int = 128, n_heads: int = 0, kappa: int = 1):
+                 xi: int, prompt_len: int, n_decode: int, group: int = 128, n_heads: int = 0, kappa: int = 1,
+                 tp: int = 1):
         self.bits = [int(b) for b in bits]
         self.stage_of_layer = [int(s) for s in stage_of_layer]
         self.n_layers = len(bits)
@@ -127,12 +128,17 @@ class Plan:
         self.prompt_len, self.n_decode, self.group = prompt_len, n_decode, group
         self._bits = (ctypes.c_int32 * self.n_layers)(*self.bits)
         self._sol = (ctypes.c_int32 * self.n_layers)(*self.stage_of_layer)
-        self.n_heads, self.kappa = n_heads, kappa
+        self.n_heads, self.kappa, self.tp = n_heads, kappa, max(1, tp)
         self.c = sq_plan(self.n_layers, self.n_stages, hidden, ffn, group, self._bits, self._sol, B, eta, xi,
-                         prompt_len, n_decode, n_heads, kappa)
+                         prompt_len, n_decode, n_heads, kappa, tp)
+
+    @property
+    def n_ranks(self) -> int:
+        return self.n_stages * self.tp
 
     def layers_of(self, rank: int) -> list[int]:
-        return [l for l, s in enumerate(self.stage_of_layer) if s == rank]
+        """layer indices held by global rank `rank` (stage rank // tp)"""
+        return [l for l, s in enumerate(self.stage_of_layer) if s == rank // self.tp]
 
 
 def sq_plan_check(plan: Plan) -> None:
@@ -162,6 +168,14 @@ class Comm:
         return cls(h.value)
 
     @classmethod
+    def mesh(cls, uid: bytes, n_stages: int, tp: int, rank: int) -> "Comm":
+        """P x tp mesh (f4): stage rings + one TP communicator per stage (sq_comm_init_mesh)."""
+        h = ctypes.c_void_p()
+        buf = (ctypes.c_uint8 * len(uid)).from_buffer_copy(uid)
+        _check(_L.sq_comm_init_mesh(ctypes.byref(h), buf, n_stages, tp, rank))
+        return cls(h.value)
+
+    @classmethod
     def nccl(cls, uid: bytes, nranks: int, rank: int) -> "Comm":
         h = ctypes.c_void_p()
         buf = (ctypes.c_uint8 * len(uid)).from_buffer_copy(uid)
@@ -181,9 +195,16 @@ def sq_comm_get_unique_id() -> bytes:
     return bytes(buf)
 
 
+def _flat(layers):
+    """list[Layer] -> itself; TP shard sets list[list[Layer]] ([tp][n_layers]) -> flattened, set-major"""
+    if layers and isinstance(layers[0], (list, tuple)):
+        return [l for s in layers for l in s], len(layers[0])
+    return layers, len(layers)
+
+
 class PipelineWorkspace:
-    def __init__(self, plan: Plan, layers: list[Layer], rank: int, device="cuda"):
-        arr = layer_array(layers)
+    def __init__(self, plan: Plan, layers, rank: int, device="cuda"):
+        arr = layer_array(_flat(layers)[0])
         n = int(_L.sq_pipeline_workspace_bytes(ctypes.byref(plan.c), arr, rank))
         if n == 0:
             raise ValueError("invalid plan/layers for workspace query")
@@ -193,12 +214,14 @@ class PipelineWorkspace:
         self.nbytes = n
 
 
-def sq_pipeline_run(plan: Plan, rank: int, layers: list[Layer], comm: Comm | None, x0: torch.Tensor | None,
+def sq_pipeline_run(plan: Plan, rank: int, layers, comm: Comm | None, x0: torch.Tensor | None,
                     out: torch.Tensor | None, ws: PipelineWorkspace, stream=None, arr=None) -> dict:
-    """a6: run the whole generation (prefill + n_decode steps) for this rank (rank -1: all stages)."""
-    arr = layer_array(layers) if arr is None else arr
+    """a6: run the whole generation (prefill + n_decode steps) for this rank (rank -1: all stages).
+    TP plans (plan.tp > 1): layers = this rank's shards, or for rank -1 the [tp][n_layers] shard sets."""
+    flat, n_layers = _flat(layers)
+    arr = layer_array(flat) if arr is None else arr
     st = sq_run_stats()
-    _check(_L.sq_pipeline_run(ctypes.byref(plan.c), rank, arr, len(layers), comm.h if comm else None, _ptr(x0),
+    _check(_L.sq_pipeline_run(ctypes.byref(plan.c), rank, arr, n_layers, comm.h if comm else None, _ptr(x0),
                               _ptr(out), ctypes.c_void_p(ws.ptr), ws.nbytes, ctypes.byref(st), _stream(stream)))
     return {"t_total_ms": st.t_total_ms, "t_prefill_ms": st.t_prefill_ms, "t_decode_ms": st.t_decode_ms,
             "tokens_per_s": st.tokens_per_s, "bytes_sent": st.bytes_sent, "gpu_launches": st.gpu_launches,

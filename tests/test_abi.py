@@ -29,7 +29,7 @@ def test_library_exports_every_declared_symbol():
 def test_host_only_functions():
     import paper_conf_cluster_zhaowplw25_b200 as sq
     L = sq.lib()
-    assert L.sq_abi_version() == 2
+    assert L.sq_abi_version() == 3
     # (4 h1^2 + 2 h1 h2) * bit/8 bytes per layer
     h1 = 9216
     for bits in (3, 4, 8, 16):

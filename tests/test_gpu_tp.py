@@ -164,3 +164,43 @@ def test_tp_argument_errors():
     R.sq_stage_forward_tp(g3, 1, torch.zeros((2, 384), device="cuda"), torch.empty((2, 384), device="cuda"),
                           R.TpWorkspace(g3, 2), 3)
     torch.cuda.synchronize()
+
+
+def _oracle_full(L, h1, h2, bits):
+    full = []
+    for l in range(L):
+        q = {}
+        for name, (n, k) in {"qkv": (3 * h1, h1), "o": (h1, h1), "fc1": (h2, h1), "fc2": (h1, h2)}.items():
+            seed = synth.weight_seed(l, name)
+            q[name] = O.QWeight(synth.weight_f16(seed, n, k), int(bits[l]), bias=synth.bias_f16(seed, n))
+        full.append(O.Layer(int(bits[l]), 0, q["qkv"], q["o"], q["fc1"], q["fc2"]))
+    return full
+
+
+@pytest.mark.parametrize("P,tp,heads,kappa", [(2, 2, 0, 1), (1, 3, 0, 1), (2, 2, 12, 2), (3, 3, 12, 1)])
+def test_pipeline_mesh_virtual(P, tp, heads, kappa):
+    # a P x tp mesh (TP inside every pipeline stage, P:236 / P:318) run whole on one device (rank -1),
+    # configs[0] shapes, against the UNSHARDED oracle pipeline (O7, or O7 with attention)
+    sq, R = sqm()
+    from paper_conf_cluster_zhaowplw25_b200 import plan as PL
+    h1, h2, L = 768, 3072, 6
+    B, eta, xi, s, n_dec = 3, 2, 2, 16, 4
+    bits = [4, 3, 16, 8, 4, 3]
+    sol = PL.partition_layers([1.0] * L, P)
+    plan = R.Plan(bits, sol, h1, h2, B, eta, xi, s, n_dec, n_heads=heads, kappa=kappa, tp=tp)
+    R.sq_plan_check(plan)
+    sets = R.build_tp_layers(L, h1, h2, bits, tp)
+    comm = R.Comm.local(P)
+    ws = R.PipelineWorkspace(plan, sets, -1)
+    x0 = synth.hidden_f32(1, B * s, h1).reshape(B, s, h1)
+    out = torch.zeros((B, 1 + n_dec, h1), dtype=torch.float32, device="cuda")
+    st = R.sq_pipeline_run(plan, -1, sets, comm, torch.from_numpy(x0).cuda(), out, ws)
+    comm.destroy()
+    full = _oracle_full(L, h1, h2, bits)
+    ref = O.pipeline_attn(full, x0.astype(np.float64), n_dec, heads) if heads else \
+        O.pipeline(full, x0.astype(np.float64), n_dec)
+    got = out.cpu().numpy()
+    for t in range(1 + n_dec):
+        assert nw(got[:, t], ref[:, t]) <= TOL, (t, nw(got[:, t], ref[:, t]))
+    if heads == 0:
+        assert st["graph_replays"] > 0   # the virtual TP decode step replays from the graph cache
