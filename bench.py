@@ -532,6 +532,10 @@ def run_ours(args, wl):
             del ws
             torch.cuda.empty_cache()
             extra["attention"] = attention_run(wl, plan, layers, arr, x0, pk)
+        if not args.no_tp and args.workload == "opt66b":
+            layers.clear()
+            torch.cuda.empty_cache()
+            extra["tp_stage"] = tp_run()
         if not args.no_bloom and args.workload == "opt66b":
             layers.clear()  # the OPT-66B model's HBM goes to the BLOOM-176B-shaped one
             torch.cuda.empty_cache()
@@ -735,6 +739,74 @@ def bloom_run(pk: dict, steps: int = 1):
     return res
 
 
+# ------------------------------------------------------------------ f4: tensor-parallel stages
+def tp_run(reps: int = 5, tps=(2, 4, 8)):
+    """SURVEY 8(f) f4 intra-node TP: 4 OPT-66B-shaped layers (bits 4/3/4/8) as one stage,
+    unsharded (sq_stage_forward) and split T ways (sq_stage_forward_tp, virtual: the T shard sets run
+    one after the other on this GPU, so time / T is one TP rank's compute).  Decode micro-batch 32 and a
+    2048-token prefill item; each call captured in a CUDA graph, median of `reps` replays.
+    eff = t(TP1) / t(TP T virtual): 1.0 means the 1/T-wide kernels keep the unsharded kernels' efficiency,
+    i.e. T ranks would run the stage T x faster before the all-reduce (not measurable on one GPU; its
+    algorithmic volume per rank is 2 x layers x tokens x h1 x 4 bytes per step, reported)."""
+    import statistics
+    import torch
+    import synth
+    from paper_conf_cluster_zhaowplw25_b200 import runtime as R
+    L, h1, h2 = 4, 9216, 36864
+    bits = [4, 3, 4, 8]
+    cases = (("decode", 1, 32), ("prefill", 0, 2048))
+
+    def timed(fn):
+        fn()
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            fn()
+        g.replay()
+        torch.cuda.synchronize()
+        ts = []
+        for _ in range(reps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            g.replay()
+            e1.record()
+            torch.cuda.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        del g
+        return statistics.median(ts)
+
+    res = {"workload": "4 OPT-66B layers (h1 9216, h2 36864), bits 4/3/4/8; decode m = 32, prefill 2048 tokens",
+           "results": []}
+    base = {}
+    g1 = R.build_layers(L, h1, h2, bits)
+    for name, phase, T_tok in cases:
+        x = torch.empty((T_tok, h1), dtype=torch.float32, device="cuda")
+        synth.device_fill_f32(x.data_ptr(), 5, 0, x.numel(), 1.0, False)
+        y = torch.empty_like(x)
+        ws = R.StageWorkspace(g1, T_tok)
+        arr = R.layer_array(g1)
+        base[name] = timed(lambda: R.sq_stage_forward(g1, phase, x, y, ws, arr=arr))
+        res["results"].append({"tp": 1, "phase": name, "ms": round(base[name], 3)})
+        del ws
+    del g1
+    torch.cuda.empty_cache()
+    for T in tps:
+        sets = R.build_tp_layers(L, h1, h2, bits, T)
+        for name, phase, T_tok in cases:
+            x = torch.empty((T_tok, h1), dtype=torch.float32, device="cuda")
+            synth.device_fill_f32(x.data_ptr(), 5, 0, x.numel(), 1.0, False)
+            y = torch.empty_like(x)
+            ws = R.TpWorkspace(sets, T_tok)
+            ms = timed(lambda: R.sq_stage_forward_tp(sets, phase, x, y, ws, T))
+            res["results"].append({"tp": T, "phase": name, "ms_all_shards": round(ms, 3),
+                                   "ms_per_rank": round(ms / T, 3), "eff": round(base[name] / ms, 3),
+                                   "allreduce_MB_per_rank": round(2 * L * T_tok * h1 * 4 / 1e6, 1)})
+            del ws
+        del sets
+        torch.cuda.empty_cache()
+    return res
+
+
 # ------------------------------------------------------------------ f3: the same run with real attention
 def attention_run(wl: dict, plan0, layers, arr, x0, pk: dict, steps: int = 1):
     """the configs[3] generation with causal attention over a KV cache (head_dim 128,
@@ -819,6 +891,7 @@ def main():
     ap.add_argument("--no-configs0", action="store_true")
     ap.add_argument("--no-attention", action="store_true")
     ap.add_argument("--no-bloom", action="store_true")
+    ap.add_argument("--no-tp", action="store_true")
     ap.add_argument("--cpu-tokens", type=int, default=8)
     ap.add_argument("--cpu-row-frac", type=int, default=8)
     args = ap.parse_args()

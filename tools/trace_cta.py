@@ -39,3 +39,9 @@ nu = int((t[4] > 0).sum())
 if nu > 2:
     print(f"CTA0 units traced {nu}: MMA issue rate {(t[4, nu - 1] - t[4, 1]) / max(nu - 2, 1):.0f} cycles/unit; "
           f"last MMA issued at {(t[4, nu - 1] - c0) / ghz / 1e3:.2f} us")
+ac = (t[9, :ns] - g0) / 1e3
+if (t[9, :ns] > 0).all():
+    print(f"accumulators complete min/med/max {ac.min():.2f}/{np.median(ac):.2f}/{ac.max():.2f} us")
+if (t[10, :ns] > 0).all():
+    cs = (t[10, :ns] - g0) / 1e3
+    print(f"cluster partials in place min/med/max {cs.min():.2f}/{np.median(cs):.2f}/{cs.max():.2f} us")
