@@ -19,12 +19,26 @@
 //  * Epilogue: the dequant warps tcgen05.ld the accumulator (lane = weight row,
 //    column = token), add bias / activation / residual, store y.
 // Warp roles: 0 = TMA producer, 1 = MMA issuer (+TMEM alloc), 2..9 = dequant (2 groups) + epilogue.
+//
+// CTA-pair variant (CG = 2, the default when n / 128 is even): the two CTAs of a (2, 1, 1) cluster
+// hold adjacent 128-row weight tiles of the same 256-token tile; each loads HALF the activation tile
+// (128 tokens) by TMA with .cta_group::2 (both halves complete on the leader's barrier) and
+// dequantizes its own rows into its own TMEM; the leader issues tcgen05.mma.cta_group::2 (M = 256,
+// N = 256, A from both CTAs' TMEM, B from both CTAs' shared memory) and commits to both CTAs'
+// barriers (multicast); the peer's dequant warps signal the leader's "A ready" barrier remotely.
+// Each SM then streams and reads half the activation bytes per MMA (the 1-CTA tile's activation
+// traffic -- TMA writes + MMA reads of B -- saturated the shared-memory port), and the pair reads the
+// activation tile from L2 once instead of twice.
 #include <cuda.h>
 
 #include <cstring>
 #include <mutex>
 
 #include "sq_tc.cuh"
+
+#ifndef SQ_GEMM_SX2
+#define SQ_GEMM_SX2 8
+#endif
 
 namespace sq {
 namespace {
@@ -33,19 +47,24 @@ using namespace tc;
 constexpr int BN = 128;   // weight rows per tile (TMEM lanes, MMA M)
 constexpr int BT = 256;   // tokens per tile (MMA N)
 constexpr int XK = 64;    // k per activation stage (one 128-B swizzle row)
-constexpr int S_X = 4;
 constexpr int S_A = 4;
 constexpr int DQ_GROUPS = 2;  // dequant warp-groups on alternating groups of k
 // ring depths S_A and S_W are multiples of DQ_GROUPS so that every slot belongs to one group
 // (consumed in order): an mbarrier parity wait can never run two phases ahead of its slot
-constexpr int X_STAGE_BYTES = BT * XK * 2;  // 32 KB
+template <int CG>
+constexpr int x_stage_bytes() { return BT / CG * XK * 2; }  // 32 KB (one CTA) / 16 KB (per CTA of a pair)
+// activation ring depth: the pair's half-size stages buy twice the stages for the same shared memory
+template <int CG>
+constexpr int x_stages() { return CG == 2 ? SQ_GEMM_SX2 : 4; }
 constexpr int TMEM_COLS = 512;
 constexpr int D_COL = 0;
 constexpr int A_COL = 256;
 constexpr int NUM_THREADS = 32 * (2 + 4 * DQ_GROUPS);
 
-template <int BITS>
+template <int BITS, int CG>
 struct Smem {
+  static constexpr int X_STAGE_BYTES = x_stage_bytes<CG>();
+  static constexpr int S_X = x_stages<CG>();
   static constexpr int W_STAGE = ((BN * GCfg<BITS>::GB + 1023) / 1024) * 1024;
   static constexpr int OFF_X = 0;
   static constexpr int OFF_W = OFF_X + S_X * X_STAGE_BYTES;
@@ -67,14 +86,60 @@ struct GemmP {
   int kg;
 };
 
-// instruction descriptor: kind::f16, A=B=f16 K-major, D=f32, M=128, N=256
-constexpr uint32_t kIdesc = make_idesc(BN, BT);
+// ---- CTA-pair (cta_group::2) primitives
+__device__ __forceinline__ uint32_t cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+// shared::cluster address of the same byte in CTA `rank` of the cluster
+__device__ __forceinline__ uint32_t mapa_u32(uint32_t local, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(local), "r"(rank));
+  return r;
+}
+// arrive on a barrier of either CTA of the pair (cluster address).  Default .release.cta semantics,
+// as CUTLASS's cluster barrier: the TMEM stores it publishes are ordered by tcgen05.wait::st +
+// tcgen05.fence::before_thread_sync, and a cluster-scope release (plus cluster-scope acquire polls
+// on the leader) put a memory barrier on every arrival and poll: measured 15-30 % slower GEMMs.
+__device__ __forceinline__ void mbar_arrive_cl(uint32_t cl_addr) {
+  asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(cl_addr) : "memory");
+}
+// TMA load by either CTA of a pair, completing on the barrier at cluster address mbar_cl (the leader's)
+__device__ __forceinline__ void tma_load_2d_cg2(void* smem_dst, const void* tmap, uint32_t mbar_cl, int32_t c0,
+                                                int32_t c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];"
+      ::"r"(smem_u32(smem_dst)), "l"(tmap), "r"(mbar_cl), "r"(c0), "r"(c1)
+      : "memory");
+}
+__device__ __forceinline__ void tc_mma_ts_cg2(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc,
+                                              uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+// commit the leader's MMAs to the barrier at the same offset in both CTAs of the pair
+__device__ __forceinline__ void tc_commit_cg2(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;"
+               ::"r"(smem_u32(bar)), "h"((uint16_t)0x3)
+               : "memory");
+}
 
-template <int BITS, int EPI>
+template <int BITS, int EPI, int CG>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
     k_gemm(const __grid_constant__ CUtensorMap tm_x, const __grid_constant__ CUtensorMap tm_w,
            const __grid_constant__ CUtensorMap tm_m, const GemmP p) {
-  using SM = Smem<BITS>;
+  using SM = Smem<BITS, CG>;
+  constexpr int X_STAGE_BYTES = SM::X_STAGE_BYTES;
+  constexpr int S_X = SM::S_X;
+  // instruction descriptor: kind::f16, A=B=f16 K-major, D=f32, M = 128 per CTA, N = 256
+  constexpr uint32_t kIdesc = make_idesc(BN * CG, BT);
   constexpr int S_W = GCfg<BITS>::S_W;
   static_assert(S_W % DQ_GROUPS == 0 && S_A % DQ_GROUPS == 0, "slots must not be shared by dequant groups");
   constexpr int GB = GCfg<BITS>::GB;
@@ -94,23 +159,36 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(smem + SM::OFF_TMEM);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int64_t n0 = (int64_t)blockIdx.y * BN;   // weight-row tile
-  const int64_t t0 = (int64_t)blockIdx.x * BT;   // token tile
+  // weight-row tile, token tile.  Pairs (cluster (2, 1, 1): tcgen05 pairs CTAs along x) take
+  // blockIdx.x = 2 x token tile + rank, blockIdx.y = row-tile pair, so consecutive CTAs still share a
+  // weight panel as in the one-CTA grid (x = token tile, y = row tile)
+  const int64_t n0 = CG == 2 ? ((int64_t)blockIdx.y * 2 + (blockIdx.x & 1)) * BN : (int64_t)blockIdx.y * BN;
+  const int64_t t0 = CG == 2 ? (int64_t)(blockIdx.x >> 1) * BT : (int64_t)blockIdx.x * BT;
   const int kg = p.kg;
+  const uint32_t rank = CG == 2 ? cluster_rank() : 0;  // CTA of the pair (0 = leader, issues the MMAs)
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < S_X; ++i) { mbar_init(&full_x[i], 1); mbar_init(&empty_x[i], 1); }
     for (int i = 0; i < S_W; ++i) { mbar_init(&full_w[i], 1); mbar_init(&empty_w[i], 4); }
-    for (int i = 0; i < S_A; ++i) { mbar_init(&full_a[i], 4); mbar_init(&empty_a[i], 1); }
+    for (int i = 0; i < S_A; ++i) { mbar_init(&full_a[i], 4 * CG); mbar_init(&empty_a[i], 1); }
     mbar_init(d_full, 1);
     fence_barrier_init();
     prefetch_tmap(&tm_x);
     prefetch_tmap(&tm_w);
     if constexpr (BITS != 16) prefetch_tmap(&tm_m);
   }
-  if (warp == 1) tmem_alloc(tmem_slot, TMEM_COLS);
+  if (warp == 1) {
+    if constexpr (CG == 2) {
+      asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                   "r"(TMEM_COLS) : "memory");
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+    } else {
+      tmem_alloc(tmem_slot, TMEM_COLS);
+    }
+  }
   tc_fence_before();
   __syncthreads();
+  if constexpr (CG == 2) cluster_sync_all();  // the peer's barriers are initialised before any remote arrive
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
 
@@ -134,14 +212,22 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         for (int h = 0; h < 2; ++h, ++it_x) {
           const int sx = it_x % S_X, rx = it_x / S_X;
           mbar_wait(&empty_x[sx], (rx & 1) ^ 1);
-          if (elect_one()) mbar_arrive_expect_tx(&full_x[sx], X_STAGE_BYTES);
-          if (elect_one()) tma_load_2d(smem + SM::OFF_X + sx * X_STAGE_BYTES, &tm_x, &full_x[sx], g * 128 + h * XK, (int32_t)t0);
+          if constexpr (CG == 2) {
+            // this CTA's half of the token tile; both halves complete on the leader's barrier
+            if (rank == 0 && elect_one()) mbar_arrive_expect_tx(&full_x[sx], 2 * X_STAGE_BYTES);
+            if (elect_one())
+              tma_load_2d_cg2(smem + SM::OFF_X + sx * X_STAGE_BYTES, &tm_x, mapa_u32(smem_u32(&full_x[sx]), 0),
+                              g * 128 + h * XK, (int32_t)(t0 + rank * (BT / 2)));
+          } else {
+            if (elect_one()) mbar_arrive_expect_tx(&full_x[sx], X_STAGE_BYTES);
+            if (elect_one()) tma_load_2d(smem + SM::OFF_X + sx * X_STAGE_BYTES, &tm_x, &full_x[sx], g * 128 + h * XK, (int32_t)t0);
+          }
         }
       }
     }
   } else if (warp == 1) {
-    // ---------------- MMA issuer (single thread)
-    {  // whole warp runs the loop; the elected leader issues tcgen05.mma / commit
+    // ---------------- MMA issuer (single thread; the pair's leader only)
+    if (CG == 1 || rank == 0) {  // whole warp runs the loop; the elected leader issues tcgen05.mma / commit
       int it_x = 0;
       for (int g = 0; g < kg; ++g) {
         const int sa = g % S_A, ra = g / S_A;
@@ -156,13 +242,17 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           for (int kk = 0; kk < XK / 16; ++kk) {
             const uint64_t bdesc = make_sw128_desc(xs + kk * 32);
             const uint32_t a_tm = tmem + A_COL + sa * 64 + h * 32 + kk * 8;
-            if (elect_one()) tc_mma_ts(tmem + D_COL, a_tm, bdesc, kIdesc, (g | h | kk) != 0);
+            if constexpr (CG == 2) {
+              if (elect_one()) tc_mma_ts_cg2(tmem + D_COL, a_tm, bdesc, kIdesc, (g | h | kk) != 0);
+            } else {
+              if (elect_one()) tc_mma_ts(tmem + D_COL, a_tm, bdesc, kIdesc, (g | h | kk) != 0);
+            }
           }
-          if (elect_one()) tc_commit(&empty_x[sx]);
+          if (elect_one()) { if constexpr (CG == 2) tc_commit_cg2(&empty_x[sx]); else tc_commit(&empty_x[sx]); }
         }
-        if (elect_one()) tc_commit(&empty_a[sa]);
+        if (elect_one()) { if constexpr (CG == 2) tc_commit_cg2(&empty_a[sa]); else tc_commit(&empty_a[sa]); }
       }
-      if (elect_one()) tc_commit(d_full);
+      if (elect_one()) { if constexpr (CG == 2) tc_commit_cg2(d_full); else tc_commit(d_full); }
     }
   } else {
     // ---------------- dequant warps (one thread per weight row; group gi takes k-groups
@@ -184,7 +274,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       __syncwarp();
       if (lane == 0) {
         mbar_arrive(&empty_w[sw]);
-        mbar_arrive(&full_a[sa]);
+        // (pair: the leader's barrier, from either CTA)
+        if constexpr (CG == 2) mbar_arrive_cl(mapa_u32(smem_u32(&full_a[sa]), 0)); else mbar_arrive(&full_a[sa]);
       }
     }
     // ---------------- epilogue (each dequant group drains half of the 256 token columns)
@@ -235,9 +326,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   }
   tc_fence_before();
   __syncthreads();
+  if constexpr (CG == 2) cluster_sync_all();  // neither CTA frees TMEM / shared memory the pair still reads
   if (warp == 1) {
     tc_fence_after();
-    tmem_dealloc(tmem, TMEM_COLS);
+    if constexpr (CG == 2)
+      asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS) : "memory");
+    else
+      tmem_dealloc(tmem, TMEM_COLS);
   }
 }
 
@@ -249,29 +344,59 @@ cudaError_t encode_2d(CUtensorMap* m, CUtensorMapDataType dt, const void* ptr, u
   return encode_nd(m, dt, ptr, 2, dims, st, box, sw);
 }
 
-template <int BITS, int EPI>
+template <int BITS, int EPI, int CG>
 cudaError_t launch_be(const CUtensorMap& tx, const CUtensorMap& tw, const CUtensorMap& tm, const GemmP& p, cudaStream_t s) {
-  auto kern = k_gemm<BITS, EPI>;
+  auto kern = k_gemm<BITS, EPI, CG>;
   static bool attr_set = false;
   if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Smem<BITS>::BYTES);
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Smem<BITS, CG>::BYTES);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
   dim3 grid((unsigned)((p.m + BT - 1) / BT), (unsigned)(p.n / BN));
-  kern<<<grid, NUM_THREADS, Smem<BITS>::BYTES, s>>>(tx, tw, tm, p);
-  return cudaGetLastError();
+  if constexpr (CG == 2) grid = dim3(2 * grid.x, grid.y / 2);
+  if constexpr (CG == 1) {
+    kern<<<grid, NUM_THREADS, Smem<BITS, CG>::BYTES, s>>>(tx, tw, tm, p);
+    return cudaGetLastError();
+  } else {
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = grid;
+    cfg.blockDim = dim3(NUM_THREADS);
+    cfg.dynamicSmemBytes = Smem<BITS, CG>::BYTES;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 2;  // the pair: adjacent 128-row weight tiles of one token tile
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kern, tx, tw, tm, p);
+  }
+}
+
+template <int BITS, int CG>
+cudaError_t launch_bc(const CUtensorMap& tx, const CUtensorMap& tw, const CUtensorMap& tm, const GemmP& p, int epi,
+                      cudaStream_t s) {
+  switch (epi) {
+    case SQ_EPI_F16: return launch_be<BITS, SQ_EPI_F16, CG>(tx, tw, tm, p, s);
+    case SQ_EPI_F16_RELU: return launch_be<BITS, SQ_EPI_F16_RELU, CG>(tx, tw, tm, p, s);
+    case SQ_EPI_F16_GELU: return launch_be<BITS, SQ_EPI_F16_GELU, CG>(tx, tw, tm, p, s);
+    default: return launch_be<BITS, SQ_EPI_F32_ACCUM, CG>(tx, tw, tm, p, s);
+  }
+}
+
+// CTA pairs when the row tiles pair up (n / 128 even); SQ_GEMM_CG=1 forces the one-CTA tile
+int gemm_cg(int64_t n) {
+  static int forced = -1;
+  if (forced < 0) { const char* e = getenv("SQ_GEMM_CG"); forced = (e && e[0] == '1') ? 1 : 0; }
+  return (forced == 1 || (n / BN) % 2) ? 1 : 2;
 }
 
 template <int BITS>
 cudaError_t launch_b(const CUtensorMap& tx, const CUtensorMap& tw, const CUtensorMap& tm, const GemmP& p, int epi,
                      cudaStream_t s) {
-  switch (epi) {
-    case SQ_EPI_F16: return launch_be<BITS, SQ_EPI_F16>(tx, tw, tm, p, s);
-    case SQ_EPI_F16_RELU: return launch_be<BITS, SQ_EPI_F16_RELU>(tx, tw, tm, p, s);
-    case SQ_EPI_F16_GELU: return launch_be<BITS, SQ_EPI_F16_GELU>(tx, tw, tm, p, s);
-    default: return launch_be<BITS, SQ_EPI_F32_ACCUM>(tx, tw, tm, p, s);
-  }
+  return gemm_cg(p.n) == 2 ? launch_bc<BITS, 2>(tx, tw, tm, p, epi, s) : launch_bc<BITS, 1>(tx, tw, tm, p, epi, s);
 }
 
 }  // namespace
@@ -281,7 +406,7 @@ cudaError_t launch_gemm(const sq_qweight& w, const __half* x, int64_t ldx, int64
   CUtensorMap tx, tw, tm;
   memset(&tm, 0, sizeof(tm));
   cudaError_t e = encode_2d(&tx, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, x, (uint64_t)w.k, (uint64_t)m, (uint64_t)ldx * 2,
-                            XK, BT, CU_TENSOR_MAP_SWIZZLE_128B);
+                            XK, BT / gemm_cg(w.n), CU_TENSOR_MAP_SWIZZLE_128B);
   if (e != cudaSuccess) return e;
   if (w.bits == 16) {
     e = encode_2d(&tw, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, w.packed, (uint64_t)w.k, (uint64_t)w.n, (uint64_t)w.k * 2, 64,
