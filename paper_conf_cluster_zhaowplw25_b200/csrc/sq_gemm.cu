@@ -20,7 +20,7 @@
 //    column = token), add bias / activation / residual, store y.
 // Warp roles: 0 = TMA producer, 1 = MMA issuer (+TMEM alloc), 2..9 = dequant (2 groups) + epilogue.
 //
-// CTA-pair variant (CG = 2, the default when n / 128 is even): the two CTAs of a (2, 1, 1) cluster
+// CTA-pair variant (CG = 2, the default when n / 128 is even and m >= 512): the two CTAs of a (2, 1, 1) cluster
 // hold adjacent 128-row weight tiles of the same 256-token tile; each loads HALF the activation tile
 // (128 tokens) by TMA with .cta_group::2 (both halves complete on the leader's barrier) and
 // dequantizes its own rows into its own TMEM; the leader issues tcgen05.mma.cta_group::2 (M = 256,
@@ -386,17 +386,20 @@ cudaError_t launch_bc(const CUtensorMap& tx, const CUtensorMap& tw, const CUtens
   }
 }
 
-// CTA pairs when the row tiles pair up (n / 128 even); SQ_GEMM_CG=1 forces the one-CTA tile
-int gemm_cg(int64_t n) {
+// CTA pairs when the row tiles pair up (n / 128 even) and the GEMM has at least two token tiles' worth
+// of tokens (a 32-token OPT-125m prefill linear took ~9 us longer as a pair: cluster launch and
+// barriers for a few CTAs); SQ_GEMM_CG=1 forces the one-CTA tile, SQ_GEMM_CG=2 pairs at any m
+int gemm_cg(int64_t n, int64_t m) {
   static int forced = -1;
-  if (forced < 0) { const char* e = getenv("SQ_GEMM_CG"); forced = (e && e[0] == '1') ? 1 : 0; }
-  return (forced == 1 || (n / BN) % 2) ? 1 : 2;
+  if (forced < 0) { const char* e = getenv("SQ_GEMM_CG"); forced = !e ? 0 : (e[0] == '1' ? 1 : (e[0] == '2' ? 2 : 0)); }
+  if (forced == 1 || (n / BN) % 2) return 1;
+  return (forced == 2 || m >= 2 * BT) ? 2 : 1;
 }
 
 template <int BITS>
 cudaError_t launch_b(const CUtensorMap& tx, const CUtensorMap& tw, const CUtensorMap& tm, const GemmP& p, int epi,
                      cudaStream_t s) {
-  return gemm_cg(p.n) == 2 ? launch_bc<BITS, 2>(tx, tw, tm, p, epi, s) : launch_bc<BITS, 1>(tx, tw, tm, p, epi, s);
+  return gemm_cg(p.n, p.m) == 2 ? launch_bc<BITS, 2>(tx, tw, tm, p, epi, s) : launch_bc<BITS, 1>(tx, tw, tm, p, epi, s);
 }
 
 }  // namespace
@@ -406,7 +409,7 @@ cudaError_t launch_gemm(const sq_qweight& w, const __half* x, int64_t ldx, int64
   CUtensorMap tx, tw, tm;
   memset(&tm, 0, sizeof(tm));
   cudaError_t e = encode_2d(&tx, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, x, (uint64_t)w.k, (uint64_t)m, (uint64_t)ldx * 2,
-                            XK, BT / gemm_cg(w.n), CU_TENSOR_MAP_SWIZZLE_128B);
+                            XK, BT / gemm_cg(w.n, m), CU_TENSOR_MAP_SWIZZLE_128B);
   if (e != cudaSuccess) return e;
   if (w.bits == 16) {
     e = encode_2d(&tw, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, w.packed, (uint64_t)w.k, (uint64_t)w.n, (uint64_t)w.k * 2, 64,

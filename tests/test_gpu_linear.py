@@ -295,3 +295,23 @@ def test_decode_mma_full_grid_sampled(bits):
     script = os.path.join(os.path.dirname(os.path.abspath(__file__)), "_decode_path_check.py")
     r = subprocess.run([sys.executable, script, "full", str(bits)], env=env, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+
+
+def test_prefill_cta_pair_bitwise(tmp_path):
+    """K3's CTA-pair tile (cta_group::2, the default for even n/128) and the one-CTA tile
+    (SQ_GEMM_CG=1) accumulate every output in the same k order: their outputs are bit-identical
+    (fp16 and fp32-residual epilogues, ragged token tiles whose second half is out of range)."""
+    import os
+    import subprocess
+    import sys
+    script = os.path.join(os.path.dirname(os.path.abspath(__file__)), "_prefill_cg_dump.py")
+    res = {}
+    for cg in ("1", "2"):
+        env = dict(os.environ, SQ_GEMM_CG=cg)
+        path = str(tmp_path / f"cg{cg}.npz")
+        r = subprocess.run([sys.executable, script, path], env=env, capture_output=True, text=True, timeout=600)
+        assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+        res[cg] = np.load(path)
+    for key in res["1"].files:
+        a, b = res["1"][key], res["2"][key]
+        assert np.array_equal(a.view(np.uint8), b.view(np.uint8)), key

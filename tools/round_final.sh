@@ -21,4 +21,11 @@ g = sq.W8Linear.from_fp16(w); x = torch.randn(m, k, device='cuda').half(); y = t
 for _ in range(4):
     xq, sx = sq.sq_quantize_act8(x); sq.sq_linear_w8a8(g, xq, sx, y, 0)
 torch.cuda.synchronize()" > /dev/null 2>&1
+timeout 300 ncu --set full --import-source on --clock-control none -k regex:k_gemm -s 3 -c 1 -o gpurun_out/final_gemm_b4_36864x9216_m4096 python tools/gemm_one.py 36864 9216 4 4096 > /dev/null 2>&1
+timeout 300 ncu --set full --import-source on --clock-control none -k regex:k_gemm -s 3 -c 1 -o gpurun_out/final_gemm_b16_27648x9216_m4096 python tools/gemm_one.py 27648 9216 16 4096 > /dev/null 2>&1
+# launch lists of one bench step (prefill window, decode window; serialised, cold cache)
+K='regex:k_gemm|k_gemv|k_layernorm|k_copy|k_xsum|k_attn|k_kv'
+B="python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu --no-gemv-sweep --no-gemm-sweep --no-configs0 --no-attention --no-bloom --no-tp"
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k "$K" -c 2100 --csv --log-file gpurun_out/final_launches_prefill.csv $B > gpurun_out/final_launch_pre.log 2>&1
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k "$K" -s 2100 -c 3000 --csv --log-file gpurun_out/final_launches_decode.csv $B > gpurun_out/final_launch_dec.log 2>&1
 tail -2 gpurun_out/final_pytest.log
