@@ -16,7 +16,7 @@ import os
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libsq.so")
+LIB_PATH = os.environ.get("SQ_LIB_PATH") or os.path.join(_HERE, "libsq.so")  # SQ_LIB_PATH: experiment builds
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} not built: run `python __graft_entry__.py build` (no CPU fallback exists)")
 _L = ctypes.CDLL(LIB_PATH)

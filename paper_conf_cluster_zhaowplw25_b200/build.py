@@ -15,8 +15,11 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
-OBJ = os.path.join(ROOT, "build", "obj")
-LIB = os.path.join(PKG, "libsq.so")
+# SQ_BUILD_TAG=<t> (experiments only): objects under build/obj_<t>, library libsq_<t>.so, loaded with
+# SQ_LIB_PATH; the product build is the untagged libsq.so
+_TAG = os.environ.get("SQ_BUILD_TAG", "")
+OBJ = os.path.join(ROOT, "build", "obj" + (f"_{_TAG}" if _TAG else ""))
+LIB = os.path.join(PKG, f"libsq_{_TAG}.so" if _TAG else "libsq.so")
 SYNTH_SRC = os.path.join(ROOT, "synth", "synth.cu")
 SYNTH_LIB = os.path.join(ROOT, "synth", "libsqsynth.so")
 

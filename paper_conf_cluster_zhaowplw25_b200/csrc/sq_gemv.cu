@@ -30,7 +30,19 @@
 namespace sq {
 namespace {
 
-constexpr int kWarps = 16;  // one 512-thread CTA per SM
+#ifndef SQ_K2_WARPS
+#define SQ_K2_WARPS 16
+#endif
+#ifndef SQ_K2_SMEM_KB
+#define SQ_K2_SMEM_KB 227
+#endif
+#ifndef SQ_K2_CPS
+#define SQ_K2_CPS 1
+#endif
+#ifndef SQ_K2_MINB
+#define SQ_K2_MINB 1
+#endif
+constexpr int kWarps = SQ_K2_WARPS;  // one 512-thread CTA per SM
 constexpr int kThreads = kWarps * 32;
 constexpr int kRows = 16;   // rows per unit (mma M)
 constexpr int kXsTok = 32;  // token slots per group in the xsum buffer
@@ -445,7 +457,7 @@ struct QRing {
   static constexpr int BARS = kWarps * 8 * 8;                     // <= 8 mbarriers per warp
   static constexpr int CH = BITS == 8 ? 2 : (BITS == 4 ? 3 : 4);  // units per slot (3.3-4.2 KB)
   static constexpr int SLOT = CH * (UB + UM);
-  static constexpr int S0 = (227 * 1024 - PART - BARS - 128) / kWarps / SLOT;
+  static constexpr int S0 = (SQ_K2_SMEM_KB * 1024 - PART - BARS - 128) / kWarps / SLOT;
   static constexpr int S = S0 > 8 ? 8 : S0;
   static constexpr int BYTES = PART + BARS + kWarps * S * SLOT;
   static_assert(S >= 2, "ring depth");
@@ -470,7 +482,7 @@ __device__ __forceinline__ void lds_codes(const uint8_t* p, uint32_t* c) {
 }
 
 template <int BITS, int TOK, int EPI>
-__global__ void __launch_bounds__(kThreads, 1) k_gemv_q(const GemvP p) {
+__global__ void __launch_bounds__(kThreads, SQ_K2_MINB) k_gemv_q(const GemvP p) {
   using RC = QRing<BITS, TOK>;
   constexpr int LU = Cfg<BITS>::LU;
   constexpr int GB = Cfg<BITS>::GB;
@@ -700,7 +712,7 @@ cudaError_t launch_b(const GemvP& p, int epi, cudaStream_t s) {
 
 // number of CTAs: one per SM (fewer for tiny problems so every warp gets >= 1 unit)
 int64_t gemv_ctas(int64_t U) {
-  const int64_t full = (int64_t)num_sms();
+  const int64_t full = (int64_t)num_sms() * SQ_K2_CPS;
   const int64_t need = (U + kWarps - 1) / kWarps;
   return need < full ? need : full;
 }

@@ -13,7 +13,8 @@ from __future__ import annotations
 
 import torch
 
-from . import QLinear, SQ_EPI_F16, SQ_EPI_F16_GELU, SQ_EPI_F16_RELU, sq_act_moments, sq_linear_prefill, sq_scale_sq_sums
+from . import (QLinear, SQ_EPI_F16, SQ_EPI_F16_GELU, SQ_EPI_F16_RELU, SQ_EPI_F32_ACCUM, sq_act_moments,
+               sq_linear_prefill, sq_scale_sq_sums)
 
 LINEARS = ("qkv", "o", "fc1", "fc2")
 
@@ -43,9 +44,9 @@ def layer_terms(layer_idx: int, h1: int, h2: int, bits_set=(3, 4, 8), act: int =
     qkv = torch.empty((calib_tokens, 3 * h1), dtype=torch.float16, device="cuda")
     sq_linear_prefill(QLinear.from_fp16(ws["qkv"], 16), a, qkv, SQ_EPI_F16)
     v = qkv[:, 2 * h1:].contiguous()
-    h = torch.empty((calib_tokens, h1), dtype=torch.float16, device="cuda")
-    sq_linear_prefill(QLinear.from_fp16(ws["o"], 16), v, h, SQ_EPI_F16)
-    h2in = _ln16(x + h.float())
+    r = x.clone()  # residual stream: the o-proj epilogue adds its product in fp32 (r += v W_o^T), as in the stage
+    sq_linear_prefill(QLinear.from_fp16(ws["o"], 16), v, r, SQ_EPI_F32_ACCUM)
+    h2in = _ln16(r)
     u = torch.empty((calib_tokens, h2), dtype=torch.float16, device="cuda")
     sq_linear_prefill(QLinear.from_fp16(ws["fc1"], 16), h2in, u, SQ_EPI_F16_RELU if act == 0 else SQ_EPI_F16_GELU)
     g = {}
