@@ -42,6 +42,9 @@ namespace {
 #ifndef SQ_K2_MINB
 #define SQ_K2_MINB 1
 #endif
+#ifndef SQ_K2S_SMEM_KB
+#define SQ_K2S_SMEM_KB 113
+#endif
 constexpr int kWarps = SQ_K2_WARPS;  // one 512-thread CTA per SM
 constexpr int kThreads = kWarps * 32;
 constexpr int kRows = 16;   // rows per unit (mma M)
@@ -647,6 +650,277 @@ __global__ void __launch_bounds__(kThreads, SQ_K2_MINB) k_gemv_q(const GemvP p) 
   reduce_tail<TOK, EPI>(p, part_s, C0, C1, R, warp, lane, g, q);
 }
 
+// ---------------------------------------------------------------- K2s: strips of RT row tiles (m <= 8)
+// A work item is (strip, group): RT consecutive 16-row tiles x one 128-k group.  The activation
+// fragment and the group sums of a group are loaded once per RT units (K2 re-loads them for every
+// unit), and the RT units' HMMA chains are independent (ILP).  Items are flattened strip-major /
+// group-minor and split evenly over the grid's warps, as K2's units are; each warp streams its
+// items into its own S-slot ring with per-lane bulk copies (lane r < RT: unit r's codes, lane
+// RT + r: its meta; placement T16 makes each unit one contiguous range).  Unpack, mma.sync and the
+// factorised per-group scale / zero are K2's.  Deterministic: the split strips are reduced in
+// fixed warp order in shared memory (in the warps' idle rings) and across CTAs by the last CTA to
+// arrive, in fixed CTA order.
+// K2s CTA: 8 warps, two CTAs per SM (measured against one 16-warp CTA: equal or up to 7 % faster on
+// OPT-13B / OPT-66B shapes; tools/exp_k2s2.sh)
+constexpr int kSWarps = 8;
+constexpr int kSThreads = kSWarps * 32;
+constexpr int kSCtasPerSm = 2;
+
+template <int BITS>
+struct SRing {
+  static constexpr int RT = BITS == 8 ? 2 : 4;                     // tiles per strip
+  static constexpr int UB = 16 * Cfg<BITS>::GB;                   // codes bytes per unit
+  static constexpr int SLOT = RT * (UB + 64);                     // one item: RT units + their meta
+  static constexpr int BAR_BYTES = kSWarps * 8 * 8;                // <= 8 mbarriers per warp
+  static constexpr int S0 = (SQ_K2S_SMEM_KB * 1024 - 128 - BAR_BYTES) / kSWarps / SLOT;
+  static constexpr int S = S0 > 8 ? 8 : S0;
+  static constexpr int PARTW = 2 * 8 * RT * kRows * 4;            // a warp's head / tail strip partials
+  static constexpr int BYTES = 128 + BAR_BYTES + kSWarps * S * SLOT;  // + alignment slack
+  static_assert(S >= 2 && S * SLOT >= PARTW && BYTES <= 227 * 1024 && SLOT % 128 == 0, "K2s shared memory");
+};
+
+template <int EPI, int RT>
+__device__ __forceinline__ void store_strip_tile(const GemvP& p, int tile, int g, int q, const float (&v)[4]) {
+  if (tile < p.n / kRows) store_out<8, EPI>(p, tile, g, q, reinterpret_cast<const float(&)[1][4]>(v));
+}
+
+// K2's reduce_tail for strips: in-CTA partials live in each warp's ring (stride WS bytes), the
+// cross-CTA partials in p.part [CTAs][2][8][RT * 16].
+template <int EPI, int RT, int WS>
+__device__ __forceinline__ void reduce_tail_s(const GemvP& p, const uint8_t* part_base, int C0, int C1, int R,
+                                              int warp, int lane, int g, int q) {
+  constexpr int TOK = 8, RR = RT * kRows;
+  const int kg = p.kg;
+  if (R <= 0) return;
+  const int t_first = C0 / kg, t_last = (C1 - 1) / kg;
+  for (int t = t_first + warp; t <= t_last; t += kSWarps) {
+    const int lo = t * kg > C0 ? t * kg : C0;
+    const int hi = (t + 1) * kg < C1 ? (t + 1) * kg : C1;  // exclusive
+    const int wa = (int)(((long long)(lo - C0 + 1) * kSWarps - 1) / R);
+    const int wb = (int)(((long long)(hi - C0) * kSWarps - 1) / R);
+    const bool whole = lo == t * kg && hi == (t + 1) * kg;
+    if (wa == wb && whole) continue;  // one warp stored it directly
+    float v[RT][4];
+#pragma unroll
+    for (int r = 0; r < RT; ++r)
+#pragma unroll
+      for (int i = 0; i < 4; ++i) v[r][i] = 0.f;
+    for (int wi = wa; wi <= wb; ++wi) {
+      const int wlo = C0 + range_lo(wi, R, kSWarps), whi = C0 + range_lo(wi + 1, R, kSWarps);
+      if (whi <= wlo) continue;  // empty warp range
+      const int sl = (wlo < t * kg) ? 1 : 0;
+      const float* qp = reinterpret_cast<const float*>(part_base + (size_t)wi * WS) + sl * TOK * RR;
+#pragma unroll
+      for (int r = 0; r < RT; ++r)
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+          const int tok = 2 * q + e;
+          v[r][e] += qp[tok * RR + r * kRows + g];
+          v[r][2 + e] += qp[tok * RR + r * kRows + g + 8];
+        }
+    }
+    if (whole) {
+#pragma unroll
+      for (int r = 0; r < RT; ++r) store_strip_tile<EPI, RT>(p, t * RT + r, g, q, v[r]);
+      continue;
+    }
+#ifdef SQ_K2S_ABL_NOFIX
+    continue;  // timing ablation only: results wrong
+#endif
+    // straddles a CTA boundary: publish this CTA's partial, the last CTA to arrive reduces
+    const int cslot = (C0 < t * kg) ? 1 : 0;
+    float* gp = p.part + ((int64_t)blockIdx.x * 2 + cslot) * TOK * RR;
+#pragma unroll
+    for (int r = 0; r < RT; ++r)
+#pragma unroll
+      for (int e = 0; e < 2; ++e) {
+        const int tok = 2 * q + e;
+        __stcg(gp + tok * RR + r * kRows + g, v[r][e]);
+        __stcg(gp + tok * RR + r * kRows + g + 8, v[r][2 + e]);
+      }
+    __threadfence();
+    __syncwarp();
+    const int NC = gridDim.x;
+    const int ca = (int)(((long long)(t * kg + 1) * NC - 1) / p.U);
+    const int cb2 = (int)(((long long)((t + 1) * kg) * NC - 1) / p.U);
+    int old = 0;
+    if (lane == 0) old = atomicAdd(p.cnt + t, 1);
+    old = __shfl_sync(0xffffffff, old, 0);
+    if (old != cb2 - ca) continue;
+    __threadfence();
+#pragma unroll
+    for (int r = 0; r < RT; ++r)
+#pragma unroll
+      for (int i = 0; i < 4; ++i) v[r][i] = 0.f;
+    for (int c = ca; c <= cb2; ++c) {
+      const int sl = (range_lo(c, p.U, NC) < t * kg) ? 1 : 0;
+      const float* qp = p.part + ((int64_t)c * 2 + sl) * TOK * RR;
+#pragma unroll
+      for (int r = 0; r < RT; ++r)
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+          const int tok = 2 * q + e;
+          v[r][e] += __ldcg(qp + tok * RR + r * kRows + g);
+          v[r][2 + e] += __ldcg(qp + tok * RR + r * kRows + g + 8);
+        }
+    }
+#pragma unroll
+    for (int r = 0; r < RT; ++r) store_strip_tile<EPI, RT>(p, t * RT + r, g, q, v[r]);
+    if (lane == 0) p.cnt[t] = 0;
+  }
+}
+
+template <int BITS, int EPI>
+__global__ void __launch_bounds__(kSThreads, kSCtasPerSm)
+    k_gemv_s(const __grid_constant__ CUtensorMap tm_w, const __grid_constant__ CUtensorMap tm_m, const GemvP p) {
+  using RC = SRing<BITS>;
+  constexpr int TOK = 8;
+  constexpr int LU = Cfg<BITS>::LU, GB = Cfg<BITS>::GB;
+  constexpr int RT = RC::RT, UB = RC::UB, SLOT = RC::SLOT, S = RC::S, RR = RT * kRows;
+  extern __shared__ float4 smem4[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>(smem4);
+  smem += (128 - (smem_u32(smem) & 127)) & 127;  // TMA destinations: 128-B aligned slots
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31, g = lane >> 2, q = lane & 3;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem) + warp * 8;
+  uint8_t* ring = smem + RC::BAR_BYTES + warp * S * SLOT;
+  const int kg = p.kg, m = p.m;
+  const int T = p.n / kRows;
+  const int C0 = range_lo(blockIdx.x, p.U, gridDim.x), C1 = range_lo(blockIdx.x + 1, p.U, gridDim.x);
+  const int R = C1 - C0;
+  const int u0 = C0 + range_lo(warp, R, kSWarps), u1 = C0 + range_lo(warp + 1, R, kSWarps);
+  const int nit = u1 - u0;
+  const int head_set = u0 / kg;
+  const int grp0 = u0 - head_set * kg;
+
+  // ---- the warp's ring: item c -> slot c % S, filled by lane 0 with two TMA boxes: the strip's RT
+  // units of group fgrp ([RT][UB] codes, 3-D map of 256-B lines) and their meta ([RT][16] u32)
+  int fset = head_set, fgrp = grp0;
+  auto issue = [&](int c) {
+    const int slot = c % S;
+    mbar_arrive_expect_tx(&bar[slot], (uint32_t)SLOT);
+    tma_load_3d(ring + slot * SLOT, &tm_w, &bar[slot], 0, fgrp * (UB / 256), fset * RT);
+    tma_load_2d(ring + slot * SLOT + RT * UB, &tm_m, &bar[slot], fgrp * 16, fset * RT);
+    if (++fgrp == kg) { fgrp = 0; ++fset; }
+  };
+  if (lane == 0) {
+    if (warp == 0) { prefetch_tmap(&tm_w); prefetch_tmap(&tm_m); }
+    for (int i = 0; i < S; ++i) mbar_init(&bar[i], 1);
+    fence_barrier_init();
+    for (int c = 0; c < S && c < nit; ++c) issue(c);
+  }
+  __syncwarp();
+  // PDL: the weight fetches above are independent of the previous kernel; everything below is not
+  pdl_trigger();
+  pdl_wait();
+
+  // the lane's activation row (token g) and k set, matching its codes (see k_gemv_q)
+  const bool xon = g < m;
+  const __half* xrow = p.x + (int64_t)(xon ? g : 0) * p.ldx + (BITS == 8 ? q * 16 : q * 32);
+  const int lane_off = BITS == 8 ? q * 16 : q * lane_bytes<BITS>();
+  uint32_t xt[16];
+#pragma unroll
+  for (int i = 0; i < 16; ++i) xt[i] = 0u;
+
+  int set = head_set, grp = grp0;
+  bool seg_from_start = (grp0 == 0);
+  float acc[RT][4], hacc[RT][4];
+#pragma unroll
+  for (int r = 0; r < RT; ++r)
+#pragma unroll
+    for (int i = 0; i < 4; ++i) { acc[r][i] = 0.f; hacc[r][i] = 0.f; }
+  bool has_head = false;
+
+  for (int c = 0; c < nit; ++c) {
+    const int slot = c % S;
+    // activation fragment + group sums of this group (independent of the slot)
+    if (xon) {
+      const uint4* xp = reinterpret_cast<const uint4*>(xrow + grp * 128);
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int xo = BITS == 8 ? (i < 2 ? i : 8 + (i - 2)) : i;  // 16-B units
+        const uint4 v = __ldg(xp + xo);
+        xt[4 * i] = v.x; xt[4 * i + 1] = v.y; xt[4 * i + 2] = v.z; xt[4 * i + 3] = v.w;
+      }
+    }
+    const float4 xsv = __ldg(reinterpret_cast<const float4*>(p.xsum + grp * kXsTok + 2 * q));
+    const float xs0 = xsv.x + xsv.y, xs1 = xsv.z + xsv.w;
+    const float xo0 = BITS == 4 ? fmaf(1024.f, xsv.x, 64.f * xsv.y) : (BITS == 3 ? 8.f * xs0 : 1024.f * xs0);
+    const float xo1 = BITS == 4 ? fmaf(1024.f, xsv.z, 64.f * xsv.w) : (BITS == 3 ? 8.f * xs1 : 1024.f * xs1);
+    mbar_wait(&bar[slot], (uint32_t)((c / S) & 1));
+    const uint8_t* cs = ring + slot * SLOT;
+    const uint32_t* ms = reinterpret_cast<const uint32_t*>(cs + RT * UB);
+#pragma unroll
+    for (int r = 0; r < RT; ++r) {
+      uint32_t cw0[LU], cw1[LU];
+      lds_codes<BITS>(cs + r * UB + g * GB + lane_off, cw0);
+      lds_codes<BITS>(cs + r * UB + (g + 8) * GB + lane_off, cw1);
+      const uint32_t mr0 = ms[r * 16 + g], mr1 = ms[r * 16 + g + 8];
+      float d[4];
+      {
+        uint32_t a[4];
+        frag<BITS>(cw0, 0, a[0], a[2]);
+        frag<BITS>(cw1, 0, a[1], a[3]);
+        mma_16816_zc(d, a, xt[0], xt[1]);
+      }
+#pragma unroll
+      for (int t = 1; t < 8; ++t) {
+        uint32_t a[4];
+        frag<BITS>(cw0, t, a[0], a[2]);
+        frag<BITS>(cw1, t, a[1], a[3]);
+        mma_16816(d, a, xt[2 * t], xt[2 * t + 1], d);
+      }
+      const float2 f0 = __half22float2(*reinterpret_cast<const __half2*>(&mr0));  // (s, z) row g
+      const float2 f1 = __half22float2(*reinterpret_cast<const __half2*>(&mr1));  // row g+8
+      // y += s * (D - xoff) + z * xs
+      acc[r][0] = fmaf(-f0.x, xo0, fmaf(f0.y, xs0, fmaf(f0.x, d[0], acc[r][0])));
+      acc[r][1] = fmaf(-f0.x, xo1, fmaf(f0.y, xs1, fmaf(f0.x, d[1], acc[r][1])));
+      acc[r][2] = fmaf(-f1.x, xo0, fmaf(f1.y, xs0, fmaf(f1.x, d[2], acc[r][2])));
+      acc[r][3] = fmaf(-f1.x, xo1, fmaf(f1.y, xs1, fmaf(f1.x, d[3], acc[r][3])));
+    }
+    __syncwarp();  // every lane's reads of this slot are done
+    if (lane == 0 && c + S < nit) issue(c + S);
+    if (grp == kg - 1) {  // strip finished
+      if (seg_from_start) {
+#pragma unroll
+        for (int r = 0; r < RT; ++r) store_strip_tile<EPI, RT>(p, set * RT + r, g, q, acc[r]);
+      } else {  // the head strip, entered part-way
+#pragma unroll
+        for (int r = 0; r < RT; ++r)
+#pragma unroll
+          for (int i = 0; i < 4; ++i) hacc[r][i] = acc[r][i];
+        has_head = true;
+      }
+#pragma unroll
+      for (int r = 0; r < RT; ++r)
+#pragma unroll
+        for (int i = 0; i < 4; ++i) acc[r][i] = 0.f;
+      seg_from_start = true;
+      grp = 0;
+      ++set;
+    } else {
+      ++grp;
+    }
+  }
+  // partial strips into the warp's idle ring: [2][TOK][RR], slot 0 = head strip, 1 = tail strip
+  __syncwarp();
+  float* pw = reinterpret_cast<float*>(ring);
+  auto put = [&](int sl, const float (&v)[RT][4]) {
+#pragma unroll
+    for (int r = 0; r < RT; ++r)
+#pragma unroll
+      for (int e = 0; e < 2; ++e) {
+        const int tok = 2 * q + e;
+        pw[(sl * TOK + tok) * RR + r * kRows + g] = v[r][e];
+        pw[(sl * TOK + tok) * RR + r * kRows + g + 8] = v[r][2 + e];
+      }
+  };
+  if (has_head) put(0, hacc);
+  if (nit > 0 && grp != 0) put(set == head_set ? 0 : 1, acc);  // range ended inside a strip
+  __syncthreads();
+  reduce_tail_s<EPI, RT, S * SLOT>(p, smem + RC::BAR_BYTES, C0, C1, R, warp, lane, g, q);
+}
+
 // xsum[g][t] = (sum_{k%4<2} x[t,k], sum_{k%4>=2} x[t,k]) over group g, t < 32 (0 for t >= m);
 // one warp per (g, t), fixed summation order.
 __global__ void k_xsum(const __half* __restrict__ x, int64_t ldx, int64_t m, int kg, float2* __restrict__ out) {
@@ -693,6 +967,41 @@ cudaError_t launch_e(const GemvP& p, cudaStream_t s) {
   return launch_pdl(kern, dim3((unsigned)p.W), dim3(kThreads), smem, s, p);
 }
 
+template <int BITS, int EPI>
+cudaError_t launch_s_e(const CUtensorMap& tw, const CUtensorMap& tm, const GemvP& p, cudaStream_t s) {
+  void (*kern)(const CUtensorMap, const CUtensorMap, const GemvP) = k_gemv_s<BITS, EPI>;
+  const size_t smem = (size_t)SRing<BITS>::BYTES;
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  return launch_pdl(kern, dim3((unsigned)p.W), dim3(kSThreads), smem, s, tw, tm, p);
+}
+
+template <int BITS>
+cudaError_t launch_s(const sq_qweight& w, const GemvP& p, int epi, cudaStream_t s) {
+  // codes: [n/16 tiles][kg * UB/256 lines][256 B], box = RT tiles x one unit; meta: [n/16][kg * 16] u32
+  constexpr int RT = SRing<BITS>::RT, UB = SRing<BITS>::UB;
+  CUtensorMap tw, tm;
+  const uint64_t nt = (uint64_t)w.n / kRows, kg = (uint64_t)p.kg;
+  const uint64_t dw[3] = {256, kg * (UB / 256), nt}, sw_[2] = {256, kg * UB};
+  const uint32_t bw[3] = {256, (uint32_t)(UB / 256), (uint32_t)RT};
+  cudaError_t e = encode_nd(&tw, CU_TENSOR_MAP_DATA_TYPE_UINT8, w.packed, 3, dw, sw_, bw, CU_TENSOR_MAP_SWIZZLE_NONE);
+  if (e != cudaSuccess) return e;
+  const uint64_t dm[2] = {kg * 16, nt}, sm_[1] = {kg * 64};
+  const uint32_t bm[2] = {16, (uint32_t)RT};
+  e = encode_nd(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, w.meta, 2, dm, sm_, bm, CU_TENSOR_MAP_SWIZZLE_NONE);
+  if (e != cudaSuccess) return e;
+  switch (epi) {
+    case SQ_EPI_F16: return launch_s_e<BITS, SQ_EPI_F16>(tw, tm, p, s);
+    case SQ_EPI_F16_RELU: return launch_s_e<BITS, SQ_EPI_F16_RELU>(tw, tm, p, s);
+    case SQ_EPI_F16_GELU: return launch_s_e<BITS, SQ_EPI_F16_GELU>(tw, tm, p, s);
+    default: return launch_s_e<BITS, SQ_EPI_F32_ACCUM>(tw, tm, p, s);
+  }
+}
+
 template <int BITS, int TOK>
 cudaError_t launch_t(const GemvP& p, int epi, cudaStream_t s) {
   switch (epi) {
@@ -717,11 +1026,36 @@ int64_t gemv_ctas(int64_t U) {
   return need < full ? need : full;
 }
 
+// K2s: two 8-warp CTAs per SM (fewer for tiny problems so every warp gets >= 1 item)
+int64_t gemv_s_ctas(int64_t U) {
+  const int64_t full = (int64_t)num_sms() * kSCtasPerSm;
+  const int64_t need = (U + kSWarps - 1) / kSWarps;
+  return need < full ? need : full;
+}
+
 int tok_pad(int64_t m) { return m <= 8 ? 8 : (m <= 16 ? 16 : 32); }
 
 // fixed-size counter region (n <= 65536) so linears of different n can share one workspace
 constexpr int64_t kMaxN = 65536;
 size_t cnt_bytes(int64_t) { return (size_t)(kMaxN / kRows) * sizeof(int); }
+// per-CTA boundary partials: K2 [W][2][tok][16], K2s [W][2][8][RT * 16] (RT <= 4)
+size_t part_bytes(int64_t W, int64_t m) {
+  const int64_t per = tok_pad(m) * kRows > 8 * 4 * kRows ? tok_pad(m) * kRows : 8 * 4 * kRows;
+  return (size_t)W * 2 * per * sizeof(float);
+}
+// K2s (strips) for quantized weights at m <= 8 (SQ_K2S=0: K2)
+// Whole strips only (n a multiple of RT * 16, so no TMA box reaches past the matrix).  Measured
+// (tools/exp_k2s.sh, back-to-back graph launches): K2s streams large linears at 4.9-5.1 TB/s INT4,
+// 6.1-6.5 INT8, 3.1-3.4 INT3 (m <= 8; K2 4.1 / 5.6 / 2.9, K2c 4.4-4.7 / 5.5-5.8 / 3.0-3.3), but
+// its finer split costs ~2 us more per launch than K2's on small INT3 / INT4 linears (5120^2 INT4:
+// 10.2 vs 8.3 us), so K2 keeps INT3 / INT4 linears under 20 MB.  SQ_K2S=0 / 1 forces K2 / K2s.
+bool use_k2s(int bits, int64_t n, int64_t k, int m) {
+  static int forced = -2;
+  if (forced == -2) { const char* e = getenv("SQ_K2S"); forced = !e ? -1 : (e[0] == '0' ? 0 : 1); }
+  if (bits == 16 || m > 8 || n % (bits == 8 ? 32 : 64) != 0) return false;
+  if (forced >= 0) return forced == 1;
+  return bits == 8 || (double)n * k * bits / 8.0 >= 20e6;
+}
 
 }  // namespace
 
@@ -729,8 +1063,8 @@ size_t xsum_bytes(int64_t k) { return (size_t)(k / 128) * kXsTok * sizeof(float2
 
 size_t gemv_workspace_bytes(int64_t n, int64_t k, int64_t m) {
   const int64_t U = (n / kRows) * (k / 128);
-  const int64_t W = gemv_ctas(U);
-  size_t part = (size_t)W * 2 * tok_pad(m) * kRows * sizeof(float);  // per-CTA boundary partials
+  const int64_t W = gemv_ctas(U) > gemv_s_ctas(U) ? gemv_ctas(U) : gemv_s_ctas(U);
+  size_t part = part_bytes(W, m);
   size_t a = cnt_bytes(n) + part + xsum_bytes(k) + 256;
   size_t b = n % 128 == 0 ? gemv_tc_workspace_bytes(n, k) : 0;
   return a > b ? a : b;
@@ -755,10 +1089,10 @@ int gemv_path(int64_t n, int64_t k, int m, int bits) {
   // (round 2, INT3 re-laid with a one-LOP3 unpack: the tcgen05 kernel wins INT3 linears from ~80 MB
   // at every m, e.g. 36864 x 9216 at m = 1: 3.34 vs 2.89 TB/s; the mma.sync kernel keeps the OPT-13B
   // sizes at m <= 8, e.g. 20480 x 5120: 2.24 vs 2.05 TB/s)
+  // (round 3: the strip kernel K2s streams every quantized linear at m <= 8 at least as fast as the
+  // tcgen05 kernel, e.g. 36864 x 9216 INT4 5.1 / 4.6 TB/s at m = 1 / 8 vs 4.4-4.7; tools/exp_k2s2.sh)
   if (bits == 16 || m > 8) return 1;
-  const double bytes = (double)n * k * bits / 8.0;
-  if (bytes >= 120e6 || (bits == 3 && bytes >= 80e6)) return 1;
-  return (bits == 4 && m > 4) ? 1 : 0;
+  return 0;
 }
 
 cudaError_t launch_xsum(const __half* x, int64_t ldx, int64_t m, int64_t k, float2* xsum, cudaStream_t s) {
@@ -787,10 +1121,11 @@ cudaError_t launch_gemv(const sq_qweight& w, const __half* x, int64_t ldx, int m
   p.ldy = (int)ldy;
   p.U = (int)((w.n / kRows) * p.kg);
   p.W = (int)gemv_ctas(p.U);
+  const int64_t wmax = gemv_ctas(p.U) > gemv_s_ctas(p.U) ? gemv_ctas(p.U) : gemv_s_ctas(p.U);  // as sized
   uint8_t* base = static_cast<uint8_t*>(ws);
   p.cnt = reinterpret_cast<int*>(base);
   p.part = reinterpret_cast<float*>(base + cnt_bytes(w.n));
-  float2* xs_ws = reinterpret_cast<float2*>(base + cnt_bytes(w.n) + (size_t)p.W * 2 * tok_pad(m) * kRows * sizeof(float));
+  float2* xs_ws = reinterpret_cast<float2*>(base + cnt_bytes(w.n) + part_bytes(wmax, m));
   if (w.bits != 16 && xsum == nullptr) {
     cudaError_t e = launch_xsum(x, ldx, m, w.k, xs_ws, s);
     if (e != cudaSuccess) return e;
@@ -800,6 +1135,19 @@ cudaError_t launch_gemv(const sq_qweight& w, const __half* x, int64_t ldx, int m
   const double bytes = (double)w.n * w.k * w.bits / 8.0 + (w.bits != 16 ? (double)w.n * (w.k / 128) * 4.0 : 0.0);
   auto t = prof_begin(KC_GEMV, bytes, 2.0 * m * w.n * w.k, s);
   cudaError_t e;
+  if (use_k2s(w.bits, w.n, w.k, m)) {
+    const int rt = w.bits == 8 ? SRing<8>::RT : SRing<4>::RT;
+    p.U = (int)(((w.n / kRows + rt - 1) / rt) * p.kg);
+    p.W = (int)gemv_s_ctas(p.U);
+    switch (w.bits) {
+      case 3: e = launch_s<3>(w, p, epi, s); break;
+      case 4: e = launch_s<4>(w, p, epi, s); break;
+      default: e = launch_s<8>(w, p, epi, s); break;
+    }
+    prof_end(t, s);
+    count_launch();
+    return e;
+  }
   switch (w.bits) {
     case 3: e = launch_b<3>(p, epi, s); break;
     case 4: e = launch_b<4>(p, epi, s); break;

@@ -231,18 +231,21 @@ def test_one_token_prefill_equals_decode_function():
     assert normwise(a, ref) <= TOL and normwise(b, ref) <= TOL
 
 
-@pytest.mark.parametrize("path", ["mma", "tc", "tc-nocluster"])
+@pytest.mark.parametrize("path", ["mma", "mma-k2", "mma-k2s", "tc", "tc-nocluster"])
 def test_decode_forced_path(path):
-    """Both decode kernels (mma.sync K2 and tcgen05 K2c) for every bit width and m in 1..32, whatever
-    the automatic choice (gemv_path) would pick: SQ_GEMV_PATH forces one (read once per process).
-    "tc-nocluster" forces K2c's global-memory split-k fix-up instead of the cluster/DSMEM reduction
-    (SQ_TC_CLUSTER=0), the fallback taken when the clusters cannot all be resident."""
+    """Every decode kernel (mma.sync K2 and its strip form K2s, tcgen05 K2c) for every bit width and m
+    in 1..32, whatever the automatic choice (gemv_path, use_k2s) would pick: SQ_GEMV_PATH forces the
+    family, SQ_K2S=0 / 1 K2 / K2s for m <= 8 (read once per process).  "tc-nocluster" forces K2c's
+    global-memory split-k fix-up instead of the cluster/DSMEM reduction (SQ_TC_CLUSTER=0), the
+    fallback taken when the clusters cannot all be resident."""
     import os
     import subprocess
     import sys
     env = dict(os.environ, SQ_GEMV_PATH=path.split("-")[0])
     if path == "tc-nocluster":
         env["SQ_TC_CLUSTER"] = "0"
+    if path in ("mma-k2", "mma-k2s"):
+        env["SQ_K2S"] = "1" if path == "mma-k2s" else "0"
     script = os.path.join(os.path.dirname(os.path.abspath(__file__)), "_decode_path_check.py")
     r = subprocess.run([sys.executable, script], env=env, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
@@ -283,15 +286,17 @@ def test_prefill_adversarial(bits, m):
     check_adversarial(y - y0, O.linear(x32, qo))
 
 
+@pytest.mark.parametrize("kern", ["k2", "k2s"])
 @pytest.mark.parametrize("bits", [3, 4, 8])
-def test_decode_mma_full_grid_sampled(bits):
-    """The mma.sync decode kernel (K2) at its configs[1] launch shape: OPT-13B fc1 (20480 x 5120) at
-    m = 1 (one 16-warp CTA per SM, units split evenly, tiles straddling CTAs -> cross-CTA fix-up),
-    forced with SQ_GEMV_PATH=mma in a subprocess; 64 sampled output rows vs the oracle."""
+def test_decode_mma_full_grid_sampled(bits, kern):
+    """The mma.sync decode kernels at the configs[1] launch shape: OPT-13B fc1 (20480 x 5120) at m = 1
+    (K2: one 16-warp CTA per SM, units split evenly; K2s: two 8-warp CTAs per SM, strip items split
+    evenly; tiles / strips straddling CTAs -> cross-CTA fix-up), forced with SQ_GEMV_PATH=mma and
+    SQ_K2S in a subprocess; 64 sampled output rows vs the oracle, and a bitwise repeat."""
     import os
     import subprocess
     import sys
-    env = dict(os.environ, SQ_GEMV_PATH="mma")
+    env = dict(os.environ, SQ_GEMV_PATH="mma", SQ_K2S="1" if kern == "k2s" else "0")
     script = os.path.join(os.path.dirname(os.path.abspath(__file__)), "_decode_path_check.py")
     r = subprocess.run([sys.executable, script, "full", str(bits)], env=env, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
