@@ -42,8 +42,14 @@ namespace {
 #ifndef SQ_K2_MINB
 #define SQ_K2_MINB 1
 #endif
+#ifndef SQ_K2S_RELACQ
+#define SQ_K2S_RELACQ 1
+#endif
 #ifndef SQ_K2S_SMEM_KB
-#define SQ_K2S_SMEM_KB 113
+#define SQ_K2S_SMEM_KB 76
+#endif
+#ifndef SQ_K2S_MINB
+#define SQ_K2S_MINB 2
 #endif
 constexpr int kWarps = SQ_K2_WARPS;  // one 512-thread CTA per SM
 constexpr int kThreads = kWarps * 32;
@@ -666,9 +672,9 @@ constexpr int kSWarps = 8;
 constexpr int kSThreads = kSWarps * 32;
 constexpr int kSCtasPerSm = 2;
 
-template <int BITS>
+template <int BITS, int RT_>
 struct SRing {
-  static constexpr int RT = BITS == 8 ? 2 : 4;                     // tiles per strip
+  static constexpr int RT = RT_;                                  // tiles per strip
   static constexpr int UB = 16 * Cfg<BITS>::GB;                   // codes bytes per unit
   static constexpr int SLOT = RT * (UB + 64);                     // one item: RT units + their meta
   static constexpr int BAR_BYTES = kSWarps * 8 * 8;                // <= 8 mbarriers per warp
@@ -738,16 +744,23 @@ __device__ __forceinline__ void reduce_tail_s(const GemvP& p, const uint8_t* par
         __stcg(gp + tok * RR + r * kRows + g, v[r][e]);
         __stcg(gp + tok * RR + r * kRows + g + 8, v[r][2 + e]);
       }
-    __threadfence();
-    __syncwarp();
     const int NC = gridDim.x;
     const int ca = (int)(((long long)(t * kg + 1) * NC - 1) / p.U);
     const int cb2 = (int)(((long long)((t + 1) * kg) * NC - 1) / p.U);
     int old = 0;
+#if SQ_K2S_RELACQ
+    __syncwarp();
+    if (lane == 0) asm volatile("atom.acq_rel.gpu.global.add.s32 %0, [%1], 1;" : "=r"(old) : "l"(p.cnt + t) : "memory");
+    old = __shfl_sync(0xffffffff, old, 0);
+    if (old != cb2 - ca) continue;
+#else
+    __threadfence();
+    __syncwarp();
     if (lane == 0) old = atomicAdd(p.cnt + t, 1);
     old = __shfl_sync(0xffffffff, old, 0);
     if (old != cb2 - ca) continue;
     __threadfence();
+#endif
 #pragma unroll
     for (int r = 0; r < RT; ++r)
 #pragma unroll
@@ -770,10 +783,10 @@ __device__ __forceinline__ void reduce_tail_s(const GemvP& p, const uint8_t* par
   }
 }
 
-template <int BITS, int EPI>
-__global__ void __launch_bounds__(kSThreads, kSCtasPerSm)
+template <int BITS, int RT_, int EPI>
+__global__ void __launch_bounds__(kSThreads, SQ_K2S_MINB)
     k_gemv_s(const __grid_constant__ CUtensorMap tm_w, const __grid_constant__ CUtensorMap tm_m, const GemvP p) {
-  using RC = SRing<BITS>;
+  using RC = SRing<BITS, RT_>;
   constexpr int TOK = 8;
   constexpr int LU = Cfg<BITS>::LU, GB = Cfg<BITS>::GB;
   constexpr int RT = RC::RT, UB = RC::UB, SLOT = RC::SLOT, S = RC::S, RR = RT * kRows;
@@ -967,10 +980,10 @@ cudaError_t launch_e(const GemvP& p, cudaStream_t s) {
   return launch_pdl(kern, dim3((unsigned)p.W), dim3(kThreads), smem, s, p);
 }
 
-template <int BITS, int EPI>
+template <int BITS, int RT, int EPI>
 cudaError_t launch_s_e(const CUtensorMap& tw, const CUtensorMap& tm, const GemvP& p, cudaStream_t s) {
-  void (*kern)(const CUtensorMap, const CUtensorMap, const GemvP) = k_gemv_s<BITS, EPI>;
-  const size_t smem = (size_t)SRing<BITS>::BYTES;
+  void (*kern)(const CUtensorMap, const CUtensorMap, const GemvP) = k_gemv_s<BITS, RT, EPI>;
+  const size_t smem = (size_t)SRing<BITS, RT>::BYTES;
   static bool attr = false;
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -980,10 +993,10 @@ cudaError_t launch_s_e(const CUtensorMap& tw, const CUtensorMap& tm, const GemvP
   return launch_pdl(kern, dim3((unsigned)p.W), dim3(kSThreads), smem, s, tw, tm, p);
 }
 
-template <int BITS>
+template <int BITS, int RT>
 cudaError_t launch_s(const sq_qweight& w, const GemvP& p, int epi, cudaStream_t s) {
   // codes: [n/16 tiles][kg * UB/256 lines][256 B], box = RT tiles x one unit; meta: [n/16][kg * 16] u32
-  constexpr int RT = SRing<BITS>::RT, UB = SRing<BITS>::UB;
+  constexpr int UB = SRing<BITS, RT>::UB;
   CUtensorMap tw, tm;
   const uint64_t nt = (uint64_t)w.n / kRows, kg = (uint64_t)p.kg;
   const uint64_t dw[3] = {256, kg * (UB / 256), nt}, sw_[2] = {256, kg * UB};
@@ -995,10 +1008,10 @@ cudaError_t launch_s(const sq_qweight& w, const GemvP& p, int epi, cudaStream_t 
   e = encode_nd(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, w.meta, 2, dm, sm_, bm, CU_TENSOR_MAP_SWIZZLE_NONE);
   if (e != cudaSuccess) return e;
   switch (epi) {
-    case SQ_EPI_F16: return launch_s_e<BITS, SQ_EPI_F16>(tw, tm, p, s);
-    case SQ_EPI_F16_RELU: return launch_s_e<BITS, SQ_EPI_F16_RELU>(tw, tm, p, s);
-    case SQ_EPI_F16_GELU: return launch_s_e<BITS, SQ_EPI_F16_GELU>(tw, tm, p, s);
-    default: return launch_s_e<BITS, SQ_EPI_F32_ACCUM>(tw, tm, p, s);
+    case SQ_EPI_F16: return launch_s_e<BITS, RT, SQ_EPI_F16>(tw, tm, p, s);
+    case SQ_EPI_F16_RELU: return launch_s_e<BITS, RT, SQ_EPI_F16_RELU>(tw, tm, p, s);
+    case SQ_EPI_F16_GELU: return launch_s_e<BITS, RT, SQ_EPI_F16_GELU>(tw, tm, p, s);
+    default: return launch_s_e<BITS, RT, SQ_EPI_F32_ACCUM>(tw, tm, p, s);
   }
 }
 
@@ -1045,16 +1058,22 @@ size_t part_bytes(int64_t W, int64_t m) {
 }
 // K2s (strips) for quantized weights at m <= 8 (SQ_K2S=0: K2)
 // Whole strips only (n a multiple of RT * 16, so no TMA box reaches past the matrix).  Measured
-// (tools/exp_k2s.sh, back-to-back graph launches): K2s streams large linears at 4.9-5.1 TB/s INT4,
-// 6.1-6.5 INT8, 3.1-3.4 INT3 (m <= 8; K2 4.1 / 5.6 / 2.9, K2c 4.4-4.7 / 5.5-5.8 / 3.0-3.3), but
-// its finer split costs ~2 us more per launch than K2's on small INT3 / INT4 linears (5120^2 INT4:
-// 10.2 vs 8.3 us), so K2 keeps INT3 / INT4 linears under 20 MB.  SQ_K2S=0 / 1 forces K2 / K2s.
+// (tools/exp_k2s9.sh, back-to-back graph launches, m = 1 / 8): K2s is as fast as K2 or faster on every
+// OPT-125m ... OPT-66B shape, e.g. 36864 x 9216 INT4 34.4 / 37.1 us vs 44.2 / 60.8, 20480 x 5120
+// INT4 15.5 / 17.0 vs 17.7 / 23.7, 768 x 3072 5.5 vs 6.0-6.5 (2304 x 768: within 0.2 us), so K2
+// remains only for n not a multiple of 32.  SQ_K2S=0 / 1 forces K2 / K2s.
+// strip width: 4 tiles (the activation fragment re-used 4x) for INT3 / INT4 linears of more than
+// 1280 tiles, else 2 (twice the items per warp; 5120^2 INT4 9.7 -> 8.0 us, 5120 x 20480 17.1 ->
+// 16.3 us, but 36864 x 9216 34.2 -> 37.8 us; tools/exp_k2s8.sh); INT8 always 2
+int k2s_rt(int bits, int64_t n) { return (bits != 8 && n / kRows > 1280) ? 4 : 2; }
+
 bool use_k2s(int bits, int64_t n, int64_t k, int m) {
   static int forced = -2;
   if (forced == -2) { const char* e = getenv("SQ_K2S"); forced = !e ? -1 : (e[0] == '0' ? 0 : 1); }
-  if (bits == 16 || m > 8 || n % (bits == 8 ? 32 : 64) != 0) return false;
+  if (bits == 16 || m > 8 || n % (16 * k2s_rt(bits, n)) != 0) return false;
+  (void)k;
   if (forced >= 0) return forced == 1;
-  return bits == 8 || (double)n * k * bits / 8.0 >= 20e6;
+  return true;
 }
 
 }  // namespace
@@ -1136,14 +1155,13 @@ cudaError_t launch_gemv(const sq_qweight& w, const __half* x, int64_t ldx, int m
   auto t = prof_begin(KC_GEMV, bytes, 2.0 * m * w.n * w.k, s);
   cudaError_t e;
   if (use_k2s(w.bits, w.n, w.k, m)) {
-    const int rt = w.bits == 8 ? SRing<8>::RT : SRing<4>::RT;
+    const int rt = k2s_rt(w.bits, w.n);
     p.U = (int)(((w.n / kRows + rt - 1) / rt) * p.kg);
     p.W = (int)gemv_s_ctas(p.U);
-    switch (w.bits) {
-      case 3: e = launch_s<3>(w, p, epi, s); break;
-      case 4: e = launch_s<4>(w, p, epi, s); break;
-      default: e = launch_s<8>(w, p, epi, s); break;
-    }
+    if (rt == 4) e = w.bits == 3 ? launch_s<3, 4>(w, p, epi, s) : launch_s<4, 4>(w, p, epi, s);
+    else if (w.bits == 3) e = launch_s<3, 2>(w, p, epi, s);
+    else if (w.bits == 4) e = launch_s<4, 2>(w, p, epi, s);
+    else e = launch_s<8, 2>(w, p, epi, s);
     prof_end(t, s);
     count_launch();
     return e;

@@ -15,7 +15,7 @@ import paper_conf_cluster_zhaowplw25_b200 as sq
 def main():
     worst = 0.0
     for bits in (3, 4, 8, 16):
-        for (n, k) in ((256, 512), (768, 768), (384, 1152)):
+        for (n, k) in ((256, 512), (768, 768), (384, 1152), (9600, 256)):
             w = synth.weight_f16(900 + n + bits, n, k)
             b = synth.bias_f16(901 + n, n)
             qo = O.QWeight(w, bits, bias=b)
