@@ -287,6 +287,19 @@ def test_prefill_adversarial(bits, m):
 
 
 @pytest.mark.parametrize("kern", ["k2", "k2s"])
+def test_decode_mma_writes_in_bounds(kern):
+    """K2 / K2s write nothing outside y's window and the workspace, and reset every split-k counter
+    (sentinel-filled buffers; the substitute for compute-sanitizer, which this pool has closed)."""
+    import os
+    import subprocess
+    import sys
+    env = dict(os.environ, SQ_GEMV_PATH="mma", SQ_K2S="1" if kern == "k2s" else "0")
+    script = os.path.join(os.path.dirname(os.path.abspath(__file__)), "_decode_path_check.py")
+    r = subprocess.run([sys.executable, script, "canary"], env=env, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+
+
+@pytest.mark.parametrize("kern", ["k2", "k2s"])
 @pytest.mark.parametrize("bits", [3, 4, 8])
 def test_decode_mma_full_grid_sampled(bits, kern):
     """The mma.sync decode kernels at the configs[1] launch shape: OPT-13B fc1 (20480 x 5120) at m = 1
