@@ -106,9 +106,13 @@ sq_status stage_forward(const sq_layer* layers, int n_layers, int phase, const f
   __half* att16 = reinterpret_cast<__half*>(base + W.att16);
   void* gws = base + W.gemv;
   const bool dec = phase == SQ_DECODE;
+  // linears of a decode step, and of a prefill micro-batch of <= 32 tokens (configs[0]'s 32-token
+  // prompt, small chunks), run on the decode kernels: the prefill GEMM's 256-token tile would be at
+  // most 1/8 full and every launch pays its TMEM / pipeline prologue (same function)
+  const bool gv = dec || T <= 32;
   auto lin = [&](const sq_qweight& w, const __half* x, int64_t ldx, void* y, int64_t ldy, int epi,
                  const float2* xsum) -> cudaError_t {
-    if (dec) return launch_gemv(w, x, ldx, (int)T, y, ldy, epi, xsum, gws, s);
+    if (gv) return launch_gemv(w, x, ldx, (int)T, y, ldy, epi, xsum, gws, s);
     return launch_gemm(w, x, ldx, T, y, ldy, epi, s);
   };
   cudaError_t e = cudaSuccess;
@@ -117,7 +121,7 @@ sq_status stage_forward(const sq_layer* layers, int n_layers, int phase, const f
     // per-group activation sums only for linears on the mma.sync decode path (K2); the tcgen05
     // decode (K2c) dequantizes the weights and needs none
     const bool q = L.bits != 16;
-    auto k2 = [&](const sq_qweight& w) { return dec && q && gemv_path(w.n, w.k, (int)T, w.bits) == 0; };
+    auto k2 = [&](const sq_qweight& w) { return gv && q && gemv_path(w.n, w.k, (int)T, w.bits) == 0; };
     const float* xr = (l == 0) ? x_in : x_out;
     const bool copy = (l == 0 && x_in != x_out);
     // a = LN(x) (layer 0 also initialises the residual buffer x_out = x_in)
@@ -232,10 +236,14 @@ sq_status stage_forward_tp(const sq_layer* sh, int n_layers, int n_sets, sq_comm
   float2* xsb = reinterpret_cast<float2*>(base + W.xsb);
   void* gws = base + W.gemv;
   const bool dec = phase == SQ_DECODE;
+  // linears of a decode step, and of a prefill micro-batch of <= 32 tokens (configs[0]'s 32-token
+  // prompt, small chunks), run on the decode kernels: the prefill GEMM's 256-token tile would be at
+  // most 1/8 full and every launch pays its TMEM / pipeline prologue (same function)
+  const bool gv = dec || T <= 32;
   const bool zero_first = comm && tp_rank > 0;  // ranks r > 0 contribute p_r only (x comes from rank 0)
   auto lin = [&](const sq_qweight& w, const __half* x, int64_t ldx, void* y, int64_t ldy, int epi,
                  const float2* xsum) -> cudaError_t {
-    if (dec) return launch_gemv(w, x, ldx, (int)T, y, ldy, epi, xsum, gws, s);
+    if (gv) return launch_gemv(w, x, ldx, (int)T, y, ldy, epi, xsum, gws, s);
     return launch_gemm(w, x, ldx, T, y, ldy, epi, s);
   };
   auto reduce = [&]() -> sq_status {
@@ -247,7 +255,7 @@ sq_status stage_forward_tp(const sq_layer* sh, int n_layers, int n_sets, sq_comm
   for (int l = 0; l < n_layers && e == cudaSuccess && st == SQ_OK; ++l) {
     const sq_layer& L0 = sh[l];
     const bool q = L0.bits != 16;
-    auto k2 = [&](const sq_qweight& w) { return dec && q && gemv_path(w.n, w.k, (int)T, w.bits) == 0; };
+    auto k2 = [&](const sq_qweight& w) { return gv && q && gemv_path(w.n, w.k, (int)T, w.bits) == 0; };
     const float* xr = (l == 0) ? x_in : x_out;
     const bool copy = (l == 0 && x_in != x_out);
     e = launch_layernorm_f16(xr, T, h1, a16, k2(L0.qkv) ? xsa : nullptr, copy ? x_in : nullptr, copy ? x_out : nullptr, s);
