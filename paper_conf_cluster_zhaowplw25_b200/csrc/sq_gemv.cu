@@ -783,7 +783,7 @@ __device__ __forceinline__ void reduce_tail_s(const GemvP& p, const uint8_t* par
   }
 }
 
-template <int BITS, int RT_, int EPI>
+template <int BITS, int RT_, int EPI, bool XS>
 __global__ void __launch_bounds__(kSThreads, SQ_K2S_MINB)
     k_gemv_s(const __grid_constant__ CUtensorMap tm_w, const __grid_constant__ CUtensorMap tm_m, const GemvP p) {
   using RC = SRing<BITS, RT_>;
@@ -856,10 +856,38 @@ __global__ void __launch_bounds__(kSThreads, SQ_K2S_MINB)
         xt[4 * i] = v.x; xt[4 * i + 1] = v.y; xt[4 * i + 2] = v.z; xt[4 * i + 3] = v.w;
       }
     }
-    const float4 xsv = __ldg(reinterpret_cast<const float4*>(p.xsum + grp * kXsTok + 2 * q));
-    const float xs0 = xsv.x + xsv.y, xs1 = xsv.z + xsv.w;
-    const float xo0 = BITS == 4 ? fmaf(1024.f, xsv.x, 64.f * xsv.y) : (BITS == 3 ? 8.f * xs0 : 1024.f * xs0);
-    const float xo1 = BITS == 4 ? fmaf(1024.f, xsv.z, 64.f * xsv.w) : (BITS == 3 ? 8.f * xs1 : 1024.f * xs1);
+    float xs0, xs1, xo0, xo1;
+    if constexpr (XS) {
+      // the group sums on the tensor core: xs = sum x (A = ones), xoff = sum off_k x (A = the unpack
+      // offsets at each fragment position: INT4 lo codes 1024 at k 2q.., hi codes 64 at k 2q+8..) --
+      // the same fragment positions as the codes, so D - xoff cancels the offsets by construction
+      constexpr uint32_t H1 = 0x3C003C00u, H1024 = 0x64006400u, H64 = 0x54005400u;
+      const uint32_t a1[4] = {H1, H1, H1, H1};
+      float ds[4];
+      mma_16816_zc(ds, a1, xt[0], xt[1]);
+#pragma unroll
+      for (int t = 1; t < 8; ++t) mma_16816(ds, a1, xt[2 * t], xt[2 * t + 1], ds);
+      xs0 = ds[0];
+      xs1 = ds[1];
+      if constexpr (BITS == 4) {
+        const uint32_t ao[4] = {H1024, H1024, H64, H64};
+        float dof[4];
+        mma_16816_zc(dof, ao, xt[0], xt[1]);
+#pragma unroll
+        for (int t = 1; t < 8; ++t) mma_16816(dof, ao, xt[2 * t], xt[2 * t + 1], dof);
+        xo0 = dof[0];
+        xo1 = dof[1];
+      } else {
+        xo0 = (BITS == 3 ? 8.f : 1024.f) * xs0;
+        xo1 = (BITS == 3 ? 8.f : 1024.f) * xs1;
+      }
+    } else {
+      const float4 xsv = __ldg(reinterpret_cast<const float4*>(p.xsum + grp * kXsTok + 2 * q));
+      xs0 = xsv.x + xsv.y;
+      xs1 = xsv.z + xsv.w;
+      xo0 = BITS == 4 ? fmaf(1024.f, xsv.x, 64.f * xsv.y) : (BITS == 3 ? 8.f * xs0 : 1024.f * xs0);
+      xo1 = BITS == 4 ? fmaf(1024.f, xsv.z, 64.f * xsv.w) : (BITS == 3 ? 8.f * xs1 : 1024.f * xs1);
+    }
     mbar_wait(&bar[slot], (uint32_t)((c / S) & 1));
     const uint8_t* cs = ring + slot * SLOT;
     const uint32_t* ms = reinterpret_cast<const uint32_t*>(cs + RT * UB);
@@ -980,9 +1008,9 @@ cudaError_t launch_e(const GemvP& p, cudaStream_t s) {
   return launch_pdl(kern, dim3((unsigned)p.W), dim3(kThreads), smem, s, p);
 }
 
-template <int BITS, int RT, int EPI>
-cudaError_t launch_s_e(const CUtensorMap& tw, const CUtensorMap& tm, const GemvP& p, cudaStream_t s) {
-  void (*kern)(const CUtensorMap, const CUtensorMap, const GemvP) = k_gemv_s<BITS, RT, EPI>;
+template <int BITS, int RT, int EPI, bool XS>
+cudaError_t launch_s_x(const CUtensorMap& tw, const CUtensorMap& tm, const GemvP& p, cudaStream_t s) {
+  void (*kern)(const CUtensorMap, const CUtensorMap, const GemvP) = k_gemv_s<BITS, RT, EPI, XS>;
   const size_t smem = (size_t)SRing<BITS, RT>::BYTES;
   static bool attr = false;
   if (!attr) {
@@ -991,6 +1019,11 @@ cudaError_t launch_s_e(const CUtensorMap& tw, const CUtensorMap& tm, const GemvP
     attr = true;
   }
   return launch_pdl(kern, dim3((unsigned)p.W), dim3(kSThreads), smem, s, tw, tm, p);
+}
+// XS: group sums computed in the kernel (p.xsum == null) or read from p.xsum
+template <int BITS, int RT, int EPI>
+cudaError_t launch_s_e(const CUtensorMap& tw, const CUtensorMap& tm, const GemvP& p, cudaStream_t s) {
+  return p.xsum ? launch_s_x<BITS, RT, EPI, false>(tw, tm, p, s) : launch_s_x<BITS, RT, EPI, true>(tw, tm, p, s);
 }
 
 template <int BITS, int RT>
@@ -1067,7 +1100,7 @@ size_t part_bytes(int64_t W, int64_t m) {
 // 16.3 us, but 36864 x 9216 34.2 -> 37.8 us; tools/exp_k2s8.sh); INT8 always 2
 int k2s_rt(int bits, int64_t n) { return (bits != 8 && n / kRows > 1280) ? 4 : 2; }
 
-bool use_k2s(int bits, int64_t n, int64_t k, int m) {
+bool k2s_rule(int bits, int64_t n, int64_t k, int m) {
   static int forced = -2;
   if (forced == -2) { const char* e = getenv("SQ_K2S"); forced = !e ? -1 : (e[0] == '0' ? 0 : 1); }
   if (bits == 16 || m > 8 || n % (16 * k2s_rt(bits, n)) != 0) return false;
@@ -1077,6 +1110,8 @@ bool use_k2s(int bits, int64_t n, int64_t k, int m) {
 }
 
 }  // namespace
+
+bool use_k2s(int bits, int64_t n, int64_t k, int m) { return k2s_rule(bits, n, k, m); }
 
 size_t xsum_bytes(int64_t k) { return (size_t)(k / 128) * kXsTok * sizeof(float2); }
 
@@ -1145,7 +1180,8 @@ cudaError_t launch_gemv(const sq_qweight& w, const __half* x, int64_t ldx, int m
   p.cnt = reinterpret_cast<int*>(base);
   p.part = reinterpret_cast<float*>(base + cnt_bytes(w.n));
   float2* xs_ws = reinterpret_cast<float2*>(base + cnt_bytes(w.n) + part_bytes(wmax, m));
-  if (w.bits != 16 && xsum == nullptr) {
+  const bool k2s = use_k2s(w.bits, w.n, w.k, m);
+  if (w.bits != 16 && xsum == nullptr && !k2s) {  // K2s computes missing group sums itself
     cudaError_t e = launch_xsum(x, ldx, m, w.k, xs_ws, s);
     if (e != cudaSuccess) return e;
     xsum = xs_ws;
@@ -1154,7 +1190,7 @@ cudaError_t launch_gemv(const sq_qweight& w, const __half* x, int64_t ldx, int m
   const double bytes = (double)w.n * w.k * w.bits / 8.0 + (w.bits != 16 ? (double)w.n * (w.k / 128) * 4.0 : 0.0);
   auto t = prof_begin(KC_GEMV, bytes, 2.0 * m * w.n * w.k, s);
   cudaError_t e;
-  if (use_k2s(w.bits, w.n, w.k, m)) {
+  if (k2s) {
     const int rt = k2s_rt(w.bits, w.n);
     p.U = (int)(((w.n / kRows + rt - 1) / rt) * p.kg);
     p.W = (int)gemv_s_ctas(p.U);

@@ -40,7 +40,8 @@ size_t gemv_tc_workspace_bytes(int64_t n, int64_t k);
 size_t gemv_tc_xsum_offset(int64_t n, int64_t k);
 cudaError_t launch_gemv_tc(const sq_qweight& w, const __half* x, int64_t ldx, int m, void* y, int64_t ldy, int epi,
                            void* ws, cudaStream_t s);
-int gemv_path(int64_t n, int64_t k, int m, int bits);  // 0 = mma.sync (K2), 1 = tcgen05 (K2c)
+int gemv_path(int64_t n, int64_t k, int m, int bits);  // 0 = mma.sync (K2 / K2s), 1 = tcgen05 (K2c)
+bool use_k2s(int bits, int64_t n, int64_t k, int m);   // within path 0: the strip kernel (own group sums)
 
 cudaError_t launch_gemm(const sq_qweight& w, const __half* x, int64_t ldx, int64_t m, void* y, int64_t ldy,
                         int epi, cudaStream_t s);

@@ -118,10 +118,11 @@ sq_status stage_forward(const sq_layer* layers, int n_layers, int phase, const f
   cudaError_t e = cudaSuccess;
   for (int l = 0; l < n_layers && e == cudaSuccess; ++l) {
     const sq_layer& L = layers[l];
-    // per-group activation sums only for linears on the mma.sync decode path (K2); the tcgen05
-    // decode (K2c) dequantizes the weights and needs none
+    // per-group activation sums only for linears on the round-1 mma.sync decode kernel (K2); the strip
+    // kernel K2s computes its own on the tensor core, the tcgen05 decode (K2c) dequantizes and needs none
     const bool q = L.bits != 16;
-    auto k2 = [&](const sq_qweight& w) { return gv && q && gemv_path(w.n, w.k, (int)T, w.bits) == 0; };
+    auto k2 = [&](const sq_qweight& w) { return gv && q && gemv_path(w.n, w.k, (int)T, w.bits) == 0 &&
+                                                   !use_k2s(w.bits, w.n, w.k, (int)T); };
     const float* xr = (l == 0) ? x_in : x_out;
     const bool copy = (l == 0 && x_in != x_out);
     // a = LN(x) (layer 0 also initialises the residual buffer x_out = x_in)
@@ -255,7 +256,8 @@ sq_status stage_forward_tp(const sq_layer* sh, int n_layers, int n_sets, sq_comm
   for (int l = 0; l < n_layers && e == cudaSuccess && st == SQ_OK; ++l) {
     const sq_layer& L0 = sh[l];
     const bool q = L0.bits != 16;
-    auto k2 = [&](const sq_qweight& w) { return gv && q && gemv_path(w.n, w.k, (int)T, w.bits) == 0; };
+    auto k2 = [&](const sq_qweight& w) { return gv && q && gemv_path(w.n, w.k, (int)T, w.bits) == 0 &&
+                                                   !use_k2s(w.bits, w.n, w.k, (int)T); };
     const float* xr = (l == 0) ? x_in : x_out;
     const bool copy = (l == 0 && x_in != x_out);
     e = launch_layernorm_f16(xr, T, h1, a16, k2(L0.qkv) ? xsa : nullptr, copy ? x_in : nullptr, copy ? x_out : nullptr, s);

@@ -30,6 +30,15 @@ def main():
                 err = float(np.abs(yy - ref).max() / np.abs(ref).max())
                 worst = max(worst, err)
                 assert err <= 2e-3, (os.environ.get("SQ_GEMV_PATH"), bits, n, k, m, err)
+                if bits != 16 and m <= 8:
+                    # group sums supplied by the caller (sq_xsum) instead of computed in the kernel
+                    xd = torch.from_numpy(x).cuda()
+                    y2 = torch.empty_like(y)
+                    sq.sq_linear_decode(qg, xd, y2, 0, xsum=sq.sq_xsum(xd))
+                    torch.cuda.synchronize()
+                    err = float(np.abs(y2.float().cpu().numpy().astype(np.float64) - ref).max() / np.abs(ref).max())
+                    worst = max(worst, err)
+                    assert err <= 2e-3, (os.environ.get("SQ_GEMV_PATH"), "xsum", bits, n, k, m, err)
                 # fp32-residual epilogue (o / fc2): y_f32 += x W~^T + bias
                 y0 = synth.act_f16(903 + m, m, n).astype(np.float32)
                 ya = torch.from_numpy(y0.copy()).cuda()
