@@ -685,17 +685,17 @@ struct SRing {
   static_assert(S >= 2 && S * SLOT >= PARTW && BYTES <= 227 * 1024 && SLOT % 128 == 0, "K2s shared memory");
 };
 
-template <int EPI, int RT>
-__device__ __forceinline__ void store_strip_tile(const GemvP& p, int tile, int g, int q, const float (&v)[4]) {
-  if (tile < p.n / kRows) store_out<8, EPI>(p, tile, g, q, reinterpret_cast<const float(&)[1][4]>(v));
+template <int EPI, int NJ>
+__device__ __forceinline__ void store_strip_tile(const GemvP& p, int tile, int g, int q, const float (&v)[NJ][4]) {
+  if (tile < p.n / kRows) store_out<8 * NJ, EPI>(p, tile, g, q, v);
 }
 
-// K2's reduce_tail for strips: in-CTA partials live in each warp's ring (stride WS bytes), the
-// cross-CTA partials in p.part [CTAs][2][8][RT * 16].
-template <int EPI, int RT, int WS>
+// K2's reduce_tail for strips: in-CTA partials live in each warp's ring (stride WS bytes) as
+// [2][32 lanes][RT][NJ] float4, the cross-CTA partials in p.part [CTAs][2][32 lanes][RT][NJ] float4.
+template <int EPI, int RT, int NJ, int WS>
 __device__ __forceinline__ void reduce_tail_s(const GemvP& p, const uint8_t* part_base, int C0, int C1, int R,
                                               int warp, int lane, int g, int q) {
-  constexpr int TOK = 8, RR = RT * kRows;
+  constexpr int PL = RT * NJ;  // float4 per lane per partial
   const int kg = p.kg;
   if (R <= 0) return;
   const int t_first = C0 / kg, t_last = (C1 - 1) / kg;
@@ -706,44 +706,38 @@ __device__ __forceinline__ void reduce_tail_s(const GemvP& p, const uint8_t* par
     const int wb = (int)(((long long)(hi - C0) * kSWarps - 1) / R);
     const bool whole = lo == t * kg && hi == (t + 1) * kg;
     if (wa == wb && whole) continue;  // one warp stored it directly
-    float v[RT][4];
+    float v[RT][NJ][4];
 #pragma unroll
     for (int r = 0; r < RT; ++r)
 #pragma unroll
-      for (int i = 0; i < 4; ++i) v[r][i] = 0.f;
+      for (int j = 0; j < NJ; ++j)
+#pragma unroll
+        for (int i = 0; i < 4; ++i) v[r][j][i] = 0.f;
     for (int wi = wa; wi <= wb; ++wi) {
       const int wlo = C0 + range_lo(wi, R, kSWarps), whi = C0 + range_lo(wi + 1, R, kSWarps);
       if (whi <= wlo) continue;  // empty warp range
       const int sl = (wlo < t * kg) ? 1 : 0;
-      const float* qp = reinterpret_cast<const float*>(part_base + (size_t)wi * WS) + sl * TOK * RR;
+      const float4* qp = reinterpret_cast<const float4*>(part_base + (size_t)wi * WS) + (sl * 32 + lane) * PL;
 #pragma unroll
       for (int r = 0; r < RT; ++r)
 #pragma unroll
-        for (int e = 0; e < 2; ++e) {
-          const int tok = 2 * q + e;
-          v[r][e] += qp[tok * RR + r * kRows + g];
-          v[r][2 + e] += qp[tok * RR + r * kRows + g + 8];
+        for (int j = 0; j < NJ; ++j) {
+          const float4 u = qp[r * NJ + j];
+          v[r][j][0] += u.x; v[r][j][1] += u.y; v[r][j][2] += u.z; v[r][j][3] += u.w;
         }
     }
     if (whole) {
 #pragma unroll
-      for (int r = 0; r < RT; ++r) store_strip_tile<EPI, RT>(p, t * RT + r, g, q, v[r]);
+      for (int r = 0; r < RT; ++r) store_strip_tile<EPI, NJ>(p, t * RT + r, g, q, v[r]);
       continue;
     }
-#ifdef SQ_K2S_ABL_NOFIX
-    continue;  // timing ablation only: results wrong
-#endif
     // straddles a CTA boundary: publish this CTA's partial, the last CTA to arrive reduces
     const int cslot = (C0 < t * kg) ? 1 : 0;
-    float* gp = p.part + ((int64_t)blockIdx.x * 2 + cslot) * TOK * RR;
+    float4* gp = reinterpret_cast<float4*>(p.part) + (((int64_t)blockIdx.x * 2 + cslot) * 32 + lane) * PL;
 #pragma unroll
     for (int r = 0; r < RT; ++r)
 #pragma unroll
-      for (int e = 0; e < 2; ++e) {
-        const int tok = 2 * q + e;
-        __stcg(gp + tok * RR + r * kRows + g, v[r][e]);
-        __stcg(gp + tok * RR + r * kRows + g + 8, v[r][2 + e]);
-      }
+      for (int j = 0; j < NJ; ++j) __stcg(gp + r * NJ + j, make_float4(v[r][j][0], v[r][j][1], v[r][j][2], v[r][j][3]));
     const int NC = gridDim.x;
     const int ca = (int)(((long long)(t * kg + 1) * NC - 1) / p.U);
     const int cb2 = (int)(((long long)((t + 1) * kg) * NC - 1) / p.U);
@@ -764,32 +758,34 @@ __device__ __forceinline__ void reduce_tail_s(const GemvP& p, const uint8_t* par
 #pragma unroll
     for (int r = 0; r < RT; ++r)
 #pragma unroll
-      for (int i = 0; i < 4; ++i) v[r][i] = 0.f;
+      for (int j = 0; j < NJ; ++j)
+#pragma unroll
+        for (int i = 0; i < 4; ++i) v[r][j][i] = 0.f;
     for (int c = ca; c <= cb2; ++c) {
       const int sl = (range_lo(c, p.U, NC) < t * kg) ? 1 : 0;
-      const float* qp = p.part + ((int64_t)c * 2 + sl) * TOK * RR;
+      const float4* qp = reinterpret_cast<const float4*>(p.part) + (((int64_t)c * 2 + sl) * 32 + lane) * PL;
 #pragma unroll
       for (int r = 0; r < RT; ++r)
 #pragma unroll
-        for (int e = 0; e < 2; ++e) {
-          const int tok = 2 * q + e;
-          v[r][e] += __ldcg(qp + tok * RR + r * kRows + g);
-          v[r][2 + e] += __ldcg(qp + tok * RR + r * kRows + g + 8);
+        for (int j = 0; j < NJ; ++j) {
+          const float4 u = __ldcg(qp + r * NJ + j);
+          v[r][j][0] += u.x; v[r][j][1] += u.y; v[r][j][2] += u.z; v[r][j][3] += u.w;
         }
     }
 #pragma unroll
-    for (int r = 0; r < RT; ++r) store_strip_tile<EPI, RT>(p, t * RT + r, g, q, v[r]);
+    for (int r = 0; r < RT; ++r) store_strip_tile<EPI, NJ>(p, t * RT + r, g, q, v[r]);
     if (lane == 0) p.cnt[t] = 0;
   }
 }
 
-template <int BITS, int RT_, int EPI, bool XS>
+// NJ = token n8 tiles: 1 (m <= 8) or 2 (m <= 16, RT = 2)
+template <int BITS, int RT_, int EPI, bool XS, int NJ>
 __global__ void __launch_bounds__(kSThreads, SQ_K2S_MINB)
     k_gemv_s(const __grid_constant__ CUtensorMap tm_w, const __grid_constant__ CUtensorMap tm_m, const GemvP p) {
   using RC = SRing<BITS, RT_>;
-  constexpr int TOK = 8;
   constexpr int LU = Cfg<BITS>::LU, GB = Cfg<BITS>::GB;
-  constexpr int RT = RC::RT, UB = RC::UB, SLOT = RC::SLOT, S = RC::S, RR = RT * kRows;
+  constexpr int RT = RC::RT, UB = RC::UB, SLOT = RC::SLOT, S = RC::S, PL = RT * NJ;
+  static_assert(S * SLOT >= 2 * 32 * PL * 16, "partials fit in the ring");
   extern __shared__ float4 smem4[];
   uint8_t* smem = reinterpret_cast<uint8_t*>(smem4);
   smem += (128 - (smem_u32(smem) & 127)) & 127;  // TMA destinations: 128-B aligned slots
@@ -798,7 +794,6 @@ __global__ void __launch_bounds__(kSThreads, SQ_K2S_MINB)
   uint64_t* bar = reinterpret_cast<uint64_t*>(smem) + warp * 8;
   uint8_t* ring = smem + RC::BAR_BYTES + warp * S * SLOT;
   const int kg = p.kg, m = p.m;
-  const int T = p.n / kRows;
   const int C0 = range_lo(blockIdx.x, p.U, gridDim.x), C1 = range_lo(blockIdx.x + 1, p.U, gridDim.x);
   const int R = C1 - C0;
   const int u0 = C0 + range_lo(warp, R, kSWarps), u1 = C0 + range_lo(warp + 1, R, kSWarps);
@@ -827,66 +822,78 @@ __global__ void __launch_bounds__(kSThreads, SQ_K2S_MINB)
   pdl_trigger();
   pdl_wait();
 
-  // the lane's activation row (token g) and k set, matching its codes (see k_gemv_q)
-  const bool xon = g < m;
-  const __half* xrow = p.x + (int64_t)(xon ? g : 0) * p.ldx + (BITS == 8 ? q * 16 : q * 32);
-  const int lane_off = BITS == 8 ? q * 16 : q * lane_bytes<BITS>();
-  uint32_t xt[16];
+  // the lane's activation rows (tokens 8j + g) and k set, matching its codes (see k_gemv_q)
+  bool xon[NJ];
+  const __half* xrow[NJ];
 #pragma unroll
-  for (int i = 0; i < 16; ++i) xt[i] = 0u;
+  for (int j = 0; j < NJ; ++j) {
+    xon[j] = 8 * j + g < m;
+    xrow[j] = p.x + (int64_t)(xon[j] ? 8 * j + g : 0) * p.ldx + (BITS == 8 ? q * 16 : q * 32);
+  }
+  const int lane_off = BITS == 8 ? q * 16 : q * lane_bytes<BITS>();
+  uint32_t xt[NJ][16];
+#pragma unroll
+  for (int j = 0; j < NJ; ++j)
+#pragma unroll
+    for (int i = 0; i < 16; ++i) xt[j][i] = 0u;
 
   int set = head_set, grp = grp0;
   bool seg_from_start = (grp0 == 0);
-  float acc[RT][4], hacc[RT][4];
+  float acc[RT][NJ][4], hacc[RT][NJ][4];
 #pragma unroll
   for (int r = 0; r < RT; ++r)
 #pragma unroll
-    for (int i = 0; i < 4; ++i) { acc[r][i] = 0.f; hacc[r][i] = 0.f; }
+    for (int j = 0; j < NJ; ++j)
+#pragma unroll
+      for (int i = 0; i < 4; ++i) { acc[r][j][i] = 0.f; hacc[r][j][i] = 0.f; }
   bool has_head = false;
 
   for (int c = 0; c < nit; ++c) {
     const int slot = c % S;
-    // activation fragment + group sums of this group (independent of the slot)
-    if (xon) {
-      const uint4* xp = reinterpret_cast<const uint4*>(xrow + grp * 128);
+    // activation fragments + group sums of this group (independent of the slot)
+    float xs0[NJ], xs1[NJ], xo0[NJ], xo1[NJ];
 #pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const int xo = BITS == 8 ? (i < 2 ? i : 8 + (i - 2)) : i;  // 16-B units
-        const uint4 v = __ldg(xp + xo);
-        xt[4 * i] = v.x; xt[4 * i + 1] = v.y; xt[4 * i + 2] = v.z; xt[4 * i + 3] = v.w;
+    for (int j = 0; j < NJ; ++j) {
+      if (xon[j]) {
+        const uint4* xp = reinterpret_cast<const uint4*>(xrow[j] + grp * 128);
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const int xo = BITS == 8 ? (i < 2 ? i : 8 + (i - 2)) : i;  // 16-B units
+          const uint4 v = __ldg(xp + xo);
+          xt[j][4 * i] = v.x; xt[j][4 * i + 1] = v.y; xt[j][4 * i + 2] = v.z; xt[j][4 * i + 3] = v.w;
+        }
       }
-    }
-    float xs0, xs1, xo0, xo1;
-    if constexpr (XS) {
-      // the group sums on the tensor core: xs = sum x (A = ones), xoff = sum off_k x (A = the unpack
-      // offsets at each fragment position: INT4 lo codes 1024 at k 2q.., hi codes 64 at k 2q+8..) --
-      // the same fragment positions as the codes, so D - xoff cancels the offsets by construction
-      constexpr uint32_t H1 = 0x3C003C00u, H1024 = 0x64006400u, H64 = 0x54005400u;
-      const uint32_t a1[4] = {H1, H1, H1, H1};
-      float ds[4];
-      mma_16816_zc(ds, a1, xt[0], xt[1]);
+      if constexpr (XS) {
+        // the group sums on the tensor core: xs = sum x (A = ones), xoff = sum off_k x (A = the unpack
+        // offsets at each fragment position: INT4 lo codes 1024 at k 2q.., hi codes 64 at k 2q+8..) --
+        // the same fragment positions as the codes, so D - xoff cancels the offsets by construction
+        constexpr uint32_t H1 = 0x3C003C00u, H1024 = 0x64006400u, H64 = 0x54005400u;
+        const uint32_t a1[4] = {H1, H1, H1, H1};
+        float ds[4];
+        mma_16816_zc(ds, a1, xt[j][0], xt[j][1]);
 #pragma unroll
-      for (int t = 1; t < 8; ++t) mma_16816(ds, a1, xt[2 * t], xt[2 * t + 1], ds);
-      xs0 = ds[0];
-      xs1 = ds[1];
-      if constexpr (BITS == 4) {
-        const uint32_t ao[4] = {H1024, H1024, H64, H64};
-        float dof[4];
-        mma_16816_zc(dof, ao, xt[0], xt[1]);
+        for (int t = 1; t < 8; ++t) mma_16816(ds, a1, xt[j][2 * t], xt[j][2 * t + 1], ds);
+        xs0[j] = ds[0];
+        xs1[j] = ds[1];
+        if constexpr (BITS == 4) {
+          const uint32_t ao[4] = {H1024, H1024, H64, H64};
+          float dof[4];
+          mma_16816_zc(dof, ao, xt[j][0], xt[j][1]);
 #pragma unroll
-        for (int t = 1; t < 8; ++t) mma_16816(dof, ao, xt[2 * t], xt[2 * t + 1], dof);
-        xo0 = dof[0];
-        xo1 = dof[1];
+          for (int t = 1; t < 8; ++t) mma_16816(dof, ao, xt[j][2 * t], xt[j][2 * t + 1], dof);
+          xo0[j] = dof[0];
+          xo1[j] = dof[1];
+        } else {
+          xo0[j] = (BITS == 3 ? 8.f : 1024.f) * xs0[j];
+          xo1[j] = (BITS == 3 ? 8.f : 1024.f) * xs1[j];
+        }
       } else {
-        xo0 = (BITS == 3 ? 8.f : 1024.f) * xs0;
-        xo1 = (BITS == 3 ? 8.f : 1024.f) * xs1;
+        const float4 xsv = __ldg(reinterpret_cast<const float4*>(p.xsum + grp * kXsTok + 8 * j + 2 * q));
+        xs0[j] = xsv.x + xsv.y;
+        xs1[j] = xsv.z + xsv.w;
+        xo0[j] = BITS == 4 ? fmaf(1024.f, xsv.x, 64.f * xsv.y) : (BITS == 3 ? 8.f * xs0[j] : 1024.f * xs0[j]);
+        xo1[j] = BITS == 4 ? fmaf(1024.f, xsv.z, 64.f * xsv.w) : (BITS == 3 ? 8.f * xs1[j] : 1024.f * xs1[j]);
       }
-    } else {
-      const float4 xsv = __ldg(reinterpret_cast<const float4*>(p.xsum + grp * kXsTok + 2 * q));
-      xs0 = xsv.x + xsv.y;
-      xs1 = xsv.z + xsv.w;
-      xo0 = BITS == 4 ? fmaf(1024.f, xsv.x, 64.f * xsv.y) : (BITS == 3 ? 8.f * xs0 : 1024.f * xs0);
-      xo1 = BITS == 4 ? fmaf(1024.f, xsv.z, 64.f * xsv.w) : (BITS == 3 ? 8.f * xs1 : 1024.f * xs1);
     }
     mbar_wait(&bar[slot], (uint32_t)((c / S) & 1));
     const uint8_t* cs = ring + slot * SLOT;
@@ -897,45 +904,50 @@ __global__ void __launch_bounds__(kSThreads, SQ_K2S_MINB)
       lds_codes<BITS>(cs + r * UB + g * GB + lane_off, cw0);
       lds_codes<BITS>(cs + r * UB + (g + 8) * GB + lane_off, cw1);
       const uint32_t mr0 = ms[r * 16 + g], mr1 = ms[r * 16 + g + 8];
-      float d[4];
-      {
-        uint32_t a[4];
-        frag<BITS>(cw0, 0, a[0], a[2]);
-        frag<BITS>(cw1, 0, a[1], a[3]);
-        mma_16816_zc(d, a, xt[0], xt[1]);
-      }
+      float d[NJ][4];
 #pragma unroll
-      for (int t = 1; t < 8; ++t) {
+      for (int t = 0; t < 8; ++t) {
         uint32_t a[4];
         frag<BITS>(cw0, t, a[0], a[2]);
         frag<BITS>(cw1, t, a[1], a[3]);
-        mma_16816(d, a, xt[2 * t], xt[2 * t + 1], d);
+#pragma unroll
+        for (int j = 0; j < NJ; ++j) {
+          if (t == 0) mma_16816_zc(d[j], a, xt[j][0], xt[j][1]);
+          else mma_16816(d[j], a, xt[j][2 * t], xt[j][2 * t + 1], d[j]);
+        }
       }
       const float2 f0 = __half22float2(*reinterpret_cast<const __half2*>(&mr0));  // (s, z) row g
       const float2 f1 = __half22float2(*reinterpret_cast<const __half2*>(&mr1));  // row g+8
       // y += s * (D - xoff) + z * xs
-      acc[r][0] = fmaf(-f0.x, xo0, fmaf(f0.y, xs0, fmaf(f0.x, d[0], acc[r][0])));
-      acc[r][1] = fmaf(-f0.x, xo1, fmaf(f0.y, xs1, fmaf(f0.x, d[1], acc[r][1])));
-      acc[r][2] = fmaf(-f1.x, xo0, fmaf(f1.y, xs0, fmaf(f1.x, d[2], acc[r][2])));
-      acc[r][3] = fmaf(-f1.x, xo1, fmaf(f1.y, xs1, fmaf(f1.x, d[3], acc[r][3])));
+#pragma unroll
+      for (int j = 0; j < NJ; ++j) {
+        acc[r][j][0] = fmaf(-f0.x, xo0[j], fmaf(f0.y, xs0[j], fmaf(f0.x, d[j][0], acc[r][j][0])));
+        acc[r][j][1] = fmaf(-f0.x, xo1[j], fmaf(f0.y, xs1[j], fmaf(f0.x, d[j][1], acc[r][j][1])));
+        acc[r][j][2] = fmaf(-f1.x, xo0[j], fmaf(f1.y, xs0[j], fmaf(f1.x, d[j][2], acc[r][j][2])));
+        acc[r][j][3] = fmaf(-f1.x, xo1[j], fmaf(f1.y, xs1[j], fmaf(f1.x, d[j][3], acc[r][j][3])));
+      }
     }
     __syncwarp();  // every lane's reads of this slot are done
     if (lane == 0 && c + S < nit) issue(c + S);
     if (grp == kg - 1) {  // strip finished
       if (seg_from_start) {
 #pragma unroll
-        for (int r = 0; r < RT; ++r) store_strip_tile<EPI, RT>(p, set * RT + r, g, q, acc[r]);
+        for (int r = 0; r < RT; ++r) store_strip_tile<EPI, NJ>(p, set * RT + r, g, q, acc[r]);
       } else {  // the head strip, entered part-way
 #pragma unroll
         for (int r = 0; r < RT; ++r)
 #pragma unroll
-          for (int i = 0; i < 4; ++i) hacc[r][i] = acc[r][i];
+          for (int j = 0; j < NJ; ++j)
+#pragma unroll
+            for (int i = 0; i < 4; ++i) hacc[r][j][i] = acc[r][j][i];
         has_head = true;
       }
 #pragma unroll
       for (int r = 0; r < RT; ++r)
 #pragma unroll
-        for (int i = 0; i < 4; ++i) acc[r][i] = 0.f;
+        for (int j = 0; j < NJ; ++j)
+#pragma unroll
+          for (int i = 0; i < 4; ++i) acc[r][j][i] = 0.f;
       seg_from_start = true;
       grp = 0;
       ++set;
@@ -943,23 +955,20 @@ __global__ void __launch_bounds__(kSThreads, SQ_K2S_MINB)
       ++grp;
     }
   }
-  // partial strips into the warp's idle ring: [2][TOK][RR], slot 0 = head strip, 1 = tail strip
+  // partial strips into the warp's idle ring: [2][32 lanes][RT][NJ] float4 (each lane's accumulators
+  // contiguous); slot 0 = head strip, 1 = tail strip
   __syncwarp();
-  float* pw = reinterpret_cast<float*>(ring);
-  auto put = [&](int sl, const float (&v)[RT][4]) {
+  float4* pw = reinterpret_cast<float4*>(ring);
+  auto put = [&](int sl, const float (&v)[RT][NJ][4]) {
 #pragma unroll
     for (int r = 0; r < RT; ++r)
 #pragma unroll
-      for (int e = 0; e < 2; ++e) {
-        const int tok = 2 * q + e;
-        pw[(sl * TOK + tok) * RR + r * kRows + g] = v[r][e];
-        pw[(sl * TOK + tok) * RR + r * kRows + g + 8] = v[r][2 + e];
-      }
+      for (int j = 0; j < NJ; ++j) pw[(sl * 32 + lane) * PL + r * NJ + j] = make_float4(v[r][j][0], v[r][j][1], v[r][j][2], v[r][j][3]);
   };
   if (has_head) put(0, hacc);
   if (nit > 0 && grp != 0) put(set == head_set ? 0 : 1, acc);  // range ended inside a strip
   __syncthreads();
-  reduce_tail_s<EPI, RT, S * SLOT>(p, smem + RC::BAR_BYTES, C0, C1, R, warp, lane, g, q);
+  reduce_tail_s<EPI, RT, NJ, S * SLOT>(p, smem + RC::BAR_BYTES, C0, C1, R, warp, lane, g, q);
 }
 
 // xsum[g][t] = (sum_{k%4<2} x[t,k], sum_{k%4>=2} x[t,k]) over group g, t < 32 (0 for t >= m);
@@ -1008,9 +1017,9 @@ cudaError_t launch_e(const GemvP& p, cudaStream_t s) {
   return launch_pdl(kern, dim3((unsigned)p.W), dim3(kThreads), smem, s, p);
 }
 
-template <int BITS, int RT, int EPI, bool XS>
+template <int BITS, int RT, int EPI, bool XS, int NJ>
 cudaError_t launch_s_x(const CUtensorMap& tw, const CUtensorMap& tm, const GemvP& p, cudaStream_t s) {
-  void (*kern)(const CUtensorMap, const CUtensorMap, const GemvP) = k_gemv_s<BITS, RT, EPI, XS>;
+  void (*kern)(const CUtensorMap, const CUtensorMap, const GemvP) = k_gemv_s<BITS, RT, EPI, XS, NJ>;
   const size_t smem = (size_t)SRing<BITS, RT>::BYTES;
   static bool attr = false;
   if (!attr) {
@@ -1023,7 +1032,11 @@ cudaError_t launch_s_x(const CUtensorMap& tw, const CUtensorMap& tm, const GemvP
 // XS: group sums computed in the kernel (p.xsum == null) or read from p.xsum
 template <int BITS, int RT, int EPI>
 cudaError_t launch_s_e(const CUtensorMap& tw, const CUtensorMap& tm, const GemvP& p, cudaStream_t s) {
-  return p.xsum ? launch_s_x<BITS, RT, EPI, false>(tw, tm, p, s) : launch_s_x<BITS, RT, EPI, true>(tw, tm, p, s);
+  if constexpr (RT == 2) {
+    if (p.m > 8)
+      return p.xsum ? launch_s_x<BITS, RT, EPI, false, 2>(tw, tm, p, s) : launch_s_x<BITS, RT, EPI, true, 2>(tw, tm, p, s);
+  }
+  return p.xsum ? launch_s_x<BITS, RT, EPI, false, 1>(tw, tm, p, s) : launch_s_x<BITS, RT, EPI, true, 1>(tw, tm, p, s);
 }
 
 template <int BITS, int RT>
@@ -1098,13 +1111,23 @@ size_t part_bytes(int64_t W, int64_t m) {
 // strip width: 4 tiles (the activation fragment re-used 4x) for INT3 / INT4 linears of more than
 // 1280 tiles, else 2 (twice the items per warp; 5120^2 INT4 9.7 -> 8.0 us, 5120 x 20480 17.1 ->
 // 16.3 us, but 36864 x 9216 34.2 -> 37.8 us; tools/exp_k2s8.sh); INT8 always 2
-int k2s_rt(int bits, int64_t n) { return (bits != 8 && n / kRows > 1280) ? 4 : 2; }
+// (m in 9..16: two token tiles, RT = 2)
+int k2s_rt(int bits, int64_t n, int m) { return (bits != 8 && m <= 8 && n / kRows > 1280) ? 4 : 2; }
+
+// m in 9..16 (two token tiles, tools/exp_k2s16.sh): K2s beats K2c only on INT8 linears up to ~120 MB
+// (20480 x 5120: 23.6-23.9 vs 25.3-25.5 us; 5120^2: 10.8-11.2 vs 13.1), and loses up to 1.6x on large or
+// INT3 / INT4 ones (HMMA-bound at RT = 2); SQ_K2S16=1 / 0 forces it on / off there.
+bool k2s16(int bits, int64_t n, int64_t k) {
+  static int forced = -2;
+  if (forced == -2) { const char* e = getenv("SQ_K2S16"); forced = !e ? -1 : (e[0] == '1' ? 1 : 0); }
+  if (forced >= 0) return forced == 1;
+  return bits == 8 && (double)n * k <= 120e6;
+}
 
 bool k2s_rule(int bits, int64_t n, int64_t k, int m) {
   static int forced = -2;
   if (forced == -2) { const char* e = getenv("SQ_K2S"); forced = !e ? -1 : (e[0] == '0' ? 0 : 1); }
-  if (bits == 16 || m > 8 || n % (16 * k2s_rt(bits, n)) != 0) return false;
-  (void)k;
+  if (bits == 16 || m > 16 || (m > 8 && !k2s16(bits, n, k)) || n % (16 * k2s_rt(bits, n, m)) != 0) return false;
   if (forced >= 0) return forced == 1;
   return true;
 }
@@ -1145,7 +1168,8 @@ int gemv_path(int64_t n, int64_t k, int m, int bits) {
   // sizes at m <= 8, e.g. 20480 x 5120: 2.24 vs 2.05 TB/s)
   // (round 3: the strip kernel K2s streams every quantized linear at m <= 8 at least as fast as the
   // tcgen05 kernel, e.g. 36864 x 9216 INT4 5.1 / 4.6 TB/s at m = 1 / 8 vs 4.4-4.7; tools/exp_k2s2.sh)
-  if (bits == 16 || m > 8) return 1;
+  if (bits == 16 || m > 16) return 1;
+  if (m > 8) return k2s_rule(bits, n, k, m) ? 0 : 1;
   return 0;
 }
 
@@ -1191,7 +1215,7 @@ cudaError_t launch_gemv(const sq_qweight& w, const __half* x, int64_t ldx, int m
   auto t = prof_begin(KC_GEMV, bytes, 2.0 * m * w.n * w.k, s);
   cudaError_t e;
   if (k2s) {
-    const int rt = k2s_rt(w.bits, w.n);
+    const int rt = k2s_rt(w.bits, w.n, m);
     p.U = (int)(((w.n / kRows + rt - 1) / rt) * p.kg);
     p.W = (int)gemv_s_ctas(p.U);
     if (rt == 4) e = w.bits == 3 ? launch_s<3, 4>(w, p, epi, s) : launch_s<4, 4>(w, p, epi, s);

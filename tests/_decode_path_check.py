@@ -20,7 +20,7 @@ def main():
             b = synth.bias_f16(901 + n, n)
             qo = O.QWeight(w, bits, bias=b)
             qg = sq.QLinear.from_fp16(torch.from_numpy(w).cuda(), bits, torch.from_numpy(b).cuda())
-            for m in (1, 3, 5, 8, 9, 32):
+            for m in (1, 3, 5, 8, 9, 16, 32):
                 x = synth.act_f16(902 + m, m, k)
                 ref = O.linear(x, qo)
                 y = torch.empty((m, n), dtype=torch.float16, device="cuda")
@@ -30,7 +30,7 @@ def main():
                 err = float(np.abs(yy - ref).max() / np.abs(ref).max())
                 worst = max(worst, err)
                 assert err <= 2e-3, (os.environ.get("SQ_GEMV_PATH"), bits, n, k, m, err)
-                if bits != 16 and m <= 8:
+                if bits != 16 and m <= 16:
                     # group sums supplied by the caller (sq_xsum) instead of computed in the kernel
                     xd = torch.from_numpy(x).cuda()
                     y2 = torch.empty_like(y)

@@ -231,7 +231,7 @@ def test_one_token_prefill_equals_decode_function():
     assert normwise(a, ref) <= TOL and normwise(b, ref) <= TOL
 
 
-@pytest.mark.parametrize("path", ["mma", "mma-k2", "mma-k2s", "tc", "tc-nocluster"])
+@pytest.mark.parametrize("path", ["mma", "mma-k2", "mma-k2s", "mma-k2s16", "tc", "tc-nocluster"])
 def test_decode_forced_path(path):
     """Every decode kernel (mma.sync K2 and its strip form K2s, tcgen05 K2c) for every bit width and m
     in 1..32, whatever the automatic choice (gemv_path, use_k2s) would pick: SQ_GEMV_PATH forces the
@@ -244,8 +244,10 @@ def test_decode_forced_path(path):
     env = dict(os.environ, SQ_GEMV_PATH=path.split("-")[0])
     if path == "tc-nocluster":
         env["SQ_TC_CLUSTER"] = "0"
-    if path in ("mma-k2", "mma-k2s"):
-        env["SQ_K2S"] = "1" if path == "mma-k2s" else "0"
+    if path.startswith("mma-k2"):
+        env["SQ_K2S"] = "1" if path.startswith("mma-k2s") else "0"
+    if path == "mma-k2s16":
+        env["SQ_K2S16"] = "1"  # m in 9..16 on K2s too (two token tiles)
     script = os.path.join(os.path.dirname(os.path.abspath(__file__)), "_decode_path_check.py")
     r = subprocess.run([sys.executable, script], env=env, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
