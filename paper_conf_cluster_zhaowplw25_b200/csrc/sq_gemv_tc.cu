@@ -383,10 +383,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
           if (elect_one()) {
             const uint32_t d_tm = tmem + D_COL + t * BT;
             const uint32_t a_tm = tmem + A_COL + sa * DCfg<BITS, UG>::A_SLOT;
+            // B descriptor as two words: the per-k-step offsets are 32-bit adds on the address word (fewer
+            // R2UR moves into the uniform registers UTCHMMA reads; 0-7 % faster, tools/exp_udesc.sh)
+            const uint32_t blo = (uint32_t)bdesc0, bhi = (uint32_t)(bdesc0 >> 32);
 #pragma unroll
             for (int kk = 0; kk < 8 * UG; ++kk)
-              tc_mma_ts(d_tm, a_tm + kk * 8, bdesc0 + (uint64_t)(((kk >> 2) * X_BLOCK + (kk & 3) * 32) >> 4),
-                        kIdescTc, (j == j0 && kk == 0) ? 0u : 1u);
+              tc_mma_ts_w(d_tm, a_tm + kk * 8, blo + (uint32_t)(((kk >> 2) * X_BLOCK + (kk & 3) * 32) >> 4), bhi,
+                          kIdescTc, (j == j0 && kk == 0) ? 0u : 1u);
             tc_commit(&empty_a[sa]);
             if (t == pp - 1) {
               tc_commit(&empty_x[sx]);
