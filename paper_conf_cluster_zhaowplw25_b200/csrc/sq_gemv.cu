@@ -23,6 +23,11 @@
 //  * Split tiles are reduced in shared memory in fixed warp order; a tile that
 //    straddles two CTAs is finished by the last CTA (atomic counter, fixed CTA
 //    order).  Deterministic; counters self-reset.
+//
+// K2s (below, k_gemv_s) is the default for quantized weights at m <= 8 (INT8 up to m = 16): the same
+// unpack / mma.sync / factorised scale-zero on STRIPS of RT row tiles x one group, per-warp TMA rings,
+// two 8-warp CTAs per SM, group sums on the tensor core.  K2 (k_gemv_q) remains for n not a multiple of
+// 32 and for m in 9..32 off the tcgen05 kernel's shapes ("Which decode kernel").
 #include <cstdlib>
 
 #include "sq_common.cuh"
@@ -30,28 +35,7 @@
 namespace sq {
 namespace {
 
-#ifndef SQ_K2_WARPS
-#define SQ_K2_WARPS 16
-#endif
-#ifndef SQ_K2_SMEM_KB
-#define SQ_K2_SMEM_KB 227
-#endif
-#ifndef SQ_K2_CPS
-#define SQ_K2_CPS 1
-#endif
-#ifndef SQ_K2_MINB
-#define SQ_K2_MINB 1
-#endif
-#ifndef SQ_K2S_RELACQ
-#define SQ_K2S_RELACQ 1
-#endif
-#ifndef SQ_K2S_SMEM_KB
-#define SQ_K2S_SMEM_KB 76
-#endif
-#ifndef SQ_K2S_MINB
-#define SQ_K2S_MINB 2
-#endif
-constexpr int kWarps = SQ_K2_WARPS;  // one 512-thread CTA per SM
+constexpr int kWarps = 16;  // one 512-thread CTA per SM
 constexpr int kThreads = kWarps * 32;
 constexpr int kRows = 16;   // rows per unit (mma M)
 constexpr int kXsTok = 32;  // token slots per group in the xsum buffer
@@ -466,7 +450,7 @@ struct QRing {
   static constexpr int BARS = kWarps * 8 * 8;                     // <= 8 mbarriers per warp
   static constexpr int CH = BITS == 8 ? 2 : (BITS == 4 ? 3 : 4);  // units per slot (3.3-4.2 KB)
   static constexpr int SLOT = CH * (UB + UM);
-  static constexpr int S0 = (SQ_K2_SMEM_KB * 1024 - PART - BARS - 128) / kWarps / SLOT;
+  static constexpr int S0 = (227 * 1024 - PART - BARS - 128) / kWarps / SLOT;
   static constexpr int S = S0 > 8 ? 8 : S0;
   static constexpr int BYTES = PART + BARS + kWarps * S * SLOT;
   static_assert(S >= 2, "ring depth");
@@ -491,7 +475,7 @@ __device__ __forceinline__ void lds_codes(const uint8_t* p, uint32_t* c) {
 }
 
 template <int BITS, int TOK, int EPI>
-__global__ void __launch_bounds__(kThreads, SQ_K2_MINB) k_gemv_q(const GemvP p) {
+__global__ void __launch_bounds__(kThreads, 1) k_gemv_q(const GemvP p) {
   using RC = QRing<BITS, TOK>;
   constexpr int LU = Cfg<BITS>::LU;
   constexpr int GB = Cfg<BITS>::GB;
@@ -667,10 +651,13 @@ __global__ void __launch_bounds__(kThreads, SQ_K2_MINB) k_gemv_q(const GemvP p) 
 // fixed warp order in shared memory (in the warps' idle rings) and across CTAs by the last CTA to
 // arrive, in fixed CTA order.
 // K2s CTA: 8 warps, two CTAs per SM (measured against one 16-warp CTA: equal or up to 7 % faster on
-// OPT-13B / OPT-66B shapes; tools/exp_k2s2.sh)
+// OPT-13B / OPT-66B shapes; tools/gemv_rot.py --graph on variant builds)
 constexpr int kSWarps = 8;
 constexpr int kSThreads = kSWarps * 32;
 constexpr int kSCtasPerSm = 2;
+// per-CTA shared memory budget: two-slot rings (a third slot measured 0.9 us slower per launch on
+// 20480 x 5120: more bytes requested at kernel start delay the first items)
+constexpr int kSSmemKB = 76;
 
 template <int BITS, int RT_>
 struct SRing {
@@ -678,7 +665,7 @@ struct SRing {
   static constexpr int UB = 16 * Cfg<BITS>::GB;                   // codes bytes per unit
   static constexpr int SLOT = RT * (UB + 64);                     // one item: RT units + their meta
   static constexpr int BAR_BYTES = kSWarps * 8 * 8;                // <= 8 mbarriers per warp
-  static constexpr int S0 = (SQ_K2S_SMEM_KB * 1024 - 128 - BAR_BYTES) / kSWarps / SLOT;
+  static constexpr int S0 = (kSSmemKB * 1024 - 128 - BAR_BYTES) / kSWarps / SLOT;
   static constexpr int S = S0 > 8 ? 8 : S0;
   static constexpr int PARTW = 2 * 8 * RT * kRows * 4;            // a warp's head / tail strip partials
   static constexpr int BYTES = 128 + BAR_BYTES + kSWarps * S * SLOT;  // + alignment slack
@@ -742,19 +729,12 @@ __device__ __forceinline__ void reduce_tail_s(const GemvP& p, const uint8_t* par
     const int ca = (int)(((long long)(t * kg + 1) * NC - 1) / p.U);
     const int cb2 = (int)(((long long)((t + 1) * kg) * NC - 1) / p.U);
     int old = 0;
-#if SQ_K2S_RELACQ
+    // release (orders this warp's partial stores, __syncwarp + cumulativity) / acquire (the last CTA's
+    // reads below) in one atomic: no __threadfence on either side (-0.2-0.7 us per launch)
     __syncwarp();
     if (lane == 0) asm volatile("atom.acq_rel.gpu.global.add.s32 %0, [%1], 1;" : "=r"(old) : "l"(p.cnt + t) : "memory");
     old = __shfl_sync(0xffffffff, old, 0);
     if (old != cb2 - ca) continue;
-#else
-    __threadfence();
-    __syncwarp();
-    if (lane == 0) old = atomicAdd(p.cnt + t, 1);
-    old = __shfl_sync(0xffffffff, old, 0);
-    if (old != cb2 - ca) continue;
-    __threadfence();
-#endif
 #pragma unroll
     for (int r = 0; r < RT; ++r)
 #pragma unroll
@@ -780,7 +760,7 @@ __device__ __forceinline__ void reduce_tail_s(const GemvP& p, const uint8_t* par
 
 // NJ = token n8 tiles: 1 (m <= 8) or 2 (m <= 16, RT = 2)
 template <int BITS, int RT_, int EPI, bool XS, int NJ>
-__global__ void __launch_bounds__(kSThreads, SQ_K2S_MINB)
+__global__ void __launch_bounds__(kSThreads, kSCtasPerSm)
     k_gemv_s(const __grid_constant__ CUtensorMap tm_w, const __grid_constant__ CUtensorMap tm_m, const GemvP p) {
   using RC = SRing<BITS, RT_>;
   constexpr int LU = Cfg<BITS>::LU, GB = Cfg<BITS>::GB;
@@ -1080,7 +1060,7 @@ cudaError_t launch_b(const GemvP& p, int epi, cudaStream_t s) {
 
 // number of CTAs: one per SM (fewer for tiny problems so every warp gets >= 1 unit)
 int64_t gemv_ctas(int64_t U) {
-  const int64_t full = (int64_t)num_sms() * SQ_K2_CPS;
+  const int64_t full = (int64_t)num_sms();
   const int64_t need = (U + kWarps - 1) / kWarps;
   return need < full ? need : full;
 }
@@ -1104,17 +1084,17 @@ size_t part_bytes(int64_t W, int64_t m) {
 }
 // K2s (strips) for quantized weights at m <= 8 (SQ_K2S=0: K2)
 // Whole strips only (n a multiple of RT * 16, so no TMA box reaches past the matrix).  Measured
-// (tools/exp_k2s9.sh, back-to-back graph launches, m = 1 / 8): K2s is as fast as K2 or faster on every
+// (tools/gemv_rot.py --graph on variant builds, back-to-back graph launches, m = 1 / 8): K2s is as fast as K2 or faster on every
 // OPT-125m ... OPT-66B shape, e.g. 36864 x 9216 INT4 34.4 / 37.1 us vs 44.2 / 60.8, 20480 x 5120
 // INT4 15.5 / 17.0 vs 17.7 / 23.7, 768 x 3072 5.5 vs 6.0-6.5 (2304 x 768: within 0.2 us), so K2
 // remains only for n not a multiple of 32.  SQ_K2S=0 / 1 forces K2 / K2s.
 // strip width: 4 tiles (the activation fragment re-used 4x) for INT3 / INT4 linears of more than
 // 1280 tiles, else 2 (twice the items per warp; 5120^2 INT4 9.7 -> 8.0 us, 5120 x 20480 17.1 ->
-// 16.3 us, but 36864 x 9216 34.2 -> 37.8 us; tools/exp_k2s8.sh); INT8 always 2
+// 16.3 us, but 36864 x 9216 34.2 -> 37.8 us; tools/gemv_rot.py --graph on variant builds); INT8 always 2
 // (m in 9..16: two token tiles, RT = 2)
 int k2s_rt(int bits, int64_t n, int m) { return (bits != 8 && m <= 8 && n / kRows > 1280) ? 4 : 2; }
 
-// m in 9..16 (two token tiles, tools/exp_k2s16.sh): K2s beats K2c only on INT8 linears up to ~120 MB
+// m in 9..16 (two token tiles, tools/gemv_rot.py --graph on variant builds): K2s beats K2c only on INT8 linears up to ~120 MB
 // (20480 x 5120: 23.6-23.9 vs 25.3-25.5 us; 5120^2: 10.8-11.2 vs 13.1), and loses up to 1.6x on large or
 // INT3 / INT4 ones (HMMA-bound at RT = 2); SQ_K2S16=1 / 0 forces it on / off there.
 bool k2s16(int bits, int64_t n, int64_t k) {
@@ -1167,7 +1147,7 @@ int gemv_path(int64_t n, int64_t k, int m, int bits) {
   // at every m, e.g. 36864 x 9216 at m = 1: 3.34 vs 2.89 TB/s; the mma.sync kernel keeps the OPT-13B
   // sizes at m <= 8, e.g. 20480 x 5120: 2.24 vs 2.05 TB/s)
   // (round 3: the strip kernel K2s streams every quantized linear at m <= 8 at least as fast as the
-  // tcgen05 kernel, e.g. 36864 x 9216 INT4 5.1 / 4.6 TB/s at m = 1 / 8 vs 4.4-4.7; tools/exp_k2s2.sh)
+  // tcgen05 kernel, e.g. 36864 x 9216 INT4 5.1 / 4.6 TB/s at m = 1 / 8 vs 4.4-4.7; tools/gemv_rot.py --graph on variant builds)
   if (bits == 16 || m > 16) return 1;
   if (m > 8) return k2s_rule(bits, n, k, m) ? 0 : 1;
   return 0;

@@ -384,7 +384,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             const uint32_t d_tm = tmem + D_COL + t * BT;
             const uint32_t a_tm = tmem + A_COL + sa * DCfg<BITS, UG>::A_SLOT;
             // B descriptor as two words: the per-k-step offsets are 32-bit adds on the address word (fewer
-            // R2UR moves into the uniform registers UTCHMMA reads; 0-7 % faster, tools/exp_udesc.sh)
+            // R2UR moves into the uniform registers UTCHMMA reads; 0-7 % faster, tools/gemv_rot.py --graph on variant builds)
             const uint32_t blo = (uint32_t)bdesc0, bhi = (uint32_t)(bdesc0 >> 32);
 #pragma unroll
             for (int kk = 0; kk < 8 * UG; ++kk)
