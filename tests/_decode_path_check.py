@@ -97,6 +97,36 @@ def full(bits):
     print("ok full", bits, err)
 
 
+def bloom(bits):
+    """configs[4] BLOOM-176B linears at their full size (fc1 57344 x 14336, fc2 14336 x 57344) on the
+    automatic decode path (K2s at m = 1 / 8, K2c at m = 32): sampled rows vs the oracle, bitwise repeat."""
+    for (n, k, name) in ((57344, 14336, "fc1"), (14336, 57344, "fc2")):
+        seed = synth.weight_seed(3, name)
+        wd = torch.empty((n, k), dtype=torch.float16, device="cuda")
+        synth.device_weight_f16(wd.data_ptr(), seed, n, k)
+        qg = sq.QLinear.from_fp16(wd, bits)
+        del wd
+        rows = np.random.default_rng(bits + n).choice(n, 32, replace=False)
+        rows[0], rows[1] = 0, n - 1
+        qo = O.QWeight(synth.weight_f16(seed, n, k, rows=rows), bits)
+        for m in (1, 8, 32):
+            x = synth.act_f16(31 + m, m, k)
+            xd = torch.from_numpy(x).cuda()
+            y = torch.empty((m, n), dtype=torch.float16, device="cuda")
+            sq.sq_linear_decode(qg, xd, y, 0)
+            y2 = torch.empty_like(y)
+            sq.sq_linear_decode(qg, xd, y2, 0)
+            torch.cuda.synchronize()
+            assert torch.equal(y, y2), ("bloom repeat", name, bits, m)
+            ref = O.linear(x, qo)
+            yy = y.float().cpu().numpy().astype(np.float64)[:, rows]
+            err = float(np.abs(yy - ref).max() / np.abs(ref).max())
+            assert err <= 2e-3, ("bloom", name, bits, m, err)
+        del qg
+        torch.cuda.empty_cache()
+    print("ok bloom", bits)
+
+
 def canary():
     """Out-of-bounds guard for the forced kernel (compute-sanitizer is closed on this pool): y is a
     strided window of a larger buffer pre-filled with a sentinel, the workspace is followed by a
@@ -137,5 +167,7 @@ if __name__ == "__main__":
         full(int(sys.argv[2]))
     elif len(sys.argv) > 1 and sys.argv[1] == "canary":
         canary()
+    elif len(sys.argv) > 2 and sys.argv[1] == "bloom":
+        bloom(int(sys.argv[2]))
     else:
         main()

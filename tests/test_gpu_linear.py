@@ -288,6 +288,18 @@ def test_prefill_adversarial(bits, m):
     check_adversarial(y - y0, O.linear(x32, qo))
 
 
+@pytest.mark.parametrize("bits", [3, 4])
+def test_decode_bloom_full_size_sampled(bits):
+    """Maximum sizes of the workloads: BLOOM-176B fc1 / fc2 (configs[4], INT3 / INT4) on the automatic
+    decode path at m = 1, 8, 32 -- 32 sampled rows vs the oracle and a bitwise repeat."""
+    import os
+    import subprocess
+    import sys
+    script = os.path.join(os.path.dirname(os.path.abspath(__file__)), "_decode_path_check.py")
+    r = subprocess.run([sys.executable, script, "bloom", str(bits)], capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+
+
 @pytest.mark.parametrize("kern", ["k2", "k2s"])
 def test_decode_mma_writes_in_bounds(kern):
     """K2 / K2s write nothing outside y's window and the workspace, and reset every split-k counter
