@@ -127,3 +127,60 @@ def profile(h1: int, h2: int, bits_set=(3, 4, 8, 16), pre_points=((1, 128), (1, 
         del copies, ws
         torch.cuda.empty_cache()
     return out
+
+
+def profile_interleaved(h1: int, h2: int, point_sets: dict, bits_set=(3, 4, 8, 16), reps: int = 5, dec_reps: int = 25,
+                        act: int = 0, n_layers: int = 8, seed: int = 0) -> dict:
+    """As ``profile``, for several named point sets at once ({"train": {"pre": [...], "dec": [...]}, "unseen":
+    ...}), every (set, bits, phase, point) measured in one seeded random order with all bit widths'
+    stages resident.  The board runs at its power limit and the clock drifts with the load history
+    (1275-1965 MHz), so profiling one set after the other puts a clock difference
+    between the fit and its validation; interleaving gives both sets the same mix of thermal states.
+    Returns {set name: [samples]}."""
+    import random
+    import torch
+    from . import SQ_DECODE, SQ_PREFILL
+    from .runtime import StageWorkspace, build_layers, layer_array, sq_stage_forward
+    max_tok = max(v * s for d in point_sets.values() for v, s in d.get("pre", ()))
+    stages = {}
+    for b in bits_set:
+        copies = build_layers(n_layers, h1, h2, [b] * n_layers, act=act)
+        stages[b] = (copies, layer_array(copies), StageWorkspace(copies, max_tok))
+    x = torch.randn(max_tok, h1, device="cuda")
+    y = torch.empty_like(x)
+    jobs = [(name, b, ph, pt) for name, d in point_sets.items() for b in bits_set for ph in ("pre", "dec")
+            for pt in d.get(ph, ())]
+    random.Random(seed).shuffle(jobs)
+    out = {name: [] for name in point_sets}
+    for name, b, phase, (v, s_or_ctx) in jobs:
+        copies, arr, ws = stages[b]
+        tokens = v * s_or_ctx if phase == "pre" else v
+        ph = SQ_PREFILL if phase == "pre" else SQ_DECODE
+        run = lambda: sq_stage_forward(copies, ph, x[:tokens], y[:tokens], ws, arr=arr)
+        if phase == "dec":
+            # decode steps replay from CUDA graphs in sq_pipeline_run: time them the same way (the
+            # ~6 launches per layer would otherwise be host-enqueue bound)
+            run()
+            torch.cuda.synchronize()
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g):
+                run()
+            run = g.replay
+        ts = []
+        # a decode step of the 8-layer stage is ~1-3 ms: more repetitions than a prefill point so the
+        # median spans the power-capped clock's swings
+        for rep in range((reps if phase == "pre" else dec_reps) + 1):
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record()
+            run()
+            e1.record()
+            torch.cuda.synchronize()
+            if rep:
+                ts.append(e0.elapsed_time(e1) / 1e3 / len(copies))
+        out[name].append({"phase": phase, "bits": int(b), "v": int(v), "s": int(s_or_ctx), "ctx": int(s_or_ctx),
+                          "t": statistics.median(ts)})
+    del stages
+    torch.cuda.empty_cache()
+    return out
+

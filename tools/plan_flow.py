@@ -43,12 +43,15 @@ def main():
 
     # ---- 1. latency cost model: fit on profiled points, validate on unseen workloads
     t0 = time.time()
-    train = CM.profile(h1, h2, pre_points=((1, 128), (1, 512), (2, 256), (2, 1024), (4, 128), (4, 512), (8, 256),
-                                            (8, 512), (16, 256), (6, 640)),
-                       dec_points=((1, 256), (2, 1024), (4, 512), (6, 128), (8, 512), (12, 256), (16, 384),
-                                   (24, 900), (32, 640), (32, 1024)))
-    unseen = CM.profile(h1, h2, pre_points=((3, 384), (5, 256), (6, 448), (12, 320)),
-                        dec_points=((3, 384), (5, 700), (12, 768), (20, 200), (28, 512)), reps=3)
+    # train and unseen points measured interleaved in one random order (same thermal / clock mix)
+    sets = CM.profile_interleaved(h1, h2, {
+        "train": {"pre": ((1, 128), (1, 512), (2, 256), (2, 1024), (4, 128), (4, 512), (8, 256), (8, 512), (16, 256),
+                          (6, 640)),
+                  "dec": ((1, 256), (2, 1024), (4, 512), (6, 128), (8, 512), (12, 256), (16, 384), (24, 900),
+                          (32, 640), (32, 1024))},
+        "unseen": {"pre": ((3, 384), (5, 256), (6, 448), (12, 320)),
+                   "dec": ((3, 384), (5, 700), (12, 768), (20, 200), (28, 512))}})
+    train, unseen = sets["train"], sets["unseen"]
     model = CM.LatencyModel.fit(train, {"gpu": torch.cuda.get_device_name(0), "h1": h1, "h2": h2})
     err_tr, err_un = model.errors(train), model.errors(unseen)
     out["costmodel"] = {"coef": json.loads(model.to_json())["coef"], "train_points": len(train),
