@@ -143,12 +143,15 @@ typedef enum {
 /* ------------------------------------------------------------------------
  * a4 — decode linear (P:57 decode phase, memory-bound per P:106/P:164):
  *   y = epi(x . W~^T), m in [1, 32] tokens (one per sequence of the decode
- *   micro-batch xi).  Streams the packed weights once with 128-bit loads,
- *   unpacks in registers, fp32 accumulation (CUDA-core unpack + mma.sync
- *   dot products, K2).
+ *   micro-batch xi).  Streams the packed weights once (TMA / bulk copies into
+ *   shared-memory rings), unpacks in registers, fp32 accumulation: mma.sync
+ *   strips for quantized weights at m <= 8 (INT8 m <= 16; K2s, K2
+ *   when n % 32 != 0), tcgen05 with the dequantized weights in tensor memory
+ *   otherwise (K2c).
  *   x_dev fp16 [m, ldx] (ldx % 8 == 0, 16-B aligned).  y_dev per epi.
  *   xsum_dev: optional float2 [k/128][32] group sums of x produced by
- *     sq_xsum (NULL: computed internally into the workspace).
+ *     sq_xsum (NULL: computed by the kernel on the tensor core (K2s) or into
+ * the workspace by sq_xsum (K2); ignored by K2c).
  *   ws_dev/ws_bytes: >= sq_linear_workspace_bytes(w, m); must be ZEROED once
  *     before first use (holds self-resetting counters); one workspace per
  *     concurrently running call.

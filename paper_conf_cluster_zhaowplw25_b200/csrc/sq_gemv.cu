@@ -640,16 +640,18 @@ __global__ void __launch_bounds__(kThreads, 1) k_gemv_q(const GemvP p) {
   reduce_tail<TOK, EPI>(p, part_s, C0, C1, R, warp, lane, g, q);
 }
 
-// ---------------------------------------------------------------- K2s: strips of RT row tiles (m <= 8)
+// ---------------------------------------------------------------- K2s: strips of RT row tiles (m <= 8;
+// INT8 m <= 16 with two token tiles)
 // A work item is (strip, group): RT consecutive 16-row tiles x one 128-k group.  The activation
-// fragment and the group sums of a group are loaded once per RT units (K2 re-loads them for every
-// unit), and the RT units' HMMA chains are independent (ILP).  Items are flattened strip-major /
-// group-minor and split evenly over the grid's warps, as K2's units are; each warp streams its
-// items into its own S-slot ring with per-lane bulk copies (lane r < RT: unit r's codes, lane
-// RT + r: its meta; placement T16 makes each unit one contiguous range).  Unpack, mma.sync and the
-// factorised per-group scale / zero are K2's.  Deterministic: the split strips are reduced in
-// fixed warp order in shared memory (in the warps' idle rings) and across CTAs by the last CTA to
-// arrive, in fixed CTA order.
+// fragment of a group is loaded once per RT units (K2 re-loads it for every unit), its group sums
+// (xs, xoff) are read from the caller's sq_xsum output or computed on the tensor core (HMMA with
+// ones / offset A fragments), and the RT units' HMMA chains are independent (ILP).  Items are
+// flattened strip-major / group-minor and split evenly over the grid's warps, as K2's units are;
+// each warp streams its items into its own S-slot ring, lane 0 issuing one 3-D TMA box of the
+// strip's RT units (T16: [tile][group lines][256 B]) and one 2-D box of their meta per item.
+// Unpack, mma.sync and the factorised per-group scale / zero are K2's.  Deterministic: the split
+// strips are reduced in fixed warp order in shared memory (in the warps' idle rings) and across
+// CTAs by the last CTA to arrive, in fixed CTA order.
 // K2s CTA: 8 warps, two CTAs per SM (measured against one 16-warp CTA: equal or up to 7 % faster on
 // OPT-13B / OPT-66B shapes; tools/gemv_rot.py --graph on variant builds)
 constexpr int kSWarps = 8;
@@ -667,9 +669,8 @@ struct SRing {
   static constexpr int BAR_BYTES = kSWarps * 8 * 8;                // <= 8 mbarriers per warp
   static constexpr int S0 = (kSSmemKB * 1024 - 128 - BAR_BYTES) / kSWarps / SLOT;
   static constexpr int S = S0 > 8 ? 8 : S0;
-  static constexpr int PARTW = 2 * 8 * RT * kRows * 4;            // a warp's head / tail strip partials
   static constexpr int BYTES = 128 + BAR_BYTES + kSWarps * S * SLOT;  // + alignment slack
-  static_assert(S >= 2 && S * SLOT >= PARTW && BYTES <= 227 * 1024 && SLOT % 128 == 0, "K2s shared memory");
+  static_assert(S >= 2 && BYTES <= 227 * 1024 && SLOT % 128 == 0, "K2s shared memory");
 };
 
 template <int EPI, int NJ>
