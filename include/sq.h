@@ -151,7 +151,7 @@ typedef enum {
  *   x_dev fp16 [m, ldx] (ldx % 8 == 0, 16-B aligned).  y_dev per epi.
  *   xsum_dev: optional float2 [k/128][32] group sums of x produced by
  *     sq_xsum (NULL: computed by the kernel on the tensor core (K2s) or into
- * the workspace by sq_xsum (K2); ignored by K2c).
+ *     the workspace by sq_xsum (K2); ignored by K2c).
  *   ws_dev/ws_bytes: >= sq_linear_workspace_bytes(w, m); must be ZEROED once
  *     before first use (holds self-resetting counters); one workspace per
  *     concurrently running call.
