@@ -131,6 +131,34 @@ __device__ __forceinline__ void frag(const uint32_t* c, int t, uint32_t& lo, uin
   }
 }
 
+// K2s's INT3 fragments: each 3-bit field read in place under its own magic exponent, one LOP3 per
+// code pair (fields at bits 0 / 3 / 6 of a 16-bit half -> 1024 / 128 / 16 + c; fields 9 / 12 via one
+// shift per word -> 1024 / 128 + c; pair 15 from the spare bits -> 1024 + c), as K2c's dequant does.
+// The per-position offsets are removed by the group correction xoff = sum off_k x_k, which K2s
+// computes on the tensor core with the same fragment positions (k3_magic as the A operand).
+__device__ __forceinline__ constexpr uint32_t k3_magic(int i) {
+  return i == 15 ? 0x64006400u : ((i % 5) % 3 == 0 ? 0x64006400u : ((i % 5) % 3 == 1 ? 0x58005800u : 0x4C004C00u));
+}
+__device__ __forceinline__ constexpr uint32_t k3_mask(int i) {
+  return i == 15 ? 0x00070007u : ((i % 5) % 3 == 0 ? 0x00070007u : ((i % 5) % 3 == 1 ? 0x00380038u : 0x01C001C0u));
+}
+__device__ __forceinline__ void frag3m(const uint32_t* c, const uint32_t* c9, uint32_t p15, int t, uint32_t& lo,
+                                       uint32_t& hi) {
+  auto pairv = [&](int i) -> uint32_t {
+    if (i == 15) return lop3_and_or(p15, 0x00070007u, 0x64006400u);
+    const uint32_t x = (i % 5) < 3 ? c[i / 5] : c9[i / 5];
+    return lop3_and_or(x, k3_mask(i), k3_magic(i));
+  };
+  lo = pairv(2 * t);
+  hi = pairv(2 * t + 1);
+}
+__device__ __forceinline__ uint32_t k3_spare(const uint32_t* c) {
+  uint32_t u;
+  asm("lop3.b32 %0, %1, %2, %3, 0xCA;" : "=r"(u) : "r"(0x00010001u), "r"(c[0] >> 15), "r"(c[1] >> 14));
+  asm("lop3.b32 %0, %1, %2, %3, 0xCA;" : "=r"(u) : "r"(0x00030003u), "r"(u), "r"(c[2] >> 13));
+  return u;
+}
+
 // predicated 16-B load (no divergent branch): dst unchanged when !pred
 __device__ __forceinline__ void ldg_v4_pred(uint32_t* d, const void* p, bool pred) {
   asm volatile(
@@ -845,29 +873,27 @@ __global__ void __launch_bounds__(kSThreads, kSCtasPerSm)
         }
       }
       if constexpr (XS) {
-        // the group sums on the tensor core: xs = sum x (A = ones), xoff = sum off_k x (A = the unpack
-        // offsets at each fragment position: INT4 lo codes 1024 at k 2q.., hi codes 64 at k 2q+8..) --
-        // the same fragment positions as the codes, so D - xoff cancels the offsets by construction
+        // the group sums on the tensor core, both from ONE 8-HMMA chain: A rows 0-7 are ones (D rows
+        // 0-7 = xs = sum x), rows 8-15 the unpack offsets at each fragment position (D rows 8-15 =
+        // xoff = sum off_k x; INT4: lo codes 1024 at k 2q.., hi codes 64 at k 2q+8..) -- the same
+        // positions as the codes, so D - xoff cancels the offsets by construction
         constexpr uint32_t H1 = 0x3C003C00u, H1024 = 0x64006400u, H64 = 0x54005400u;
-        const uint32_t a1[4] = {H1, H1, H1, H1};
         float ds[4];
-        mma_16816_zc(ds, a1, xt[j][0], xt[j][1]);
 #pragma unroll
-        for (int t = 1; t < 8; ++t) mma_16816(ds, a1, xt[j][2 * t], xt[j][2 * t + 1], ds);
+        for (int t = 0; t < 8; ++t) {
+          uint32_t ao[4];
+          ao[0] = H1;
+          ao[2] = H1;
+          if constexpr (BITS == 4) { ao[1] = H1024; ao[3] = H64; }
+          else if constexpr (BITS == 3) { ao[1] = k3_magic(2 * t); ao[3] = k3_magic(2 * t + 1); }
+          else { ao[1] = H1024; ao[3] = H1024; }
+          if (t == 0) mma_16816_zc(ds, ao, xt[j][0], xt[j][1]);
+          else mma_16816(ds, ao, xt[j][2 * t], xt[j][2 * t + 1], ds);
+        }
         xs0[j] = ds[0];
         xs1[j] = ds[1];
-        if constexpr (BITS == 4) {
-          const uint32_t ao[4] = {H1024, H1024, H64, H64};
-          float dof[4];
-          mma_16816_zc(dof, ao, xt[j][0], xt[j][1]);
-#pragma unroll
-          for (int t = 1; t < 8; ++t) mma_16816(dof, ao, xt[j][2 * t], xt[j][2 * t + 1], dof);
-          xo0[j] = dof[0];
-          xo1[j] = dof[1];
-        } else {
-          xo0[j] = (BITS == 3 ? 8.f : 1024.f) * xs0[j];
-          xo1[j] = (BITS == 3 ? 8.f : 1024.f) * xs1[j];
-        }
+        xo0[j] = ds[2];
+        xo1[j] = ds[3];
       } else {
         const float4 xsv = __ldg(reinterpret_cast<const float4*>(p.xsum + grp * kXsTok + 8 * j + 2 * q));
         xs0[j] = xsv.x + xsv.y;
@@ -886,11 +912,23 @@ __global__ void __launch_bounds__(kSThreads, kSCtasPerSm)
       lds_codes<BITS>(cs + r * UB + (g + 8) * GB + lane_off, cw1);
       const uint32_t mr0 = ms[r * 16 + g], mr1 = ms[r * 16 + g + 8];
       float d[NJ][4];
+      uint32_t c90[3], c91[3], s150 = 0, s151 = 0;
+      if constexpr (BITS == 3) {
+#pragma unroll
+        for (int w = 0; w < 3; ++w) { c90[w] = cw0[w] >> 9; c91[w] = cw1[w] >> 9; }
+        s150 = k3_spare(cw0);
+        s151 = k3_spare(cw1);
+      }
 #pragma unroll
       for (int t = 0; t < 8; ++t) {
         uint32_t a[4];
-        frag<BITS>(cw0, t, a[0], a[2]);
-        frag<BITS>(cw1, t, a[1], a[3]);
+        if constexpr (BITS == 3) {
+          frag3m(cw0, c90, s150, t, a[0], a[2]);
+          frag3m(cw1, c91, s151, t, a[1], a[3]);
+        } else {
+          frag<BITS>(cw0, t, a[0], a[2]);
+          frag<BITS>(cw1, t, a[1], a[3]);
+        }
 #pragma unroll
         for (int j = 0; j < NJ; ++j) {
           if (t == 0) mma_16816_zc(d[j], a, xt[j][0], xt[j][1]);
@@ -1013,11 +1051,14 @@ cudaError_t launch_s_x(const CUtensorMap& tw, const CUtensorMap& tm, const GemvP
 // XS: group sums computed in the kernel (p.xsum == null) or read from p.xsum
 template <int BITS, int RT, int EPI>
 cudaError_t launch_s_e(const CUtensorMap& tw, const CUtensorMap& tm, const GemvP& p, cudaStream_t s) {
+  // INT3 always computes its own sums (its per-position offsets 1024 / 128 / 16 are not the caller's
+  // two-way split)
+  const bool own = p.xsum == nullptr || BITS == 3;
   if constexpr (RT == 2) {
     if (p.m > 8)
-      return p.xsum ? launch_s_x<BITS, RT, EPI, false, 2>(tw, tm, p, s) : launch_s_x<BITS, RT, EPI, true, 2>(tw, tm, p, s);
+      return own ? launch_s_x<BITS, RT, EPI, true, 2>(tw, tm, p, s) : launch_s_x<BITS, RT, EPI, false, 2>(tw, tm, p, s);
   }
-  return p.xsum ? launch_s_x<BITS, RT, EPI, false, 1>(tw, tm, p, s) : launch_s_x<BITS, RT, EPI, true, 1>(tw, tm, p, s);
+  return own ? launch_s_x<BITS, RT, EPI, true, 1>(tw, tm, p, s) : launch_s_x<BITS, RT, EPI, false, 1>(tw, tm, p, s);
 }
 
 template <int BITS, int RT>
