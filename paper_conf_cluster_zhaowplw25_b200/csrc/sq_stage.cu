@@ -123,12 +123,14 @@ sq_status stage_forward(const sq_layer* layers, int n_layers, int phase, const f
     const bool q = L.bits != 16;
     auto k2 = [&](const sq_qweight& w) { return gv && q && gemv_path(w.n, w.k, (int)T, w.bits) == 0 &&
                                                    !use_k2s(w.bits, w.n, w.k, (int)T); };
+    // LayerNorm's group sums (free: it holds the row) feed K2 and K2s alike
+    auto lnxs = [&](const sq_qweight& w) { return gv && q && gemv_path(w.n, w.k, (int)T, w.bits) == 0; };
     const float* xr = (l == 0) ? x_in : x_out;
     const bool copy = (l == 0 && x_in != x_out);
     // a = LN(x) (layer 0 also initialises the residual buffer x_out = x_in)
-    e = launch_layernorm_f16(xr, T, h1, a16, k2(L.qkv) ? xs : nullptr, copy ? x_in : nullptr, copy ? x_out : nullptr, s);
+    e = launch_layernorm_f16(xr, T, h1, a16, lnxs(L.qkv) ? xs : nullptr, copy ? x_in : nullptr, copy ? x_out : nullptr, s);
     if (e) break;
-    e = lin(L.qkv, a16, h1, qkv16, 3 * h1, SQ_EPI_F16, k2(L.qkv) ? xs : nullptr);
+    e = lin(L.qkv, a16, h1, qkv16, 3 * h1, SQ_EPI_F16, lnxs(L.qkv) ? xs : nullptr);
     if (e) break;
     // attention: the R12 stub attn = v = qkv[:, 2h1:3h1], or causal attention over the KV cache (f3)
     const __half* v = qkv16 + 2 * h1;
@@ -147,9 +149,9 @@ sq_status stage_forward(const sq_layer* layers, int n_layers, int phase, const f
     }
     e = lin(L.o, v, ldv, x_out, h1, SQ_EPI_F32_ACCUM, k2(L.o) ? xs : nullptr);
     if (e) break;
-    e = launch_layernorm_f16(x_out, T, h1, a16, k2(L.fc1) ? xs : nullptr, nullptr, nullptr, s);
+    e = launch_layernorm_f16(x_out, T, h1, a16, lnxs(L.fc1) ? xs : nullptr, nullptr, nullptr, s);
     if (e) break;
-    e = lin(L.fc1, a16, h1, u16, h2, L.act == 0 ? SQ_EPI_F16_RELU : SQ_EPI_F16_GELU, k2(L.fc1) ? xs : nullptr);
+    e = lin(L.fc1, a16, h1, u16, h2, L.act == 0 ? SQ_EPI_F16_RELU : SQ_EPI_F16_GELU, lnxs(L.fc1) ? xs : nullptr);
     if (e) break;
     if (k2(L.fc2)) {
       e = launch_xsum(u16, h2, T, h2, xs, s);
@@ -258,13 +260,15 @@ sq_status stage_forward_tp(const sq_layer* sh, int n_layers, int n_sets, sq_comm
     const bool q = L0.bits != 16;
     auto k2 = [&](const sq_qweight& w) { return gv && q && gemv_path(w.n, w.k, (int)T, w.bits) == 0 &&
                                                    !use_k2s(w.bits, w.n, w.k, (int)T); };
+    // LayerNorm's group sums (free: it holds the row) feed K2 and K2s alike
+    auto lnxs = [&](const sq_qweight& w) { return gv && q && gemv_path(w.n, w.k, (int)T, w.bits) == 0; };
     const float* xr = (l == 0) ? x_in : x_out;
     const bool copy = (l == 0 && x_in != x_out);
-    e = launch_layernorm_f16(xr, T, h1, a16, k2(L0.qkv) ? xsa : nullptr, copy ? x_in : nullptr, copy ? x_out : nullptr, s);
+    e = launch_layernorm_f16(xr, T, h1, a16, lnxs(L0.qkv) ? xsa : nullptr, copy ? x_in : nullptr, copy ? x_out : nullptr, s);
     if (e) break;
     for (int r = 0; r < n_sets && !e; ++r) {
       const sq_layer& L = sh[r * n_layers + l];
-      e = lin(L.qkv, a16, h1, qkv16, 3 * h1s, SQ_EPI_F16, k2(L.qkv) ? xsa : nullptr);
+      e = lin(L.qkv, a16, h1, qkv16, 3 * h1s, SQ_EPI_F16, lnxs(L.qkv) ? xsa : nullptr);
       if (e) break;
       const __half* v = qkv16 + 2 * h1s;
       int64_t ldv = 3 * h1s;
@@ -282,11 +286,11 @@ sq_status stage_forward_tp(const sq_layer* sh, int n_layers, int n_sets, sq_comm
       e = lin(L.o, v, ldv, x_out, h1, SQ_EPI_F32_ACCUM, k2(L.o) ? xsb : nullptr);
     }
     if (e || (st = reduce())) break;
-    e = launch_layernorm_f16(x_out, T, h1, a16, k2(L0.fc1) ? xsa : nullptr, nullptr, nullptr, s);
+    e = launch_layernorm_f16(x_out, T, h1, a16, lnxs(L0.fc1) ? xsa : nullptr, nullptr, nullptr, s);
     if (e) break;
     for (int r = 0; r < n_sets && !e; ++r) {
       const sq_layer& L = sh[r * n_layers + l];
-      e = lin(L.fc1, a16, h1, u16, h2s, L.act == 0 ? SQ_EPI_F16_RELU : SQ_EPI_F16_GELU, k2(L.fc1) ? xsa : nullptr);
+      e = lin(L.fc1, a16, h1, u16, h2s, L.act == 0 ? SQ_EPI_F16_RELU : SQ_EPI_F16_GELU, lnxs(L.fc1) ? xsa : nullptr);
       if (e) break;
       if (k2(L.fc2) && (e = launch_xsum(u16, h2s, T, h2s, xsb, s))) break;
       if (zero_first && (e = cudaMemsetAsync(x_out, 0, (size_t)T * h1 * sizeof(float), s))) break;
