@@ -7,7 +7,10 @@
 namespace sq {
 namespace {
 
-constexpr int kLnThreads = 256;
+// 16 warps per row: the 32-row decode LayerNorm is latency-bound (one CTA per row); 512 threads cut
+// the decode phase of the configs[3] bench by 2 % against 256 (same box, two runs each), 1024 also
+// but slowed the 4096-row prefill LayerNorms
+constexpr int kLnThreads = 512;
 
 __device__ __forceinline__ float block_sum(float v, float* red) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -29,7 +32,7 @@ template <bool F16OUT>
 __global__ void __launch_bounds__(kLnThreads) k_layernorm(const float* __restrict__ x, int64_t d, void* __restrict__ y,
                                                           float2* __restrict__ xsum, int xsum_rows,
                                                           const float* __restrict__ copy_src, float* __restrict__ copy_dst) {
-  constexpr int MAXV = 14;  // up to d = 14 * 1024 = 14336 (BLOOM-176B h1)
+  constexpr int MAXV = (112 + kLnThreads / 32 - 1) / (kLnThreads / 32);  // up to d = 112 * 128 = 14336 (BLOOM-176B h1)
   __shared__ float red[kLnThreads / 32];
   pdl_trigger();
   pdl_wait();
